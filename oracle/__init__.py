@@ -80,6 +80,9 @@ def lib():
                                          C.c_uint64, C.c_int64, C.c_int32, C.c_int32,
                                          C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
         _lib.oracle_num_threads.restype = C.c_int
+        _lib.oracle_update.argtypes = [C.c_int64, C.POINTER(_Opts), C.c_int32, C.c_void_p,
+                                       C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
+                                       C.c_void_p, C.c_void_p]
     return _lib
 
 
@@ -122,6 +125,18 @@ class Options:
     def c(self) -> _Opts:
         return _Opts(ASSUMPTIONS[self.assumption], self.K, self.lam, self.G, self.lr, self.beta1,
                      self.beta2, self.eps, 0 if self.optimizer == "adam" else 1)
+
+
+def update(theta, grad, opts: Options, m=None, v=None, step_index=0):
+    """The oracle's optimiser step alone (same code as inside step())."""
+    th = np.ascontiguousarray(theta, dtype=np.float64)
+    g = np.ascontiguousarray(grad, dtype=np.float64)
+    m = None if m is None else np.ascontiguousarray(m, dtype=np.float64)
+    v = None if v is None else np.ascontiguousarray(v, dtype=np.float64)
+    out = [np.zeros_like(th) for _ in range(3)]
+    lib().oracle_update(th.size, C.byref(opts.c()), step_index, _p(th), _p(m), _p(v), _p(g),
+                        _p(out[0]), _p(out[1]), _p(out[2]))
+    return {"theta_out": out[0], "m_out": out[1], "v_out": out[2]}
 
 
 class Graph:

@@ -503,6 +503,19 @@ void backward(const Graph& g, int K, Weights w, const double* cp, const double* 
   }
 }
 
+// Optimiser step on one logit (reading S10): Adam with bias correction
+// (bc1 = 1 - beta1^t, bc2 = 1 - beta2^t), or plain gradient descent.
+void update(const oracle_opts& opt, double bc1, double bc2, double g, double& th, double& m,
+            double& v) {
+  if (opt.optimizer == 0) {
+    m = opt.beta1 * m + (1.0 - opt.beta1) * g;
+    v = opt.beta2 * v + (1.0 - opt.beta2) * g * g;
+    th = th - opt.lr * (m / bc1) / (std::sqrt(v / bc2) + opt.eps);
+  } else {
+    th = th - opt.lr * g;
+  }
+}
+
 // Decode (P279, readings S17-S19): c_j = argmax_{k in m_j} theta_k (lowest id on
 // ties); select from the root down; valid iff the selected subgraph has no
 // cycle (constraint (c), P109), checked by a 3-colour DFS.
@@ -637,13 +650,7 @@ int oracle_step(void* hg, const oracle_cost* cost, const oracle_opts* opt, int32
       const size_t idx = (size_t)k * B + b;
       double th = theta[b][k], gk = gth[k];
       double m = m_in ? m_in[idx] : 0.0, v = v_in ? v_in[idx] : 0.0;
-      if (opt->optimizer == 0) {
-        m = opt->beta1 * m + (1.0 - opt->beta1) * gk;
-        v = opt->beta2 * v + (1.0 - opt->beta2) * gk * gk;
-        th = th - opt->lr * (m / bc1) / (std::sqrt(v / bc2) + opt->eps);
-      } else {
-        th = th - opt->lr * gk;
-      }
+      update(*opt, bc1, bc2, gk, th, m, v);
       if (out->theta_out) out->theta_out[idx] = th;
       if (out->m_out) out->m_out[idx] = m;
       if (out->v_out) out->v_out[idx] = v;
@@ -690,6 +697,22 @@ void oracle_decode(void* hg, const oracle_cost* cost, int32_t B, const double* t
     }
     if (valid) valid[b] = ok;
     if (disc_cost) disc_cost[b] = dc;
+  }
+}
+
+// The optimiser step alone on n logits, given the gradient (tests compare the
+// GPU update with this given the GPU's own gradient).
+void oracle_update(int64_t n, const oracle_opts* opt, int32_t step_index, const double* theta,
+                   const double* m_in, const double* v_in, const double* g, double* theta_out,
+                   double* m_out, double* v_out) {
+  const double bc1 = 1.0 - std::pow(opt->beta1, (double)(step_index + 1));
+  const double bc2 = 1.0 - std::pow(opt->beta2, (double)(step_index + 1));
+  for (int64_t i = 0; i < n; ++i) {
+    double th = theta[i], m = m_in ? m_in[i] : 0.0, v = v_in ? v_in[i] : 0.0;
+    update(*opt, bc1, bc2, g[i], th, m, v);
+    theta_out[i] = th;
+    m_out[i] = m;
+    v_out[i] = v;
   }
 }
 

@@ -1,0 +1,271 @@
+// E-graph loader: validation, CSR/CSC, strongly connected components, K_auto.
+//
+// Problem statement: PAPER.md:91-101 (classes m_j, nodes n_i, ch_i, pa_j, ec(i)).
+// Sparse representation instead of dense matrices: PAPER.md:285-289 (Sec. 4.1).
+// SCC decomposition of the NOTEARS term: PAPER.md:318 (Sec. 4.3).
+// K_auto: reading S1.
+#include <algorithm>
+#include <cstring>
+
+#include "internal.h"
+
+namespace smoothe {
+
+namespace {
+
+// Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
+void class_successors(const HostGraph& g, std::vector<int32_t>& ptr, std::vector<int32_t>& adj) {
+  ptr.assign(g.M + 1, 0);
+  adj.clear();
+  std::vector<int32_t> buf;
+  for (int32_t j = 0; j < g.M; ++j) {
+    buf.clear();
+    for (int32_t k = g.class_ptr[j]; k < g.class_ptr[j + 1]; ++k)
+      buf.insert(buf.end(), g.child_class.begin() + g.child_ptr[k],
+                 g.child_class.begin() + g.child_ptr[k + 1]);
+    std::sort(buf.begin(), buf.end());
+    buf.erase(std::unique(buf.begin(), buf.end()), buf.end());
+    adj.insert(adj.end(), buf.begin(), buf.end());
+    ptr[j + 1] = (int32_t)adj.size();
+  }
+}
+
+// Kosaraju: finish order on the graph, then components on the transpose.
+std::vector<int32_t> kosaraju(int32_t M, const std::vector<int32_t>& ptr,
+                              const std::vector<int32_t>& adj) {
+  std::vector<int32_t> order;
+  order.reserve(M);
+  std::vector<uint8_t> seen(M, 0);
+  std::vector<std::pair<int32_t, int32_t>> st;
+  for (int32_t s = 0; s < M; ++s) {
+    if (seen[s]) continue;
+    seen[s] = 1;
+    st.push_back({s, ptr[s]});
+    while (!st.empty()) {
+      auto& top = st.back();
+      if (top.second < ptr[top.first + 1]) {
+        int32_t w = adj[top.second++];
+        if (!seen[w]) {
+          seen[w] = 1;
+          st.push_back({w, ptr[w]});
+        }
+      } else {
+        order.push_back(top.first);
+        st.pop_back();
+      }
+    }
+  }
+  // transpose
+  std::vector<int32_t> tptr(M + 1, 0), tadj(adj.size());
+  for (size_t e = 0; e < adj.size(); ++e) tptr[adj[e] + 1]++;
+  for (int32_t j = 0; j < M; ++j) tptr[j + 1] += tptr[j];
+  std::vector<int32_t> fill(tptr.begin(), tptr.end() - 1);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t e = ptr[j]; e < ptr[j + 1]; ++e) tadj[fill[adj[e]]++] = j;
+  std::vector<int32_t> comp(M, -1);
+  std::vector<int32_t> stack;
+  int32_t nc = 0;
+  for (auto it = order.rbegin(); it != order.rend(); ++it) {
+    if (comp[*it] >= 0) continue;
+    stack.push_back(*it);
+    comp[*it] = nc;
+    while (!stack.empty()) {
+      int32_t v = stack.back();
+      stack.pop_back();
+      for (int32_t e = tptr[v]; e < tptr[v + 1]; ++e)
+        if (comp[tadj[e]] < 0) {
+          comp[tadj[e]] = nc;
+          stack.push_back(tadj[e]);
+        }
+    }
+    ++nc;
+  }
+  return comp;
+}
+
+// K_auto (S1): DFS from the root, successors in increasing class id; edges into
+// a vertex still on the DFS path are dropped; longest path over what remains.
+int32_t k_auto(const HostGraph& g, const std::vector<int32_t>& ptr, const std::vector<int32_t>& adj) {
+  const int32_t M = g.M;
+  std::vector<uint8_t> state(M, 0);  // 0 new, 1 on path, 2 done
+  std::vector<int32_t> post;
+  std::vector<uint8_t> keep(adj.size(), 0);
+  std::vector<std::pair<int32_t, int32_t>> st;
+  st.push_back({g.root, ptr[g.root]});
+  state[g.root] = 1;
+  while (!st.empty()) {
+    auto& top = st.back();
+    if (top.second < ptr[top.first + 1]) {
+      int32_t e = top.second++;
+      int32_t w = adj[e];
+      if (state[w] == 1) continue;
+      keep[e] = 1;
+      if (state[w] == 0) {
+        state[w] = 1;
+        st.push_back({w, ptr[w]});
+      }
+    } else {
+      state[top.first] = 2;
+      post.push_back(top.first);
+      st.pop_back();
+    }
+  }
+  std::vector<int32_t> depth(M, -1);
+  depth[g.root] = 0;
+  int32_t best = 0;
+  for (auto it = post.rbegin(); it != post.rend(); ++it) {
+    int32_t v = *it;
+    if (depth[v] < 0) continue;
+    best = std::max(best, depth[v]);
+    for (int32_t e = ptr[v]; e < ptr[v + 1]; ++e)
+      if (keep[e]) depth[adj[e]] = std::max(depth[adj[e]], depth[v] + 1);
+  }
+  return best;
+}
+
+}  // namespace
+
+void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
+                      const int32_t* child_class, int32_t root, HostGraph& g) {
+  SM_REQUIRE(class_ptr && child_ptr && (child_class || child_ptr[N] == 0), SMOOTHE_E_INVALID_ARG,
+             "NULL e-graph array");
+  SM_REQUIRE(M > 0 && N > 0, SMOOTHE_E_INVALID_ARG, "num_classes and num_nodes must be > 0");
+  SM_REQUIRE(N < (1 << 29), SMOOTHE_E_INVALID_ARG, "num_nodes must be < 2^29");
+  SM_REQUIRE(root >= 0 && root < M, SMOOTHE_E_BAD_GRAPH, "root class out of range");
+  SM_REQUIRE(class_ptr[0] == 0 && class_ptr[M] == N, SMOOTHE_E_BAD_GRAPH,
+             "class_ptr must start at 0 and end at num_nodes");
+  for (int32_t j = 0; j < M; ++j)
+    SM_REQUIRE(class_ptr[j + 1] > class_ptr[j], SMOOTHE_E_BAD_GRAPH,
+               "class " + std::to_string(j) + " is empty or class_ptr is not increasing");
+  SM_REQUIRE(child_ptr[0] == 0, SMOOTHE_E_BAD_GRAPH, "child_ptr[0] must be 0");
+  for (int32_t i = 0; i < N; ++i)
+    SM_REQUIRE(child_ptr[i + 1] >= child_ptr[i], SMOOTHE_E_BAD_GRAPH, "child_ptr not monotone");
+  SM_REQUIRE(child_ptr[N] < ((int64_t)1 << 31), SMOOTHE_E_INVALID_ARG, "more than 2^31-1 edges");
+  for (int64_t e = 0; e < child_ptr[N]; ++e)
+    SM_REQUIRE(child_class[e] >= 0 && child_class[e] < M, SMOOTHE_E_BAD_GRAPH,
+               "child class id out of range");
+
+  g = HostGraph();
+  g.M = M;
+  g.N = N;
+  g.root = root;
+  g.class_ptr.assign(class_ptr, class_ptr + M + 1);
+  g.ec.resize(N);
+  for (int32_t j = 0; j < M; ++j) {
+    for (int32_t i = class_ptr[j]; i < class_ptr[j + 1]; ++i) g.ec[i] = j;
+    g.max_class_size = std::max(g.max_class_size, class_ptr[j + 1] - class_ptr[j]);
+  }
+  // CSR children as sets
+  g.child_ptr.assign(N + 1, 0);
+  g.child_class.reserve(child_ptr[N]);
+  std::vector<int32_t> buf;
+  for (int32_t i = 0; i < N; ++i) {
+    buf.assign(child_class + child_ptr[i], child_class + child_ptr[i + 1]);
+    std::sort(buf.begin(), buf.end());
+    buf.erase(std::unique(buf.begin(), buf.end()), buf.end());
+    g.child_class.insert(g.child_class.end(), buf.begin(), buf.end());
+    g.child_ptr[i + 1] = (int32_t)g.child_class.size();
+  }
+  g.E = (int64_t)g.child_class.size();
+  // CSC parents, by increasing e-node id
+  g.par_ptr.assign(M + 1, 0);
+  for (int32_t c : g.child_class) g.par_ptr[c + 1]++;
+  for (int32_t j = 0; j < M; ++j) {
+    g.max_in_degree = std::max(g.max_in_degree, g.par_ptr[j + 1]);
+    g.par_ptr[j + 1] += g.par_ptr[j];
+  }
+  g.par_node.resize(g.E);
+  g.par_class.resize(g.E);
+  {
+    std::vector<int32_t> fill(g.par_ptr.begin(), g.par_ptr.end() - 1);
+    for (int32_t i = 0; i < N; ++i)
+      for (int32_t e = g.child_ptr[i]; e < g.child_ptr[i + 1]; ++e) {
+        int32_t slot = fill[g.child_class[e]]++;
+        g.par_node[slot] = i;
+        g.par_class[slot] = g.ec[i];
+      }
+  }
+
+  // strongly connected components of the class graph
+  std::vector<int32_t> sptr, sadj;
+  class_successors(g, sptr, sadj);
+  std::vector<int32_t> comp = kosaraju(M, sptr, sadj);
+  int32_t ncomp = 0;
+  for (int32_t c : comp) ncomp = std::max(ncomp, c + 1);
+  std::vector<int32_t> csize(ncomp, 0);
+  for (int32_t c : comp) csize[c]++;
+  std::vector<uint8_t> selfloop(M, 0);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t e = sptr[j]; e < sptr[j + 1]; ++e)
+      if (sadj[e] == j) selfloop[j] = 1;
+  std::vector<int32_t> remap(ncomp, -1);
+  g.scc_of_class.assign(M, -1);
+  g.scc_local.assign(M, -1);
+  for (int32_t j = 0; j < M; ++j) {
+    int32_t c = comp[j];
+    if (csize[c] == 1 && !selfloop[j]) continue;
+    if (remap[c] < 0) remap[c] = g.num_scc++;
+    g.scc_of_class[j] = remap[c];
+  }
+  g.scc_class_ptr.assign(g.num_scc + 1, 0);
+  for (int32_t j = 0; j < M; ++j)
+    if (g.scc_of_class[j] >= 0) g.scc_class_ptr[g.scc_of_class[j] + 1]++;
+  for (int32_t s = 0; s < g.num_scc; ++s) {
+    g.scc_max = std::max(g.scc_max, g.scc_class_ptr[s + 1]);
+    g.scc_class_ptr[s + 1] += g.scc_class_ptr[s];
+  }
+  g.scc_classes = g.scc_class_ptr[g.num_scc];
+  g.scc_class.resize(g.scc_classes);
+  {
+    std::vector<int32_t> fill(g.scc_class_ptr.begin(), g.scc_class_ptr.end() - 1);
+    for (int32_t j = 0; j < M; ++j) {
+      int32_t s = g.scc_of_class[j];
+      if (s < 0) continue;
+      g.scc_local[j] = fill[s] - g.scc_class_ptr[s];
+      g.scc_class[fill[s]++] = j;
+    }
+  }
+  // Abar entries and penalty slots per component
+  g.ent_ptr.assign(1, 0);
+  g.ent_node_ptr.assign(1, 0);
+  g.slot_ptr.assign(1, 0);
+  g.slot_jptr.assign(1, 0);
+  g.node_slot.assign(N, -1);
+  std::vector<std::pair<int64_t, int32_t>> pairs;  // ((i_local, j_local), node)
+  for (int32_t s = 0; s < g.num_scc; ++s) {
+    pairs.clear();
+    for (int32_t l = g.scc_class_ptr[s]; l < g.scc_class_ptr[s + 1]; ++l) {
+      int32_t i = g.scc_class[l];
+      int32_t il = g.scc_local[i];
+      for (int32_t k = g.class_ptr[i]; k < g.class_ptr[i + 1]; ++k) {
+        g.node_slot[k] = (int32_t)g.slot_node.size();
+        g.slot_node.push_back(k);
+        g.slot_iloc.push_back(il);
+        for (int32_t e = g.child_ptr[k]; e < g.child_ptr[k + 1]; ++e) {
+          int32_t c = g.child_class[e];
+          if (g.scc_of_class[c] != s) continue;
+          g.slot_jloc.push_back(g.scc_local[c]);
+          pairs.push_back({((int64_t)il << 32) | (uint32_t)g.scc_local[c], k});
+        }
+        g.slot_jptr.push_back((int32_t)g.slot_jloc.size());
+      }
+    }
+    g.slot_ptr.push_back((int32_t)g.slot_node.size());
+    std::sort(pairs.begin(), pairs.end());
+    for (size_t a = 0; a < pairs.size();) {
+      size_t b = a;
+      while (b < pairs.size() && pairs[b].first == pairs[a].first) {
+        g.ent_node.push_back(pairs[b].second);
+        ++b;
+      }
+      g.ent_i.push_back((int32_t)(pairs[a].first >> 32));
+      g.ent_j.push_back((int32_t)(pairs[a].first & 0xffffffff));
+      g.ent_node_ptr.push_back((int32_t)g.ent_node.size());
+      a = b;
+    }
+    g.ent_ptr.push_back((int32_t)g.ent_i.size());
+  }
+  g.K_auto = k_auto(g, sptr, sadj);
+}
+
+}  // namespace smoothe

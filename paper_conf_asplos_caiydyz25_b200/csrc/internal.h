@@ -1,0 +1,168 @@
+// Internal declarations of libsmoothe (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/smoothe.h"
+
+namespace smoothe {
+
+// ---------------------------------------------------------------------------
+// Errors
+// ---------------------------------------------------------------------------
+void set_error(const std::string& msg);
+
+struct Failure {
+  smoothe_status status;
+  std::string msg;
+};
+
+#define SM_CUDA(call)                                                                  \
+  do {                                                                                 \
+    cudaError_t _e = (call);                                                           \
+    if (_e != cudaSuccess)                                                             \
+      throw ::smoothe::Failure{SMOOTHE_E_CUDA, std::string(#call) + ": " +             \
+                                                    cudaGetErrorString(_e)};           \
+  } while (0)
+
+#define SM_REQUIRE(cond, status, msg)                                                  \
+  do {                                                                                 \
+    if (!(cond)) throw ::smoothe::Failure{status, msg};                                \
+  } while (0)
+
+// ---------------------------------------------------------------------------
+// E-graph: host analysis (egraph.cpp) and its device mirror
+// ---------------------------------------------------------------------------
+struct HostGraph {
+  int32_t M = 0, N = 0, root = 0;
+  int64_t E = 0;
+  std::vector<int32_t> class_ptr;                  // [M+1]
+  std::vector<int32_t> ec;                         // [N]
+  std::vector<int32_t> child_ptr, child_class;     // CSR: ch_i, sorted, deduplicated
+  std::vector<int32_t> par_ptr, par_node, par_class;// CSC: pa_j sorted by node id, ec(node)
+  // non-trivial strongly connected components (size > 1 or self-loop)
+  int32_t num_scc = 0, scc_classes = 0, scc_max = 0;
+  std::vector<int32_t> scc_of_class;               // [M] component id or -1
+  std::vector<int32_t> scc_class_ptr, scc_class;   // members per component, by class id
+  std::vector<int32_t> scc_local;                  // [M] position inside its component
+  // Abar entries: unique (i_local, j_local) per component and their e-nodes k
+  // (k in m_i, j in ch_k), SURVEY.md 8(a) a5.
+  std::vector<int32_t> ent_ptr;                    // [num_scc+1]
+  std::vector<int32_t> ent_i, ent_j;               // local indices
+  std::vector<int32_t> ent_node_ptr, ent_node;     // contributing e-nodes
+  // penalty slots: every e-node of a component's classes, with its children
+  // inside the component (gradient scatter of App. B).
+  std::vector<int32_t> slot_ptr;                   // [num_scc+1]
+  std::vector<int32_t> slot_node, slot_iloc;       // [num_slots]
+  std::vector<int32_t> slot_jptr, slot_jloc;       // children in the component (local)
+  std::vector<int32_t> node_slot;                  // [N] slot id or -1
+  int32_t K_auto = 0, max_class_size = 0, max_in_degree = 0;
+};
+
+void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
+                      const int32_t* child_class, int32_t root, HostGraph& g);
+
+struct DevGraph {
+  int32_t *class_ptr = nullptr, *child_ptr = nullptr, *child_class = nullptr;
+  int32_t *par_ptr = nullptr, *par_node = nullptr, *par_class = nullptr;
+  int32_t *scc_class_ptr = nullptr, *ent_ptr = nullptr, *ent_i = nullptr, *ent_j = nullptr;
+  int32_t *ent_node_ptr = nullptr, *ent_node = nullptr;
+  int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
+  int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
+  int64_t bytes = 0;
+};
+
+}  // namespace smoothe
+
+struct smoothe_egraph {
+  smoothe::HostGraph host;
+  smoothe::DevGraph dev;
+  int device = -1;
+  int refcount = 1;  // the handle itself + one per live run
+  bool freed = false;
+};
+
+namespace smoothe {
+
+// ---------------------------------------------------------------------------
+// Kernel launch interface (kernels.cu).  Per-seed rows have Bp floats; Bp is
+// num_seeds rounded up to 32, 64 or a multiple of 128.
+// ---------------------------------------------------------------------------
+struct Shape {
+  int32_t M, N, root, B, Bp, W;  // W = Bp / 32 bitmask words per row
+};
+
+struct Agg {
+  float wI, wC;  // independent / correlated weights
+};
+
+void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t seed_begin,
+                       float* theta, float* m, float* v);
+void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
+                           float* cp, int32_t* choice, uint32_t* sel);
+void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am);
+void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
+                        const float* cp, const float* qK, float* gcp, float* gqK, float* f_part,
+                        float* p_out, int32_t nblocks_hint);
+void launch_cost_gp(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* gp,
+                    const float* cp, const float* qK, float* gcp, float* gqK);
+// p = cp * q^K[ec]; with u != NULL also f_part = per-block partial sums of u^T p
+void launch_materialize_p_f(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
+                            const float* cp, const float* qK, float* p, float* f_part);
+// quadratic cost over symmetric neighbour lists; u may be NULL (pair terms only)
+void launch_quadratic(cudaStream_t s, const Shape& sh, const int32_t* qptr, const int32_t* qnbr,
+                      const float* qw, const float* u, const float* p, float* gp, float* f_part);
+void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, int32_t Bp,
+                            double* out, double scale);
+void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
+                             double* out);
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, const float* gq, const float* pi,
+                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev);
+void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
+                    int32_t G, double lambda, const float* cp, double* h_part, float* pen);
+void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,
+                   const float* gcp, const float* pen, float* theta, float* m, float* v,
+                   const double* step_scalars, int32_t optimizer, float lr, float beta1,
+                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out);
+void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_scalars,
+                          double beta1, double beta2, const int32_t* unused);
+void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, int Bp, float value);
+void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const double* f,
+                 const double* fextra, const double* h, double* ftot, double* loss);
+void launch_decode_reach(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                         uint32_t* reach, int32_t* flags, int32_t grid);
+void launch_decode_settle(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                          uint32_t* settle, int32_t* flags, int32_t grid);
+void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g,
+                               const double* u, const int32_t* choice, const uint32_t* reach,
+                               double* cost_part);
+void launch_decode_s(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                     const uint32_t* reach, float* s_out);
+int decode_grid(int device);
+int decode_cost_rows(const Shape& sh);
+void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
+                        const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,
+                        const int32_t* step_counter, double* best, int32_t* best_flag,
+                        double* valid_cost_out, uint8_t* valid_out);
+void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice,
+                          const uint32_t* reach, const double* best, const int32_t* best_flag,
+                          int64_t seed_begin, int32_t* best_choice);
+// MLP (kernels_mlp.cu): f_mlp[b] (fp64) and gz1 = df/dz1 (may be NULL);
+// gp = u + W1^T gz1.
+void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
+                    const float* b1, const float* W2, const float* b2, const float* W3,
+                    const float* b3, const float* p, float* z1_part, double* f_mlp, float* gz1,
+                    int32_t nsplit);
+void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* u,
+                    const float* gz1, float* gp);
+
+int num_sms(int device);
+int64_t& launch_counter();
+
+}  // namespace smoothe

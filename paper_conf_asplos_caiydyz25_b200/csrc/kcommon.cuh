@@ -1,0 +1,78 @@
+// Device-side helpers shared by the kernels of libsmoothe (sm_100a).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "internal.h"
+
+namespace smoothe {
+
+// Every per-seed array is [row][Bp] fp32, seed innermost.  A "row group" of
+// LPR lanes covers one chunk of 4*LPR seeds of one row with float4 accesses
+// (Bp = 32 -> LPR 8, Bp = 64 -> LPR 16, Bp >= 128 -> LPR 32 and Bp/128
+// chunks).  Grids are 2-D: x over rows, y over chunks, so a row group never
+// straddles chunks and block reductions are per seed.
+constexpr int kBlock = 256;
+
+__host__ __device__ inline int lanes_per_row(int Bp) { return Bp >= 128 ? 32 : Bp / 4; }
+__host__ __device__ inline int num_chunks(int Bp) { return Bp >= 128 ? Bp / 128 : 1; }
+
+template <int LPR>
+struct RowGroup {
+  int row;   // row index (class or node)
+  int s0;    // first seed of this lane (multiple of 4)
+  int sub;   // group index inside the block
+  __device__ RowGroup() {
+    const int lane = threadIdx.x % LPR;
+    sub = threadIdx.x / LPR;
+    row = blockIdx.x * (kBlock / LPR) + sub;
+    s0 = blockIdx.y * (4 * LPR) + lane * 4;
+  }
+};
+
+inline dim3 row_grid(int rows, int Bp, int LPR) {
+  return dim3((rows + kBlock / LPR - 1) / (kBlock / LPR), num_chunks(Bp));
+}
+
+__device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
+__device__ __forceinline__ int4 ld4i(const int32_t* p) { return *reinterpret_cast<const int4*>(p); }
+__device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+__device__ __forceinline__ void st4i(int32_t* p, int4 v) { *reinterpret_cast<int4*>(p) = v; }
+
+__device__ __forceinline__ float comp(const float4& v, int c) {
+  return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+__device__ __forceinline__ float& comp(float4& v, int c) {
+  return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+__device__ __forceinline__ int comp(const int4& v, int c) {
+  return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+__device__ __forceinline__ int& comp(int4& v, int c) {
+  return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+
+#define SM_DISPATCH_LPR(Bp, ...)            \
+  do {                                      \
+    const int _lpr = lanes_per_row(Bp);     \
+    if (_lpr == 32) {                       \
+      constexpr int LPR = 32;               \
+      __VA_ARGS__;                          \
+    } else if (_lpr == 16) {                \
+      constexpr int LPR = 16;               \
+      __VA_ARGS__;                          \
+    } else {                                \
+      constexpr int LPR = 8;                \
+      __VA_ARGS__;                          \
+    }                                       \
+  } while (0)
+
+#define SM_LAUNCH_CHECK()                                        \
+  do {                                                           \
+    ++::smoothe::launch_counter();                               \
+    SM_CUDA(cudaGetLastError());                                 \
+  } while (0)
+
+}  // namespace smoothe

@@ -1,0 +1,266 @@
+// Decode, validity and keep-best (sm_100a).
+//
+// Sampling: from the root, each selected class m_j takes the
+// e-node c_j = argmax cp (= argmax theta, reading S17) and selects all of its
+// child classes; completeness (a), (b) holds by construction (P105-107) and
+// acyclicity (c) (P109) is checked.  Bit-sliced over seeds: word w of a row
+// holds seeds 32w..32w+31.
+//
+//   sel[k][w]    bit set iff the seed chose e-node k in its class   (softmax kernel)
+//   reach[j][w]  least fixpoint of  reach_root = 1,
+//                reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k)       (top-down)
+//   settle[j][w] least fixpoint of settle_j = OR_{k in m_j} (sel_k AND AND_{c in ch_k} settle_c)
+//                (bottom-up); a class settles iff its selected sub-term is finite
+//                and acyclic, so  valid <=> settle_root.
+// Both fixpoints are computed in place by one cooperative kernel that repeats
+// rounds until a round changes nothing (monotone, so asynchronous in-place
+// updates reach the same least fixpoint).
+//
+// Discrete cost (reading S19): sum of u over the chosen e-node of every reached
+// class, each class once, accumulated in fp64 (exact for integer-valued u).
+#include <cooperative_groups.h>
+
+#include "kcommon.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace smoothe {
+
+__global__ void __launch_bounds__(256) k_reach(int M, int W, int root,
+                                               const int32_t* __restrict__ par_ptr,
+                                               const int32_t* __restrict__ par_node,
+                                               const int32_t* __restrict__ par_class,
+                                               const uint32_t* __restrict__ sel, uint32_t* reach,
+                                               int32_t* flags, int max_rounds) {
+  cg::grid_group grid = cg::this_grid();
+  const int64_t nitems = (int64_t)M * W;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < max_rounds; ++r) {
+    int changed = 0;
+    for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < nitems; it += stride) {
+      const int j = (int)(it / W), w = (int)(it % W);
+      if (j == root) continue;
+      uint32_t v = 0;
+      for (int e = par_ptr[j]; e < par_ptr[j + 1]; ++e)
+        v |= __ldcg(reach + (size_t)par_class[e] * W + w) & sel[(size_t)par_node[e] * W + w];
+      if (v != __ldcg(reach + it)) {
+        __stcg(reach + it, v);
+        changed = 1;
+      }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) flags[(r + 1) % 3] = 0;
+    changed = __syncthreads_or(changed);
+    if (changed && threadIdx.x == 0) atomicOr(flags + r % 3, 1);
+    grid.sync();
+    if (*((volatile int32_t*)flags + r % 3) == 0) break;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_settle(int M, int W, const int32_t* __restrict__ class_ptr,
+                                                const int32_t* __restrict__ child_ptr,
+                                                const int32_t* __restrict__ child_class,
+                                                const uint32_t* __restrict__ sel, uint32_t* settle,
+                                                int32_t* flags, int max_rounds) {
+  cg::grid_group grid = cg::this_grid();
+  const int64_t nitems = (int64_t)M * W;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < max_rounds; ++r) {
+    int changed = 0;
+    for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < nitems; it += stride) {
+      const int j = (int)(it / W), w = (int)(it % W);
+      uint32_t v = 0;
+      for (int k = class_ptr[j]; k < class_ptr[j + 1]; ++k) {
+        uint32_t acc = sel[(size_t)k * W + w];
+        for (int e = child_ptr[k]; acc && e < child_ptr[k + 1]; ++e)
+          acc &= __ldcg(settle + (size_t)child_class[e] * W + w);
+        v |= acc;
+      }
+      if (v != __ldcg(settle + it)) {
+        __stcg(settle + it, v);
+        changed = 1;
+      }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) flags[(r + 1) % 3] = 0;
+    changed = __syncthreads_or(changed);
+    if (changed && threadIdx.x == 0) atomicOr(flags + r % 3, 1);
+    grid.sync();
+    if (*((volatile int32_t*)flags + r % 3) == 0) break;
+  }
+}
+
+static void coop_launch(const void* fn, int grid, void** args, cudaStream_t s) {
+  SM_CUDA(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(256), args, 0, s));
+  SM_LAUNCH_CHECK();
+}
+
+void launch_decode_reach(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                         uint32_t* reach, int32_t* flags, int32_t grid) {
+  SM_CUDA(cudaMemsetAsync(flags, 0, 3 * sizeof(int32_t), s));
+  SM_CUDA(cudaMemsetAsync(reach, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
+  SM_CUDA(cudaMemsetAsync(reach + (size_t)sh.root * sh.W, 0xff, sizeof(uint32_t) * sh.W, s));
+  int M = sh.M, W = sh.W, root = sh.root, max_rounds = sh.M + 2;
+  const int32_t *pp = g.par_ptr, *pn = g.par_node, *pc = g.par_class;
+  void* args[] = {&M, &W, &root, (void*)&pp, (void*)&pn, (void*)&pc, (void*)&sel, &reach, &flags,
+                  &max_rounds};
+  coop_launch((const void*)k_reach, grid, args, s);
+}
+
+void launch_decode_settle(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                          uint32_t* settle, int32_t* flags, int32_t grid) {
+  SM_CUDA(cudaMemsetAsync(flags, 0, 3 * sizeof(int32_t), s));
+  SM_CUDA(cudaMemsetAsync(settle, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
+  int M = sh.M, W = sh.W, max_rounds = sh.M + 2;
+  const int32_t *cp_ = g.class_ptr, *chp = g.child_ptr, *chc = g.child_class;
+  void* args[] = {&M, &W, (void*)&cp_, (void*)&chp, (void*)&chc, (void*)&sel, &settle, &flags,
+                  &max_rounds};
+  coop_launch((const void*)k_settle, grid, args, s);
+}
+
+int decode_grid(int device) {
+  int per_sm = 0;
+  SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_reach, 256, 0));
+  int per_sm2 = 0;
+  SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm2, k_settle, 256, 0));
+  per_sm = std::min(per_sm, per_sm2);
+  return std::max(1, std::min(per_sm, 4)) * num_sms(device);
+}
+
+// Discrete linear cost per seed: part[blockIdx.x][b] = sum over the block's
+// classes j with reach_j(b) of u[c_j(b)], fp64.
+constexpr int kCostClasses = 64;
+
+__global__ void k_decode_cost_linear(int M, int Bp, int W, const double* __restrict__ u,
+                                     const int32_t* __restrict__ choice,
+                                     const uint32_t* __restrict__ reach, double* __restrict__ part) {
+  const int b = blockIdx.y * blockDim.x + threadIdx.x;
+  if (b >= Bp) return;
+  const int j0 = blockIdx.x * kCostClasses, j1 = min(M, j0 + kCostClasses);
+  double acc = 0.0;
+  for (int j = j0; j < j1; ++j)
+    if ((reach[(size_t)j * W + (b >> 5)] >> (b & 31)) & 1u) acc += u[choice[(size_t)j * Bp + b]];
+  part[(size_t)blockIdx.x * Bp + b] = acc;
+}
+
+void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph&, const double* u,
+                               const int32_t* choice, const uint32_t* reach, double* cost_part) {
+  const int tpb = sh.Bp < 128 ? sh.Bp : 128;
+  const dim3 grid((sh.M + kCostClasses - 1) / kCostClasses, sh.Bp / tpb);
+  k_decode_cost_linear<<<grid, tpb, 0, s>>>(sh.M, sh.Bp, sh.W, u, choice, reach, cost_part);
+  SM_LAUNCH_CHECK();
+}
+
+int decode_cost_rows(const Shape& sh) { return (sh.M + kCostClasses - 1) / kCostClasses; }
+
+// s[k][b] = 1 iff class ec(k) is reached and chose k (the binary s of P99).
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_decode_s(int M, int Bp, int W,
+                                                     const int32_t* __restrict__ class_ptr,
+                                                     const uint32_t* __restrict__ sel,
+                                                     const uint32_t* __restrict__ reach,
+                                                     float* __restrict__ s_out) {
+  const RowGroup<LPR> rg;
+  if (rg.row >= M) return;
+  const int w = rg.s0 >> 5, sh = rg.s0 & 31;
+  const uint32_t r = reach[(size_t)rg.row * W + w];
+  for (int k = class_ptr[rg.row]; k < class_ptr[rg.row + 1]; ++k) {
+    const uint32_t bits = (r & sel[(size_t)k * W + w]) >> sh;
+    st4(s_out + (size_t)k * Bp + rg.s0,
+        make_float4((float)(bits & 1u), (float)((bits >> 1) & 1u), (float)((bits >> 2) & 1u),
+                    (float)((bits >> 3) & 1u)));
+  }
+}
+
+void launch_decode_s(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
+                     const uint32_t* reach, float* s_out) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_decode_s<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, sh.W, g.class_ptr,
+                                                                 sel, reach, s_out);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Keep-best (P297, readings S18, S20): the lowest (cost, step, global seed) of
+// the valid samples.  best = {cost, step, seed, steps since improvement}.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_best_update(
+    int B, int W, int root, const uint32_t* __restrict__ settle, const double* __restrict__ dcost,
+    const double* __restrict__ dextra, int64_t seed_begin, int32_t* __restrict__ counter,
+    double* __restrict__ best, int32_t* __restrict__ flag, double* __restrict__ cost_out,
+    uint8_t* __restrict__ valid_out) {
+  __shared__ double sc[256];
+  __shared__ int sb[256];
+  double bc = INFINITY;
+  int bb = 0x7fffffff;
+  for (int b = threadIdx.x; b < B; b += blockDim.x) {
+    const bool ok = (settle[(size_t)root * W + (b >> 5)] >> (b & 31)) & 1u;
+    const double c = ok ? dcost[b] + (dextra ? dextra[b] : 0.0) : INFINITY;
+    if (cost_out) cost_out[b] = c;
+    if (valid_out) valid_out[b] = ok ? 1 : 0;
+    if (c < bc) {
+      bc = c;
+      bb = b;
+    }
+  }
+  sc[threadIdx.x] = bc;
+  sb[threadIdx.x] = bb;
+  __syncthreads();
+  for (int off = blockDim.x / 2; off > 0; off >>= 1) {
+    if (threadIdx.x < off) {
+      const double c2 = sc[threadIdx.x + off];
+      const int b2 = sb[threadIdx.x + off];
+      if (c2 < sc[threadIdx.x] || (c2 == sc[threadIdx.x] && b2 < sb[threadIdx.x])) {
+        sc[threadIdx.x] = c2;
+        sb[threadIdx.x] = b2;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const int step = *counter;
+    if (sc[0] < best[0]) {
+      best[0] = sc[0];
+      best[1] = (double)step;
+      best[2] = (double)(seed_begin + sb[0]);
+      best[3] = 0.0;
+      *flag = 1;
+    } else {
+      best[3] += 1.0;
+      *flag = 0;
+    }
+    *counter = step + 1;
+  }
+}
+
+void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
+                        const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,
+                        const int32_t* step_counter, double* best, int32_t* best_flag,
+                        double* valid_cost_out, uint8_t* valid_out) {
+  k_best_update<<<1, 256, 0, s>>>(sh.B, sh.W, sh.root, settle, dcost_lin, dcost_extra, seed_begin,
+                                  const_cast<int32_t*>(step_counter), best, best_flag,
+                                  valid_cost_out, valid_out);
+  SM_LAUNCH_CHECK();
+}
+
+__global__ void k_best_snapshot(int M, int Bp, int W, const int32_t* __restrict__ choice,
+                                const uint32_t* __restrict__ reach, const double* __restrict__ best,
+                                const int32_t* __restrict__ flag, int64_t seed_begin,
+                                int32_t* __restrict__ best_choice) {
+  if (*flag == 0) return;
+  const int b = (int)((int64_t)best[2] - seed_begin);
+  for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < M; j += gridDim.x * blockDim.x) {
+    const bool r = (reach[(size_t)j * W + (b >> 5)] >> (b & 31)) & 1u;
+    best_choice[j] = r ? choice[(size_t)j * Bp + b] : -1;
+  }
+}
+
+void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice,
+                          const uint32_t* reach, const double* best, const int32_t* best_flag,
+                          int64_t seed_begin, int32_t* best_choice) {
+  const int grid = std::min((sh.M + 255) / 256, 148 * 4);
+  k_best_snapshot<<<grid, 256, 0, s>>>(sh.M, sh.Bp, sh.W, choice, reach, best, best_flag,
+                                       seed_begin, best_choice);
+  SM_LAUNCH_CHECK();
+}
+
+}  // namespace smoothe

@@ -1,0 +1,642 @@
+// Step kernels of the seed-parallel SmoothE gradient step (sm_100a).
+//
+//   theta init (Philox4x32-10, reading S9)
+//   segmented softmax + argmax + decode selection masks
+//   forward Jacobi sweep of Eqs. 5-7                      PAPER.md:201-223 (schedule 215)
+//   linear / quadratic cost + backward initialisation     PAPER.md:101, 156; reading S24
+//   reverse sweep (hand-derived reverse mode)
+//   softmax backward fused with Adam                      PAPER.md:275-277; reading S10
+//
+// All per-seed arrays are [row][Bp] fp32 (seed innermost): every gather of a
+// parent/child row is a contiguous 16-byte-per-lane access (kcommon.cuh).
+// Products, differences and the max that the reverse sweep must reproduce
+// bit-for-bit use explicit round-to-nearest intrinsics (no FMA contraction).
+#include <algorithm>
+#include <cfloat>
+
+#include "kcommon.cuh"
+
+namespace smoothe {
+
+// ---------------------------------------------------------------------------
+// theta = (x >> 8) * 2^-23 - 1, x = Philox4x32-10(key, ctr = (node, seed))[0]
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t philox_x0(uint64_t key, uint64_t node, uint64_t seed) {
+  uint32_t c0 = (uint32_t)node, c1 = (uint32_t)(node >> 32);
+  uint32_t c2 = (uint32_t)seed, c3 = (uint32_t)(seed >> 32);
+  uint32_t k0 = (uint32_t)key, k1 = (uint32_t)(key >> 32);
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    if (r) {
+      k0 += 0x9E3779B9u;
+      k1 += 0xBB67AE85u;
+    }
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+    const uint32_t n0 = hi1 ^ c1 ^ k0, n2 = hi0 ^ c3 ^ k1;
+    c0 = n0;
+    c1 = lo1;
+    c2 = n2;
+    c3 = lo0;
+  }
+  return c0;
+}
+
+__global__ void k_theta_init(int64_t total, int Bp, int B, uint64_t key, int64_t seed_begin,
+                             float* __restrict__ theta, float* __restrict__ m, float* __restrict__ v) {
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (int64_t)gridDim.x * blockDim.x) {
+    const int b = (int)(idx % Bp);
+    const int64_t node = idx / Bp;
+    float t = 0.f;
+    if (b < B) {
+      const uint32_t x = philox_x0(key, (uint64_t)node, (uint64_t)(seed_begin + b));
+      t = (float)(x >> 8) * 0x1p-23f - 1.0f;  // exact: 24-bit grid
+    }
+    theta[idx] = t;
+    m[idx] = 0.f;
+    v[idx] = 0.f;
+  }
+}
+
+void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t seed_begin,
+                       float* theta, float* m, float* v) {
+  const int64_t total = (int64_t)sh.N * sh.Bp;
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 16);
+  k_theta_init<<<grid, 256, 0, s>>>(total, sh.Bp, sh.B, key, seed_begin, theta, m, v);
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Segmented softmax within each e-class (Eq. 3b), the decode choice
+// c_j = argmax_{k in m_j} theta_k (lowest id on ties, reading S17) and the
+// selection masks sel[k][w] (bit l = seed 32w+l chose e-node k).
+// One warp per (class, <=4 words of 32 seeds); lane l owns seed 32w+l so a
+// ballot yields the mask word directly.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(kBlock) k_softmax_argmax(int M, int Bp, int W, int nw,
+                                                           const int32_t* __restrict__ class_ptr,
+                                                           const float* __restrict__ theta,
+                                                           float* __restrict__ cp,
+                                                           int32_t* __restrict__ choice,
+                                                           uint32_t* __restrict__ sel) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int nwc = W / nw;
+  const int j = warp / nwc;
+  if (j >= M) return;
+  const int w0 = (warp % nwc) * nw;
+  const int k0 = class_ptr[j], k1 = class_ptr[j + 1];
+  float mx[4], sum[4];
+  int am[4];
+#pragma unroll
+  for (int s = 0; s < 4; ++s) {
+    mx[s] = -FLT_MAX;
+    sum[s] = 0.f;
+    am[s] = k0;
+  }
+  for (int k = k0; k < k1; ++k) {
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+      if (s < nw) {
+        const float t = theta[(size_t)k * Bp + 32 * (w0 + s) + lane];
+        if (t > mx[s]) {
+          mx[s] = t;
+          am[s] = k;
+        }
+      }
+    }
+  }
+  for (int k = k0; k < k1; ++k) {
+#pragma unroll
+    for (int s = 0; s < 4; ++s)
+      if (s < nw) sum[s] += expf(theta[(size_t)k * Bp + 32 * (w0 + s) + lane] - mx[s]);
+  }
+  for (int k = k0; k < k1; ++k) {
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+      if (s < nw) {
+        const size_t idx = (size_t)k * Bp + 32 * (w0 + s) + lane;
+        cp[idx] = expf(theta[idx] - mx[s]) / sum[s];
+        const uint32_t bits = __ballot_sync(0xffffffffu, am[s] == k);
+        if (lane == 0) sel[(size_t)k * W + w0 + s] = bits;
+      }
+    }
+  }
+#pragma unroll
+  for (int s = 0; s < 4; ++s)
+    if (s < nw) choice[(size_t)j * Bp + 32 * (w0 + s) + lane] = am[s];
+}
+
+void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
+                           float* cp, int32_t* choice, uint32_t* sel) {
+  const int nw = sh.W < 4 ? sh.W : 4;
+  const int64_t warps = (int64_t)sh.M * (sh.W / nw);
+  const int grid = (int)((warps * 32 + kBlock - 1) / kBlock);
+  k_softmax_argmax<<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, sh.W, nw, g.class_ptr, theta, cp, choice, sel);
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Forward sweep t (readings S2-S4, S6-S8):
+//   p^t_k = cp_k * q^{t-1}_{ec(k)}                                      (Eq. 5)
+//   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
+// Also keeps, for the reverse sweep, the product over the non-zero factors
+// (pi), and am = (lowest arg-max e-node << 2) | min(#zero factors, 3).
+// One row group per (class, seed chunk): a CSC pull over the parents.
+// ---------------------------------------------------------------------------
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_sweep_forward(
+    int M, int Bp, int root, const int32_t* __restrict__ par_ptr,
+    const int32_t* __restrict__ par_node, const int32_t* __restrict__ par_class, float wI, float wC,
+    const float* __restrict__ cp, const float* __restrict__ q_prev, float* __restrict__ q,
+    float* __restrict__ pi, int32_t* __restrict__ am) {
+  const RowGroup<LPR> rg;
+  const int j = rg.row;
+  if (j >= M || j == root) return;
+  const int e0 = par_ptr[j], e1 = par_ptr[j + 1];
+  float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
+  float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
+  int4 arg = make_int4(-1, -1, -1, -1);
+  int4 zc = make_int4(0, 0, 0, 0);
+#pragma unroll 4
+  for (int e = e0; e < e1; ++e) {
+    const int k = __ldg(par_node + e);
+    const int c = __ldg(par_class + e);
+    const float4 cv = ld4(cp + (size_t)k * Bp + rg.s0);
+    const float4 qv = ld4(q_prev + (size_t)c * Bp + rg.s0);
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const float p = __fmul_rn(comp(cv, x), comp(qv, x));
+      const float f = __fsub_rn(1.f, p);
+      if (f == 0.f) comp(zc, x) += 1;
+      else comp(prod, x) = __fmul_rn(comp(prod, x), f);
+      if (p > comp(mx, x)) {
+        comp(mx, x) = p;
+        comp(arg, x) = k;
+      }
+    }
+  }
+  float4 qo;
+  int4 ao;
+#pragma unroll
+  for (int x = 0; x < 4; ++x) {
+    const float P = comp(zc, x) > 0 ? 0.f : comp(prod, x);
+    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
+    comp(ao, x) = (comp(arg, x) << 2) | min(comp(zc, x), 3);
+  }
+  const size_t o = (size_t)j * Bp + rg.s0;
+  st4(q + o, qo);
+  if (pi) st4(pi + o, prod);
+  st4i(am + o, ao);
+}
+
+void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.par_ptr, g.par_node, g.par_class, a.wI, a.wC, cp, q_prev, q, pi, am);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Linear cost f_b = sum_i u_i p_i with p = cp * q^K[ec] (P101), fused with the
+// backward initialisation (App. C step 1-2): g_cp_i = u_i q^K_{ec(i)},
+// g_q^K_j = sum_{i in m_j} u_i cp_i (0 at the root).  Per-block partial sums
+// of f go to f_part[blockIdx.x][Bp] (reduced in fp64 by k_reduce_rows).
+// ---------------------------------------------------------------------------
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_cost_linear(
+    int M, int Bp, int root, const int32_t* __restrict__ class_ptr, const float* __restrict__ u,
+    const float* __restrict__ cp, const float* __restrict__ qK, float* __restrict__ gcp,
+    float* __restrict__ gqK, float* __restrict__ f_part, float* __restrict__ p_out) {
+  __shared__ float4 red[kBlock / LPR][LPR];
+  const RowGroup<LPR> rg;
+  float4 facc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (rg.row < M) {
+    const int j = rg.row;
+    const float4 qv = ld4(qK + (size_t)j * Bp + rg.s0);
+    float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) {
+      const float ui = __ldg(u + i);
+      const size_t o = (size_t)i * Bp + rg.s0;
+      const float4 cv = ld4(cp + o);
+      float4 p, gc;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        comp(p, x) = __fmul_rn(comp(cv, x), comp(qv, x));
+        comp(facc, x) += ui * comp(p, x);
+        comp(gc, x) = ui * comp(qv, x);
+        comp(gq, x) += ui * comp(cv, x);
+      }
+      st4(gcp + o, gc);
+      if (p_out) st4(p_out + o, p);
+    }
+    if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
+    st4(gqK + (size_t)j * Bp + rg.s0, gq);
+  }
+  red[rg.sub][threadIdx.x % LPR] = facc;
+  __syncthreads();
+  if (threadIdx.x < LPR) {
+    float4 acc = red[0][threadIdx.x];
+    for (int r = 1; r < kBlock / LPR; ++r) {
+      const float4 v = red[r][threadIdx.x];
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    st4(f_part + (size_t)blockIdx.x * Bp + rg.s0, acc);
+  }
+}
+
+void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
+                        const float* cp, const float* qK, float* gcp, float* gqK, float* f_part,
+                        float* p_out, int32_t) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_cost_linear<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.class_ptr, u, cp, qK, gcp, gqK, f_part, p_out);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// p = cp * q^K[ec] materialised for the non-linear cost models; with u, also
+// the per-block partial sums of the linear part u^T p (P409: f = f_lin + f_nl).
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_materialize_p(int M, int Bp,
+                                                          const int32_t* __restrict__ class_ptr,
+                                                          const float* __restrict__ u,
+                                                          const float* __restrict__ cp,
+                                                          const float* __restrict__ qK,
+                                                          float* __restrict__ p,
+                                                          float* __restrict__ f_part) {
+  __shared__ float4 red[kBlock / LPR][LPR];
+  const RowGroup<LPR> rg;
+  float4 facc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (rg.row < M) {
+    const float4 qv = ld4(qK + (size_t)rg.row * Bp + rg.s0);
+    for (int i = class_ptr[rg.row]; i < class_ptr[rg.row + 1]; ++i) {
+      const size_t o = (size_t)i * Bp + rg.s0;
+      const float4 cv = ld4(cp + o);
+      const float ui = u ? __ldg(u + i) : 0.f;
+      float4 pv;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        comp(pv, x) = __fmul_rn(comp(cv, x), comp(qv, x));
+        comp(facc, x) += ui * comp(pv, x);
+      }
+      st4(p + o, pv);
+    }
+  }
+  if (!f_part) return;
+  red[rg.sub][threadIdx.x % LPR] = facc;
+  __syncthreads();
+  if (threadIdx.x < LPR) {
+    float4 acc = red[0][threadIdx.x];
+    for (int r = 1; r < kBlock / LPR; ++r) {
+      const float4 v = red[r][threadIdx.x];
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    st4(f_part + (size_t)blockIdx.x * Bp + rg.s0, acc);
+  }
+}
+
+void launch_materialize_p_f(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
+                            const float* cp, const float* qK, float* p, float* f_part) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_materialize_p<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, g.class_ptr, u,
+                                                                      cp, qK, p, f_part);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+__global__ void k_fill_rows(float* base, int64_t stride, int count, int Bp, float value) {
+  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < count * Bp; idx += gridDim.x * blockDim.x)
+    base[(size_t)(idx / Bp) * stride + idx % Bp] = value;
+}
+
+void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, int Bp, float value) {
+  if (count <= 0) return;
+  const int grid = std::min((count * Bp + 255) / 256, 1024);
+  k_fill_rows<<<grid, 256, 0, s>>>(base, stride, count, Bp, value);
+  SM_LAUNCH_CHECK();
+}
+
+// ftot[b] = f[b] + fextra[b];  L = sum_b ftot[b] + lambda * sum_g G h_g  (Eq. 10a; S12)
+__global__ void k_loss(int B, int G, int ngroups, double lambda, const double* __restrict__ f,
+                       const double* __restrict__ fextra, const double* __restrict__ h,
+                       double* __restrict__ ftot, double* __restrict__ loss) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  double L = 0.0;
+  for (int b = 0; b < B; ++b) {
+    const double v = f[b] + (fextra ? fextra[b] : 0.0);
+    ftot[b] = v;
+    L += v;
+  }
+  if (h)
+    for (int g = 0; g < ngroups; ++g) L += lambda * G * h[g];
+  *loss = L;
+}
+
+void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const double* f,
+                 const double* fextra, const double* h, double* ftot, double* loss) {
+  k_loss<<<1, 32, 0, s>>>(B, G, ngroups, lambda, f, fextra, h, ftot, loss);
+  SM_LAUNCH_CHECK();
+}
+
+// Backward initialisation from a general g_p = df/dp (quadratic / MLP).
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_cost_gp(int M, int Bp, int root,
+                                                    const int32_t* __restrict__ class_ptr,
+                                                    const float* __restrict__ gp,
+                                                    const float* __restrict__ cp,
+                                                    const float* __restrict__ qK,
+                                                    float* __restrict__ gcp, float* __restrict__ gqK) {
+  const RowGroup<LPR> rg;
+  if (rg.row >= M) return;
+  const int j = rg.row;
+  const float4 qv = ld4(qK + (size_t)j * Bp + rg.s0);
+  float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) {
+    const size_t o = (size_t)i * Bp + rg.s0;
+    const float4 gv = ld4(gp + o), cv = ld4(cp + o);
+    float4 gc;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      comp(gc, x) = comp(gv, x) * comp(qv, x);
+      comp(gq, x) += comp(gv, x) * comp(cv, x);
+    }
+    st4(gcp + o, gc);
+  }
+  if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
+  st4(gqK + (size_t)j * Bp + rg.s0, gq);
+}
+
+void launch_cost_gp(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* gp,
+                    const float* cp, const float* qK, float* gcp, float* gqK) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_cost_gp<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, sh.root, g.class_ptr,
+                                                                gp, cp, qK, gcp, gqK);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// Quadratic cost (reading S24) over a symmetric neighbour list of the pairs:
+//   f = sum_i p_i (u_i + 1/2 sum_{k in nbr(i)} w_ik p_k),   g_p_i = u_i + sum_k w_ik p_k.
+// Rows are e-nodes.  Also used on the 0/1 decode vector s (exact for integer u, w).
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_cost_quadratic(int N, int Bp,
+                                                           const int32_t* __restrict__ qptr,
+                                                           const int32_t* __restrict__ qnbr,
+                                                           const float* __restrict__ qw,
+                                                           const float* __restrict__ u,
+                                                           const float* __restrict__ p,
+                                                           float* __restrict__ gp,
+                                                           float* __restrict__ f_part) {
+  __shared__ float4 red[kBlock / LPR][LPR];
+  const RowGroup<LPR> rg;
+  float4 facc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (rg.row < N) {
+    const int i = rg.row;
+    const float ui = u ? u[i] : 0.f;
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int e = qptr[i]; e < qptr[i + 1]; ++e) {
+      const float w = __ldg(qw + e);
+      const float4 pk = ld4(p + (size_t)__ldg(qnbr + e) * Bp + rg.s0);
+#pragma unroll
+      for (int x = 0; x < 4; ++x) comp(acc, x) += w * comp(pk, x);
+    }
+    const float4 pi = ld4(p + (size_t)i * Bp + rg.s0);
+    float4 g;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      comp(g, x) = ui + comp(acc, x);
+      comp(facc, x) = comp(pi, x) * (ui + 0.5f * comp(acc, x));
+    }
+    if (gp) st4(gp + (size_t)i * Bp + rg.s0, g);
+  }
+  red[rg.sub][threadIdx.x % LPR] = facc;
+  __syncthreads();
+  if (threadIdx.x < LPR) {
+    float4 acc = red[0][threadIdx.x];
+    for (int r = 1; r < kBlock / LPR; ++r) {
+      const float4 v = red[r][threadIdx.x];
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    st4(f_part + (size_t)blockIdx.x * Bp + rg.s0, acc);
+  }
+}
+
+void launch_quadratic(cudaStream_t s, const Shape& sh, const int32_t* qptr, const int32_t* qnbr,
+                      const float* qw, const float* u, const float* p, float* gp, float* f_part) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_cost_quadratic<LPR><<<row_grid(sh.N, sh.Bp, LPR), kBlock, 0, s>>>(sh.N, sh.Bp, qptr, qnbr, qw,
+                                                                       u, p, gp, f_part);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// out[b] = scale * sum_r part[r][b], fp64, fixed order (deterministic).
+__global__ void k_reduce_rows(const float* __restrict__ part, int nrows, int Bp,
+                              double* __restrict__ out, double scale) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= Bp) return;
+  double acc = 0.0;
+  for (int r = 0; r < nrows; ++r) acc += (double)part[(size_t)r * Bp + b];
+  out[b] = acc * scale;
+}
+
+void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, int32_t Bp,
+                            double* out, double scale) {
+  k_reduce_rows<<<(Bp + 127) / 128, 128, 0, s>>>(part, nrows, Bp, out, scale);
+  SM_LAUNCH_CHECK();
+}
+
+__global__ void k_reduce_rows_d(const double* __restrict__ part, int nrows, int Bp,
+                                double* __restrict__ out) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= Bp) return;
+  double acc = 0.0;
+  for (int r = 0; r < nrows; ++r) acc += part[(size_t)r * Bp + b];
+  out[b] = acc;
+}
+
+void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
+                             double* out) {
+  k_reduce_rows_d<<<(Bp + 127) / 128, 128, 0, s>>>(part, nrows, Bp, out);
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Reverse sweep t, one row group per class j':
+// for every e-node k in m_j' (contiguous):
+//   p_k    = cp_k q^{t-1}_{j'}  (recomputed bit-identically to the forward sweep)
+//   g_p^t_k = sum_{j in ch_k} g_q^t_j (wI excl_{jk} + wC [k = a^t_j])
+//   excl_{jk} = prod_{k' in pa_j, k' != k} (1 - p^t_k'): the stored product of
+//   the non-zero factors divided by k's own factor (the same fp32 value, so the
+//   quotient is exact to a few ulp); with one zero factor it is the stored
+//   product if k's factor is that zero, else 0; with two or more zeros it is 0.
+//   g_cp_k += g_p^t_k q^{t-1}_{j'};   g_q^{t-1}_{j'} = sum_k g_p^t_k cp_k (0 at root)
+// Deterministic: no atomics, every output row has one owner.
+// ---------------------------------------------------------------------------
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_sweep_reverse(
+    int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
+    const int32_t* __restrict__ child_ptr, const int32_t* __restrict__ child_class, float wI,
+    float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
+    const float* __restrict__ gq, const float* __restrict__ pi, const int32_t* __restrict__ am,
+    float* __restrict__ gcp, float* __restrict__ gq_prev) {
+  const RowGroup<LPR> rg;
+  const int jp = rg.row;
+  if (jp >= M) return;
+  const float4 qp = ld4(q_prev + (size_t)jp * Bp + rg.s0);
+  float4 gqacc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int k = class_ptr[jp]; k < class_ptr[jp + 1]; ++k) {
+    const size_t ok = (size_t)k * Bp + rg.s0;
+    const float4 cv = ld4(cp + ok);
+    float4 om;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+    float4 gp = make_float4(0.f, 0.f, 0.f, 0.f);
+    const int e0 = child_ptr[k], e1 = child_ptr[k + 1];
+#pragma unroll 2
+    for (int e = e0; e < e1; ++e) {
+      const size_t oj = (size_t)__ldg(child_class + e) * Bp + rg.s0;
+      const float4 g = ld4(gq + oj);
+      const int4 a = ld4i(am + oj);
+      float4 P = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (wI != 0.f) P = ld4(pi + oj);
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        const int av = comp(a, x);
+        const int zc = av & 3;
+        float D = (av >> 2) == k ? wC : 0.f;
+        if (wI != 0.f) {
+          const float o = comp(om, x);
+          float excl = 0.f;
+          if (zc == 0) excl = __fdiv_rn(comp(P, x), o);
+          else if (zc == 1 && o == 0.f) excl = comp(P, x);
+          D += wI * excl;
+        }
+        comp(gp, x) += comp(g, x) * D;
+      }
+    }
+    float4 gc = ld4(gcp + ok);
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      comp(gc, x) += comp(gp, x) * comp(qp, x);
+      comp(gqacc, x) += comp(gp, x) * comp(cv, x);
+    }
+    st4(gcp + ok, gc);
+  }
+  if (gq_prev) {
+    if (jp == root) gqacc = make_float4(0.f, 0.f, 0.f, 0.f);
+    st4(gq_prev + (size_t)jp * Bp + rg.s0, gqacc);
+  }
+}
+
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, const float* gq, const float* pi,
+                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_sweep_reverse<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.class_ptr, g.child_ptr, g.child_class, a.wI, a.wC, cp, q_prev, gq,
+        pi, am, gcp, write_gq_prev ? gq_prev : nullptr);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Step scalars: Adam bias corrections for step number t = counter + 1 (fp64).
+// ---------------------------------------------------------------------------
+__global__ void k_step_prologue(const int32_t* __restrict__ counter, double* __restrict__ scal,
+                                double beta1, double beta2) {
+  const double t = (double)(*counter + 1);
+  scal[0] = 1.0 / (1.0 - pow(beta1, t));
+  scal[1] = 1.0 / (1.0 - pow(beta2, t));
+}
+
+void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_scalars,
+                          double beta1, double beta2, const int32_t*) {
+  k_step_prologue<<<1, 1, 0, s>>>(step_counter, step_scalars, beta1, beta2);
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Softmax backward fused with the optimiser (P277; reading S10), per class:
+//   g_tot_k = g_cp_k + pen_k(group)                      (App. B penalty term)
+//   g_theta_k = cp_k (g_tot_k - sum_{k' in m_j} cp_k' g_tot_k')
+//   Adam: m = b1 m + (1-b1) g; v = b2 v + (1-b2) g^2;
+//         theta -= lr (m c1) / (sqrt(v c2) + eps),  c1,2 = 1/(1 - b1,2^t)
+// ---------------------------------------------------------------------------
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_update(
+    int M, int Bp, int G, int ngroups, const int32_t* __restrict__ class_ptr,
+    const int32_t* __restrict__ node_slot, const float* __restrict__ cp,
+    const float* __restrict__ gcp, const float* __restrict__ pen, float* __restrict__ theta,
+    float* __restrict__ m, float* __restrict__ v, const double* __restrict__ scal, int optimizer,
+    float lr, float beta1, float beta2, float eps, float* __restrict__ gth_out,
+    float* __restrict__ gcp_out) {
+  const RowGroup<LPR> rg;
+  if (rg.row >= M) return;
+  const int j = rg.row;
+  const int k0 = class_ptr[j], k1 = class_ptr[j + 1];
+  int grp[4];
+#pragma unroll
+  for (int x = 0; x < 4; ++x) grp[x] = min((rg.s0 + x) / G, ngroups - 1);
+  auto gtot = [&](int k, float4 gc) {
+    const int slot = node_slot ? __ldg(node_slot + k) : -1;
+    if (slot >= 0) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) comp(gc, x) += pen[(size_t)slot * ngroups + grp[x]];
+    }
+    return gc;
+  };
+  float4 ssum = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int k = k0; k < k1; ++k) {
+    const size_t o = (size_t)k * Bp + rg.s0;
+    const float4 cv = ld4(cp + o);
+    const float4 gt = gtot(k, ld4(gcp + o));
+#pragma unroll
+    for (int x = 0; x < 4; ++x) comp(ssum, x) += comp(cv, x) * comp(gt, x);
+  }
+  const float c1 = (float)scal[0], c2 = (float)scal[1];
+  for (int k = k0; k < k1; ++k) {
+    const size_t o = (size_t)k * Bp + rg.s0;
+    const float4 cv = ld4(cp + o);
+    const float4 gt = gtot(k, ld4(gcp + o));
+    float4 th = ld4(theta + o), mv = ld4(m + o), vv = ld4(v + o), gth;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const float g = comp(cv, x) * (comp(gt, x) - comp(ssum, x));
+      comp(gth, x) = g;
+      if (optimizer == 0) {
+        const float mn = beta1 * comp(mv, x) + (1.f - beta1) * g;
+        const float vn = beta2 * comp(vv, x) + (1.f - beta2) * (g * g);
+        comp(mv, x) = mn;
+        comp(vv, x) = vn;
+        comp(th, x) = comp(th, x) - lr * (mn * c1) / (sqrtf(vn * c2) + eps);
+      } else {
+        comp(th, x) = comp(th, x) - lr * g;
+      }
+    }
+    st4(theta + o, th);
+    st4(m + o, mv);
+    st4(v + o, vv);
+    if (gth_out) st4(gth_out + o, gth);
+    if (gcp_out) st4(gcp_out + o, gt);
+  }
+}
+
+void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,
+                   const float* gcp, const float* pen, float* theta, float* m, float* v,
+                   const double* step_scalars, int32_t optimizer, float lr, float beta1,
+                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out) {
+  const int ngroups = (sh.B + G - 1) / G;
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_update<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, G, ngroups, g.class_ptr, pen ? g.node_slot : nullptr, cp, gcp, pen, theta, m,
+        v, step_scalars, optimizer, lr, beta1, beta2, eps, grad_theta_out, grad_cp_out);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+}  // namespace smoothe

@@ -1,0 +1,880 @@
+// libsmoothe runtime: the C ABI of include/smoothe.h.
+//
+// One optimisation step (Sec. 3.5) is a fixed sequence of
+// kernel launches on the run's private stream (captured once into a CUDA graph
+// and replayed, unless profiling):
+//
+//   prologue      Adam bias corrections of this step            (S10)
+//   softmax       cp = softmax(theta), c_j = argmax theta, sel   (Eq. 3b, P277, P279)
+//   forward x K   q^t from q^{t-1}                               (Eqs. 5-7, P215)
+//   cost          f(p), backward initialisation                  (P101, P409, P425)
+//   penalty       NOTEARS per (SCC, group)                       (Eqs. 8-11, P318-325)
+//   reverse x K   g_cp, g_q                                      (App. C)
+//   update        softmax backward + Adam                        (P277)
+//   decode        reach, settle, discrete cost                   (P279, P103-111)
+//   best          keep the best (cost, step, seed)               (P297, S20)
+#include <algorithm>
+#include <array>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <mutex>
+#include <new>
+
+#include "internal.h"
+
+namespace smoothe {
+
+static thread_local std::string g_last_error;
+void set_error(const std::string& msg) { g_last_error = msg; }
+
+int64_t& launch_counter() {
+  static int64_t counter = 0;
+  return counter;
+}
+
+int num_sms(int device) {
+  static int cached[64] = {0};
+  if (device >= 0 && device < 64 && cached[device]) return cached[device];
+  int n = 0;
+  SM_CUDA(cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, device));
+  if (device >= 0 && device < 64) cached[device] = n;
+  return n;
+}
+
+template <typename T>
+static T* dalloc(std::vector<void*>& owned, size_t count) {
+  if (count == 0) count = 1;
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, count * sizeof(T));
+  if (e == cudaErrorMemoryAllocation) {
+    (void)cudaGetLastError();
+    throw Failure{SMOOTHE_E_OOM, "cudaMalloc of " + std::to_string(count * sizeof(T)) + " bytes failed"};
+  }
+  SM_CUDA(e);
+  owned.push_back(p);
+  return static_cast<T*>(p);
+}
+
+template <typename T>
+static T* upload(std::vector<void*>& owned, const std::vector<T>& v, int64_t* bytes = nullptr) {
+  T* d = dalloc<T>(owned, v.size());
+  if (!v.empty()) SM_CUDA(cudaMemcpy(d, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
+  if (bytes) *bytes += (int64_t)(v.size() * sizeof(T));
+  return d;
+}
+
+}  // namespace smoothe
+
+using namespace smoothe;
+
+struct smoothe_egraph_dev_owner {
+  std::vector<void*> owned;
+};
+
+struct smoothe_run {
+  smoothe_egraph* g = nullptr;
+  smoothe_options opt{};
+  Shape sh{};
+  int K = 0, G = 1, ngroups = 1, device = 0, cost_kind = 0, H1 = 0, H2 = 0, nsplit = 0;
+  int coop_grid = 0, f_rows = 0, dcost_rows = 0;
+  Agg agg{0.f, 0.f};
+  cudaStream_t stream = nullptr;
+  std::vector<void*> owned;
+  // state
+  float *theta = nullptr, *m = nullptr, *v = nullptr, *cp = nullptr, *gcp = nullptr;
+  float *qstack = nullptr, *pistack = nullptr;
+  int32_t* astack = nullptr;
+  float* gq[2] = {nullptr, nullptr};
+  float* f_part = nullptr;
+  double *f = nullptr, *fextra = nullptr, *ftot = nullptr, *h_part = nullptr, *h = nullptr,
+         *loss = nullptr;
+  float* pen = nullptr;
+  int32_t* choice = nullptr;
+  uint32_t *sel = nullptr, *reach = nullptr, *settle = nullptr;
+  int32_t* flags = nullptr;
+  double *dcost_part = nullptr, *dcost = nullptr, *dextra = nullptr;
+  double* best = nullptr;
+  int32_t *best_flag = nullptr, *best_choice = nullptr, *counter = nullptr;
+  double* scal = nullptr;
+  // cost model
+  float* u_f = nullptr;
+  double* u_d = nullptr;
+  int32_t *q_ptr = nullptr, *q_nbr = nullptr;
+  float* q_w = nullptr;
+  float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr, *W3 = nullptr, *b3 = nullptr;
+  float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *gz1 = nullptr;
+  double* fmlp_s = nullptr;
+  // debug outputs (set only during smoothe_debug_step)
+  float *dbg_p = nullptr, *dbg_gth = nullptr, *dbg_gcp = nullptr;
+  double* dbg_dcost = nullptr;
+  uint8_t* dbg_valid = nullptr;
+  bool debug = false;
+  // timing / profiling
+  cudaEvent_t ev_start = nullptr;
+  std::vector<cudaEvent_t> ev_step;
+  std::chrono::steady_clock::time_point t_create;
+  bool profiling = false;
+  std::vector<std::array<cudaEvent_t, SMOOTHE_NUM_PHASES + 1>> prof_ev;
+  std::vector<cudaEvent_t> prof_pool;
+  size_t prof_pool_used = 0;
+  int64_t prof_launch[SMOOTHE_NUM_PHASES] = {0};
+  int64_t prof_launch_total = 0, prof_steps = 0;
+  // graph
+  cudaGraphExec_t graph_exec = nullptr;
+  bool graph_failed = false;
+  bool poisoned = false;
+  int steps_run = 0;
+};
+
+namespace {
+
+template <typename F>
+smoothe_status guarded(smoothe_run* run, F&& fn) {
+  try {
+    fn();
+    return SMOOTHE_OK;
+  } catch (const Failure& f) {
+    set_error(f.msg);
+    if (run && f.status == SMOOTHE_E_CUDA) run->poisoned = true;
+    return f.status;
+  } catch (const std::bad_alloc&) {
+    set_error("host allocation failed");
+    return SMOOTHE_E_OOM;
+  } catch (...) {
+    set_error("unknown internal error");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+}
+
+void check_run(smoothe_run* run) {
+  SM_REQUIRE(run != nullptr, SMOOTHE_E_INVALID_ARG, "NULL run");
+  SM_REQUIRE(!run->poisoned, SMOOTHE_E_STATE, "run is poisoned by an earlier CUDA error");
+  SM_CUDA(cudaSetDevice(run->device));
+}
+
+cudaEvent_t pool_event(smoothe_run* r) {
+  if (r->prof_pool_used == r->prof_pool.size()) {
+    cudaEvent_t e;
+    SM_CUDA(cudaEventCreate(&e));
+    r->prof_pool.push_back(e);
+  }
+  return r->prof_pool[r->prof_pool_used++];
+}
+
+// Record the boundary event before `phase` when profiling.
+struct PhaseMarks {
+  smoothe_run* r;
+  std::array<cudaEvent_t, SMOOTHE_NUM_PHASES + 1> ev{};
+  int64_t last = 0;
+  int cur = -1;
+  explicit PhaseMarks(smoothe_run* run) : r(run) {}
+  void mark(int phase) {
+    if (!r->profiling) return;
+    if (cur >= 0) r->prof_launch[cur] += launch_counter() - last;
+    last = launch_counter();
+    cur = phase;
+    ev[phase] = pool_event(r);
+    SM_CUDA(cudaEventRecord(ev[phase], r->stream));
+  }
+  void finish() {
+    if (!r->profiling) return;
+    r->prof_launch[cur] += launch_counter() - last;
+    ev[SMOOTHE_NUM_PHASES] = pool_event(r);
+    SM_CUDA(cudaEventRecord(ev[SMOOTHE_NUM_PHASES], r->stream));
+    r->prof_ev.push_back(ev);
+  }
+};
+
+void enqueue_step(smoothe_run* r) {
+  const Shape& sh = r->sh;
+  const DevGraph& g = r->g->dev;
+  const HostGraph& hg = r->g->host;
+  cudaStream_t s = r->stream;
+  const size_t MB = (size_t)sh.M * sh.Bp;
+  const int K = r->K;
+  const int64_t l0 = launch_counter();
+  PhaseMarks pm(r);
+
+  pm.mark(SMOOTHE_PHASE_SOFTMAX);
+  launch_step_prologue(s, r->counter, r->scal, r->opt.beta1, r->opt.beta2, nullptr);
+  launch_softmax_argmax(s, sh, g, r->theta, r->cp, r->choice, r->sel);
+
+  pm.mark(SMOOTHE_PHASE_FORWARD);
+  for (int t = 1; t <= K; ++t)
+    launch_sweep_forward(s, sh, g, r->agg, r->cp, r->qstack + (size_t)(t - 1) * MB,
+                         r->qstack + (size_t)t * MB,
+                         r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
+                         r->astack + (size_t)(t - 1) * MB);
+
+  pm.mark(SMOOTHE_PHASE_COST);
+  const float* qK = r->qstack + (size_t)K * MB;
+  float* gqK = r->gq[K & 1];
+  if (r->cost_kind == SMOOTHE_COST_LINEAR) {
+    launch_cost_linear(s, sh, g, r->u_f, r->cp, qK, r->gcp, gqK, r->f_part,
+                       r->debug ? r->dbg_p : nullptr, 0);
+    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+  } else if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
+    launch_materialize_p_f(s, sh, g, nullptr, r->cp, qK, r->p, nullptr);
+    launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, r->u_f, r->p, r->gp, r->f_part);
+    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+    launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
+  } else {
+    launch_materialize_p_f(s, sh, g, r->u_f, r->cp, qK, r->p, r->f_part);
+    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+    launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
+                   r->z1_part, r->fextra, r->gz1, r->nsplit);
+    launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
+    launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
+  }
+
+  pm.mark(SMOOTHE_PHASE_PENALTY);
+  if (hg.num_scc > 0) {
+    launch_notears(s, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen);
+    launch_reduce_rows_f64d(s, r->h_part, hg.num_scc, r->ngroups, r->h);
+  }
+  launch_loss(s, sh.B, r->G, r->ngroups, r->opt.lambda, r->f,
+              r->cost_kind == SMOOTHE_COST_MLP ? r->fextra : nullptr, hg.num_scc > 0 ? r->h : nullptr,
+              r->ftot, r->loss);
+
+  pm.mark(SMOOTHE_PHASE_REVERSE);
+  for (int t = K; t >= 1; --t)
+    launch_sweep_reverse(s, sh, g, r->agg, r->cp, r->qstack + (size_t)(t - 1) * MB, r->gq[t & 1],
+                         r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
+                         r->astack + (size_t)(t - 1) * MB, r->gcp, r->gq[(t - 1) & 1], t > 1);
+
+  pm.mark(SMOOTHE_PHASE_UPDATE);
+  launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
+                r->v, r->scal, r->opt.optimizer, (float)r->opt.lr, (float)r->opt.beta1,
+                (float)r->opt.beta2, (float)r->opt.eps, r->debug ? r->dbg_gth : nullptr,
+                r->debug ? r->dbg_gcp : nullptr);
+
+  pm.mark(SMOOTHE_PHASE_DECODE);
+  launch_decode_reach(s, sh, g, r->sel, r->reach, r->flags, r->coop_grid);
+  launch_decode_settle(s, sh, g, r->sel, r->settle, r->flags + 4, r->coop_grid);
+  launch_decode_cost_linear(s, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
+  launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost);
+  const double* dextra = nullptr;
+  if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
+    launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
+    launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, nullptr, r->sbin, nullptr, r->f_part);
+    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->dextra, 1.0);
+    dextra = r->dextra;
+  } else if (r->cost_kind == SMOOTHE_COST_MLP) {
+    launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
+    launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
+                   r->z1_part, r->dextra, nullptr, r->nsplit);
+    dextra = r->dextra;
+  }
+
+  pm.mark(SMOOTHE_PHASE_BEST);
+  launch_best_update(s, sh, r->settle, r->dcost, dextra, r->opt.seed_begin, r->counter, r->best,
+                     r->best_flag, r->debug ? r->dbg_dcost : nullptr,
+                     r->debug ? r->dbg_valid : nullptr);
+  launch_best_snapshot(s, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
+                       r->best_choice);
+  pm.finish();
+  if (r->profiling) {
+    r->prof_launch_total += launch_counter() - l0;
+    r->prof_steps += 1;
+  }
+}
+
+void run_one_step(smoothe_run* r) {
+  const bool use_graph = r->opt.use_graphs && !r->profiling && !r->debug && !r->graph_failed;
+  if (use_graph && !r->graph_exec) {
+    cudaGraph_t graph = nullptr;
+    const int64_t before = launch_counter();
+    bool ok = cudaStreamBeginCapture(r->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+    if (ok) {
+      try {
+        enqueue_step(r);
+      } catch (const Failure&) {
+        ok = false;
+      }
+      cudaError_t e = cudaStreamEndCapture(r->stream, &graph);
+      ok = ok && e == cudaSuccess && graph != nullptr;
+    }
+    if (ok) ok = cudaGraphInstantiate(&r->graph_exec, graph, 0) == cudaSuccess;
+    if (graph) cudaGraphDestroy(graph);
+    launch_counter() = before;
+    if (!ok) {
+      (void)cudaGetLastError();
+      r->graph_exec = nullptr;
+      r->graph_failed = true;  // fall back to direct launches (still all on the GPU)
+    }
+  }
+  if (use_graph && r->graph_exec) {
+    SM_CUDA(cudaGraphLaunch(r->graph_exec, r->stream));
+  } else {
+    enqueue_step(r);
+  }
+  if ((size_t)r->steps_run < r->ev_step.size()) {
+    SM_CUDA(cudaEventRecord(r->ev_step[r->steps_run], r->stream));
+  }
+  r->steps_run++;
+}
+
+void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
+  const Shape& sh = r->sh;
+  const HostGraph& hg = r->g->host;
+  auto& o = r->owned;
+  const size_t NB = (size_t)sh.N * sh.Bp, MB = (size_t)sh.M * sh.Bp;
+  r->theta = dalloc<float>(o, NB);
+  r->m = dalloc<float>(o, NB);
+  r->v = dalloc<float>(o, NB);
+  r->cp = dalloc<float>(o, NB);
+  r->gcp = dalloc<float>(o, NB);
+  r->qstack = dalloc<float>(o, (size_t)(r->K + 1) * MB);
+  if (r->agg.wI != 0.f) r->pistack = dalloc<float>(o, std::max<size_t>(1, (size_t)r->K * MB));
+  r->astack = dalloc<int32_t>(o, std::max<size_t>(1, (size_t)r->K * MB));
+  r->gq[0] = dalloc<float>(o, MB);
+  r->gq[1] = dalloc<float>(o, MB);
+  const int rows_per_block_min = 256 / 32;  // kBlock / LPR(32): fewest rows per block
+  r->f_rows = (std::max(sh.M, sh.N) + rows_per_block_min - 1) / rows_per_block_min + 1;
+  r->f_part = dalloc<float>(o, (size_t)r->f_rows * sh.Bp);
+  r->f = dalloc<double>(o, sh.Bp);
+  r->fextra = dalloc<double>(o, sh.Bp);
+  r->ftot = dalloc<double>(o, sh.Bp);
+  r->h_part = dalloc<double>(o, (size_t)std::max(1, hg.num_scc) * r->ngroups);
+  r->h = dalloc<double>(o, r->ngroups);
+  r->loss = dalloc<double>(o, 1);
+  r->pen = dalloc<float>(o, std::max<size_t>(1, hg.slot_node.size() * (size_t)r->ngroups));
+  r->choice = dalloc<int32_t>(o, MB);
+  r->sel = dalloc<uint32_t>(o, (size_t)sh.N * sh.W);
+  r->reach = dalloc<uint32_t>(o, (size_t)sh.M * sh.W);
+  r->settle = dalloc<uint32_t>(o, (size_t)sh.M * sh.W);
+  r->flags = dalloc<int32_t>(o, 8);
+  r->dcost_rows = decode_cost_rows(sh);
+  r->dcost_part = dalloc<double>(o, (size_t)r->dcost_rows * sh.Bp);
+  r->dcost = dalloc<double>(o, sh.Bp);
+  r->dextra = dalloc<double>(o, sh.Bp);
+  r->best = dalloc<double>(o, 4);
+  r->best_flag = dalloc<int32_t>(o, 1);
+  r->best_choice = dalloc<int32_t>(o, sh.M);
+  r->counter = dalloc<int32_t>(o, 1);
+  r->scal = dalloc<double>(o, 2);
+  r->dbg_p = nullptr;
+
+  // cost model
+  std::vector<float> uf(sh.N);
+  std::vector<double> ud(cost->u, cost->u + sh.N);
+  for (int i = 0; i < sh.N; ++i) uf[i] = (float)cost->u[i];
+  r->u_f = upload(o, uf);
+  r->u_d = upload(o, ud);
+  if (r->cost_kind != SMOOTHE_COST_LINEAR) {
+    r->p = dalloc<float>(o, NB);
+    r->gp = dalloc<float>(o, NB);
+    r->sbin = dalloc<float>(o, NB);
+  }
+  if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
+    // symmetric neighbour lists: pair (i, j, w) appears as j in nbr(i) and i in nbr(j)
+    std::vector<int32_t> ptr(sh.N + 1, 0);
+    for (int64_t e = 0; e < cost->quad_nnz; ++e) {
+      ptr[cost->quad_i[e] + 1]++;
+      ptr[cost->quad_j[e] + 1]++;
+    }
+    for (int i = 0; i < sh.N; ++i) ptr[i + 1] += ptr[i];
+    std::vector<int32_t> nbr(ptr[sh.N]), fill(ptr.begin(), ptr.end() - 1);
+    std::vector<float> w(ptr[sh.N]);
+    for (int64_t e = 0; e < cost->quad_nnz; ++e) {
+      const int a = cost->quad_i[e], b = cost->quad_j[e];
+      w[fill[a]] = (float)cost->quad_w[e];
+      nbr[fill[a]++] = b;
+      w[fill[b]] = (float)cost->quad_w[e];
+      nbr[fill[b]++] = a;
+    }
+    r->q_ptr = upload(o, ptr);
+    r->q_nbr = upload(o, nbr);
+    r->q_w = upload(o, w);
+  }
+  if (r->cost_kind == SMOOTHE_COST_MLP) {
+    const int H1 = r->H1, H2 = r->H2;
+    r->W1 = upload(o, std::vector<float>(cost->W1, cost->W1 + (size_t)H1 * sh.N));
+    r->b1 = upload(o, std::vector<float>(cost->b1, cost->b1 + H1));
+    r->W2 = upload(o, std::vector<float>(cost->W2, cost->W2 + (size_t)H2 * H1));
+    r->b2 = upload(o, std::vector<float>(cost->b2, cost->b2 + H2));
+    r->W3 = upload(o, std::vector<float>(cost->W3, cost->W3 + H2));
+    r->b3 = upload(o, std::vector<float>(cost->b3, cost->b3 + 1));
+    r->nsplit = std::max(1, std::min(2 * num_sms(r->device), (sh.N + 255) / 256));
+    r->z1_part = dalloc<float>(o, (size_t)r->nsplit * H1 * sh.Bp);
+    r->gz1 = dalloc<float>(o, (size_t)H1 * sh.Bp);
+  }
+}
+
+void init_state(smoothe_run* r) {
+  const Shape& sh = r->sh;
+  cudaStream_t s = r->stream;
+  const size_t MB = (size_t)sh.M * sh.Bp;
+  launch_theta_init(s, sh, r->opt.rng_key, r->opt.seed_begin, r->theta, r->m, r->v);
+  SM_CUDA(cudaMemsetAsync(r->qstack, 0, sizeof(float) * (size_t)(r->K + 1) * MB, s));
+  launch_fill_rows(s, r->qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K + 1, sh.Bp, 1.0f);
+  if (r->pistack) {
+    SM_CUDA(cudaMemsetAsync(r->pistack, 0, sizeof(float) * (size_t)r->K * MB, s));
+    launch_fill_rows(s, r->pistack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K, sh.Bp, 1.0f);
+  }
+  SM_CUDA(cudaMemsetAsync(r->astack, 0, sizeof(int32_t) * std::max<size_t>(1, (size_t)r->K * MB), s));
+  SM_CUDA(cudaMemsetAsync(r->gq[0], 0, sizeof(float) * MB, s));
+  SM_CUDA(cudaMemsetAsync(r->gq[1], 0, sizeof(float) * MB, s));
+  SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
+  SM_CUDA(cudaMemsetAsync(r->fextra, 0, sizeof(double) * sh.Bp, s));
+  SM_CUDA(cudaMemsetAsync(r->counter, 0, sizeof(int32_t), s));
+  const double init_best[4] = {INFINITY, -1.0, -1.0, 0.0};
+  SM_CUDA(cudaMemcpyAsync(r->best, init_best, sizeof(init_best), cudaMemcpyHostToDevice, s));
+  SM_CUDA(cudaMemsetAsync(r->best_choice, 0xff, sizeof(int32_t) * sh.M, s));
+  SM_CUDA(cudaStreamSynchronize(s));
+}
+
+void copy_rows_d2h(float* dst, const float* src, int rows, int B, int Bp, cudaStream_t s) {
+  if (!dst) return;
+  SM_CUDA(cudaMemcpy2DAsync(dst, sizeof(float) * B, src, sizeof(float) * Bp, sizeof(float) * B,
+                            rows, cudaMemcpyDeviceToHost, s));
+}
+
+void copy_rows_h2d(float* dst, const float* src, int rows, int B, int Bp, cudaStream_t s) {
+  SM_CUDA(cudaMemcpy2DAsync(dst, sizeof(float) * Bp, src, sizeof(float) * B, sizeof(float) * B,
+                            rows, cudaMemcpyHostToDevice, s));
+}
+
+}  // namespace
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+const char* smoothe_last_error(void) { return g_last_error.c_str(); }
+const char* smoothe_version(void) { return "smoothe-b200 0.1 (sm_100a)"; }
+
+smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const int32_t* class_ptr,
+                                   const int64_t* child_ptr, const int32_t* child_class,
+                                   int32_t root_class, int device_ordinal, smoothe_egraph** out) {
+  if (!out) {
+    set_error("NULL out");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+  *out = nullptr;
+  smoothe_egraph* g = nullptr;
+  auto owner = new (std::nothrow) smoothe_egraph_dev_owner();
+  smoothe_status st = guarded(nullptr, [&] {
+    g = new smoothe_egraph();
+    build_host_graph(num_classes, num_nodes, class_ptr, child_ptr, child_class, root_class, g->host);
+    g->device = device_ordinal;
+    if (device_ordinal >= 0) {
+      int ndev = 0;
+      SM_CUDA(cudaGetDeviceCount(&ndev));
+      SM_REQUIRE(device_ordinal < ndev, SMOOTHE_E_INVALID_ARG, "device ordinal out of range");
+      SM_CUDA(cudaSetDevice(device_ordinal));
+      cudaDeviceProp prop;
+      SM_CUDA(cudaGetDeviceProperties(&prop, device_ordinal));
+      SM_REQUIRE(prop.major == 10, SMOOTHE_E_CUDA,
+                 "libsmoothe is built for sm_100a; device has sm_" + std::to_string(prop.major) +
+                     std::to_string(prop.minor));
+      auto& o = owner->owned;
+      const HostGraph& h = g->host;
+      DevGraph& d = g->dev;
+      int64_t& b = d.bytes;
+      d.class_ptr = upload(o, h.class_ptr, &b);
+      d.child_ptr = upload(o, h.child_ptr, &b);
+      d.child_class = upload(o, h.child_class, &b);
+      d.par_ptr = upload(o, h.par_ptr, &b);
+      d.par_node = upload(o, h.par_node, &b);
+      d.par_class = upload(o, h.par_class, &b);
+      d.scc_class_ptr = upload(o, h.scc_class_ptr, &b);
+      d.ent_ptr = upload(o, h.ent_ptr, &b);
+      d.ent_i = upload(o, h.ent_i, &b);
+      d.ent_j = upload(o, h.ent_j, &b);
+      d.ent_node_ptr = upload(o, h.ent_node_ptr, &b);
+      d.ent_node = upload(o, h.ent_node, &b);
+      d.slot_ptr = upload(o, h.slot_ptr, &b);
+      d.slot_node = upload(o, h.slot_node, &b);
+      d.slot_iloc = upload(o, h.slot_iloc, &b);
+      d.slot_jptr = upload(o, h.slot_jptr, &b);
+      d.slot_jloc = upload(o, h.slot_jloc, &b);
+      d.node_slot = upload(o, h.node_slot, &b);
+    }
+  });
+  if (st != SMOOTHE_OK) {
+    if (owner) {
+      for (void* p : owner->owned) cudaFree(p);
+      delete owner;
+    }
+    delete g;
+    return st;
+  }
+  delete owner;  // the allocations now belong to g->dev (freed by smoothe_free_egraph)
+  *out = g;
+  return SMOOTHE_OK;
+}
+
+smoothe_status smoothe_egraph_get_info(const smoothe_egraph* g, smoothe_egraph_info* out) {
+  if (!g || !out) {
+    set_error("NULL argument");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+  const HostGraph& h = g->host;
+  out->num_classes = h.M;
+  out->num_nodes = h.N;
+  out->num_edges = h.E;
+  out->root = h.root;
+  out->K_auto = h.K_auto;
+  out->num_scc = h.num_scc;
+  out->scc_classes = h.scc_classes;
+  out->scc_max = h.scc_max;
+  out->max_class_size = h.max_class_size;
+  out->max_in_degree = h.max_in_degree;
+  out->device = g->device;
+  out->device_bytes = g->dev.bytes;
+  return SMOOTHE_OK;
+}
+
+smoothe_status smoothe_egraph_get_scc(const smoothe_egraph* g, int32_t* scc_of_class) {
+  if (!g || !scc_of_class) {
+    set_error("NULL argument");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+  std::memcpy(scc_of_class, g->host.scc_of_class.data(), sizeof(int32_t) * g->host.M);
+  return SMOOTHE_OK;
+}
+
+smoothe_status smoothe_options_default(smoothe_options* opt) {
+  if (!opt) {
+    set_error("NULL options");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+  std::memset(opt, 0, sizeof(*opt));
+  opt->assumption = SMOOTHE_AGG_HYBRID;
+  opt->prop_iters = -1;
+  opt->lambda = 1.0;
+  opt->penalty_group = 1;
+  opt->lr = 0.1;
+  opt->beta1 = 0.9;
+  opt->beta2 = 0.999;
+  opt->eps = 1e-8;
+  opt->optimizer = 0;
+  opt->use_graphs = 1;
+  return SMOOTHE_OK;
+}
+
+smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* cost,
+                                  int32_t num_seeds, const smoothe_options* opt,
+                                  smoothe_run** out) {
+  if (!out) {
+    set_error("NULL out");
+    return SMOOTHE_E_INVALID_ARG;
+  }
+  *out = nullptr;
+  smoothe_run* r = new (std::nothrow) smoothe_run();
+  if (!r) return SMOOTHE_E_OOM;
+  smoothe_status st = guarded(nullptr, [&] {
+    SM_REQUIRE(g && cost && opt && cost->u, SMOOTHE_E_INVALID_ARG, "NULL argument");
+    SM_REQUIRE(g->device >= 0, SMOOTHE_E_STATE, "host-only e-graph (device_ordinal = -1)");
+    SM_REQUIRE(num_seeds > 0, SMOOTHE_E_INVALID_ARG, "num_seeds must be > 0");
+    SM_REQUIRE(opt->penalty_group > 0 && num_seeds % opt->penalty_group == 0,
+               SMOOTHE_E_INVALID_ARG, "penalty_group must divide num_seeds (S13)");
+    SM_REQUIRE(opt->assumption >= 0 && opt->assumption <= 2, SMOOTHE_E_INVALID_ARG, "bad assumption");
+    SM_REQUIRE(opt->optimizer == 0 || opt->optimizer == 1, SMOOTHE_E_INVALID_ARG, "bad optimizer");
+    SM_REQUIRE(cost->kind >= 0 && cost->kind <= 2, SMOOTHE_E_INVALID_ARG, "bad cost kind");
+    SM_REQUIRE(g->host.scc_max <= 64, SMOOTHE_E_INVALID_ARG,
+               "strongly connected components larger than 64 classes are not supported yet");
+    r->g = g;
+    r->opt = *opt;
+    r->device = g->device;
+    SM_CUDA(cudaSetDevice(r->device));
+    const HostGraph& hg = g->host;
+    Shape& sh = r->sh;
+    sh.M = hg.M;
+    sh.N = hg.N;
+    sh.root = hg.root;
+    sh.B = num_seeds;
+    sh.Bp = num_seeds <= 32 ? 32 : num_seeds <= 64 ? 64 : ((num_seeds + 127) / 128) * 128;
+    sh.W = sh.Bp / 32;
+    r->K = opt->prop_iters < 0 ? hg.K_auto : opt->prop_iters;
+    r->G = opt->penalty_group;
+    r->ngroups = num_seeds / r->G;
+    r->agg = opt->assumption == SMOOTHE_AGG_INDEPENDENT   ? Agg{1.f, 0.f}
+             : opt->assumption == SMOOTHE_AGG_CORRELATED ? Agg{0.f, 1.f}
+                                                          : Agg{0.5f, 0.5f};
+    r->cost_kind = cost->kind;
+    if (cost->kind == SMOOTHE_COST_QUADRATIC) {
+      SM_REQUIRE(cost->quad_nnz >= 0 && (cost->quad_nnz == 0 || (cost->quad_i && cost->quad_j && cost->quad_w)),
+                 SMOOTHE_E_INVALID_ARG, "quadratic pairs missing");
+      for (int64_t e = 0; e < cost->quad_nnz; ++e)
+        SM_REQUIRE(cost->quad_i[e] >= 0 && cost->quad_i[e] < sh.N && cost->quad_j[e] >= 0 &&
+                       cost->quad_j[e] < sh.N && cost->quad_i[e] != cost->quad_j[e],
+                   SMOOTHE_E_INVALID_ARG, "bad quadratic pair");
+    }
+    if (cost->kind == SMOOTHE_COST_MLP) {
+      SM_REQUIRE(cost->W1 && cost->b1 && cost->W2 && cost->b2 && cost->W3 && cost->b3,
+                 SMOOTHE_E_INVALID_ARG, "MLP weights missing");
+      SM_REQUIRE(cost->mlp_hidden1 > 0 && cost->mlp_hidden1 <= 64 && cost->mlp_hidden2 > 0 &&
+                     cost->mlp_hidden2 <= 16,
+                 SMOOTHE_E_INVALID_ARG, "MLP hidden sizes must be <= 64 and <= 16");
+      r->H1 = cost->mlp_hidden1;
+      r->H2 = cost->mlp_hidden2;
+    }
+    SM_CUDA(cudaStreamCreateWithFlags(&r->stream, cudaStreamNonBlocking));
+    r->coop_grid = decode_grid(r->device);
+    alloc_state(r, cost);
+    SM_CUDA(cudaEventCreate(&r->ev_start));
+    r->ev_step.resize(4096);
+    for (auto& e : r->ev_step) SM_CUDA(cudaEventCreate(&e));
+    r->t_create = std::chrono::steady_clock::now();
+    SM_CUDA(cudaEventRecord(r->ev_start, r->stream));
+    init_state(r);
+    g->refcount++;
+  });
+  if (st != SMOOTHE_OK) {
+    for (void* p : r->owned) cudaFree(p);
+    if (r->stream) cudaStreamDestroy(r->stream);
+    delete r;
+    return st;
+  }
+  *out = r;
+  return SMOOTHE_OK;
+}
+
+smoothe_status smoothe_run_steps(smoothe_run* run, int32_t steps) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(steps >= 0, SMOOTHE_E_INVALID_ARG, "steps must be >= 0");
+    cudaStream_t user = (cudaStream_t)run->opt.cuda_stream;
+    cudaEvent_t join = nullptr;
+    if (user) {  // order after the caller's stream
+      SM_CUDA(cudaEventCreateWithFlags(&join, cudaEventDisableTiming));
+      SM_CUDA(cudaEventRecord(join, user));
+      SM_CUDA(cudaStreamWaitEvent(run->stream, join, 0));
+    }
+    const bool checks = run->opt.patience > 0 || run->opt.time_limit_s > 0;
+    for (int32_t i = 0; i < steps; ++i) {
+      run_one_step(run);
+      if (checks && ((i + 1) % 8 == 0 || i + 1 == steps)) {
+        double best[4];
+        SM_CUDA(cudaMemcpyAsync(best, run->best, sizeof(best), cudaMemcpyDeviceToHost, run->stream));
+        SM_CUDA(cudaStreamSynchronize(run->stream));
+        if (run->opt.patience > 0 && best[3] >= run->opt.patience) break;
+        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - run->t_create).count();
+        if (run->opt.time_limit_s > 0 && el >= run->opt.time_limit_s) break;
+      }
+    }
+    if (user) {
+      SM_CUDA(cudaEventRecord(join, run->stream));
+      SM_CUDA(cudaStreamWaitEvent(user, join, 0));
+      SM_CUDA(cudaEventDestroy(join));
+    }
+  });
+}
+
+smoothe_status smoothe_run_synchronize(smoothe_run* run) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+  });
+}
+
+smoothe_status smoothe_optimize(smoothe_egraph* g, const smoothe_cost_model* cost, int32_t num_seeds,
+                                int32_t steps, const smoothe_options* opt, smoothe_run** out) {
+  smoothe_status st = smoothe_run_create(g, cost, num_seeds, opt, out);
+  if (st != SMOOTHE_OK) return st;
+  st = smoothe_run_steps(*out, steps);
+  if (st != SMOOTHE_OK) return st;
+  return smoothe_run_synchronize(*out);
+}
+
+smoothe_status smoothe_extract(smoothe_run* run, int32_t* choice, smoothe_summary* out) {
+  bool valid = false;
+  smoothe_status st = guarded(run, [&] {
+    check_run(run);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+    double best[4], loss = 0.0;
+    SM_CUDA(cudaMemcpy(best, run->best, sizeof(best), cudaMemcpyDeviceToHost));
+    SM_CUDA(cudaMemcpy(&loss, run->loss, sizeof(double), cudaMemcpyDeviceToHost));
+    valid = std::isfinite(best[0]);
+    if (choice) SM_CUDA(cudaMemcpy(choice, run->best_choice, sizeof(int32_t) * run->sh.M, cudaMemcpyDeviceToHost));
+    if (out) {
+      std::memset(out, 0, sizeof(*out));
+      out->best_cost = best[0];
+      out->best_step = (int32_t)best[1];
+      out->best_seed = (int64_t)best[2];
+      out->valid = valid ? 1 : 0;
+      out->steps_run = run->steps_run;
+      out->K = run->K;
+      out->last_loss = loss;
+      float ms = 0.f;
+      const int bs = out->best_step;
+      if (valid && bs >= 0 && (size_t)bs < run->ev_step.size() && bs < run->steps_run) {
+        SM_CUDA(cudaEventElapsedTime(&ms, run->ev_start, run->ev_step[bs]));
+        out->time_to_best_s = ms * 1e-3;
+      } else {
+        out->time_to_best_s = -1.0;
+      }
+      const int last = std::min<int>(run->steps_run, (int)run->ev_step.size()) - 1;
+      if (last >= 0) {
+        SM_CUDA(cudaEventElapsedTime(&ms, run->ev_start, run->ev_step[last]));
+        out->step_time_s = ms * 1e-3 / (last + 1);
+      }
+    }
+  });
+  if (st == SMOOTHE_OK && !valid) {
+    set_error("no valid extraction sampled");
+    return SMOOTHE_E_NO_VALID;
+  }
+  return st;
+}
+
+smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const float* m_in,
+                                  const float* v_in, int32_t step_index, smoothe_debug_out* dump) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(dump != nullptr, SMOOTHE_E_INVALID_ARG, "NULL dump");
+    SM_REQUIRE(step_index >= 0, SMOOTHE_E_INVALID_ARG, "step_index must be >= 0");
+    const Shape& sh = run->sh;
+    cudaStream_t s = run->stream;
+    const size_t NB = (size_t)sh.N * sh.Bp;
+    if (theta_in) copy_rows_h2d(run->theta, theta_in, sh.N, sh.B, sh.Bp, s);
+    if (m_in) copy_rows_h2d(run->m, m_in, sh.N, sh.B, sh.Bp, s);
+    else SM_CUDA(cudaMemsetAsync(run->m, 0, sizeof(float) * NB, s));
+    if (v_in) copy_rows_h2d(run->v, v_in, sh.N, sh.B, sh.Bp, s);
+    else SM_CUDA(cudaMemsetAsync(run->v, 0, sizeof(float) * NB, s));
+    SM_CUDA(cudaMemcpyAsync(run->counter, &step_index, sizeof(int32_t), cudaMemcpyHostToDevice, s));
+    // debug scratch
+    std::vector<void*> scratch;
+    run->dbg_p = run->cost_kind == SMOOTHE_COST_LINEAR ? dalloc<float>(scratch, NB) : nullptr;
+    run->dbg_gth = dalloc<float>(scratch, NB);
+    run->dbg_gcp = dalloc<float>(scratch, NB);
+    run->dbg_dcost = dalloc<double>(scratch, sh.Bp);
+    run->dbg_valid = dalloc<uint8_t>(scratch, sh.Bp);
+    std::vector<float> theta_keep;
+    run->debug = true;
+    try {
+      // the step overwrites theta; keep the input's cp etc. from the step itself
+      enqueue_step(run);
+    } catch (...) {
+      run->debug = false;
+      for (void* p : scratch) cudaFree(p);
+      throw;
+    }
+    run->debug = false;
+    const size_t MB = (size_t)sh.M * sh.Bp;
+    const float* pdev = run->cost_kind == SMOOTHE_COST_LINEAR ? run->dbg_p : run->p;
+    copy_rows_d2h(dump->cp, run->cp, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->qK, run->qstack + (size_t)run->K * MB, sh.M, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->p, pdev, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->grad_cp, run->dbg_gcp, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->grad_theta, run->dbg_gth, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->theta_out, run->theta, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->m_out, run->m, sh.N, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->v_out, run->v, sh.N, sh.B, sh.Bp, s);
+    if (dump->qstack)
+      copy_rows_d2h(dump->qstack, run->qstack, (run->K + 1) * sh.M, sh.B, sh.Bp, s);
+    if (dump->f) SM_CUDA(cudaMemcpyAsync(dump->f, run->ftot, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
+    if (dump->h) {
+      if (run->g->host.num_scc > 0)
+        SM_CUDA(cudaMemcpyAsync(dump->h, run->h, sizeof(double) * run->ngroups, cudaMemcpyDeviceToHost, s));
+      else
+        std::memset(dump->h, 0, sizeof(double) * run->ngroups);
+    }
+    if (dump->loss) SM_CUDA(cudaMemcpyAsync(dump->loss, run->loss, sizeof(double), cudaMemcpyDeviceToHost, s));
+    if (dump->choice)
+      SM_CUDA(cudaMemcpy2DAsync(dump->choice, sizeof(int32_t) * sh.B, run->choice, sizeof(int32_t) * sh.Bp,
+                                sizeof(int32_t) * sh.B, sh.M, cudaMemcpyDeviceToHost, s));
+    if (dump->valid) SM_CUDA(cudaMemcpyAsync(dump->valid, run->dbg_valid, sh.B, cudaMemcpyDeviceToHost, s));
+    if (dump->disc_cost)
+      SM_CUDA(cudaMemcpyAsync(dump->disc_cost, run->dbg_dcost, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
+    std::vector<uint32_t> rbits;
+    if (dump->reached) {
+      rbits.resize((size_t)sh.M * sh.W);
+      SM_CUDA(cudaMemcpyAsync(rbits.data(), run->reach, sizeof(uint32_t) * rbits.size(), cudaMemcpyDeviceToHost, s));
+    }
+    SM_CUDA(cudaStreamSynchronize(s));
+    if (dump->reached)
+      for (int j = 0; j < sh.M; ++j)
+        for (int b = 0; b < sh.B; ++b)
+          dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
+    for (void* p : scratch) SM_CUDA(cudaFree(p));
+    run->dbg_p = run->dbg_gth = run->dbg_gcp = nullptr;
+    run->dbg_dcost = nullptr;
+    run->dbg_valid = nullptr;
+    run->steps_run++;
+  });
+}
+
+smoothe_status smoothe_get_theta(smoothe_run* run, float* theta) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(theta, SMOOTHE_E_INVALID_ARG, "NULL theta");
+    copy_rows_d2h(theta, run->theta, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+  });
+}
+
+smoothe_status smoothe_run_profile(smoothe_run* run, int32_t enable) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+    run->profiling = enable != 0;
+    run->prof_ev.clear();
+    run->prof_pool_used = 0;
+    std::memset(run->prof_launch, 0, sizeof(run->prof_launch));
+    run->prof_launch_total = 0;
+    run->prof_steps = 0;
+  });
+}
+
+smoothe_status smoothe_run_get_profile(smoothe_run* run, smoothe_profile* out) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(out, SMOOTHE_E_INVALID_ARG, "NULL out");
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+    std::memset(out, 0, sizeof(*out));
+    for (const auto& ev : run->prof_ev) {
+      for (int ph = 0; ph < SMOOTHE_NUM_PHASES; ++ph) {
+        float ms = 0.f;
+        SM_CUDA(cudaEventElapsedTime(&ms, ev[ph], ev[ph + 1]));
+        out->phase_ms[ph] += ms;
+      }
+    }
+    for (int ph = 0; ph < SMOOTHE_NUM_PHASES; ++ph) out->phase_launches[ph] = run->prof_launch[ph];
+    out->steps = run->prof_steps;
+    out->launches = run->prof_launch_total;
+    out->num_seeds_padded = run->sh.Bp;
+  });
+}
+
+void smoothe_free_run(smoothe_run* run) {
+  if (!run) return;
+  cudaSetDevice(run->device);
+  cudaStreamSynchronize(run->stream);
+  if (run->graph_exec) cudaGraphExecDestroy(run->graph_exec);
+  for (void* p : run->owned) cudaFree(p);
+  for (auto e : run->ev_step) cudaEventDestroy(e);
+  for (auto e : run->prof_pool) cudaEventDestroy(e);
+  if (run->ev_start) cudaEventDestroy(run->ev_start);
+  if (run->stream) cudaStreamDestroy(run->stream);
+  if (run->g) {
+    run->g->refcount--;
+    if (run->g->freed && run->g->refcount == 0) smoothe_free_egraph(run->g);
+  }
+  delete run;
+}
+
+void smoothe_free_egraph(smoothe_egraph* g) {
+  if (!g) return;
+  g->freed = true;
+  if (g->refcount > 1) {  // runs still alive: freed when the last one goes
+    g->refcount--;
+    return;
+  }
+  // device arrays
+  DevGraph& d = g->dev;
+  if (g->device >= 0) {
+    cudaSetDevice(g->device);
+    void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
+                    d.scc_class_ptr, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
+                    d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot};
+    for (void* p : ptrs) cudaFree(p);
+  }
+  delete g;
+}
+
+}  // extern "C"

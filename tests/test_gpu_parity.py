@@ -1,0 +1,260 @@
+"""GPU path (libsmoothe.so through its C ABI) vs the fp64 oracle, element by
+element on the same seeded inputs (SURVEY.md 8(c) parity protocol).
+
+Bars (BASELINE.json north_star):
+* bit-exact: theta initialisation, decoded choices, reached sets, validity,
+  integer discrete costs (linear / quadratic with integer u, w);
+* |gpu - ref| <= 1e-6 + 1e-4 |ref| for cp, q^K, p, f, h, loss, g_cp;
+* g_theta = cp (g_cp - sum cp g_cp) cancels by construction, so its bound is
+  1e-6 + 1e-4 * (magnitude of the terms combined): cp (|g_cp| + sum cp |g_cp|);
+* the optimiser update is compared given the GPU's own gradient (Adam divides
+  by sqrt(v) and amplifies gradient rounding near g = 0).
+"""
+import numpy as np
+import pytest
+
+from gen import CONFIGS, fig1c_fixture, make_config, random_tiny
+
+pytestmark = pytest.mark.gpu
+
+AGGS = ["independent", "correlated", "hybrid"]
+RTOL, ATOL = 1e-4, 1e-6
+
+
+@pytest.fixture(scope="module")
+def sm():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_asplos_caiydyz25_b200 as pkg
+    pkg.lib()
+    return pkg
+
+
+def close(name, got, ref, scale=None, rtol=RTOL, atol=ATOL):
+    got = np.asarray(got, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    scale = np.abs(ref) if scale is None else scale
+    err = np.abs(got - ref) - (atol + rtol * scale)
+    bad = np.argwhere(err > 0)
+    assert bad.size == 0, (f"{name}: {len(bad)} of {ref.size} outside tolerance; first "
+                           f"{bad[:3].tolist()} got {got[tuple(bad[0])]} ref {ref[tuple(bad[0])]}")
+
+
+def class_sums(eg, x):
+    """sum over the e-nodes of each class, broadcast back to the e-nodes."""
+    ec = eg.ec()
+    out = np.zeros((eg.num_classes,) + x.shape[1:])
+    np.add.at(out, ec, x)
+    return out[ec]
+
+
+def compare_step(sm, orc, eg, B, G, agg="hybrid", lam=1.0, theta=None, m=None, v=None,
+                 step_index=0, K=-1, seed=0, cols=None, lr=0.1):
+    g = sm.load_egraph_from(eg, device=0)
+    Kr = g.K_auto if K < 0 else K
+    opts = sm.Options(assumption=agg, prop_iters=K, lam=lam, penalty_group=G, lr=lr, rng_key=3)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), B, opts)
+    rng = np.random.default_rng(seed)
+    if theta is None:
+        theta = rng.uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
+    d = run.debug_step(theta, m, v, step_index=step_index)
+    cols = slice(None) if cols is None else cols
+    th = theta[:, cols].astype(np.float64)
+    og = orc.Graph(eg)
+    assert og.K_auto == g.K_auto
+    oo = orc.Options(assumption=agg, K=Kr, lam=lam, G=G, lr=lr)
+    o = og.step(th, oo, m=None if m is None else m[:, cols], v=None if v is None else v[:, cols],
+                step_index=step_index)
+    sel = lambda a: a[:, cols]
+    close("cp", sel(d["cp"]), o["cp"])
+    close("p", sel(d["p"]), o["p"])
+    close("f", d["f"][cols], o["f"])
+    nb = th.shape[1]
+    close("h", d["h"][: nb // G], o["h"])            # cols always start at seed 0
+    close("grad_cp", sel(d["grad_cp"]), o["grad_cp"])
+    cpo, gco = o["cp"], o["grad_cp"]
+    gscale = cpo * (np.abs(gco) + class_sums(eg, cpo * np.abs(gco)))
+    close("grad_theta", sel(d["grad_theta"]), o["grad_theta"], scale=gscale)
+    assert np.array_equal(sel(d["choice"]), o["choice"])
+    assert np.array_equal(sel(d["reached"]), o["reached"])
+    assert np.array_equal(d["valid"][cols], o["valid"])
+    ok = o["valid"] == 1
+    if eg.mlp is None:
+        assert np.array_equal(d["disc_cost"][cols][ok], o["disc_cost"][ok])
+    else:
+        close("disc_cost", d["disc_cost"][cols][ok], o["disc_cost"][ok])
+    assert np.all(np.isinf(d["disc_cost"][cols][~ok]))
+    # optimiser given the GPU gradient
+    u = orc.update(th, sel(d["grad_theta"]), oo, m=None if m is None else m[:, cols],
+                   v=None if v is None else v[:, cols], step_index=step_index)
+    for k in ("theta_out", "m_out", "v_out"):
+        close(k, sel(d[k]), u[k], rtol=2e-5, atol=1e-6)
+    if cols == slice(None):
+        close("loss", d["loss"], o["loss"])
+    run.close()
+    g.close()
+    return d, o
+
+
+def test_theta_init_bitexact(sm, orc):
+    eg = make_config("C2")
+    g = sm.load_egraph_from(eg)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), 96,
+                        sm.Options(rng_key=0x5EED0002, seed_begin=5, penalty_group=8))
+    th = run.theta()
+    ref = orc.theta_init(0x5EED0002, 5, 96, eg.num_nodes)
+    assert np.array_equal(th.astype(np.float64), ref)
+
+
+@pytest.mark.parametrize("agg", AGGS)
+def test_fig1c_step(sm, orc, agg):
+    eg = fig1c_fixture()
+    rng = np.random.default_rng(1)
+    th = rng.uniform(-1, 1, (10, 4)).astype(np.float32)
+    d, o = compare_step(sm, orc, eg, 4, 2, agg, theta=th)
+    # the paper's closed form on the GPU path too
+    c1, c4 = d["cp"][1], d["cp"][4]
+    assert np.allclose(d["f"], 19 + 13 * c1 - 5 * c1 * c4, rtol=1e-6)
+
+
+@pytest.mark.parametrize("agg", AGGS)
+@pytest.mark.parametrize("kind", ["tree", "dag", "cyclic"])
+def test_tiny_families(sm, orc, agg, kind):
+    for s in range(6):
+        eg = random_tiny(3000 + s, kind, num_classes=8)
+        # B = 33: ragged (padded to 64 internally), 11 penalty groups of 3
+        compare_step(sm, orc, eg, 33, 3, agg, lam=0.7, seed=s, K=3 + s % 4)
+
+
+def test_tiny_second_adam_step(sm, orc):
+    eg = random_tiny(3100, "cyclic")
+    rng = np.random.default_rng(2)
+    B = 8
+    m = rng.normal(0, 0.1, (eg.num_nodes, B)).astype(np.float32)
+    v = rng.uniform(0, 0.05, (eg.num_nodes, B)).astype(np.float32)
+    compare_step(sm, orc, eg, B, 4, m=m, v=v, step_index=6)
+
+
+def test_one_hot_and_ties(sm, orc):
+    """Degenerate inputs: one-hot logits (cp in {0,1}, q = 1 exactly, zero
+    factors in the product), exact logit ties (lowest id wins)."""
+    eg = random_tiny(3200, "cyclic", num_classes=8)
+    rng = np.random.default_rng(3)
+    B = 32
+    th = np.zeros((eg.num_nodes, B), np.float32)
+    ec = eg.ec()
+    for j in range(eg.num_classes):
+        idx = np.where(ec == j)[0]
+        for b in range(B):
+            if b % 3 == 0:
+                th[rng.choice(idx), b] = 1e4      # one-hot
+            elif b % 3 == 1:
+                th[idx, b] = 0.25                 # all tied
+            else:
+                th[idx, b] = rng.uniform(-1, 1, idx.size)
+    compare_step(sm, orc, eg, B, 4, theta=th, lam=0.5)
+
+
+@pytest.mark.parametrize("B,G", [(64, 8), (100, 10), (200, 8)])
+def test_c2_full(sm, orc, B, G):
+    compare_step(sm, orc, make_config("C2"), B, G, seed=B)
+
+
+@pytest.mark.parametrize("agg", ["independent", "correlated"])
+def test_c2_aggregators(sm, orc, agg):
+    compare_step(sm, orc, make_config("C2"), 64, 8, agg, seed=5)
+
+
+def test_c3_quadratic_full(sm, orc):
+    spec = CONFIGS["C3"]
+    compare_step(sm, orc, make_config("C3"), spec["seeds_per_gpu"], spec["group"], seed=3)
+
+
+def test_c5_mlp_full(sm, orc):
+    spec = CONFIGS["C5"]
+    compare_step(sm, orc, make_config("C5"), spec["seeds_per_gpu"], spec["group"], seed=4)
+
+
+def test_c4_full_size_first_group(sm, orc):
+    """C4 at the bench launch configuration (128 seeds, G = 16): the oracle
+    recomputes the first penalty group (16 seeds) exactly."""
+    spec = CONFIGS["C4"]
+    B, G = spec["seeds_per_gpu"], spec["group"]
+    compare_step(sm, orc, make_config("C4"), B, G, seed=6, cols=slice(0, G))
+
+
+def test_graphs_and_direct_launches_identical(sm):
+    eg = make_config("C2")
+    outs = []
+    for use_graphs in (True, False):
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), 64,
+                            sm.Options(penalty_group=8, rng_key=11, use_graphs=use_graphs))
+        run.steps(12)
+        outs.append((run.theta(), run.extract()))
+        run.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][1][0], outs[1][1][0])
+    assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
+
+
+def test_seed_sharding_bit_identical(sm):
+    """8(e): a run of 64 seeds equals two runs of 32 seeds (seed_begin 0, 32)
+    seed by seed, and the lexicographic best of the shards is the full best."""
+    eg = make_config("C2")
+    g = sm.load_egraph_from(eg)
+    cost = sm.CostModel.from_input(eg)
+    full = sm.run_create(g, cost, 64, sm.Options(penalty_group=8, rng_key=5))
+    full.steps(15)
+    tf = full.theta()
+    cf, sf = full.extract()
+    halves = []
+    for sb in (0, 32):
+        r = sm.run_create(g, cost, 32, sm.Options(penalty_group=8, rng_key=5, seed_begin=sb))
+        r.steps(15)
+        halves.append((r.theta(), r.extract()))
+    assert np.array_equal(np.concatenate([halves[0][0], halves[1][0]], axis=1), tf)
+    bests = sorted((h[1][1]["best_cost"], h[1][1]["best_step"], h[1][1]["best_seed"], i)
+                   for i, h in enumerate(halves))
+    c, st, seed, i = bests[0]
+    assert (c, st, seed) == (sf["best_cost"], sf["best_step"], sf["best_seed"])
+    assert np.array_equal(halves[i][1][0], cf)
+
+
+def test_best_of_seeds_fig1c(sm):
+    eg = fig1c_fixture()
+    g = sm.load_egraph_from(eg)
+    run = sm.optimize(g, sm.CostModel.from_input(eg), 16, 100,
+                      sm.Options(prop_iters=4, lam=1.0, penalty_group=4, rng_key=0x5EED0001))
+    choice, s = run.extract()
+    assert s["valid"] == 1 and s["best_cost"] == 19.0
+    assert choice[1] == 2 and choice[3] == -1
+    assert s["steps_run"] == 100 and s["time_to_best_s"] > 0
+
+
+def test_extracted_solution_is_valid(sm, orc):
+    from oracle import brute
+    eg = make_config("C2")
+    g = sm.load_egraph_from(eg)
+    run = sm.optimize(g, sm.CostModel.from_input(eg), 64, 30,
+                      sm.Options(penalty_group=8, rng_key=9))
+    choice, s = run.extract()
+    assert s["valid"] == 1
+    # the extraction: every selected class's chosen node lies in it, its child
+    # classes are selected, no cycle, and the cost is the sum of u
+    sel = np.where(choice >= 0)[0]
+    ch = {int(j): int(choice[j]) for j in sel}
+    r = brute.reach(eg, [ch.get(j, int(eg.class_ptr[j])) for j in range(eg.num_classes)])
+    assert r == set(ch)
+    assert brute.acyclic(eg, [ch.get(j, int(eg.class_ptr[j])) for j in range(eg.num_classes)], r)
+    assert sum(eg.u[ch[j]] for j in ch) == s["best_cost"]
+
+
+def test_patience_stops_early(sm):
+    eg = fig1c_fixture()
+    g = sm.load_egraph_from(eg)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), 4,
+                        sm.Options(prop_iters=4, penalty_group=4, patience=16))
+    run.steps(1000)
+    _, s = run.extract()
+    assert s["steps_run"] < 1000
