@@ -191,7 +191,10 @@ def run_ours(args):
     Bl, G = spec["seeds_per_gpu"], spec["group"]
     lam = float(np.mean(eg.u))      # reading S11: lambda = mean(u)
     cost = sm.CostModel.from_input(eg)
-    stream = torch.cuda.current_stream()
+    # a real (non-legacy) stream: the library orders its private stream after
+    # this one and this one after its work, so events here bracket the steps
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     opts = sm.Options(assumption="hybrid", prop_iters=-1, lam=lam, penalty_group=G, lr=0.1,
                       rng_key=key, seed_begin=rank * Bl, cuda_stream=stream.cuda_stream,
                       use_graphs=True)
@@ -249,6 +252,10 @@ def run_ours(args):
             "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
             "step_alg_GBps": bm["step"] * Bl * N / (step_ms * 1e-3) / 1e9}
 
+    run.close()
+    g.close()
+    torch.cuda.synchronize()
+
     # e2e: the C-ABI calls with host buffers: load (H2D) + optimize (init + steps) + extract (D2H)
     e2e = None
     if not args.no_e2e:
@@ -300,8 +307,6 @@ def run_ours(args):
             "roofline": roof, "e2e": e2e, "cpu_baseline": cb, "clocks": ck,
         }
         print(json.dumps(line), flush=True)
-    run.close()
-    g.close()
     if world > 1:
         dist.destroy_process_group()
     return 0

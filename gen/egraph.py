@@ -247,6 +247,13 @@ def synth_egraph(name: str, N: int, M: int, d: float, D: int, *, seed: int,
         keep = ~drop
         owner, child, isback = owner[keep], child[keep], isback[keep]
 
+    # an upward edge that closes no cycle would only stretch the acyclic skeleton
+    # beyond D levels: keep back edges inside strongly connected components only
+    A = csr_matrix((np.ones(owner.size, dtype=np.int8), (ec[owner], child)), shape=(M, M))
+    _, lab = connected_components(A, directed=True, connection="strong")
+    keep = ~isback | (lab[ec[owner]] == lab[child])
+    owner, child, isback = owner[keep], child[keep], isback[keep]
+
     ptr_ns, child_ns = _csr(owner, child, N)
     cnt_all = np.diff(ptr_ns)[src]
     child_ptr = np.zeros(N + 1, dtype=np.int64)

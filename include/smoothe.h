@@ -201,6 +201,9 @@ typedef struct {
   uint8_t *valid;      /* [B]                                                  */
   double *disc_cost;   /* [B]     f_b(s), +inf when invalid                    */
   float *qstack;       /* [(K+1)][M][B] or NULL                                */
+  int32_t *route;      /* [K][M][B] e-node the max of sweep t routed to, i.e.  */
+                       /* the lowest id attaining the fp32 max (reading S7);  */
+                       /* -1 for classes without parents; NULL = skip         */
 } smoothe_debug_out;
 
 SMOOTHE_API smoothe_status smoothe_debug_step(smoothe_run *run, const float *theta_in, const float *m_in,

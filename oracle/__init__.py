@@ -53,7 +53,8 @@ class _Opts(C.Structure):
 class _Dump(C.Structure):
     _fields_ = [(n, C.c_void_p) for n in
                 ("cp", "qstack", "p", "f", "h", "loss", "grad_cp", "grad_theta", "theta_out",
-                 "m_out", "v_out", "choice", "valid", "disc_cost", "reached")]
+                 "m_out", "v_out", "choice", "valid", "disc_cost", "reached", "route",
+                 "route_invalid")]
 
 
 def lib():
@@ -191,8 +192,11 @@ class Graph:
         lib().oracle_graph_scc(self.h, _p(out))
         return out
 
-    def step(self, theta, opts: Options, m=None, v=None, step_index=0, qstack=False):
-        """One step for B seeds; theta [N][B] (any float dtype; upcast exactly)."""
+    def step(self, theta, opts: Options, m=None, v=None, step_index=0, qstack=False, route=None):
+        """One step for B seeds; theta [N][B] (any float dtype; upcast exactly).
+
+        route [K][M][B] int32 (optional): the max-routing decisions of the
+        system under test; the oracle validates and uses them (backward())."""
         theta = np.ascontiguousarray(theta, dtype=np.float64)
         N, B = theta.shape
         assert N == self.N
@@ -209,6 +213,12 @@ class Graph:
         }
         if qstack:
             out["qstack"] = np.zeros((K + 1, self.M, B))
+        out["route_invalid"] = np.zeros(B, dtype=np.int64)
+        keep = None
+        if route is not None:
+            keep = np.ascontiguousarray(route, dtype=np.int32)
+            assert keep.shape == (K, self.M, B)
+            out["route"] = keep
         d = _Dump(**{k: _p(a) for k, a in out.items()})
         rc = lib().oracle_step(self.h, C.byref(self.cost), C.byref(opts.c()), B, _p(theta), _p(m),
                                _p(v), step_index, C.byref(d))

@@ -126,50 +126,40 @@ void compute_scc(Graph& g) {
   }
 }
 
-// K_auto (reading S1): longest root path, in class hops, of the class graph
-// restricted to classes reachable from the root, after deleting the back edges
-// of a DFS from the root that visits successors in increasing class id.
+// K_auto (reading S1): the longest path from the root's component
+// in the condensation of the class graph (every strongly connected component
+// contracted to one vertex; one hop per edge between components).  On a DAG
+// every component is a single class, so this is the exact depth D at which the
+// parallel schedule reaches its fixed point (P213, P215).
 int compute_K_auto(const Graph& g) {
-  const int M = g.M;
-  std::vector<std::vector<int>> succ(M);
-  for (int j = 0; j < M; ++j) {
+  int ncomp = 0;
+  for (int c : g.scc_of) ncomp = std::max(ncomp, c + 1);
+  std::vector<std::vector<int>> succ(ncomp);
+  std::vector<int> indeg(ncomp, 0);
+  for (int j = 0; j < g.M; ++j)
     for (int k = g.class_begin[j]; k < g.class_end[j]; ++k)
-      for (int c : g.ch[k]) succ[j].push_back(c);
-    std::sort(succ[j].begin(), succ[j].end());
-    succ[j].erase(std::unique(succ[j].begin(), succ[j].end()), succ[j].end());
-  }
-  std::vector<int> color(M, 0);  // 0 white, 1 grey (on stack), 2 black
-  std::vector<int> order;        // post-order
-  std::vector<std::vector<int>> dag(M);
-  std::vector<std::pair<int, size_t>> st;
-  st.push_back({g.root, 0});
-  color[g.root] = 1;
-  while (!st.empty()) {
-    int v = st.back().first;
-    size_t& pos = st.back().second;
-    if (pos < succ[v].size()) {
-      int w = succ[v][pos++];
-      if (color[w] == 1) continue;  // back edge: deleted
-      dag[v].push_back(w);
-      if (color[w] == 0) {
-        color[w] = 1;
-        st.push_back({w, 0});
+      for (int c : g.ch[k]) {
+        const int a = g.scc_of[j], b = g.scc_of[c];
+        if (a != b) succ[a].push_back(b);
       }
-    } else {
-      color[v] = 2;
-      order.push_back(v);
-      st.pop_back();
-    }
+  for (auto& s : succ) {
+    std::sort(s.begin(), s.end());
+    s.erase(std::unique(s.begin(), s.end()), s.end());
+    for (int b : s) indeg[b]++;
   }
-  // longest path from the root over the DAG, in reverse post-order
-  std::vector<int> dist(M, -1);
-  dist[g.root] = 0;
+  // Kahn's topological order of the condensation, longest distance from the root
+  std::vector<int> order, dist(ncomp, -1);
+  for (int a = 0; a < ncomp; ++a)
+    if (indeg[a] == 0) order.push_back(a);
+  for (size_t i = 0; i < order.size(); ++i)
+    for (int b : succ[order[i]])
+      if (--indeg[b] == 0) order.push_back(b);
+  dist[g.scc_of[g.root]] = 0;
   int best = 0;
-  for (auto it = order.rbegin(); it != order.rend(); ++it) {
-    int v = *it;
-    if (dist[v] < 0) continue;
-    best = std::max(best, dist[v]);
-    for (int w : dag[v]) dist[w] = std::max(dist[w], dist[v] + 1);
+  for (int a : order) {
+    if (dist[a] < 0) continue;
+    best = std::max(best, dist[a]);
+    for (int b : succ[a]) dist[b] = std::max(dist[b], dist[a] + 1);
   }
   return best;
 }
@@ -292,6 +282,8 @@ struct oracle_dump {
   uint8_t* valid;      // [B]
   double* disc_cost;   // [B]      f_b(s), +inf when invalid
   uint8_t* reached;    // [M][B]
+  const int32_t* route;   // INPUT [K][M][B] or NULL: max-routing decisions to use (see backward)
+  int64_t* route_invalid; // [B] routes that are not near-maximising parents
 };
 
 void* oracle_graph_new(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -466,8 +458,17 @@ double cost_and_grad(const Graph& g, const oracle_cost& c, const double* p, doub
 // Reverse mode of the sweeps.  Exclusive products are
 // formed from prefix and suffix products: no division (reading S8); the max
 // routes to the lowest e-node id among the maximisers (reading S7).
+//
+// The arg-max of the correlated term is a floating-point DECISION.  When
+// `route` is given ([K][M] with stride `rstride` per class, the e-node each
+// sweep's max routed to, as decided by the system under test in its own
+// precision), the oracle uses it -- after checking that it is a valid
+// subgradient choice: a parent of the class whose p is a maximiser up to the
+// parity tolerance of p (1e-4 relative + 1e-6 absolute: fp32 rounding, which
+// is absolute where 1 - prod cancels); violations are counted in *invalid.
 void backward(const Graph& g, int K, Weights w, const double* cp, const double* qstack,
-              const double* gp, double* gcp) {
+              const double* gp, double* gcp, const int32_t* route = nullptr,
+              size_t rstride = 1, int64_t* invalid = nullptr) {
   const int M = g.M, N = g.N;
   const double* qK = qstack + (size_t)K * M;
   std::vector<double> gq(M, 0.0), gq_prev(M), gpt(N), pt(N);
@@ -490,6 +491,19 @@ void backward(const Graph& g, int K, Weights w, const double* cp, const double* 
       size_t amax = 0;
       for (size_t a = 1; a < n; ++a)
         if (pt[pa[a]] > pt[pa[amax]]) amax = a;  // strict: lowest id wins ties
+      if (route && w.wC != 0.0) {
+        const int r = route[((size_t)(t - 1) * M + j) * rstride];
+        const double mx = pt[pa[amax]];
+        size_t pos = n;
+        for (size_t a = 0; a < n; ++a)
+          if (pa[a] == r) pos = a;
+        // valid iff the routed parent attains the max within the parity bar
+        // (1e-4 relative + 1e-6 absolute, the fp32-vs-fp64 tolerance of p)
+        if (pos == n || pt[r] < mx - (1e-4 * mx + 1e-6)) {
+          if (invalid) ++*invalid;
+        }
+        if (pos < n) amax = pos;
+      }
       for (size_t a = 0; a < n; ++a) {
         double D = w.wI * (pre[a] * suf[a + 1]) + w.wC * (a == amax ? 1.0 : 0.0);
         gpt[pa[a]] += gq[j] * D;
@@ -630,7 +644,10 @@ int oracle_step(void* hg, const oracle_cost* cost, const oracle_opts* opt, int32
     std::vector<double> q((size_t)(K + 1) * M), p(N), gp(N), gcp(N), gth(N);
     forward(g, K, w, cp[b].data(), q.data(), p.data());
     fvals[b] = cost_and_grad(g, *cost, p.data(), gp.data());
-    backward(g, K, w, cp[b].data(), q.data(), gp.data(), gcp.data());
+    int64_t bad = 0;
+    backward(g, K, w, cp[b].data(), q.data(), gp.data(), gcp.data(),
+             out->route ? out->route + b : nullptr, (size_t)B, &bad);
+    if (out->route_invalid) out->route_invalid[b] = bad;
     const int gi = b / G;
     for (int k = 0; k < N; ++k) gcp[k] += pen[gi][k];
     // softmax backward: g_theta_i = cp_i (g_cp_i - sum_{k in m_ec(i)} cp_k g_cp_k)

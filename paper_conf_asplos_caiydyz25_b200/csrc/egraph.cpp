@@ -83,44 +83,46 @@ std::vector<int32_t> kosaraju(int32_t M, const std::vector<int32_t>& ptr,
   return comp;
 }
 
-// K_auto (S1): DFS from the root, successors in increasing class id; edges into
-// a vertex still on the DFS path are dropped; longest path over what remains.
-int32_t k_auto(const HostGraph& g, const std::vector<int32_t>& ptr, const std::vector<int32_t>& adj) {
-  const int32_t M = g.M;
-  std::vector<uint8_t> state(M, 0);  // 0 new, 1 on path, 2 done
-  std::vector<int32_t> post;
-  std::vector<uint8_t> keep(adj.size(), 0);
+// K_auto (S1): longest path from the root's component in the condensation of
+// the class graph (components contracted, one hop per inter-component edge).
+// Memoised DFS over the condensation from the root component.
+int32_t k_auto(const HostGraph& g, const std::vector<int32_t>& ptr, const std::vector<int32_t>& adj,
+               const std::vector<int32_t>& comp) {
+  int32_t nc = 0;
+  for (int32_t c : comp) nc = std::max(nc, c + 1);
+  // condensation adjacency (duplicates are harmless for a longest path)
+  std::vector<int32_t> cptr(nc + 1, 0), cadj;
+  std::vector<std::vector<int32_t>> tmp(nc);
+  for (int32_t j = 0; j < g.M; ++j)
+    for (int32_t e = ptr[j]; e < ptr[j + 1]; ++e)
+      if (comp[adj[e]] != comp[j]) tmp[comp[j]].push_back(comp[adj[e]]);
+  for (int32_t a = 0; a < nc; ++a) {
+    cadj.insert(cadj.end(), tmp[a].begin(), tmp[a].end());
+    cptr[a + 1] = (int32_t)cadj.size();
+  }
+  // height(a) = longest path starting at a; the answer is height(root component)
+  std::vector<int32_t> height(nc, -1);
   std::vector<std::pair<int32_t, int32_t>> st;
-  st.push_back({g.root, ptr[g.root]});
-  state[g.root] = 1;
+  const int32_t r = comp[g.root];
+  st.push_back({r, cptr[r]});
+  height[r] = -2;  // in progress
   while (!st.empty()) {
     auto& top = st.back();
-    if (top.second < ptr[top.first + 1]) {
-      int32_t e = top.second++;
-      int32_t w = adj[e];
-      if (state[w] == 1) continue;
-      keep[e] = 1;
-      if (state[w] == 0) {
-        state[w] = 1;
-        st.push_back({w, ptr[w]});
+    if (top.second < cptr[top.first + 1]) {
+      const int32_t b = cadj[top.second++];
+      if (height[b] == -1) {
+        height[b] = -2;
+        st.push_back({b, cptr[b]});
       }
     } else {
-      state[top.first] = 2;
-      post.push_back(top.first);
+      int32_t h = 0;
+      for (int32_t e = cptr[top.first]; e < cptr[top.first + 1]; ++e)
+        h = std::max(h, height[cadj[e]] + 1);
+      height[top.first] = h;
       st.pop_back();
     }
   }
-  std::vector<int32_t> depth(M, -1);
-  depth[g.root] = 0;
-  int32_t best = 0;
-  for (auto it = post.rbegin(); it != post.rend(); ++it) {
-    int32_t v = *it;
-    if (depth[v] < 0) continue;
-    best = std::max(best, depth[v]);
-    for (int32_t e = ptr[v]; e < ptr[v + 1]; ++e)
-      if (keep[e]) depth[adj[e]] = std::max(depth[adj[e]], depth[v] + 1);
-  }
-  return best;
+  return height[r];
 }
 
 }  // namespace
@@ -265,7 +267,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     }
     g.ent_ptr.push_back((int32_t)g.ent_i.size());
   }
-  g.K_auto = k_auto(g, sptr, sadj);
+  g.K_auto = k_auto(g, sptr, sadj, comp);
 }
 
 }  // namespace smoothe

@@ -77,7 +77,7 @@ struct smoothe_run {
   smoothe_options opt{};
   Shape sh{};
   int K = 0, G = 1, ngroups = 1, device = 0, cost_kind = 0, H1 = 0, H2 = 0, nsplit = 0;
-  int coop_grid = 0, f_rows = 0, dcost_rows = 0;
+  int coop_grid = 0, f_rows = 0, dcost_rows = 0, rows_M = 0, rows_N = 0;
   Agg agg{0.f, 0.f};
   cudaStream_t stream = nullptr;
   std::vector<void*> owned;
@@ -213,15 +213,15 @@ void enqueue_step(smoothe_run* r) {
   if (r->cost_kind == SMOOTHE_COST_LINEAR) {
     launch_cost_linear(s, sh, g, r->u_f, r->cp, qK, r->gcp, gqK, r->f_part,
                        r->debug ? r->dbg_p : nullptr, 0);
-    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0);
   } else if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
     launch_materialize_p_f(s, sh, g, nullptr, r->cp, qK, r->p, nullptr);
     launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, r->u_f, r->p, r->gp, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->f, 1.0);
     launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
   } else {
     launch_materialize_p_f(s, sh, g, r->u_f, r->cp, qK, r->p, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0);
     launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
                    r->z1_part, r->fextra, r->gz1, r->nsplit);
     launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
@@ -258,7 +258,7 @@ void enqueue_step(smoothe_run* r) {
   if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
     launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
     launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, nullptr, r->sbin, nullptr, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->f_rows, sh.Bp, r->dextra, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->dextra, 1.0);
     dextra = r->dextra;
   } else if (r->cost_kind == SMOOTHE_COST_MLP) {
     launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
@@ -332,6 +332,11 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->gq[1] = dalloc<float>(o, MB);
   const int rows_per_block_min = 256 / 32;  // kBlock / LPR(32): fewest rows per block
   r->f_rows = (std::max(sh.M, sh.N) + rows_per_block_min - 1) / rows_per_block_min + 1;
+  {  // rows of partial sums each row-group kernel writes (its grid.x)
+    const int per = 256 / (sh.Bp >= 128 ? 32 : sh.Bp / 4);
+    r->rows_M = (sh.M + per - 1) / per;
+    r->rows_N = (sh.N + per - 1) / per;
+  }
   r->f_part = dalloc<float>(o, (size_t)r->f_rows * sh.Bp);
   r->f = dalloc<double>(o, sh.Bp);
   r->fextra = dalloc<double>(o, sh.Bp);
@@ -781,6 +786,9 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     if (dump->valid) SM_CUDA(cudaMemcpyAsync(dump->valid, run->dbg_valid, sh.B, cudaMemcpyDeviceToHost, s));
     if (dump->disc_cost)
       SM_CUDA(cudaMemcpyAsync(dump->disc_cost, run->dbg_dcost, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
+    if (dump->route && run->K > 0)
+      SM_CUDA(cudaMemcpy2DAsync(dump->route, sizeof(int32_t) * sh.B, run->astack, sizeof(int32_t) * sh.Bp,
+                                sizeof(int32_t) * sh.B, (size_t)run->K * sh.M, cudaMemcpyDeviceToHost, s));
     std::vector<uint32_t> rbits;
     if (dump->reached) {
       rbits.resize((size_t)sh.M * sh.W);
@@ -791,6 +799,14 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       for (int j = 0; j < sh.M; ++j)
         for (int b = 0; b < sh.B; ++b)
           dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
+    if (dump->route) {  // unpack (arg << 2) | zero-count; the root row is not a decision
+      const size_t n = (size_t)run->K * sh.M * sh.B;
+      for (size_t i = 0; i < n; ++i) dump->route[i] >>= 2;
+      for (int t = 0; t < run->K; ++t)
+        for (int b = 0; b < sh.B; ++b) dump->route[((size_t)t * sh.M + sh.root) * sh.B + b] = -1;
+    }
+    if ((size_t)run->steps_run < run->ev_step.size())
+      SM_CUDA(cudaEventRecord(run->ev_step[run->steps_run], s));
     for (void* p : scratch) SM_CUDA(cudaFree(p));
     run->dbg_p = run->dbg_gth = run->dbg_gcp = nullptr;
     run->dbg_dcost = nullptr;

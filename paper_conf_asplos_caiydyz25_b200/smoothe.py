@@ -63,7 +63,7 @@ class _Summary(C.Structure):
 class _Dump(C.Structure):
     _fields_ = [(n, C.c_void_p) for n in
                 ("cp", "qK", "p", "grad_cp", "grad_theta", "theta_out", "m_out", "v_out", "f", "h",
-                 "loss", "choice", "reached", "valid", "disc_cost", "qstack")]
+                 "loss", "choice", "reached", "valid", "disc_cost", "qstack", "route")]
 
 
 class _Profile(C.Structure):
@@ -279,7 +279,7 @@ class Run:
         _check(lib().smoothe_get_theta(self._h, _p(out)))
         return out
 
-    def debug_step(self, theta=None, m=None, v=None, step_index=0, qstack=False):
+    def debug_step(self, theta=None, m=None, v=None, step_index=0, qstack=False, route=False):
         N, M, B = self.egraph.N, self.egraph.M, self.B
         G = self.options.penalty_group
         out = {k: np.zeros((N, B), np.float32) for k in
@@ -290,6 +290,8 @@ class Run:
                    disc_cost=np.zeros(B))
         if qstack:
             out["qstack"] = np.zeros((self.K + 1, M, B), np.float32)
+        if route:
+            out["route"] = np.zeros((self.K, M, B), np.int32)
         d = _Dump(**{k: _p(a) for k, a in out.items()})
         th, mm, vv = _c(theta, np.float32), _c(m, np.float32), _c(v, np.float32)
         _check(lib().smoothe_debug_step(self._h, _p(th), _p(mm), _p(vv), int(step_index), C.byref(d)))

@@ -57,20 +57,23 @@ def compare_step(sm, orc, eg, B, G, agg="hybrid", lam=1.0, theta=None, m=None, v
     rng = np.random.default_rng(seed)
     if theta is None:
         theta = rng.uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
-    d = run.debug_step(theta, m, v, step_index=step_index)
+    d = run.debug_step(theta, m, v, step_index=step_index, route=True)
     cols = slice(None) if cols is None else cols
     th = theta[:, cols].astype(np.float64)
     og = orc.Graph(eg)
     assert og.K_auto == g.K_auto
     oo = orc.Options(assumption=agg, K=Kr, lam=lam, G=G, lr=lr)
+    # the max's arg-max is a floating-point decision: the oracle takes the
+    # kernel's (fp32) routing, checks each is a maximising parent, and uses it
     o = og.step(th, oo, m=None if m is None else m[:, cols], v=None if v is None else v[:, cols],
-                step_index=step_index)
+                step_index=step_index, route=d["route"][:, :, cols])
     sel = lambda a: a[:, cols]
     close("cp", sel(d["cp"]), o["cp"])
     close("p", sel(d["p"]), o["p"])
     close("f", d["f"][cols], o["f"])
     nb = th.shape[1]
     close("h", d["h"][: nb // G], o["h"])            # cols always start at seed 0
+    assert o["route_invalid"].sum() == 0, "GPU routed a max to a non-maximising parent"
     close("grad_cp", sel(d["grad_cp"]), o["grad_cp"])
     cpo, gco = o["cp"], o["grad_cp"]
     gscale = cpo * (np.abs(gco) + class_sums(eg, cpo * np.abs(gco)))

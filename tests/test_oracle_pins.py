@@ -580,3 +580,64 @@ def test_generator_anchor_extraction_valid(orc):
     assert d["valid"][0] == 1
     assert g.K_auto >= eg.meta["levels"]
     assert g.num_scc > 0
+
+
+# ---------------------------------------------------------------- routing input (decisions)
+def own_routes(eg, o, K):
+    """lowest-id arg-max parent per (sweep, class, seed) from the oracle's own q-stack."""
+    pa = brute.parents(eg)
+    ec = eg.ec()
+    B = o["cp"].shape[1]
+    r = np.full((K, eg.num_classes, B), -1, np.int32)
+    for t in range(1, K + 1):
+        for j in range(eg.num_classes):
+            if j == eg.root or not pa[j]:
+                continue
+            for b in range(B):
+                p = [o["cp"][k, b] * o["qstack"][t - 1, ec[k], b] for k in pa[j]]
+                r[t - 1, j, b] = pa[j][int(np.argmax(p))]
+    return r
+
+
+def test_route_input_validated_and_used(orc):
+    eg = random_tiny(4000, "cyclic", num_classes=8)
+    g = orc.Graph(eg)
+    rng = np.random.default_rng(21)
+    th = rng.uniform(-1, 1, (eg.num_nodes, 3))
+    opts = orc.Options(assumption="hybrid", K=4, lam=0.5, G=1)
+    o = g.step(th, opts, qstack=True)
+    r = own_routes(eg, o, 4)
+    o2 = g.step(th, opts, route=r)
+    assert o2["route_invalid"].sum() == 0
+    assert np.array_equal(o2["grad_theta"], o["grad_theta"])
+    # a non-maximising route is reported and changes the gradient
+    pa = brute.parents(eg)
+    t, j = next((t, j) for t in range(4) for j in range(eg.num_classes)
+                if len(pa[j]) >= 2 and o["qstack"][t, :, 0].max() > 0 and r[t, j, 0] >= 0
+                and max(o["cp"][k, 0] * o["qstack"][t, eg.ec()[k], 0] for k in pa[j]) > 0)
+    others = [k for k in pa[j] if k != r[t, j, 0]]
+    bad = r.copy()
+    bad[t, j, 0] = others[0]
+    o3 = g.step(th, opts, route=bad)
+    p_other = o["cp"][others[0], 0] * o["qstack"][t, eg.ec()[others[0]], 0]
+    p_max = o["cp"][r[t, j, 0], 0] * o["qstack"][t, eg.ec()[r[t, j, 0]], 0]
+    if p_other < p_max * (1 - 1e-5):
+        assert o3["route_invalid"][0] >= 1
+
+
+def test_update_entry_matches_torch(orc):
+    import torch
+    rng = np.random.default_rng(22)
+    th = rng.normal(size=50)
+    grads = [rng.normal(size=50) for _ in range(3)]
+    p = torch.nn.Parameter(torch.tensor(th))
+    opt = torch.optim.Adam([p], lr=0.05, eps=1e-8)
+    opts = orc.Options(lr=0.05)
+    m = v = None
+    cur = th
+    for s, g in enumerate(grads):
+        p.grad = torch.tensor(g)
+        opt.step()
+        u = orc.update(cur, g, opts, m=m, v=v, step_index=s)
+        cur, m, v = u["theta_out"], u["m_out"], u["v_out"]
+    assert np.allclose(p.detach().numpy(), cur, rtol=0, atol=1e-14)
