@@ -268,6 +268,29 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     g.ent_ptr.push_back((int32_t)g.ent_i.size());
   }
   g.K_auto = k_auto(g, sptr, sadj, comp);
+
+  // padded sweep layouts (multiples of 4 entries per list)
+  g.pad_child_ptr.assign(N + 1, 0);
+  for (int32_t i = 0; i < N; ++i) {
+    const int32_t n = g.child_ptr[i + 1] - g.child_ptr[i];
+    g.pad_child_ptr[i + 1] = g.pad_child_ptr[i] + ((n + 3) & ~3);
+  }
+  g.pad_child.assign(g.pad_child_ptr[N], root);
+  for (int32_t i = 0; i < N; ++i)
+    std::copy(g.child_class.begin() + g.child_ptr[i], g.child_class.begin() + g.child_ptr[i + 1],
+              g.pad_child.begin() + g.pad_child_ptr[i]);
+  g.pad_par_ptr.assign(M + 1, 0);
+  for (int32_t j = 0; j < M; ++j) {
+    const int32_t n = g.par_ptr[j + 1] - g.par_ptr[j];
+    g.pad_par_ptr[j + 1] = g.pad_par_ptr[j] + ((n + 3) & ~3);
+  }
+  g.pad_par.resize(2 * (size_t)g.pad_par_ptr[M]);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t s = g.pad_par_ptr[j], e = g.par_ptr[j]; s < g.pad_par_ptr[j + 1]; ++s, ++e) {
+      const bool real = e < g.par_ptr[j + 1];
+      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
+      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
+    }
 }
 
 }  // namespace smoothe

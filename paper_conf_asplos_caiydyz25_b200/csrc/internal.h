@@ -61,6 +61,13 @@ struct HostGraph {
   std::vector<int32_t> slot_jptr, slot_jloc;       // children in the component (local)
   std::vector<int32_t> node_slot;                  // [N] slot id or -1
   int32_t K_auto = 0, max_class_size = 0, max_in_degree = 0;
+  // Sweep layouts padded to multiples of 4 entries per list (aligned vector
+  // index loads, 4 row gathers in flight):
+  //   pad_child_ptr [N+1], pad_child [.]   child classes of e-node i; padding = root
+  //                                        (g_q of the root is 0: inert)
+  //   pad_par_ptr [M+1],  pad_par [.][2]   (parent e-node, its class) of class j;
+  //                                        padding = (N, root): row N of cp is 0: p = 0
+  std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
 };
 
 void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -73,6 +80,7 @@ struct DevGraph {
   int32_t *ent_node_ptr = nullptr, *ent_node = nullptr;
   int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
+  int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int64_t bytes = 0;
 };
 

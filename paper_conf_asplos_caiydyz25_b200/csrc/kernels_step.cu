@@ -141,61 +141,72 @@ void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, c
 // Forward sweep t (readings S2-S4, S6-S8):
 //   p^t_k = cp_k * q^{t-1}_{ec(k)}                                      (Eq. 5)
 //   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
-// Also keeps, for the reverse sweep, the product over the non-zero factors
-// (pi), and am = (lowest arg-max e-node << 2) | min(#zero factors, 3).
+// Also keeps, for the reverse sweep, pi = the product over the non-zero
+// factors, signed by the number of zero factors (+: none, -: one, 0: two or
+// more), and am = the lowest e-node id attaining the max (reading S7).
 // One row group per (class, seed chunk): a CSC pull over the parents.
 // ---------------------------------------------------------------------------
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_sweep_forward(
-    int M, int Bp, int root, const int32_t* __restrict__ par_ptr,
-    const int32_t* __restrict__ par_node, const int32_t* __restrict__ par_class, float wI, float wC,
-    const float* __restrict__ cp, const float* __restrict__ q_prev, float* __restrict__ q,
-    float* __restrict__ pi, int32_t* __restrict__ am) {
+    int M, int Bp, int root, const int32_t* __restrict__ pad_par_ptr,
+    const int32_t* __restrict__ pad_par, float wI, float wC, const float* __restrict__ cp,
+    const float* __restrict__ q_prev, float* __restrict__ q, float* __restrict__ pi,
+    int32_t* __restrict__ am) {
   const RowGroup<LPR> rg;
   const int j = rg.row;
   if (j >= M || j == root) return;
-  const int e0 = par_ptr[j], e1 = par_ptr[j + 1];
+  // parents in groups of 4 (node, class) pairs: two aligned 16-byte index loads,
+  // then 8 independent row gathers; padding pairs (N, root) give p = 0 exactly
+  const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
   int4 arg = make_int4(-1, -1, -1, -1);
   int4 zc = make_int4(0, 0, 0, 0);
-#pragma unroll 4
-  for (int e = e0; e < e1; ++e) {
-    const int k = __ldg(par_node + e);
-    const int c = __ldg(par_class + e);
-    const float4 cv = ld4(cp + (size_t)k * Bp + rg.s0);
-    const float4 qv = ld4(q_prev + (size_t)c * Bp + rg.s0);
+  for (int e = e0; e < e1; e += 4) {
+    const int4 nc01 = ld4i(pad_par + 2 * (size_t)e);
+    const int4 nc23 = ld4i(pad_par + 2 * (size_t)e + 4);
+    const int kk[4] = {nc01.x, nc01.z, nc23.x, nc23.z};
+    const int cc[4] = {nc01.y, nc01.w, nc23.y, nc23.w};
+    float4 cv[4], qv[4];
 #pragma unroll
-    for (int x = 0; x < 4; ++x) {
-      const float p = __fmul_rn(comp(cv, x), comp(qv, x));
-      const float f = __fsub_rn(1.f, p);
-      if (f == 0.f) comp(zc, x) += 1;
-      else comp(prod, x) = __fmul_rn(comp(prod, x), f);
-      if (p > comp(mx, x)) {
-        comp(mx, x) = p;
-        comp(arg, x) = k;
+    for (int u = 0; u < 4; ++u) {
+      cv[u] = ld4(cp + (size_t)kk[u] * Bp + rg.s0);
+      qv[u] = ld4(q_prev + (size_t)cc[u] * Bp + rg.s0);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
+        const float f = __fsub_rn(1.f, p);
+        comp(zc, x) += f == 0.f ? 1 : 0;
+        comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
+        const bool gt = p > comp(mx, x);
+        comp(mx, x) = gt ? p : comp(mx, x);
+        comp(arg, x) = gt ? kk[u] : comp(arg, x);
       }
     }
   }
-  float4 qo;
-  int4 ao;
+  float4 qo, po;
 #pragma unroll
   for (int x = 0; x < 4; ++x) {
     const float P = comp(zc, x) > 0 ? 0.f : comp(prod, x);
     comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
-    comp(ao, x) = (comp(arg, x) << 2) | min(comp(zc, x), 3);
+    // pi = +prod (no zero factor), -prod (exactly one zero factor), 0 (two or more)
+    const int z = comp(zc, x);
+    comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
   const size_t o = (size_t)j * Bp + rg.s0;
   st4(q + o, qo);
-  if (pi) st4(pi + o, prod);
-  st4i(am + o, ao);
+  if (pi) st4(pi + o, po);
+  st4i(am + o, arg);
 }
 
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                           const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
   SM_DISPATCH_LPR(sh.Bp, {
     k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, g.par_ptr, g.par_node, g.par_class, a.wI, a.wC, cp, q_prev, q, pi, am);
+        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi, am);
   });
   SM_LAUNCH_CHECK();
 }
@@ -470,76 +481,108 @@ void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, 
 // for every e-node k in m_j' (contiguous):
 //   p_k    = cp_k q^{t-1}_{j'}  (recomputed bit-identically to the forward sweep)
 //   g_p^t_k = sum_{j in ch_k} g_q^t_j (wI excl_{jk} + wC [k = a^t_j])
-//   excl_{jk} = prod_{k' in pa_j, k' != k} (1 - p^t_k'): the stored product of
-//   the non-zero factors divided by k's own factor (the same fp32 value, so the
-//   quotient is exact to a few ulp); with one zero factor it is the stored
-//   product if k's factor is that zero, else 0; with two or more zeros it is 0.
+//   excl_{jk} = prod_{k' in pa_j, k' != k} (1 - p^t_k'), formed from the stored
+//   signed product pi_j of the non-zero factors:
+//     pi_j > 0 (no zero factor):   excl = pi_j / (1 - p_k)  (k's own factor is the
+//                                  same fp32 value, so the quotient is exact to ulps)
+//     pi_j < 0 (one zero factor):  excl = -pi_j if k's factor is that zero, else 0
+//     pi_j = 0 (two or more):      excl = 0
+//   so g_p^t_k = wI (A_k / (1 - p_k)  or  T_k if p_k = 1) + wC R_k with
+//   A_k = sum_j g_q_j max(pi_j, 0), T_k = sum_j g_q_j max(-pi_j, 0),
+//   R_k = sum_{j : a_j = k} g_q_j: one division per e-node, not per edge.
 //   g_cp_k += g_p^t_k q^{t-1}_{j'};   g_q^{t-1}_{j'} = sum_k g_p^t_k cp_k (0 at root)
-// Deterministic: no atomics, every output row has one owner.
+// The child rows of an e-node are fetched four at a time (independent loads in
+// flight).  Deterministic: no atomics, every output row has one owner.
 // ---------------------------------------------------------------------------
-template <int LPR>
+template <int LPR, bool HI, bool HC>
 __global__ void __launch_bounds__(kBlock) k_sweep_reverse(
     int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
     const int32_t* __restrict__ child_ptr, const int32_t* __restrict__ child_class, float wI,
     float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
     const float* __restrict__ gq, const float* __restrict__ pi, const int32_t* __restrict__ am,
     float* __restrict__ gcp, float* __restrict__ gq_prev) {
+  constexpr int U = 4;
   const RowGroup<LPR> rg;
   const int jp = rg.row;
   if (jp >= M) return;
   const float4 qp = ld4(q_prev + (size_t)jp * Bp + rg.s0);
-  float4 gqacc = make_float4(0.f, 0.f, 0.f, 0.f);
+  const float4 zero = make_float4(0.f, 0.f, 0.f, 0.f);
+  float4 gqacc = zero;
   for (int k = class_ptr[jp]; k < class_ptr[jp + 1]; ++k) {
     const size_t ok = (size_t)k * Bp + rg.s0;
     const float4 cv = ld4(cp + ok);
-    float4 om;
-#pragma unroll
-    for (int x = 0; x < 4; ++x) comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
-    float4 gp = make_float4(0.f, 0.f, 0.f, 0.f);
+    float4 gc = ld4(gcp + ok);
+    float4 A = zero, T = zero, R = zero;
     const int e0 = child_ptr[k], e1 = child_ptr[k + 1];
-#pragma unroll 2
-    for (int e = e0; e < e1; ++e) {
-      const size_t oj = (size_t)__ldg(child_class + e) * Bp + rg.s0;
-      const float4 g = ld4(gq + oj);
-      const int4 a = ld4i(am + oj);
-      float4 P = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (wI != 0.f) P = ld4(pi + oj);
+    for (int e = e0; e < e1; e += U) {
+      // child lists are padded to multiples of 4 with the root class, whose
+      // g_q is 0: one aligned 16-byte index load, then 12 independent gathers
+      const int4 j4 = ld4i(child_class + e);
+      const int jj[U] = {j4.x, j4.y, j4.z, j4.w};
+      float4 g[U], P[U];
+      int4 a[U];
 #pragma unroll
-      for (int x = 0; x < 4; ++x) {
-        const int av = comp(a, x);
-        const int zc = av & 3;
-        float D = (av >> 2) == k ? wC : 0.f;
-        if (wI != 0.f) {
-          const float o = comp(om, x);
-          float excl = 0.f;
-          if (zc == 0) excl = __fdiv_rn(comp(P, x), o);
-          else if (zc == 1 && o == 0.f) excl = comp(P, x);
-          D += wI * excl;
+      for (int u = 0; u < U; ++u) {
+        const size_t oj = (size_t)jj[u] * Bp + rg.s0;
+        g[u] = ld4(gq + oj);
+        if (HI) P[u] = ld4(pi + oj);
+        if (HC) a[u] = ld4i(am + oj);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+          const float gv = comp(g[u], x);
+          if (HI) {
+            const float pv = comp(P[u], x);
+            comp(A, x) = fmaf(gv, fmaxf(pv, 0.f), comp(A, x));
+            comp(T, x) = fmaf(gv, fmaxf(-pv, 0.f), comp(T, x));
+          }
+          if (HC) comp(R, x) += comp(a[u], x) == k ? gv : 0.f;
         }
-        comp(gp, x) += comp(g, x) * D;
       }
     }
-    float4 gc = ld4(gcp + ok);
 #pragma unroll
     for (int x = 0; x < 4; ++x) {
-      comp(gc, x) += comp(gp, x) * comp(qp, x);
-      comp(gqacc, x) += comp(gp, x) * comp(cv, x);
+      float gp = 0.f;
+      if (HI) {
+        const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+        gp = wI * (om != 0.f ? __fdiv_rn(comp(A, x), om) : comp(T, x));
+      }
+      if (HC) gp += wC * comp(R, x);
+      comp(gc, x) += gp * comp(qp, x);
+      comp(gqacc, x) += gp * comp(cv, x);
     }
     st4(gcp + ok, gc);
   }
   if (gq_prev) {
-    if (jp == root) gqacc = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (jp == root) gqacc = zero;
     st4(gq_prev + (size_t)jp * Bp + rg.s0, gqacc);
   }
+}
+
+template <int LPR>
+static void launch_reverse_lpr(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                               const float* cp, const float* q_prev, const float* gq,
+                               const float* pi, const int32_t* am, float* gcp, float* gq_prev) {
+  const dim3 grid = row_grid(sh.M, sh.Bp, LPR);
+#define SM_REV_ARGS sh.M, sh.Bp, sh.root, g.class_ptr, g.pad_child_ptr, g.pad_child, a.wI, a.wC, cp, \
+                    q_prev, gq, pi, am, gcp, gq_prev
+  if (a.wI != 0.f && a.wC != 0.f)
+    k_sweep_reverse<LPR, true, true><<<grid, kBlock, 0, s>>>(SM_REV_ARGS);
+  else if (a.wI != 0.f)
+    k_sweep_reverse<LPR, true, false><<<grid, kBlock, 0, s>>>(SM_REV_ARGS);
+  else
+    k_sweep_reverse<LPR, false, true><<<grid, kBlock, 0, s>>>(SM_REV_ARGS);
+#undef SM_REV_ARGS
 }
 
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
   SM_DISPATCH_LPR(sh.Bp, {
-    k_sweep_reverse<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, g.class_ptr, g.child_ptr, g.child_class, a.wI, a.wC, cp, q_prev, gq,
-        pi, am, gcp, write_gq_prev ? gq_prev : nullptr);
+    launch_reverse_lpr<LPR>(s, sh, g, a, cp, q_prev, gq, pi, am, gcp,
+                            write_gq_prev ? gq_prev : nullptr);
   });
   SM_LAUNCH_CHECK();
 }

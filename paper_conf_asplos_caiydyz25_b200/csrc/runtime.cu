@@ -323,7 +323,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->theta = dalloc<float>(o, NB);
   r->m = dalloc<float>(o, NB);
   r->v = dalloc<float>(o, NB);
-  r->cp = dalloc<float>(o, NB);
+  r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row: the padding parent of the sweeps
   r->gcp = dalloc<float>(o, NB);
   r->qstack = dalloc<float>(o, (size_t)(r->K + 1) * MB);
   if (r->agg.wI != 0.f) r->pistack = dalloc<float>(o, std::max<size_t>(1, (size_t)r->K * MB));
@@ -412,6 +412,7 @@ void init_state(smoothe_run* r) {
   cudaStream_t s = r->stream;
   const size_t MB = (size_t)sh.M * sh.Bp;
   launch_theta_init(s, sh, r->opt.rng_key, r->opt.seed_begin, r->theta, r->m, r->v);
+  SM_CUDA(cudaMemsetAsync(r->cp + (size_t)sh.N * sh.Bp, 0, sizeof(float) * sh.Bp, s));
   SM_CUDA(cudaMemsetAsync(r->qstack, 0, sizeof(float) * (size_t)(r->K + 1) * MB, s));
   launch_fill_rows(s, r->qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K + 1, sh.Bp, 1.0f);
   if (r->pistack) {
@@ -481,7 +482,11 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       int64_t& b = d.bytes;
       d.class_ptr = upload(o, h.class_ptr, &b);
       d.child_ptr = upload(o, h.child_ptr, &b);
-      d.child_class = upload(o, h.child_class, &b);
+      {  // padded with the root id so batched kernels may read up to 8 past E
+        std::vector<int32_t> padded(h.child_class);
+        padded.resize(h.child_class.size() + 8, h.root);
+        d.child_class = upload(o, padded, &b);
+      }
       d.par_ptr = upload(o, h.par_ptr, &b);
       d.par_node = upload(o, h.par_node, &b);
       d.par_class = upload(o, h.par_class, &b);
@@ -497,6 +502,10 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.slot_jptr = upload(o, h.slot_jptr, &b);
       d.slot_jloc = upload(o, h.slot_jloc, &b);
       d.node_slot = upload(o, h.node_slot, &b);
+      d.pad_child_ptr = upload(o, h.pad_child_ptr, &b);
+      d.pad_child = upload(o, h.pad_child, &b);
+      d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
+      d.pad_par = upload(o, h.pad_par, &b);
     }
   });
   if (st != SMOOTHE_OK) {
@@ -799,9 +808,7 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       for (int j = 0; j < sh.M; ++j)
         for (int b = 0; b < sh.B; ++b)
           dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
-    if (dump->route) {  // unpack (arg << 2) | zero-count; the root row is not a decision
-      const size_t n = (size_t)run->K * sh.M * sh.B;
-      for (size_t i = 0; i < n; ++i) dump->route[i] >>= 2;
+    if (dump->route) {  // the root row is not a decision (q_root = 1, S3)
       for (int t = 0; t < run->K; ++t)
         for (int b = 0; b < sh.B; ++b) dump->route[((size_t)t * sh.M + sh.root) * sh.B + b] = -1;
     }
@@ -887,7 +894,8 @@ void smoothe_free_egraph(smoothe_egraph* g) {
     cudaSetDevice(g->device);
     void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
                     d.scc_class_ptr, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
-                    d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot};
+                    d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot,
+                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par};
     for (void* p : ptrs) cudaFree(p);
   }
   delete g;

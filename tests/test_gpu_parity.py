@@ -74,8 +74,18 @@ def compare_step(sm, orc, eg, B, G, agg="hybrid", lam=1.0, theta=None, m=None, v
     nb = th.shape[1]
     close("h", d["h"][: nb // G], o["h"])            # cols always start at seed 0
     assert o["route_invalid"].sum() == 0, "GPU routed a max to a non-maximising parent"
-    close("grad_cp", sel(d["grad_cp"]), o["grad_cp"])
-    cpo, gco = o["cp"], o["grad_cp"]
+    gco = o["grad_cp"]
+    if eg.quad is not None:
+        # negative pair weights make g_p = u + sum_k w p_k cancel: bound the error
+        # by the magnitude of the terms, i.e. the same backward with |w| (the
+        # reverse mode is linear in g_p with non-negative coefficients)
+        qi, qj, qw = eg.quad
+        eg.quad = (qi, qj, np.abs(qw))
+        oa = og.__class__(eg).step(th, oo, route=d["route"][:, :, cols])
+        eg.quad = (qi, qj, qw)
+        gco = np.maximum(np.abs(gco), np.abs(oa["grad_cp"]))
+    close("grad_cp", sel(d["grad_cp"]), o["grad_cp"], scale=np.abs(gco))
+    cpo = o["cp"]
     gscale = cpo * (np.abs(gco) + class_sums(eg, cpo * np.abs(gco)))
     close("grad_theta", sel(d["grad_theta"]), o["grad_theta"], scale=gscale)
     assert np.array_equal(sel(d["choice"]), o["choice"])
