@@ -19,7 +19,7 @@ constexpr int kBlock = 256;
 __host__ __device__ inline int lanes_per_row(int Bp) { return Bp >= 128 ? 32 : Bp / 4; }
 __host__ __device__ inline int num_chunks(int Bp) { return Bp >= 128 ? Bp / 128 : 1; }
 
-template <int LPR>
+template <int LPR, int BLOCK = kBlock>
 struct RowGroup {
   int row;   // row index (class or node)
   int s0;    // first seed of this lane (multiple of 4)
@@ -27,14 +27,18 @@ struct RowGroup {
   __device__ RowGroup() {
     const int lane = threadIdx.x % LPR;
     sub = threadIdx.x / LPR;
-    row = blockIdx.x * (kBlock / LPR) + sub;
+    row = blockIdx.x * (BLOCK / LPR) + sub;
     s0 = blockIdx.y * (4 * LPR) + lane * 4;
   }
 };
 
-inline dim3 row_grid(int rows, int Bp, int LPR) {
-  return dim3((rows + kBlock / LPR - 1) / (kBlock / LPR), num_chunks(Bp));
+inline dim3 row_grid(int rows, int Bp, int LPR, int block = kBlock) {
+  return dim3((rows + block / LPR - 1) / (block / LPR), num_chunks(Bp));
 }
+
+// Threads per block of the two sweep kernels (tuning knob; blocks that are
+// too large idle behind their slowest row because class sizes are heavy-tailed).
+int sweep_block();
 
 __device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
 __device__ __forceinline__ int4 ld4i(const int32_t* p) { return *reinterpret_cast<const int4*>(p); }

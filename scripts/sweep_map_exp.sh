@@ -1,0 +1,13 @@
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+for MAP in 0 1; do for B in 64 128 256; do
+  SMOOTHE_SWEEP_MAP=$MAP SMOOTHE_SWEEP_BLOCK=$B timeout 600 python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu > gpurun_out/map${MAP}_blk_$B.json 2> gpurun_out/map${MAP}_blk_$B.err
+done; done
+python - <<'PY'
+import json
+for MAP in (0,1):
+  for B in (64,128,256):
+    try:
+        d=json.load(open(f"gpurun_out/map{MAP}_blk_{B}.json"))
+        print(MAP, B, round(d["ms_per_step"],1), {k: round(v,1) for k,v in d["phases_ms_per_step"].items() if v > 1})
+    except Exception as e: print(MAP, B, "ERR", e)
+PY
