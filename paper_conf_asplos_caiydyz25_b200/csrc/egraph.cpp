@@ -276,9 +276,13 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     g.pad_child_ptr[i + 1] = g.pad_child_ptr[i] + ((n + 3) & ~3);
   }
   g.pad_child.assign(g.pad_child_ptr[N], root);
-  for (int32_t i = 0; i < N; ++i)
+  g.pad_batch_node.resize(g.pad_child_ptr[N] / 4);
+  for (int32_t i = 0; i < N; ++i) {
     std::copy(g.child_class.begin() + g.child_ptr[i], g.child_class.begin() + g.child_ptr[i + 1],
               g.pad_child.begin() + g.pad_child_ptr[i]);
+    for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
+      g.pad_batch_node[b] = i;
+  }
   g.pad_par_ptr.assign(M + 1, 0);
   for (int32_t j = 0; j < M; ++j) {
     const int32_t n = g.par_ptr[j + 1] - g.par_ptr[j];

@@ -68,6 +68,7 @@ struct HostGraph {
   //   pad_par_ptr [M+1],  pad_par [.][2]   (parent e-node, its class) of class j;
   //                                        padding = (N, root): row N of cp is 0: p = 0
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
+  std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
 };
 
 void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -81,6 +82,7 @@ struct DevGraph {
   int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
+  int32_t *pad_batch_node = nullptr;
   int64_t bytes = 0;
 };
 

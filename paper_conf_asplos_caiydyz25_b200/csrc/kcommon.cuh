@@ -36,10 +36,6 @@ inline dim3 row_grid(int rows, int Bp, int LPR, int block = kBlock) {
   return dim3((rows + block / LPR - 1) / (block / LPR), num_chunks(Bp));
 }
 
-// Threads per block of the two sweep kernels (tuning knob; blocks that are
-// too large idle behind their slowest row because class sizes are heavy-tailed).
-int sweep_block();
-
 __device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
 __device__ __forceinline__ int4 ld4i(const int32_t* p) { return *reinterpret_cast<const int4*>(p); }
 __device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }

@@ -2,19 +2,14 @@
 //
 //   theta init (Philox4x32-10, reading S9)
 //   segmented softmax + argmax + decode selection masks
-//   forward Jacobi sweep of Eqs. 5-7                      PAPER.md:201-223 (schedule 215)
 //   linear / quadratic cost + backward initialisation     PAPER.md:101, 156; reading S24
-//   reverse sweep (hand-derived reverse mode)
 //   softmax backward fused with Adam                      PAPER.md:275-277; reading S10
 //
 // All per-seed arrays are [row][Bp] fp32 (seed innermost): every gather of a
 // parent/child row is a contiguous 16-byte-per-lane access (kcommon.cuh).
-// Products, differences and the max that the reverse sweep must reproduce
-// bit-for-bit use explicit round-to-nearest intrinsics (no FMA contraction).
+// The two propagation sweeps live in kernels_sweep.cu.
 #include <algorithm>
 #include <cfloat>
-#include <cstdlib>
-#include <unordered_map>
 
 #include "kcommon.cuh"
 
@@ -136,169 +131,6 @@ void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, c
   const int64_t warps = (int64_t)sh.M * (sh.W / nw);
   const int grid = (int)((warps * 32 + kBlock - 1) / kBlock);
   k_softmax_argmax<<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, sh.W, nw, g.class_ptr, theta, cp, choice, sel);
-  SM_LAUNCH_CHECK();
-}
-
-// ---------------------------------------------------------------------------
-// Forward sweep t (readings S2-S4, S6-S8):
-//   p^t_k = cp_k * q^{t-1}_{ec(k)}                                      (Eq. 5)
-//   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
-// Also keeps, for the reverse sweep, pi = the product over the non-zero
-// factors, signed by the number of zero factors (+: none, -: one, 0: two or
-// more), and am = the lowest e-node id attaining the max (reading S7).
-// One row group per (class, seed chunk): a CSC pull over the parents.
-// ---------------------------------------------------------------------------
-
-// Row-to-block mappings of the sweeps.  MAP 0: consecutive row groups of a
-// block take consecutive rows, blocks spread round-robin over the SMs.  MAP 1:
-// a persistent grid (a few blocks per SM), each block owns one contiguous range
-// of rows, so an SM's L1 sees neighbouring classes, whose parent / child rows
-// overlap (the generator's and real e-graphs' locality).
-template <int MAP>
-__device__ __forceinline__ void block_rows(int M, int groups, int& r0, int& r1) {
-  if (MAP == 0) {
-    r0 = blockIdx.x * groups;
-    r1 = min(M, r0 + groups);
-  } else {
-    const int per = (M + gridDim.x - 1) / gridDim.x;
-    r0 = min(M, blockIdx.x * per);
-    r1 = min(M, r0 + per);
-  }
-}
-
-template <int LPR>
-__device__ __forceinline__ void forward_row(
-    int j, int s0, int Bp, const int32_t* __restrict__ pad_par_ptr,
-    const int32_t* __restrict__ pad_par, float wI, float wC, const float* __restrict__ cp,
-    const float* __restrict__ q_prev, float* __restrict__ q, float* __restrict__ pi,
-    int32_t* __restrict__ am) {
-  // parents in groups of 4 (node, class) pairs: two aligned 16-byte index loads,
-  // then 8 independent row gathers; padding pairs (N, root) give p = 0 exactly
-  const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
-  float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
-  float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
-  int4 arg = make_int4(-1, -1, -1, -1);
-  int4 zc = make_int4(0, 0, 0, 0);
-  int4 n01 = make_int4(0, 0, 0, 0), n23 = n01;
-  if (e0 < e1) {
-    n01 = ld4i(pad_par + 2 * (size_t)e0);
-    n23 = ld4i(pad_par + 2 * (size_t)e0 + 4);
-  }
-  for (int e = e0; e < e1; e += 4) {
-    const int4 nc01 = n01, nc23 = n23;
-    if (e + 4 < e1) {  // next batch's (node, class) pairs, one step ahead
-      n01 = ld4i(pad_par + 2 * (size_t)e + 8);
-      n23 = ld4i(pad_par + 2 * (size_t)e + 12);
-    }
-    const int kk[4] = {nc01.x, nc01.z, nc23.x, nc23.z};
-    const int cc[4] = {nc01.y, nc01.w, nc23.y, nc23.w};
-    float4 cv[4], qv[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      cv[u] = ld4(cp + (size_t)kk[u] * Bp + s0);
-      qv[u] = ld4(q_prev + (size_t)cc[u] * Bp + s0);
-    }
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-#pragma unroll
-      for (int x = 0; x < 4; ++x) {
-        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
-        const float f = __fsub_rn(1.f, p);
-        comp(zc, x) += f == 0.f ? 1 : 0;
-        comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
-        const bool gt = p > comp(mx, x);
-        comp(mx, x) = gt ? p : comp(mx, x);
-        comp(arg, x) = gt ? kk[u] : comp(arg, x);
-      }
-    }
-  }
-  float4 qo, po;
-#pragma unroll
-  for (int x = 0; x < 4; ++x) {
-    const float P = comp(zc, x) > 0 ? 0.f : comp(prod, x);
-    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
-    // pi = +prod (no zero factor), -prod (exactly one zero factor), 0 (two or more)
-    const int z = comp(zc, x);
-    comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
-  }
-  const size_t o = (size_t)j * Bp + s0;
-  st4(q + o, qo);
-  if (pi) st4(pi + o, po);
-  st4i(am + o, arg);
-}
-
-template <int LPR, int BLOCK, int MAP>
-__global__ void __launch_bounds__(BLOCK) k_sweep_forward(
-    int M, int Bp, int root, const int32_t* __restrict__ pad_par_ptr,
-    const int32_t* __restrict__ pad_par, float wI, float wC, const float* __restrict__ cp,
-    const float* __restrict__ q_prev, float* __restrict__ q, float* __restrict__ pi,
-    int32_t* __restrict__ am) {
-  constexpr int groups = BLOCK / LPR;
-  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
-  int r0, r1;
-  block_rows<MAP>(M, groups, r0, r1);
-  for (int j = r0 + (int)threadIdx.x / LPR; j < r1; j += groups)
-    if (j != root) forward_row<LPR>(j, s0, Bp, pad_par_ptr, pad_par, wI, wC, cp, q_prev, q, pi, am);
-}
-
-int sweep_block() {
-  static int blk = [] {
-    const char* e = getenv("SMOOTHE_SWEEP_BLOCK");
-    const int v = e ? atoi(e) : 64;
-    return (v == 64 || v == 128 || v == 256) ? v : 64;
-  }();
-  return blk;
-}
-
-int sweep_map() {
-  static int map = [] {
-    const char* e = getenv("SMOOTHE_SWEEP_MAP");
-    return e ? (atoi(e) != 0) : 0;
-  }();
-  return map;
-}
-
-// grid of a sweep launch: one block per row group set (MAP 0) or a persistent
-// grid of `resident` blocks per SM (MAP 1)
-template <typename Kern>
-static dim3 sweep_grid(Kern kern, int map, int rows, int Bp, int LPR, int block) {
-  if (map == 0) return row_grid(rows, Bp, LPR, block);
-  static std::unordered_map<const void*, int> occupancy;  // per kernel instantiation
-  int dev = 0;
-  SM_CUDA(cudaGetDevice(&dev));
-  auto it = occupancy.find((const void*)kern);
-  if (it == occupancy.end()) {
-    int b = 0;
-    SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, block, 0));
-    it = occupancy.emplace((const void*)kern, b).first;
-  }
-  const int per_sm = it->second;
-  const int want = std::max(1, per_sm) * num_sms(dev);
-  const int most = (rows + block / LPR - 1) / (block / LPR);  // never fewer rows than groups
-  return dim3(std::max(1, std::min(want, most)), num_chunks(Bp));
-}
-
-void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
-                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
-#define SM_FWD_LAUNCH(BLK, MAP)                                                                \
-  do {                                                                                         \
-    auto kern = k_sweep_forward<LPR, BLK, MAP>;                                                \
-    kern<<<sweep_grid(kern, MAP, sh.M, sh.Bp, LPR, BLK), BLK, 0, s>>>(                         \
-        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi, am);    \
-  } while (0)
-  const int blk = sweep_block(), map = sweep_map();
-  SM_DISPATCH_LPR(sh.Bp, {
-    if (map == 0) {
-      if (blk == 64 && LPR == 32) SM_FWD_LAUNCH(64, 0);
-      else if (blk <= 128) SM_FWD_LAUNCH(128, 0);
-      else SM_FWD_LAUNCH(256, 0);
-    } else {
-      if (blk == 64 && LPR == 32) SM_FWD_LAUNCH(64, 1);
-      else if (blk <= 128) SM_FWD_LAUNCH(128, 1);
-      else SM_FWD_LAUNCH(256, 1);
-    }
-  });
-#undef SM_FWD_LAUNCH
   SM_LAUNCH_CHECK();
 }
 
@@ -564,164 +396,6 @@ __global__ void k_reduce_rows_d(const double* __restrict__ part, int nrows, int 
 void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
                              double* out) {
   k_reduce_rows_d<<<(Bp + 127) / 128, 128, 0, s>>>(part, nrows, Bp, out);
-  SM_LAUNCH_CHECK();
-}
-
-// ---------------------------------------------------------------------------
-// Reverse sweep t, one row group per class j':
-// for every e-node k in m_j' (contiguous):
-//   p_k    = cp_k q^{t-1}_{j'}  (recomputed bit-identically to the forward sweep)
-//   g_p^t_k = sum_{j in ch_k} g_q^t_j (wI excl_{jk} + wC [k = a^t_j])
-//   excl_{jk} = prod_{k' in pa_j, k' != k} (1 - p^t_k'), formed from the stored
-//   signed product pi_j of the non-zero factors:
-//     pi_j > 0 (no zero factor):   excl = pi_j / (1 - p_k)  (k's own factor is the
-//                                  same fp32 value, so the quotient is exact to ulps)
-//     pi_j < 0 (one zero factor):  excl = -pi_j if k's factor is that zero, else 0
-//     pi_j = 0 (two or more):      excl = 0
-//   so g_p^t_k = wI (A_k / (1 - p_k)  or  T_k if p_k = 1) + wC R_k with
-//   A_k = sum_j g_q_j max(pi_j, 0), T_k = sum_j g_q_j max(-pi_j, 0),
-//   R_k = sum_{j : a_j = k} g_q_j: one division per e-node, not per edge.
-//   g_cp_k += g_p^t_k q^{t-1}_{j'};   g_q^{t-1}_{j'} = sum_k g_p^t_k cp_k (0 at root)
-// The child rows of an e-node are fetched four at a time (independent loads in
-// flight).  Deterministic: no atomics, every output row has one owner.
-// ---------------------------------------------------------------------------
-template <int LPR, bool HI, bool HC>
-__device__ __forceinline__ void reverse_row(
-    int jp, int s0, int Bp, int root, const int32_t* __restrict__ class_ptr,
-    const int32_t* __restrict__ child_ptr, const int32_t* __restrict__ child_class, float wI,
-    float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
-    const float* __restrict__ gq, const float* __restrict__ pi, const int32_t* __restrict__ am,
-    float* __restrict__ gcp, float* __restrict__ gq_prev) {
-  constexpr int U = 4;
-  const float4 qp = ld4(q_prev + (size_t)jp * Bp + s0);
-  const float4 zero = make_float4(0.f, 0.f, 0.f, 0.f);
-  float4 gqacc = zero;
-  // The padded child lists of the class's e-nodes are one contiguous range,
-  // walked in batches of 4 (each batch belongs to one e-node).  The next batch's
-  // index vector and the next e-node's cp / g_cp rows are fetched one step
-  // ahead, so only the row gathers' latency is exposed.  Leaves (no children)
-  // get g_p = 0 and are skipped.
-  const int eb = child_ptr[class_ptr[jp]], ee = child_ptr[class_ptr[jp + 1]];
-  if (eb < ee) {
-    int k = class_ptr[jp];
-    while (child_ptr[k + 1] == child_ptr[k]) ++k;
-    int kend = child_ptr[k + 1];
-    size_t ok = (size_t)k * Bp + s0;
-    float4 cv = ld4(cp + ok);
-    float4 gc = ld4(gcp + ok);
-    float4 A = zero, T = zero, R = zero;
-    int4 j4 = ld4i(child_class + eb);
-    for (int e = eb; e < ee; e += U) {
-      const int jj[U] = {j4.x, j4.y, j4.z, j4.w};
-      if (e + U < ee) j4 = ld4i(child_class + e + U);
-      float4 g[U], P[U];
-      int4 a[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const size_t oj = (size_t)jj[u] * Bp + s0;
-        g[u] = ld4(gq + oj);
-        if (HI) P[u] = ld4(pi + oj);
-        if (HC) a[u] = ld4i(am + oj);
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-#pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          const float gv = comp(g[u], x);
-          if (HI) {
-            const float pv = comp(P[u], x);
-            comp(A, x) = fmaf(gv, fmaxf(pv, 0.f), comp(A, x));
-            comp(T, x) = fmaf(gv, fmaxf(-pv, 0.f), comp(T, x));
-          }
-          if (HC) comp(R, x) += comp(a[u], x) == k ? gv : 0.f;
-        }
-      }
-      if (e + U == kend) {  // last batch of e-node k: finalise it
-#pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          float gp = 0.f;
-          if (HI) {
-            const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
-            gp = wI * (om != 0.f ? __fdiv_rn(comp(A, x), om) : comp(T, x));
-          }
-          if (HC) gp += wC * comp(R, x);
-          comp(gc, x) += gp * comp(qp, x);
-          comp(gqacc, x) += gp * comp(cv, x);
-        }
-        st4(gcp + ok, gc);
-        if (e + U < ee) {  // next e-node with children
-          ++k;
-          while (child_ptr[k + 1] == child_ptr[k]) ++k;
-          kend = child_ptr[k + 1];
-          ok = (size_t)k * Bp + s0;
-          cv = ld4(cp + ok);
-          gc = ld4(gcp + ok);
-          A = zero;
-          T = zero;
-          R = zero;
-        }
-      }
-    }
-  }
-  if (gq_prev) {
-    if (jp == root) gqacc = zero;
-    st4(gq_prev + (size_t)jp * Bp + s0, gqacc);
-  }
-}
-
-template <int LPR, bool HI, bool HC, int BLOCK, int MAP>
-__global__ void __launch_bounds__(BLOCK) k_sweep_reverse(
-    int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
-    const int32_t* __restrict__ child_ptr, const int32_t* __restrict__ child_class, float wI,
-    float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
-    const float* __restrict__ gq, const float* __restrict__ pi, const int32_t* __restrict__ am,
-    float* __restrict__ gcp, float* __restrict__ gq_prev) {
-  constexpr int groups = BLOCK / LPR;
-  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
-  int r0, r1;
-  block_rows<MAP>(M, groups, r0, r1);
-  for (int j = r0 + (int)threadIdx.x / LPR; j < r1; j += groups)
-    reverse_row<LPR, HI, HC>(j, s0, Bp, root, class_ptr, child_ptr, child_class, wI, wC, cp,
-                             q_prev, gq, pi, am, gcp, gq_prev);
-}
-
-template <int LPR, int BLK, int MAP>
-static void launch_reverse_lpr(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
-                               const float* cp, const float* q_prev, const float* gq,
-                               const float* pi, const int32_t* am, float* gcp, float* gq_prev) {
-#define SM_REV_ARGS sh.M, sh.Bp, sh.root, g.class_ptr, g.pad_child_ptr, g.pad_child, a.wI, a.wC, cp, \
-                    q_prev, gq, pi, am, gcp, gq_prev
-#define SM_REV_LAUNCH(HI, HC)                                                                  \
-  do {                                                                                         \
-    auto kern = k_sweep_reverse<LPR, HI, HC, BLK, MAP>;                                        \
-    kern<<<sweep_grid(kern, MAP, sh.M, sh.Bp, LPR, BLK), BLK, 0, s>>>(SM_REV_ARGS);            \
-  } while (0)
-  if (a.wI != 0.f && a.wC != 0.f) SM_REV_LAUNCH(true, true);
-  else if (a.wI != 0.f) SM_REV_LAUNCH(true, false);
-  else SM_REV_LAUNCH(false, true);
-#undef SM_REV_LAUNCH
-#undef SM_REV_ARGS
-}
-
-void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
-                          const float* cp, const float* q_prev, const float* gq, const float* pi,
-                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
-  const int blk = sweep_block(), map = sweep_map();
-  float* out = write_gq_prev ? gq_prev : nullptr;
-#define SM_REV_BLK(MAP)                                                                        \
-  do {                                                                                         \
-    if (blk == 64 && LPR == 32)                                                                \
-      launch_reverse_lpr<LPR, 64, MAP>(s, sh, g, a, cp, q_prev, gq, pi, am, gcp, out);         \
-    else if (blk <= 128)                                                                       \
-      launch_reverse_lpr<LPR, 128, MAP>(s, sh, g, a, cp, q_prev, gq, pi, am, gcp, out);        \
-    else                                                                                       \
-      launch_reverse_lpr<LPR, 256, MAP>(s, sh, g, a, cp, q_prev, gq, pi, am, gcp, out);        \
-  } while (0)
-  SM_DISPATCH_LPR(sh.Bp, {
-    if (map == 0) SM_REV_BLK(0);
-    else SM_REV_BLK(1);
-  });
-#undef SM_REV_BLK
   SM_LAUNCH_CHECK();
 }
 

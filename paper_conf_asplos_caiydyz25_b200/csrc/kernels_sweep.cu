@@ -1,0 +1,228 @@
+// The two propagation sweeps of one SmoothE step (sm_100a): the forward
+// Jacobi sweep of Eqs. 5-7 and its reverse mode.  Together they are ~90% of a
+// step on deep graphs (2K launches per step), so their design is driven by
+// measurement:
+//
+//  * seed-innermost rows: a row group of LPR lanes owns one class row of
+//    4*LPR seeds (float4 per lane), so every parent / child gather is a
+//    contiguous 512-byte access at 128 seeds;
+//  * parent / child lists padded to multiples of 4 with inert entries, read as
+//    aligned 16-byte index vectors one batch ahead, four row gathers per
+//    array in flight per row group;
+//  * 64-thread blocks, rows assigned round-robin across SMs (the concurrent
+//    class "wavefront" shares parent / child rows through L2; contiguous
+//    per-block ranges measured 1.3-1.8x slower);
+//  * no division in the inner loops: the reverse sweep forms one reciprocal per
+//    e-node (an IEEE divide per edge or per node cost ~30% of the sweep);
+//  * deterministic: every output row has exactly one owner, no atomics.
+#include "kcommon.cuh"
+
+namespace smoothe {
+
+constexpr int kSweepBlock = 64;
+
+// ---------------------------------------------------------------------------
+// Forward sweep t (readings S2-S4, S6-S8):
+//   p^t_k = cp_k * q^{t-1}_{ec(k)}                                      (Eq. 5)
+//   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
+// and, for the reverse sweep, pi = the product over the non-zero factors signed
+// by the number of zero factors (+: none, -: exactly one, 0: two or more), and
+// am = the lowest e-node id attaining the max (reading S7).  Products, the
+// difference 1 - p and the max use explicit round-to-nearest intrinsics so the
+// reverse sweep can recompute 1 - p_k bit for bit.
+// ---------------------------------------------------------------------------
+template <int LPR>
+__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
+    int M, int Bp, int root, const int32_t* __restrict__ pad_par_ptr,
+    const int32_t* __restrict__ pad_par, float wI, float wC, const float* __restrict__ cp,
+    const float* __restrict__ q_prev, float* __restrict__ q, float* __restrict__ pi,
+    int32_t* __restrict__ am) {
+  const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
+  if (j >= M || j == root) return;
+  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
+  // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
+  // row N of cp, so p = 0: factor 1 and never a new max
+  const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
+  float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
+  float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
+  int4 arg = make_int4(-1, -1, -1, -1);
+  int4 zc = make_int4(0, 0, 0, 0);
+  int4 n01 = make_int4(0, 0, 0, 0), n23 = n01;
+  if (e0 < e1) {
+    n01 = ld4i(pad_par + 2 * (size_t)e0);
+    n23 = ld4i(pad_par + 2 * (size_t)e0 + 4);
+  }
+  for (int e = e0; e < e1; e += 4) {
+    const int kk[4] = {n01.x, n01.z, n23.x, n23.z};
+    const int cc[4] = {n01.y, n01.w, n23.y, n23.w};
+    if (e + 4 < e1) {  // next batch's pairs, one step ahead
+      n01 = ld4i(pad_par + 2 * (size_t)e + 8);
+      n23 = ld4i(pad_par + 2 * (size_t)e + 12);
+    }
+    float4 cv[4], qv[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      cv[u] = ld4(cp + (size_t)kk[u] * Bp + s0);
+      qv[u] = ld4(q_prev + (size_t)cc[u] * Bp + s0);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
+        const float f = __fsub_rn(1.f, p);
+        comp(zc, x) += f == 0.f ? 1 : 0;
+        comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
+        const bool gt = p > comp(mx, x);
+        comp(mx, x) = gt ? p : comp(mx, x);
+        comp(arg, x) = gt ? kk[u] : comp(arg, x);
+      }
+    }
+  }
+  float4 qo, po;
+#pragma unroll
+  for (int x = 0; x < 4; ++x) {
+    const int z = comp(zc, x);
+    const float P = z > 0 ? 0.f : comp(prod, x);
+    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
+    comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
+  }
+  const size_t o = (size_t)j * Bp + s0;
+  st4(q + o, qo);
+  if (pi) st4(pi + o, po);
+  st4i(am + o, arg);
+}
+
+void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi, am);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------
+// Reverse sweep t, one row group per class j'; for
+// every e-node k in m_j' (contiguous), with p_k = cp_k q^{t-1}_{j'} recomputed
+// bit-identically to the forward sweep and om = 1 - p_k:
+//   g_p^t_k = sum_{j in ch_k} g_q^t_j (wI excl_{jk} + wC [k = a^t_j])
+//   excl_{jk} = prod_{k' in pa_j, k' != k} (1 - p^t_k'):
+//     pi_j > 0 (no zero factor):  pi_j / om   (k's own factor is the same fp32
+//                                 value, so the quotient is exact to ~ulps)
+//     pi_j < 0 (one zero factor): -pi_j if om = 0 (k's factor is that zero), else 0
+//     pi_j = 0 (two or more):     0
+//   so g_p = wI (A / om  or  T if om = 0) + wC R with A = sum_j g_j max(pi_j, 0),
+//   T = sum_j g_j max(-pi_j, 0), R = sum_{j: a_j = k} g_j;
+//   g_cp_k += g_p^t_k q^{t-1}_{j'};   g_q^{t-1}_{j'} = sum_k g_p^t_k cp_k (0 at root).
+// The class's padded child lists form one contiguous run of 4-wide batches;
+// pad_batch_node gives each batch's e-node, so e-node boundaries are known one
+// batch ahead (no dependent pointer chasing) and the next e-node's cp / g_cp
+// rows are requested before the current one is finished.  Leaves own no batch
+// (g_p = 0, nothing to update).
+// ---------------------------------------------------------------------------
+template <int LPR, bool HI, bool HC>
+__global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
+    int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
+    const int32_t* __restrict__ pad_child_ptr, const int32_t* __restrict__ pad_child,
+    const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
+    const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
+    const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev) {
+  const int jp = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
+  if (jp >= M) return;
+  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
+  const float4 zero = make_float4(0.f, 0.f, 0.f, 0.f);
+  const float4 qp = ld4(q_prev + (size_t)jp * Bp + s0);
+  float4 gqacc = zero;
+  const int bb = pad_child_ptr[class_ptr[jp]] >> 2, be = pad_child_ptr[class_ptr[jp + 1]] >> 2;
+  if (bb < be) {
+    int k = pad_batch_node[bb];
+    size_t ok = (size_t)k * Bp + s0;
+    float4 cv = ld4(cp + ok), gc = ld4(gcp + ok);
+    float4 cvn = zero, gcn = zero;  // next e-node's rows, requested early
+    float4 A = zero, T = zero, R = zero;
+    int4 j4 = ld4i(pad_child + 4 * (size_t)bb);
+    int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
+    for (int b = bb; b < be; ++b) {
+      const int jj[4] = {j4.x, j4.y, j4.z, j4.w};
+      const int knext = kn;  // e-node of batch b+1 (-1: none)
+      if (b + 1 < be) {
+        j4 = ld4i(pad_child + 4 * (size_t)(b + 1));
+        kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
+      }
+      if (knext >= 0 && knext != k) {  // batch b is k's last: prefetch the next e-node
+        const size_t on = (size_t)knext * Bp + s0;
+        cvn = ld4(cp + on);
+        gcn = ld4(gcp + on);
+      }
+      float4 g[4], P[4];
+      int4 a[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const size_t oj = (size_t)jj[u] * Bp + s0;
+        g[u] = ld4(gq + oj);
+        if (HI) P[u] = ld4(pi + oj);
+        if (HC) a[u] = ld4i(am + oj);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+          const float gv = comp(g[u], x);
+          if (HI) {
+            const float pv = comp(P[u], x);
+            comp(A, x) = fmaf(gv, fmaxf(pv, 0.f), comp(A, x));
+            comp(T, x) = fmaf(gv, fmaxf(-pv, 0.f), comp(T, x));
+          }
+          if (HC) comp(R, x) += comp(a[u], x) == k ? gv : 0.f;
+        }
+      }
+      if (knext != k) {  // finalise e-node k
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+          float gp = 0.f;
+          if (HI) {
+            const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+            gp = wI * (om != 0.f ? __fdividef(comp(A, x), om) : comp(T, x));
+          }
+          if (HC) gp += wC * comp(R, x);
+          comp(gc, x) += gp * comp(qp, x);
+          comp(gqacc, x) += gp * comp(cv, x);
+        }
+        st4(gcp + ok, gc);
+        if (knext >= 0) {
+          k = knext;
+          ok = (size_t)k * Bp + s0;
+          cv = cvn;
+          gc = gcn;
+          A = zero;
+          T = zero;
+          R = zero;
+        }
+      }
+    }
+  }
+  if (gq_prev) {
+    if (jp == root) gqacc = zero;
+    st4(gq_prev + (size_t)jp * Bp + s0, gqacc);
+  }
+}
+
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                          const float* cp, const float* q_prev, const float* gq, const float* pi,
+                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
+  float* out = write_gq_prev ? gq_prev : nullptr;
+#define SM_REV(HI, HC)                                                                         \
+  k_sweep_reverse<LPR, HI, HC><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>( \
+      sh.M, sh.Bp, sh.root, g.class_ptr, g.pad_child_ptr, g.pad_child, g.pad_batch_node, a.wI,  \
+      a.wC, cp, q_prev, gq, pi, am, gcp, out)
+  SM_DISPATCH_LPR(sh.Bp, {
+    if (a.wI != 0.f && a.wC != 0.f) SM_REV(true, true);
+    else if (a.wI != 0.f) SM_REV(true, false);
+    else SM_REV(false, true);
+  });
+#undef SM_REV
+  SM_LAUNCH_CHECK();
+}
+
+}  // namespace smoothe

@@ -506,6 +506,7 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_child = upload(o, h.pad_child, &b);
       d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
       d.pad_par = upload(o, h.pad_par, &b);
+      d.pad_batch_node = upload(o, h.pad_batch_node, &b);
     }
   });
   if (st != SMOOTHE_OK) {
@@ -895,7 +896,7 @@ void smoothe_free_egraph(smoothe_egraph* g) {
     void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
                     d.scc_class_ptr, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
                     d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot,
-                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par};
+                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par, d.pad_batch_node};
     for (void* p : ptrs) cudaFree(p);
   }
   delete g;

@@ -15,7 +15,7 @@ from dataclasses import dataclass, field
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsmoothe.so")
+LIB_PATH = os.environ.get("SMOOTHE_LIB") or os.path.join(_HERE, "libsmoothe.so")
 
 OK, E_INVALID_ARG, E_BAD_GRAPH, E_OOM, E_CUDA, E_NO_VALID, E_STATE = range(7)
 STATUS_NAMES = ["OK", "E_INVALID_ARG", "E_BAD_GRAPH", "E_OOM", "E_CUDA", "E_NO_VALID", "E_STATE"]
