@@ -113,7 +113,8 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 //     pi_j < 0 (one zero factor): -pi_j if om = 0 (k's factor is that zero), else 0
 //     pi_j = 0 (two or more):     0
 //   so g_p = wI (A / om  or  T if om = 0) + wC R with A = sum_j g_j max(pi_j, 0),
-//   T = sum_j g_j max(-pi_j, 0), R = sum_{j: a_j = k} g_j;
+//   T = sum_j g_j max(-pi_j, 0), R = sum_{j: a_j = k} g_j (carried in one
+//   accumulator, see below);
 //   g_cp_k += g_p^t_k q^{t-1}_{j'};   g_q^{t-1}_{j'} = sum_k g_p^t_k cp_k (0 at root).
 // The class's padded child lists form one contiguous run of 4-wide batches;
 // pad_batch_node gives each batch's e-node, so e-node boundaries are known one
@@ -122,7 +123,7 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // (g_p = 0, nothing to update).
 // ---------------------------------------------------------------------------
 template <int LPR, bool HI, bool HC>
-__global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
+__global__ void __launch_bounds__(kSweepBlock, 16) k_sweep_reverse(
     int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
     const int32_t* __restrict__ pad_child_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
@@ -138,9 +139,16 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
   if (bb < be) {
     int k = pad_batch_node[bb];
     size_t ok = (size_t)k * Bp + s0;
-    float4 cv = ld4(cp + ok), gc = ld4(gcp + ok);
-    float4 cvn = zero, gcn = zero;  // next e-node's rows, requested early
-    float4 A = zero, T = zero, R = zero;
+    float4 cv = ld4(cp + ok);
+    float4 cvn = zero;  // next e-node's cp row, requested one batch early
+    // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
+    // three terms: X = sum_j g_j (wI max(s pi_j, 0) + wC [a_j = k] r) with
+    // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
+    // (then g_p = X).
+    float4 om;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+    float4 X = zero;
     int4 j4 = ld4i(pad_child + 4 * (size_t)bb);
     int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
     for (int b = bb; b < be; ++b) {
@@ -150,11 +158,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
         j4 = ld4i(pad_child + 4 * (size_t)(b + 1));
         kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
       }
-      if (knext >= 0 && knext != k) {  // batch b is k's last: prefetch the next e-node
-        const size_t on = (size_t)knext * Bp + s0;
-        cvn = ld4(cp + on);
-        gcn = ld4(gcp + on);
-      }
+      if (knext >= 0 && knext != k) cvn = ld4(cp + (size_t)knext * Bp + s0);
       float4 g[4], P[4];
       int4 a[4];
 #pragma unroll
@@ -168,24 +172,18 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
       for (int u = 0; u < 4; ++u) {
 #pragma unroll
         for (int x = 0; x < 4; ++x) {
-          const float gv = comp(g[u], x);
-          if (HI) {
-            const float pv = comp(P[u], x);
-            comp(A, x) = fmaf(gv, fmaxf(pv, 0.f), comp(A, x));
-            comp(T, x) = fmaf(gv, fmaxf(-pv, 0.f), comp(T, x));
-          }
-          if (HC) comp(R, x) += comp(a[u], x) == k ? gv : 0.f;
+          const bool nz = comp(om, x) != 0.f;
+          float w = 0.f;
+          if (HI) w = wI * fmaxf(nz ? comp(P[u], x) : -comp(P[u], x), 0.f);
+          if (HC) w += comp(a[u], x) == k ? (HI && nz ? wC * comp(om, x) : wC) : 0.f;
+          comp(X, x) = fmaf(comp(g[u], x), w, comp(X, x));
         }
       }
       if (knext != k) {  // finalise e-node k
+        float4 gc = ld4(gcp + ok);
 #pragma unroll
         for (int x = 0; x < 4; ++x) {
-          float gp = 0.f;
-          if (HI) {
-            const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
-            gp = wI * (om != 0.f ? __fdividef(comp(A, x), om) : comp(T, x));
-          }
-          if (HC) gp += wC * comp(R, x);
+          const float gp = HI && comp(om, x) != 0.f ? __fdividef(comp(X, x), comp(om, x)) : comp(X, x);
           comp(gc, x) += gp * comp(qp, x);
           comp(gqacc, x) += gp * comp(cv, x);
         }
@@ -194,10 +192,10 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_reverse(
           k = knext;
           ok = (size_t)k * Bp + s0;
           cv = cvn;
-          gc = gcn;
-          A = zero;
-          T = zero;
-          R = zero;
+#pragma unroll
+          for (int x = 0; x < 4; ++x)
+            comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+          X = zero;
         }
       }
     }
