@@ -269,6 +269,54 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   }
   g.K_auto = k_auto(g, sptr, sadj, comp);
 
+  // decode schedule: condensation levels reachable from the root (Kahn order)
+  {
+    std::vector<std::vector<int32_t>> cadj(ncomp);
+    for (int32_t j = 0; j < M; ++j)
+      for (int32_t e = sptr[j]; e < sptr[j + 1]; ++e)
+        if (comp[sadj[e]] != comp[j]) cadj[comp[j]].push_back(comp[sadj[e]]);
+    std::vector<uint8_t> seen(ncomp, 0);
+    std::vector<int32_t> stack{comp[root]};
+    seen[comp[root]] = 1;
+    while (!stack.empty()) {
+      const int32_t a = stack.back();
+      stack.pop_back();
+      for (int32_t b : cadj[a])
+        if (!seen[b]) {
+          seen[b] = 1;
+          stack.push_back(b);
+        }
+    }
+    std::vector<int32_t> indeg(ncomp, 0), depth(ncomp, -1), order;
+    for (int32_t a = 0; a < ncomp; ++a)
+      if (seen[a])
+        for (int32_t b : cadj[a]) indeg[b]++;
+    order.push_back(comp[root]);
+    depth[comp[root]] = 0;
+    for (size_t i = 0; i < order.size(); ++i) {
+      const int32_t a = order[i];
+      for (int32_t b : cadj[a]) {
+        depth[b] = std::max(depth[b], depth[a] + 1);
+        if (--indeg[b] == 0) order.push_back(b);
+      }
+    }
+    for (int32_t d : depth) g.num_levels = std::max(g.num_levels, d + 1);
+    std::vector<int32_t> first(ncomp, -1);  // one class per component
+    for (int32_t j = M - 1; j >= 0; --j) first[comp[j]] = j;
+    g.lvl_ptr.assign(g.num_levels + 1, 0);
+    for (int32_t a = 0; a < ncomp; ++a)
+      if (depth[a] >= 0) g.lvl_ptr[depth[a] + 1]++;
+    for (int32_t L = 0; L < g.num_levels; ++L) g.lvl_ptr[L + 1] += g.lvl_ptr[L];
+    g.lvl_item.resize(g.lvl_ptr[g.num_levels]);
+    std::vector<int32_t> fill(g.lvl_ptr.begin(), g.lvl_ptr.end() - 1);
+    for (int32_t a = 0; a < ncomp; ++a) {
+      if (depth[a] < 0) continue;
+      const int32_t j = first[a];
+      const int32_t s = g.scc_of_class[j];
+      g.lvl_item[fill[depth[a]]++] = s >= 0 ? -(s + 1) : j;
+    }
+  }
+
   // padded sweep layouts (multiples of 4 entries per list)
   g.pad_child_ptr.assign(N + 1, 0);
   for (int32_t i = 0; i < N; ++i) {

@@ -69,6 +69,12 @@ struct HostGraph {
   //                                        padding = (N, root): row N of cp is 0: p = 0
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
+  // Decode schedule: levels of the SCC condensation reachable from the root
+  // (level = longest path from the root's component).  Items of level L are
+  // lvl_item[lvl_ptr[L] .. lvl_ptr[L+1]): a class id j >= 0 (trivial
+  // component) or -(s+1) for the non-trivial SCC s.
+  int32_t num_levels = 0;
+  std::vector<int32_t> lvl_ptr, lvl_item;
 };
 
 void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -77,12 +83,13 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
 struct DevGraph {
   int32_t *class_ptr = nullptr, *child_ptr = nullptr, *child_class = nullptr;
   int32_t *par_ptr = nullptr, *par_node = nullptr, *par_class = nullptr;
-  int32_t *scc_class_ptr = nullptr, *ent_ptr = nullptr, *ent_i = nullptr, *ent_j = nullptr;
+  int32_t *scc_class_ptr = nullptr, *scc_class = nullptr, *ent_ptr = nullptr, *ent_i = nullptr, *ent_j = nullptr;
   int32_t *ent_node_ptr = nullptr, *ent_node = nullptr;
   int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t *pad_batch_node = nullptr;
+  int32_t *lvl_ptr = nullptr, *lvl_item = nullptr;
   int64_t bytes = 0;
 };
 
@@ -127,10 +134,11 @@ void launch_materialize_p_f(cudaStream_t s, const Shape& sh, const DevGraph& g, 
 // quadratic cost over symmetric neighbour lists; u may be NULL (pair terms only)
 void launch_quadratic(cudaStream_t s, const Shape& sh, const int32_t* qptr, const int32_t* qnbr,
                       const float* qw, const float* u, const float* p, float* gp, float* f_part);
+// deterministic fp64 column sums; scratch holds 128 x Bp doubles
 void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, int32_t Bp,
-                            double* out, double scale);
+                            double* out, double scale, double* scratch);
 void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
-                             double* out);
+                             double* out, double* scratch);
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev);
@@ -145,10 +153,10 @@ void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_sc
 void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, int Bp, float value);
 void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const double* f,
                  const double* fextra, const double* h, double* ftot, double* loss);
-void launch_decode_reach(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
-                         uint32_t* reach, int32_t* flags, int32_t grid);
-void launch_decode_settle(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
-                          uint32_t* settle, int32_t* flags, int32_t grid);
+// reached sets and validity masks (kernels_decode.cu); valid_out[W]
+void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
+                   const uint32_t* sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out,
+                   int32_t grid);
 void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g,
                                const double* u, const int32_t* choice, const uint32_t* reach,
                                double* cost_part);

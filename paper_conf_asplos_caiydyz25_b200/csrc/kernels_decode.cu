@@ -9,12 +9,8 @@
 //   sel[k][w]    bit set iff the seed chose e-node k in its class   (softmax kernel)
 //   reach[j][w]  least fixpoint of  reach_root = 1,
 //                reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k)       (top-down)
-//   settle[j][w] least fixpoint of settle_j = OR_{k in m_j} (sel_k AND AND_{c in ch_k} settle_c)
-//                (bottom-up); a class settles iff its selected sub-term is finite
-//                and acyclic, so  valid <=> settle_root.
-// Both fixpoints are computed in place by one cooperative kernel that repeats
-// rounds until a round changes nothing (monotone, so asynchronous in-place
-// updates reach the same least fixpoint).
+//   valid[w]     no selected cycle: checked per strongly connected component
+//                (k_decode_levels below).
 //
 // Discrete cost (reading S19): sum of u over the chosen e-node of every reached
 // class, each class once, accumulated in fp64 (exact for integer-valued u).
@@ -26,66 +22,106 @@ namespace cg = cooperative_groups;
 
 namespace smoothe {
 
-__global__ void __launch_bounds__(256) k_reach(int M, int W, int root,
-                                               const int32_t* __restrict__ par_ptr,
-                                               const int32_t* __restrict__ par_node,
-                                               const int32_t* __restrict__ par_class,
-                                               const uint32_t* __restrict__ sel, uint32_t* reach,
-                                               int32_t* flags, int max_rounds) {
-  cg::grid_group grid = cg::this_grid();
-  const int64_t nitems = (int64_t)M * W;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int r = 0; r < max_rounds; ++r) {
-    int changed = 0;
-    for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < nitems; it += stride) {
-      const int j = (int)(it / W), w = (int)(it % W);
-      if (j == root) continue;
-      uint32_t v = 0;
-      for (int e = par_ptr[j]; e < par_ptr[j + 1]; ++e)
-        v |= __ldcg(reach + (size_t)par_class[e] * W + w) & sel[(size_t)par_node[e] * W + w];
-      if (v != __ldcg(reach + it)) {
-        __stcg(reach + it, v);
-        changed = 1;
-      }
-    }
-    if (blockIdx.x == 0 && threadIdx.x == 0) flags[(r + 1) % 3] = 0;
-    changed = __syncthreads_or(changed);
-    if (changed && threadIdx.x == 0) atomicOr(flags + r % 3, 1);
-    grid.sync();
-    if (*((volatile int32_t*)flags + r % 3) == 0) break;
-  }
-}
+// One cooperative kernel computes the reached sets and the validity masks,
+// level by level over the condensation of the e-class graph (levels from the
+// loader: longest path from the root's strongly connected component):
+//  * a class in a trivial component has all its parents at lower levels, so
+//    reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k) is final in one pass;
+//  * a non-trivial SCC is iterated to its local fixpoint by one warp per
+//    (SCC, 32-seed word) (lanes = classes, |S| <= 64);
+//  * every cycle of a selection lies inside one SCC, so the selection is valid
+//    iff, in every SCC, the reached classes settle bottom-up within the SCC:
+//    settle_j = !reach_j OR OR_{k in m_j} (sel_k AND AND_{c in ch_k cap S} settle_c).
+//    Unsettled reached classes mark their seeds invalid (bit-OR atomics:
+//    order-independent, deterministic).
+// One grid barrier per level; each class is evaluated once per level pass.
+constexpr int kDecodeWarps = 8;
 
-__global__ void __launch_bounds__(256) k_settle(int M, int W, const int32_t* __restrict__ class_ptr,
-                                                const int32_t* __restrict__ child_ptr,
-                                                const int32_t* __restrict__ child_class,
-                                                const uint32_t* __restrict__ sel, uint32_t* settle,
-                                                int32_t* flags, int max_rounds) {
+__global__ void __launch_bounds__(256) k_decode_levels(
+    int W, int root, int num_levels, const int32_t* __restrict__ lvl_ptr,
+    const int32_t* __restrict__ lvl_item, const int32_t* __restrict__ par_ptr,
+    const int32_t* __restrict__ par_node, const int32_t* __restrict__ par_class,
+    const int32_t* __restrict__ class_ptr, const int32_t* __restrict__ scc_class_ptr,
+    const int32_t* __restrict__ scc_class, const int32_t* __restrict__ node_slot,
+    const int32_t* __restrict__ slot_jptr, const int32_t* __restrict__ slot_jloc,
+    const uint32_t* __restrict__ sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out) {
+  __shared__ uint32_t st[kDecodeWarps][64];
   cg::grid_group grid = cg::this_grid();
-  const int64_t nitems = (int64_t)M * W;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int r = 0; r < max_rounds; ++r) {
-    int changed = 0;
-    for (int64_t it = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; it < nitems; it += stride) {
-      const int j = (int)(it / W), w = (int)(it % W);
-      uint32_t v = 0;
-      for (int k = class_ptr[j]; k < class_ptr[j + 1]; ++k) {
-        uint32_t acc = sel[(size_t)k * W + w];
-        for (int e = child_ptr[k]; acc && e < child_ptr[k + 1]; ++e)
-          acc &= __ldcg(settle + (size_t)child_class[e] * W + w);
-        v |= acc;
-      }
-      if (v != __ldcg(settle + it)) {
-        __stcg(settle + it, v);
-        changed = 1;
-      }
+  const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int64_t gwarp = gtid >> 5, nwarps = nthreads >> 5;
+  auto pull = [&](int j, int w) {
+    uint32_t v = 0;
+    for (int e = par_ptr[j]; e < par_ptr[j + 1]; ++e)
+      v |= __ldcg(reach + (size_t)par_class[e] * W + w) & sel[(size_t)par_node[e] * W + w];
+    return v;
+  };
+  for (int L = 0; L < num_levels; ++L) {
+    const int i0 = lvl_ptr[L];
+    const int64_t nitems = (int64_t)(lvl_ptr[L + 1] - i0) * W;
+    // trivial components: one thread per (class, word)
+    for (int64_t it = gtid; it < nitems; it += nthreads) {
+      const int j = lvl_item[i0 + it / W];
+      const int w = (int)(it % W);
+      if (j < 0 || j == root) continue;
+      __stcg(reach + (size_t)j * W + w, pull(j, w));
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) flags[(r + 1) % 3] = 0;
-    changed = __syncthreads_or(changed);
-    if (changed && threadIdx.x == 0) atomicOr(flags + r % 3, 1);
+    // non-trivial SCCs: one warp per (SCC, word)
+    for (int64_t it = gwarp; it < nitems; it += nwarps) {
+      const int item = lvl_item[i0 + it / W];
+      const int w = (int)(it % W);
+      if (item >= 0) continue;
+      const int s = -item - 1, c0 = scc_class_ptr[s], n = scc_class_ptr[s + 1] - c0;
+      bool changed = true;
+      while (__any_sync(0xffffffffu, changed)) {  // local reach fixpoint (monotone)
+        changed = false;
+        for (int l = lane; l < n; l += 32) {
+          const int j = scc_class[c0 + l];
+          const uint32_t v = j == root ? 0xffffffffu : pull(j, w);
+          if (v != __ldcg(reach + (size_t)j * W + w)) {
+            __stcg(reach + (size_t)j * W + w, v);
+            changed = true;
+          }
+        }
+        __syncwarp();
+      }
+      uint32_t r[2] = {0, 0};
+      for (int l = lane, x = 0; l < n; l += 32, ++x) {
+        r[x] = __ldcg(reach + (size_t)scc_class[c0 + l] * W + w);
+        st[wib][l] = ~r[x];  // unreached classes count as settled
+      }
+      __syncwarp();
+      changed = true;
+      while (__any_sync(0xffffffffu, changed)) {  // local settle fixpoint (monotone)
+        changed = false;
+        for (int l = lane; l < n; l += 32) {
+          const int j = scc_class[c0 + l];
+          uint32_t v = st[wib][l];
+          const int q0 = node_slot[class_ptr[j]];
+          for (int k = class_ptr[j]; k < class_ptr[j + 1]; ++k) {
+            const int q = q0 + (k - class_ptr[j]);
+            uint32_t acc = sel[(size_t)k * W + w];
+            for (int e = slot_jptr[q]; acc && e < slot_jptr[q + 1]; ++e) acc &= st[wib][slot_jloc[e]];
+            v |= acc;
+          }
+          if (v != st[wib][l]) {
+            st[wib][l] = v;
+            changed = true;
+          }
+        }
+        __syncwarp();
+      }
+      uint32_t bad = 0;
+      for (int l = lane, x = 0; l < n; l += 32, ++x) bad |= r[x] & ~st[wib][l];
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+      if (lane == 0 && bad) atomicOr(invalid + w, bad);
+      __syncwarp();
+    }
     grid.sync();
-    if (*((volatile int32_t*)flags + r % 3) == 0) break;
   }
+  if (gtid < W) valid_out[gtid] = ~__ldcg(invalid + gtid);
 }
 
 static void coop_launch(const void* fn, int grid, void** args, cudaStream_t s) {
@@ -93,35 +129,24 @@ static void coop_launch(const void* fn, int grid, void** args, cudaStream_t s) {
   SM_LAUNCH_CHECK();
 }
 
-void launch_decode_reach(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
-                         uint32_t* reach, int32_t* flags, int32_t grid) {
-  SM_CUDA(cudaMemsetAsync(flags, 0, 3 * sizeof(int32_t), s));
+void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
+                   const uint32_t* sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out,
+                   int32_t grid) {
+  SM_CUDA(cudaMemsetAsync(invalid, 0, sizeof(uint32_t) * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach + (size_t)sh.root * sh.W, 0xff, sizeof(uint32_t) * sh.W, s));
-  int M = sh.M, W = sh.W, root = sh.root, max_rounds = sh.M + 2;
-  const int32_t *pp = g.par_ptr, *pn = g.par_node, *pc = g.par_class;
-  void* args[] = {&M, &W, &root, (void*)&pp, (void*)&pn, (void*)&pc, (void*)&sel, &reach, &flags,
-                  &max_rounds};
-  coop_launch((const void*)k_reach, grid, args, s);
-}
-
-void launch_decode_settle(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
-                          uint32_t* settle, int32_t* flags, int32_t grid) {
-  SM_CUDA(cudaMemsetAsync(flags, 0, 3 * sizeof(int32_t), s));
-  SM_CUDA(cudaMemsetAsync(settle, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
-  int M = sh.M, W = sh.W, max_rounds = sh.M + 2;
-  const int32_t *cp_ = g.class_ptr, *chp = g.child_ptr, *chc = g.child_class;
-  void* args[] = {&M, &W, (void*)&cp_, (void*)&chp, (void*)&chc, (void*)&sel, &settle, &flags,
-                  &max_rounds};
-  coop_launch((const void*)k_settle, grid, args, s);
+  int W = sh.W, root = sh.root, L = hg.num_levels;
+  void* args[] = {&W, &root, &L, (void*)&g.lvl_ptr, (void*)&g.lvl_item, (void*)&g.par_ptr,
+                  (void*)&g.par_node, (void*)&g.par_class, (void*)&g.class_ptr,
+                  (void*)&g.scc_class_ptr, (void*)&g.scc_class, (void*)&g.node_slot,
+                  (void*)&g.slot_jptr, (void*)&g.slot_jloc, (void*)&sel, &reach, &invalid,
+                  &valid_out};
+  coop_launch((const void*)k_decode_levels, grid, args, s);
 }
 
 int decode_grid(int device) {
   int per_sm = 0;
-  SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_reach, 256, 0));
-  int per_sm2 = 0;
-  SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm2, k_settle, 256, 0));
-  per_sm = std::min(per_sm, per_sm2);
+  SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decode_levels, 256, 0));
   return std::max(1, std::min(per_sm, 4)) * num_sms(device);
 }
 

@@ -368,35 +368,59 @@ void launch_quadratic(cudaStream_t s, const Shape& sh, const int32_t* qptr, cons
   SM_LAUNCH_CHECK();
 }
 
-// out[b] = scale * sum_r part[r][b], fp64, fixed order (deterministic).
-__global__ void k_reduce_rows(const float* __restrict__ part, int nrows, int Bp,
-                              double* __restrict__ out, double scale) {
+// out[b] = scale * sum_r part[r][b] in fp64, in a fixed order (deterministic,
+// bit-identical run to run): stage 1 sums interleaved rows of each of S slices
+// (32 seeds x 8 row strides per block, fixed-order smem combine), stage 2 sums
+// the S slice totals in order.
+constexpr int kRedSlices = 128;
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_reduce_rows_s1(const T* __restrict__ part, int nrows, int Bp,
+                                                        int per, double* __restrict__ scratch) {
+  __shared__ double red[8][32];
+  const int b = blockIdx.x * 32 + (threadIdx.x & 31);
+  const int ty = threadIdx.x >> 5;
+  const int r0 = blockIdx.y * per, r1 = min(nrows, r0 + per);
+  double acc = 0.0;
+  if (b < Bp)
+    for (int r = r0 + ty; r < r1; r += 8) acc += (double)part[(size_t)r * Bp + b];
+  red[ty][threadIdx.x & 31] = acc;
+  __syncthreads();
+  if (ty == 0 && b < Bp) {
+    double t = red[0][threadIdx.x];
+    for (int i = 1; i < 8; ++i) t += red[i][threadIdx.x];
+    scratch[(size_t)blockIdx.y * Bp + b] = t;
+  }
+}
+
+__global__ void k_reduce_rows_s2(const double* __restrict__ scratch, int S, int Bp,
+                                 double* __restrict__ out, double scale) {
   const int b = blockIdx.x * blockDim.x + threadIdx.x;
   if (b >= Bp) return;
   double acc = 0.0;
-  for (int r = 0; r < nrows; ++r) acc += (double)part[(size_t)r * Bp + b];
+  for (int i = 0; i < S; ++i) acc += scratch[(size_t)i * Bp + b];
   out[b] = acc * scale;
 }
 
-void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, int32_t Bp,
-                            double* out, double scale) {
-  k_reduce_rows<<<(Bp + 127) / 128, 128, 0, s>>>(part, nrows, Bp, out, scale);
+template <typename T>
+static void reduce_rows(cudaStream_t s, const T* part, int nrows, int Bp, double* out, double scale,
+                        double* scratch) {
+  const int S = std::max(1, std::min(kRedSlices, (nrows + 63) / 64));
+  const int per = (nrows + S - 1) / S;
+  k_reduce_rows_s1<T><<<dim3((Bp + 31) / 32, S), 256, 0, s>>>(part, nrows, Bp, per, scratch);
+  SM_LAUNCH_CHECK();
+  k_reduce_rows_s2<<<(Bp + 127) / 128, 128, 0, s>>>(scratch, S, Bp, out, scale);
   SM_LAUNCH_CHECK();
 }
 
-__global__ void k_reduce_rows_d(const double* __restrict__ part, int nrows, int Bp,
-                                double* __restrict__ out) {
-  const int b = blockIdx.x * blockDim.x + threadIdx.x;
-  if (b >= Bp) return;
-  double acc = 0.0;
-  for (int r = 0; r < nrows; ++r) acc += part[(size_t)r * Bp + b];
-  out[b] = acc;
+void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, int32_t Bp,
+                            double* out, double scale, double* scratch) {
+  reduce_rows<float>(s, part, nrows, Bp, out, scale, scratch);
 }
 
 void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
-                             double* out) {
-  k_reduce_rows_d<<<(Bp + 127) / 128, 128, 0, s>>>(part, nrows, Bp, out);
-  SM_LAUNCH_CHECK();
+                             double* out, double* scratch) {
+  reduce_rows<double>(s, part, nrows, Bp, out, 1.0, scratch);
 }
 
 // ---------------------------------------------------------------------------

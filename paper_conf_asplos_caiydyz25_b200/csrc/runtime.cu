@@ -91,12 +91,13 @@ struct smoothe_run {
          *loss = nullptr;
   float* pen = nullptr;
   int32_t* choice = nullptr;
-  uint32_t *sel = nullptr, *reach = nullptr, *settle = nullptr;
+  uint32_t *sel = nullptr, *reach = nullptr, *settle = nullptr, *invalid = nullptr;
   int32_t* flags = nullptr;
   double *dcost_part = nullptr, *dcost = nullptr, *dextra = nullptr;
   double* best = nullptr;
   int32_t *best_flag = nullptr, *best_choice = nullptr, *counter = nullptr;
   double* scal = nullptr;
+  double* red_scratch = nullptr;  // 128 x Bp, reductions
   // cost model
   float* u_f = nullptr;
   double* u_d = nullptr;
@@ -213,15 +214,15 @@ void enqueue_step(smoothe_run* r) {
   if (r->cost_kind == SMOOTHE_COST_LINEAR) {
     launch_cost_linear(s, sh, g, r->u_f, r->cp, qK, r->gcp, gqK, r->f_part,
                        r->debug ? r->dbg_p : nullptr, 0);
-    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0, r->red_scratch);
   } else if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
     launch_materialize_p_f(s, sh, g, nullptr, r->cp, qK, r->p, nullptr);
     launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, r->u_f, r->p, r->gp, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->f, 1.0, r->red_scratch);
     launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
   } else {
     launch_materialize_p_f(s, sh, g, r->u_f, r->cp, qK, r->p, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0, r->red_scratch);
     launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
                    r->z1_part, r->fextra, r->gz1, r->nsplit);
     launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
@@ -231,7 +232,7 @@ void enqueue_step(smoothe_run* r) {
   pm.mark(SMOOTHE_PHASE_PENALTY);
   if (hg.num_scc > 0) {
     launch_notears(s, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen);
-    launch_reduce_rows_f64d(s, r->h_part, hg.num_scc, r->ngroups, r->h);
+    launch_reduce_rows_f64d(s, r->h_part, hg.num_scc, r->ngroups, r->h, r->red_scratch);
   }
   launch_loss(s, sh.B, r->G, r->ngroups, r->opt.lambda, r->f,
               r->cost_kind == SMOOTHE_COST_MLP ? r->fextra : nullptr, hg.num_scc > 0 ? r->h : nullptr,
@@ -250,15 +251,15 @@ void enqueue_step(smoothe_run* r) {
                 r->debug ? r->dbg_gcp : nullptr);
 
   pm.mark(SMOOTHE_PHASE_DECODE);
-  launch_decode_reach(s, sh, g, r->sel, r->reach, r->flags, r->coop_grid);
-  launch_decode_settle(s, sh, g, r->sel, r->settle, r->flags + 4, r->coop_grid);
+  launch_decode(s, sh, hg, g, r->sel, r->reach, r->invalid, r->settle + (size_t)sh.root * sh.W,
+                r->coop_grid);
   launch_decode_cost_linear(s, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
-  launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost);
+  launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost, r->red_scratch);
   const double* dextra = nullptr;
   if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
     launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
     launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, nullptr, r->sbin, nullptr, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->dextra, 1.0);
+    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->dextra, 1.0, r->red_scratch);
     dextra = r->dextra;
   } else if (r->cost_kind == SMOOTHE_COST_MLP) {
     launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
@@ -350,6 +351,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->reach = dalloc<uint32_t>(o, (size_t)sh.M * sh.W);
   r->settle = dalloc<uint32_t>(o, (size_t)sh.M * sh.W);
   r->flags = dalloc<int32_t>(o, 8);
+  r->invalid = dalloc<uint32_t>(o, sh.W);
   r->dcost_rows = decode_cost_rows(sh);
   r->dcost_part = dalloc<double>(o, (size_t)r->dcost_rows * sh.Bp);
   r->dcost = dalloc<double>(o, sh.Bp);
@@ -359,6 +361,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->best_choice = dalloc<int32_t>(o, sh.M);
   r->counter = dalloc<int32_t>(o, 1);
   r->scal = dalloc<double>(o, 2);
+  r->red_scratch = dalloc<double>(o, (size_t)128 * sh.Bp);
   r->dbg_p = nullptr;
 
   // cost model
@@ -491,6 +494,7 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.par_node = upload(o, h.par_node, &b);
       d.par_class = upload(o, h.par_class, &b);
       d.scc_class_ptr = upload(o, h.scc_class_ptr, &b);
+      d.scc_class = upload(o, h.scc_class, &b);
       d.ent_ptr = upload(o, h.ent_ptr, &b);
       d.ent_i = upload(o, h.ent_i, &b);
       d.ent_j = upload(o, h.ent_j, &b);
@@ -507,6 +511,8 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
       d.pad_par = upload(o, h.pad_par, &b);
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
+      d.lvl_ptr = upload(o, h.lvl_ptr, &b);
+      d.lvl_item = upload(o, h.lvl_item, &b);
     }
   });
   if (st != SMOOTHE_OK) {
@@ -894,9 +900,10 @@ void smoothe_free_egraph(smoothe_egraph* g) {
   if (g->device >= 0) {
     cudaSetDevice(g->device);
     void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
-                    d.scc_class_ptr, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
+                    d.scc_class_ptr, d.scc_class, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
                     d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot,
-                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par, d.pad_batch_node};
+                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par, d.pad_batch_node,
+                    d.lvl_ptr, d.lvl_item};
     for (void* p : ptrs) cudaFree(p);
   }
   delete g;
