@@ -301,19 +301,27 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       }
     }
     for (int32_t d : depth) g.num_levels = std::max(g.num_levels, d + 1);
-    std::vector<int32_t> first(ncomp, -1);  // one class per component
-    for (int32_t j = M - 1; j >= 0; --j) first[comp[j]] = j;
-    g.lvl_ptr.assign(g.num_levels + 1, 0);
-    for (int32_t a = 0; a < ncomp; ++a)
-      if (depth[a] >= 0) g.lvl_ptr[depth[a] + 1]++;
-    for (int32_t L = 0; L < g.num_levels; ++L) g.lvl_ptr[L + 1] += g.lvl_ptr[L];
-    g.lvl_item.resize(g.lvl_ptr[g.num_levels]);
-    std::vector<int32_t> fill(g.lvl_ptr.begin(), g.lvl_ptr.end() - 1);
-    for (int32_t a = 0; a < ncomp; ++a) {
-      if (depth[a] < 0) continue;
-      const int32_t j = first[a];
-      const int32_t s = g.scc_of_class[j];
-      g.lvl_item[fill[depth[a]]++] = s >= 0 ? -(s + 1) : j;
+    g.lvl_cptr.assign(g.num_levels + 1, 0);
+    g.lvl_sptr.assign(g.num_levels + 1, 0);
+    for (int32_t j = 0; j < M; ++j)
+      if (depth[comp[j]] >= 0) g.lvl_cptr[depth[comp[j]] + 1]++;
+    for (int32_t s = 0; s < g.num_scc; ++s) {
+      const int32_t d = depth[comp[g.scc_class[g.scc_class_ptr[s]]]];
+      if (d >= 0) g.lvl_sptr[d + 1]++;
+    }
+    for (int32_t L = 0; L < g.num_levels; ++L) {
+      g.lvl_cptr[L + 1] += g.lvl_cptr[L];
+      g.lvl_sptr[L + 1] += g.lvl_sptr[L];
+    }
+    g.lvl_class.resize(g.lvl_cptr[g.num_levels]);
+    g.lvl_scc.resize(g.lvl_sptr[g.num_levels]);
+    std::vector<int32_t> cf(g.lvl_cptr.begin(), g.lvl_cptr.end() - 1);
+    std::vector<int32_t> sf(g.lvl_sptr.begin(), g.lvl_sptr.end() - 1);
+    for (int32_t j = 0; j < M; ++j)
+      if (depth[comp[j]] >= 0) g.lvl_class[cf[depth[comp[j]]]++] = j;
+    for (int32_t s = 0; s < g.num_scc; ++s) {
+      const int32_t d = depth[comp[g.scc_class[g.scc_class_ptr[s]]]];
+      if (d >= 0) g.lvl_scc[sf[d]++] = s;
     }
   }
 

@@ -70,11 +70,11 @@ struct HostGraph {
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
   // Decode schedule: levels of the SCC condensation reachable from the root
-  // (level = longest path from the root's component).  Items of level L are
-  // lvl_item[lvl_ptr[L] .. lvl_ptr[L+1]): a class id j >= 0 (trivial
-  // component) or -(s+1) for the non-trivial SCC s.
+  // (level = longest path from the root's component).  Level L holds the
+  // classes lvl_class[lvl_cptr[L] .. lvl_cptr[L+1]) and the non-trivial SCCs
+  // lvl_scc[lvl_sptr[L] .. lvl_sptr[L+1]).
   int32_t num_levels = 0;
-  std::vector<int32_t> lvl_ptr, lvl_item;
+  std::vector<int32_t> lvl_cptr, lvl_class, lvl_sptr, lvl_scc;
 };
 
 void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -83,13 +83,13 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
 struct DevGraph {
   int32_t *class_ptr = nullptr, *child_ptr = nullptr, *child_class = nullptr;
   int32_t *par_ptr = nullptr, *par_node = nullptr, *par_class = nullptr;
-  int32_t *scc_class_ptr = nullptr, *scc_class = nullptr, *ent_ptr = nullptr, *ent_i = nullptr, *ent_j = nullptr;
+  int32_t *scc_class_ptr = nullptr, *scc_class = nullptr, *scc_of_class = nullptr, *ent_ptr = nullptr, *ent_i = nullptr, *ent_j = nullptr;
   int32_t *ent_node_ptr = nullptr, *ent_node = nullptr;
   int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t *pad_batch_node = nullptr;
-  int32_t *lvl_ptr = nullptr, *lvl_item = nullptr;
+  int32_t *lvl_cptr = nullptr, *lvl_class = nullptr, *lvl_sptr = nullptr, *lvl_scc = nullptr;
   int64_t bytes = 0;
 };
 

@@ -26,9 +26,11 @@ namespace smoothe {
 // level by level over the condensation of the e-class graph (levels from the
 // loader: longest path from the root's strongly connected component):
 //  * a class in a trivial component has all its parents at lower levels, so
-//    reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k) is final in one pass;
-//  * a non-trivial SCC is iterated to its local fixpoint by one warp per
-//    (SCC, 32-seed word) (lanes = classes, |S| <= 64);
+//    reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k) is final in one pass
+//    (one warp per (class, 32-seed word), lanes over the parents);
+//  * a non-trivial SCC (one warp per (SCC, word)) ORs in its external parents
+//    once, then iterates its internal edges to the local fixpoint in shared
+//    memory (|S| <= 64);
 //  * every cycle of a selection lies inside one SCC, so the selection is valid
 //    iff, in every SCC, the reached classes settle bottom-up within the SCC:
 //    settle_j = !reach_j OR OR_{k in m_j} (sel_k AND AND_{c in ch_k cap S} settle_c).
@@ -36,60 +38,115 @@ namespace smoothe {
 //    order-independent, deterministic).
 // One grid barrier per level; each class is evaluated once per level pass.
 constexpr int kDecodeWarps = 8;
+constexpr int kDecodeMaxEnt = 192;    // intra-SCC edge entries cached in shared memory
+constexpr int kDecodeMaxNodes = 384;  // SCC e-nodes staged in shared memory
+constexpr int kDecodeMaxChild = 512;  // their internal child entries
 
 __global__ void __launch_bounds__(256) k_decode_levels(
-    int W, int root, int num_levels, const int32_t* __restrict__ lvl_ptr,
-    const int32_t* __restrict__ lvl_item, const int32_t* __restrict__ par_ptr,
+    int W, int root, int num_levels, const int32_t* __restrict__ lvl_cptr,
+    const int32_t* __restrict__ lvl_class, const int32_t* __restrict__ lvl_sptr,
+    const int32_t* __restrict__ lvl_scc, const int32_t* __restrict__ par_ptr,
     const int32_t* __restrict__ par_node, const int32_t* __restrict__ par_class,
     const int32_t* __restrict__ class_ptr, const int32_t* __restrict__ scc_class_ptr,
-    const int32_t* __restrict__ scc_class, const int32_t* __restrict__ node_slot,
+    const int32_t* __restrict__ scc_class, const int32_t* __restrict__ scc_of_class,
+    const int32_t* __restrict__ ent_ptr, const int32_t* __restrict__ ent_i,
+    const int32_t* __restrict__ ent_j, const int32_t* __restrict__ ent_node_ptr,
+    const int32_t* __restrict__ ent_node, const int32_t* __restrict__ node_slot,
+    const int32_t* __restrict__ slot_ptr, const int32_t* __restrict__ slot_node,
     const int32_t* __restrict__ slot_jptr, const int32_t* __restrict__ slot_jloc,
     const uint32_t* __restrict__ sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out) {
-  __shared__ uint32_t st[kDecodeWarps][64];
+  __shared__ uint32_t rs[kDecodeWarps][64];            // reach words of the SCC's classes
+  __shared__ uint32_t st[kDecodeWarps][64];            // settle words
+  __shared__ uint32_t es[kDecodeWarps][kDecodeMaxEnt]; // OR of sel over each intra-SCC entry
+  __shared__ uint32_t qs[kDecodeWarps][kDecodeMaxNodes];     // sel word of each SCC e-node
+  __shared__ uint16_t qp[kDecodeWarps][kDecodeMaxNodes + 1]; // its internal children: offsets
+  __shared__ uint8_t qc[kDecodeWarps][kDecodeMaxChild];      //   ... and local class ids
   cg::grid_group grid = cg::this_grid();
-  const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const int64_t gwarp = gtid >> 5, nwarps = nthreads >> 5;
-  auto pull = [&](int j, int w) {
-    uint32_t v = 0;
-    for (int e = par_ptr[j]; e < par_ptr[j + 1]; ++e)
-      v |= __ldcg(reach + (size_t)par_class[e] * W + w) & sel[(size_t)par_node[e] * W + w];
-    return v;
-  };
+  const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int L = 0; L < num_levels; ++L) {
-    const int i0 = lvl_ptr[L];
-    const int64_t nitems = (int64_t)(lvl_ptr[L + 1] - i0) * W;
-    // trivial components: one thread per (class, word)
-    for (int64_t it = gtid; it < nitems; it += nthreads) {
-      const int j = lvl_item[i0 + it / W];
+    // phase A: every class of the level ORs in its parents outside its own SCC
+    // (all final: they sit at lower levels); one warp per (class, word), lanes
+    // over the parents.  For trivial classes this is the final reach.
+    const int c0l = lvl_cptr[L];
+    const int64_t nA = (int64_t)(lvl_cptr[L + 1] - c0l) * W;
+    for (int64_t it = gwarp; it < nA; it += nwarps) {
+      const int j = lvl_class[c0l + it / W];
       const int w = (int)(it % W);
-      if (j < 0 || j == root) continue;
-      __stcg(reach + (size_t)j * W + w, pull(j, w));
+      if (j == root) continue;
+      const int sj = scc_of_class[j];
+      uint32_t v = 0;
+      for (int e = par_ptr[j] + lane; e < par_ptr[j + 1]; e += 32) {
+        const int pc = par_class[e];
+        if (sj < 0 || scc_of_class[pc] != sj)
+          v |= __ldcg(reach + (size_t)pc * W + w) & sel[(size_t)par_node[e] * W + w];
+      }
+      v = __reduce_or_sync(0xffffffffu, v);
+      if (lane == 0) __stcg(reach + (size_t)j * W + w, v);
     }
-    // non-trivial SCCs: one warp per (SCC, word)
-    for (int64_t it = gwarp; it < nitems; it += nwarps) {
-      const int item = lvl_item[i0 + it / W];
+    const int s0l = lvl_sptr[L];
+    const int64_t nB = (int64_t)(lvl_sptr[L + 1] - s0l) * W;
+    if (nB == 0) {
+      grid.sync();
+      continue;
+    }
+    grid.sync();
+    // phase B: non-trivial SCCs, one warp per (SCC, word): internal edges to
+    // the local reach fixpoint, then the local settle (acyclicity) check
+    for (int64_t it = gwarp; it < nB; it += nwarps) {
+      const int s = lvl_scc[s0l + it / W];
       const int w = (int)(it % W);
-      if (item >= 0) continue;
-      const int s = -item - 1, c0 = scc_class_ptr[s], n = scc_class_ptr[s + 1] - c0;
+      const int c0 = scc_class_ptr[s], n = scc_class_ptr[s + 1] - c0;
+      for (int l = lane; l < n; l += 32) {
+        const int j = scc_class[c0 + l];
+        rs[wib][l] = j == root ? 0xffffffffu : __ldcg(reach + (size_t)j * W + w);
+      }
+      const int e0 = ent_ptr[s], ne = ent_ptr[s + 1] - e0;
+      for (int e = lane; e < ne && e < kDecodeMaxEnt; e += 32) {
+        uint32_t m = 0;
+        for (int a = ent_node_ptr[e0 + e]; a < ent_node_ptr[e0 + e + 1]; ++a)
+          m |= sel[(size_t)ent_node[a] * W + w];
+        es[wib][e] = m;
+      }
+      __syncwarp();
       bool changed = true;
-      while (__any_sync(0xffffffffu, changed)) {  // local reach fixpoint (monotone)
+      while (__any_sync(0xffffffffu, changed)) {  // r_j |= r_i & sel(i -> j), monotone
         changed = false;
-        for (int l = lane; l < n; l += 32) {
-          const int j = scc_class[c0 + l];
-          const uint32_t v = j == root ? 0xffffffffu : pull(j, w);
-          if (v != __ldcg(reach + (size_t)j * W + w)) {
-            __stcg(reach + (size_t)j * W + w, v);
+        for (int e = lane; e < ne; e += 32) {
+          uint32_t m;
+          if (e < kDecodeMaxEnt) {
+            m = es[wib][e];
+          } else {
+            m = 0;
+            for (int a = ent_node_ptr[e0 + e]; a < ent_node_ptr[e0 + e + 1]; ++a)
+              m |= sel[(size_t)ent_node[a] * W + w];
+          }
+          const int ji = ent_j[e0 + e];
+          const uint32_t add = rs[wib][ent_i[e0 + e]] & m & ~rs[wib][ji];
+          if (add) {
+            atomicOr(&rs[wib][ji], add);
             changed = true;
           }
         }
         __syncwarp();
       }
-      uint32_t r[2] = {0, 0};
-      for (int l = lane, x = 0; l < n; l += 32, ++x) {
-        r[x] = __ldcg(reach + (size_t)scc_class[c0 + l] * W + w);
-        st[wib][l] = ~r[x];  // unreached classes count as settled
+      for (int l = lane; l < n; l += 32) {
+        __stcg(reach + (size_t)scc_class[c0 + l] * W + w, rs[wib][l]);
+        st[wib][l] = ~rs[wib][l];  // unreached classes count as settled
+      }
+      // stage the SCC's e-nodes (selection word, internal children) in shared
+      // memory when they fit, so the settle passes touch no global memory
+      const int q_begin = slot_ptr[s], nq = slot_ptr[s + 1] - q_begin;
+      const int ch_begin = slot_jptr[q_begin], nch = slot_jptr[q_begin + nq] - ch_begin;
+      const bool staged = nq <= kDecodeMaxNodes && nch <= kDecodeMaxChild;
+      if (staged) {
+        for (int q = lane; q < nq; q += 32) {
+          qs[wib][q] = sel[(size_t)slot_node[q_begin + q] * W + w];
+          qp[wib][q + 1] = (uint16_t)(slot_jptr[q_begin + q + 1] - ch_begin);
+        }
+        if (lane == 0) qp[wib][0] = 0;
+        for (int e = lane; e < nch; e += 32) qc[wib][e] = (uint8_t)slot_jloc[ch_begin + e];
       }
       __syncwarp();
       changed = true;
@@ -98,11 +155,18 @@ __global__ void __launch_bounds__(256) k_decode_levels(
         for (int l = lane; l < n; l += 32) {
           const int j = scc_class[c0 + l];
           uint32_t v = st[wib][l];
-          const int q0 = node_slot[class_ptr[j]];
-          for (int k = class_ptr[j]; k < class_ptr[j + 1]; ++k) {
-            const int q = q0 + (k - class_ptr[j]);
-            uint32_t acc = sel[(size_t)k * W + w];
-            for (int e = slot_jptr[q]; acc && e < slot_jptr[q + 1]; ++e) acc &= st[wib][slot_jloc[e]];
+          const int q0 = node_slot[class_ptr[j]] - q_begin, nk = class_ptr[j + 1] - class_ptr[j];
+          for (int t = 0; t < nk && v != 0xffffffffu; ++t) {
+            const int q = q0 + t;
+            uint32_t acc;
+            if (staged) {
+              acc = qs[wib][q] & ~v;
+              for (int e = qp[wib][q]; acc && e < qp[wib][q + 1]; ++e) acc &= st[wib][qc[wib][e]];
+            } else {
+              acc = sel[(size_t)slot_node[q_begin + q] * W + w] & ~v;
+              for (int e = slot_jptr[q_begin + q]; acc && e < slot_jptr[q_begin + q + 1]; ++e)
+                acc &= st[wib][slot_jloc[e]];
+            }
             v |= acc;
           }
           if (v != st[wib][l]) {
@@ -113,14 +177,14 @@ __global__ void __launch_bounds__(256) k_decode_levels(
         __syncwarp();
       }
       uint32_t bad = 0;
-      for (int l = lane, x = 0; l < n; l += 32, ++x) bad |= r[x] & ~st[wib][l];
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+      for (int l = lane; l < n; l += 32) bad |= rs[wib][l] & ~st[wib][l];
+      bad = __reduce_or_sync(0xffffffffu, bad);
       if (lane == 0 && bad) atomicOr(invalid + w, bad);
       __syncwarp();
     }
     grid.sync();
   }
+  const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (gtid < W) valid_out[gtid] = ~__ldcg(invalid + gtid);
 }
 
@@ -136,11 +200,14 @@ void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const D
   SM_CUDA(cudaMemsetAsync(reach, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach + (size_t)sh.root * sh.W, 0xff, sizeof(uint32_t) * sh.W, s));
   int W = sh.W, root = sh.root, L = hg.num_levels;
-  void* args[] = {&W, &root, &L, (void*)&g.lvl_ptr, (void*)&g.lvl_item, (void*)&g.par_ptr,
+  void* args[] = {&W, &root, &L, (void*)&g.lvl_cptr, (void*)&g.lvl_class, (void*)&g.lvl_sptr,
+                  (void*)&g.lvl_scc, (void*)&g.par_ptr,
                   (void*)&g.par_node, (void*)&g.par_class, (void*)&g.class_ptr,
-                  (void*)&g.scc_class_ptr, (void*)&g.scc_class, (void*)&g.node_slot,
-                  (void*)&g.slot_jptr, (void*)&g.slot_jloc, (void*)&sel, &reach, &invalid,
-                  &valid_out};
+                  (void*)&g.scc_class_ptr, (void*)&g.scc_class, (void*)&g.scc_of_class,
+                  (void*)&g.ent_ptr, (void*)&g.ent_i, (void*)&g.ent_j, (void*)&g.ent_node_ptr,
+                  (void*)&g.ent_node, (void*)&g.node_slot, (void*)&g.slot_ptr,
+                  (void*)&g.slot_node, (void*)&g.slot_jptr,
+                  (void*)&g.slot_jloc, (void*)&sel, &reach, &invalid, &valid_out};
   coop_launch((const void*)k_decode_levels, grid, args, s);
 }
 

@@ -495,6 +495,7 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.par_class = upload(o, h.par_class, &b);
       d.scc_class_ptr = upload(o, h.scc_class_ptr, &b);
       d.scc_class = upload(o, h.scc_class, &b);
+      d.scc_of_class = upload(o, h.scc_of_class, &b);
       d.ent_ptr = upload(o, h.ent_ptr, &b);
       d.ent_i = upload(o, h.ent_i, &b);
       d.ent_j = upload(o, h.ent_j, &b);
@@ -511,8 +512,10 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
       d.pad_par = upload(o, h.pad_par, &b);
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
-      d.lvl_ptr = upload(o, h.lvl_ptr, &b);
-      d.lvl_item = upload(o, h.lvl_item, &b);
+      d.lvl_cptr = upload(o, h.lvl_cptr, &b);
+      d.lvl_class = upload(o, h.lvl_class, &b);
+      d.lvl_sptr = upload(o, h.lvl_sptr, &b);
+      d.lvl_scc = upload(o, h.lvl_scc, &b);
     }
   });
   if (st != SMOOTHE_OK) {
@@ -900,10 +903,10 @@ void smoothe_free_egraph(smoothe_egraph* g) {
   if (g->device >= 0) {
     cudaSetDevice(g->device);
     void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
-                    d.scc_class_ptr, d.scc_class, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
+                    d.scc_class_ptr, d.scc_class, d.scc_of_class, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
                     d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot,
                     d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par, d.pad_batch_node,
-                    d.lvl_ptr, d.lvl_item};
+                    d.lvl_cptr, d.lvl_class, d.lvl_sptr, d.lvl_scc};
     for (void* p : ptrs) cudaFree(p);
   }
   delete g;
