@@ -39,6 +39,11 @@ inline dim3 row_grid(int rows, int Bp, int LPR, int block = kBlock) {
 __device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
 __device__ __forceinline__ int4 ld4i(const int32_t* p) { return *reinterpret_cast<const int4*>(p); }
 __device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+// evict-first ("streaming") variants for rows touched once per launch, so they
+// do not displace the rows that are gathered many times from L2
+__device__ __forceinline__ float4 ldcs4(const float* p) { return __ldcs(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ void stcs4(float* p, float4 v) { __stcs(reinterpret_cast<float4*>(p), v); }
+__device__ __forceinline__ void stcs4i(int32_t* p, int4 v) { __stcs(reinterpret_cast<int4*>(p), v); }
 __device__ __forceinline__ void st4i(int32_t* p, int4 v) { *reinterpret_cast<int4*>(p) = v; }
 
 __device__ __forceinline__ float comp(const float4& v, int c) {

@@ -89,8 +89,8 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   }
   const size_t o = (size_t)j * Bp + s0;
   st4(q + o, qo);
-  if (pi) st4(pi + o, po);
-  st4i(am + o, arg);
+  if (pi) stcs4(pi + o, po);
+  stcs4i(am + o, arg);
 }
 
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
@@ -123,7 +123,7 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // (g_p = 0, nothing to update).
 // ---------------------------------------------------------------------------
 template <int LPR, bool HI, bool HC>
-__global__ void __launch_bounds__(kSweepBlock, 16) k_sweep_reverse(
+__global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
     int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
     const int32_t* __restrict__ pad_child_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
@@ -139,8 +139,9 @@ __global__ void __launch_bounds__(kSweepBlock, 16) k_sweep_reverse(
   if (bb < be) {
     int k = pad_batch_node[bb];
     size_t ok = (size_t)k * Bp + s0;
-    float4 cv = ld4(cp + ok);
-    float4 cvn = zero;  // next e-node's cp row, requested one batch early
+    float4 cv = ldcs4(cp + ok);
+    float4 cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
+    float4 gc = ldcs4(gcp + ok);
     // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
     // three terms: X = sum_j g_j (wI max(s pi_j, 0) + wC [a_j = k] r) with
     // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
@@ -149,24 +150,33 @@ __global__ void __launch_bounds__(kSweepBlock, 16) k_sweep_reverse(
 #pragma unroll
     for (int x = 0; x < 4; ++x) comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
     float4 X = zero;
-    int4 j4 = ld4i(pad_child + 4 * (size_t)bb);
-    int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
-    for (int b = bb; b < be; ++b) {
-      const int jj[4] = {j4.x, j4.y, j4.z, j4.w};
-      const int knext = kn;  // e-node of batch b+1 (-1: none)
-      if (b + 1 < be) {
-        j4 = ld4i(pad_child + 4 * (size_t)(b + 1));
-        kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
-      }
-      if (knext >= 0 && knext != k) cvn = ld4(cp + (size_t)knext * Bp + s0);
-      float4 g[4], P[4];
-      int4 a[4];
+    // batch b's rows are in (g, P, a); batch b+1's are requested before batch b
+    // is consumed (double buffering), indices two batches ahead
+    auto fetch = [&](int4 j, float4* g, float4* P, int4* a) {
+      const int jj[4] = {j.x, j.y, j.z, j.w};
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const size_t oj = (size_t)jj[u] * Bp + s0;
         g[u] = ld4(gq + oj);
         if (HI) P[u] = ld4(pi + oj);
         if (HC) a[u] = ld4i(am + oj);
+      }
+    };
+    float4 g[4], P[4], g1[4], P1[4];
+    int4 a[4], a1[4];
+    fetch(ld4i(pad_child + 4 * (size_t)bb), g, P, a);
+    int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(root, root, root, root);
+    int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
+    for (int b = bb; b < be; ++b) {
+      const int knext = kn;  // e-node of batch b+1 (-1: none)
+      if (b + 1 < be) {
+        fetch(j4, g1, P1, a1);
+        if (b + 2 < be) j4 = ld4i(pad_child + 4 * (size_t)(b + 2));
+        kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
+      }
+      if (knext >= 0 && knext != k) {
+        cvn = ldcs4(cp + (size_t)knext * Bp + s0);
+        gcn = ldcs4(gcp + (size_t)knext * Bp + s0);
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
@@ -179,19 +189,25 @@ __global__ void __launch_bounds__(kSweepBlock, 16) k_sweep_reverse(
           comp(X, x) = fmaf(comp(g[u], x), w, comp(X, x));
         }
       }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        g[u] = g1[u];
+        P[u] = P1[u];
+        a[u] = a1[u];
+      }
       if (knext != k) {  // finalise e-node k
-        float4 gc = ld4(gcp + ok);
 #pragma unroll
         for (int x = 0; x < 4; ++x) {
           const float gp = HI && comp(om, x) != 0.f ? __fdividef(comp(X, x), comp(om, x)) : comp(X, x);
           comp(gc, x) += gp * comp(qp, x);
           comp(gqacc, x) += gp * comp(cv, x);
         }
-        st4(gcp + ok, gc);
+        stcs4(gcp + ok, gc);
         if (knext >= 0) {
           k = knext;
           ok = (size_t)k * Bp + s0;
           cv = cvn;
+          gc = gcn;
 #pragma unroll
           for (int x = 0; x < 4; ++x)
             comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
