@@ -122,48 +122,95 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // rows are requested before the current one is finished.  Leaves own no batch
 // (g_p = 0, nothing to update).
 // ---------------------------------------------------------------------------
-template <int LPR, bool HI, bool HC>
+// V seeds per lane (V = 1, 2, 4: 32 lanes always own one class row slice of
+// 32 V seeds, so no warp mixes classes; Bp > 128 uses V = 4 and Bp/128 slices).
+template <int V>
+struct Vec {
+  float v[V];
+};
+template <int V>
+struct IVec {
+  int v[V];
+};
+template <int V>
+__device__ __forceinline__ Vec<V> ldv(const float* p) {
+  Vec<V> r;
+  if (V == 4) *reinterpret_cast<float4*>(r.v) = *reinterpret_cast<const float4*>(p);
+  else if (V == 2) *reinterpret_cast<float2*>(r.v) = *reinterpret_cast<const float2*>(p);
+  else r.v[0] = *p;
+  return r;
+}
+template <int V>
+__device__ __forceinline__ Vec<V> ldv_cs(const float* p) {
+  Vec<V> r;
+  if (V == 4) *reinterpret_cast<float4*>(r.v) = __ldcs(reinterpret_cast<const float4*>(p));
+  else if (V == 2) *reinterpret_cast<float2*>(r.v) = __ldcs(reinterpret_cast<const float2*>(p));
+  else r.v[0] = __ldcs(p);
+  return r;
+}
+template <int V>
+__device__ __forceinline__ IVec<V> ldiv(const int32_t* p) {
+  IVec<V> r;
+  if (V == 4) *reinterpret_cast<int4*>(r.v) = *reinterpret_cast<const int4*>(p);
+  else if (V == 2) *reinterpret_cast<int2*>(r.v) = *reinterpret_cast<const int2*>(p);
+  else r.v[0] = *p;
+  return r;
+}
+template <int V>
+__device__ __forceinline__ void stv(float* p, const Vec<V>& x) {
+  if (V == 4) *reinterpret_cast<float4*>(p) = *reinterpret_cast<const float4*>(x.v);
+  else if (V == 2) *reinterpret_cast<float2*>(p) = *reinterpret_cast<const float2*>(x.v);
+  else *p = x.v[0];
+}
+template <int V>
+__device__ __forceinline__ void stv_cs(float* p, const Vec<V>& x) {
+  if (V == 4) __stcs(reinterpret_cast<float4*>(p), *reinterpret_cast<const float4*>(x.v));
+  else if (V == 2) __stcs(reinterpret_cast<float2*>(p), *reinterpret_cast<const float2*>(x.v));
+  else __stcs(p, x.v[0]);
+}
+
+template <int V, bool HI, bool HC>
 __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
     int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
     const int32_t* __restrict__ pad_child_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev) {
-  const int jp = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
+  const int jp = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
   if (jp >= M) return;
-  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
-  const float4 zero = make_float4(0.f, 0.f, 0.f, 0.f);
-  const float4 qp = ld4(q_prev + (size_t)jp * Bp + s0);
-  float4 gqacc = zero;
+  const int s0 = blockIdx.y * (32 * V) + (threadIdx.x % 32) * V;
+  Vec<V> zero;
+#pragma unroll
+  for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
+  const Vec<V> qp = ldv<V>(q_prev + (size_t)jp * Bp + s0);
+  Vec<V> gqacc = zero;
   const int bb = pad_child_ptr[class_ptr[jp]] >> 2, be = pad_child_ptr[class_ptr[jp + 1]] >> 2;
   if (bb < be) {
     int k = pad_batch_node[bb];
     size_t ok = (size_t)k * Bp + s0;
-    float4 cv = ldcs4(cp + ok);
-    float4 cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
-    float4 gc = ldcs4(gcp + ok);
+    Vec<V> cv = ldv_cs<V>(cp + ok), gc = ldv_cs<V>(gcp + ok);
+    Vec<V> cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
     // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
     // three terms: X = sum_j g_j (wI max(s pi_j, 0) + wC [a_j = k] r) with
     // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
     // (then g_p = X).
-    float4 om;
+    Vec<V> om, X = zero;
 #pragma unroll
-    for (int x = 0; x < 4; ++x) comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
-    float4 X = zero;
+    for (int x = 0; x < V; ++x) om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
     // batch b's rows are in (g, P, a); batch b+1's are requested before batch b
     // is consumed (double buffering), indices two batches ahead
-    auto fetch = [&](int4 j, float4* g, float4* P, int4* a) {
+    Vec<V> g[4], P[4], g1[4], P1[4];
+    IVec<V> a[4], a1[4];
+    auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) {
       const int jj[4] = {j.x, j.y, j.z, j.w};
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const size_t oj = (size_t)jj[u] * Bp + s0;
-        g[u] = ld4(gq + oj);
-        if (HI) P[u] = ld4(pi + oj);
-        if (HC) a[u] = ld4i(am + oj);
+        gg[u] = ldv<V>(gq + oj);
+        if (HI) PP[u] = ldv<V>(pi + oj);
+        if (HC) aa[u] = ldiv<V>(am + oj);
       }
     };
-    float4 g[4], P[4], g1[4], P1[4];
-    int4 a[4], a1[4];
     fetch(ld4i(pad_child + 4 * (size_t)bb), g, P, a);
     int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(root, root, root, root);
     int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
@@ -175,42 +222,41 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
         kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
       }
       if (knext >= 0 && knext != k) {
-        cvn = ldcs4(cp + (size_t)knext * Bp + s0);
-        gcn = ldcs4(gcp + (size_t)knext * Bp + s0);
+        cvn = ldv_cs<V>(cp + (size_t)knext * Bp + s0);
+        gcn = ldv_cs<V>(gcp + (size_t)knext * Bp + s0);
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
 #pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          const bool nz = comp(om, x) != 0.f;
+        for (int x = 0; x < V; ++x) {
+          const bool nz = om.v[x] != 0.f;
           float w = 0.f;
-          if (HI) w = wI * fmaxf(nz ? comp(P[u], x) : -comp(P[u], x), 0.f);
-          if (HC) w += comp(a[u], x) == k ? (HI && nz ? wC * comp(om, x) : wC) : 0.f;
-          comp(X, x) = fmaf(comp(g[u], x), w, comp(X, x));
+          if (HI) w = wI * fmaxf(nz ? P[u].v[x] : -P[u].v[x], 0.f);
+          if (HC) w += a[u].v[x] == k ? (HI && nz ? wC * om.v[x] : wC) : 0.f;
+          X.v[x] = fmaf(g[u].v[x], w, X.v[x]);
         }
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         g[u] = g1[u];
-        P[u] = P1[u];
-        a[u] = a1[u];
+        if (HI) P[u] = P1[u];
+        if (HC) a[u] = a1[u];
       }
       if (knext != k) {  // finalise e-node k
 #pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          const float gp = HI && comp(om, x) != 0.f ? __fdividef(comp(X, x), comp(om, x)) : comp(X, x);
-          comp(gc, x) += gp * comp(qp, x);
-          comp(gqacc, x) += gp * comp(cv, x);
+        for (int x = 0; x < V; ++x) {
+          const float gp = HI && om.v[x] != 0.f ? __fdividef(X.v[x], om.v[x]) : X.v[x];
+          gc.v[x] += gp * qp.v[x];
+          gqacc.v[x] += gp * cv.v[x];
         }
-        stcs4(gcp + ok, gc);
+        stv_cs<V>(gcp + ok, gc);
         if (knext >= 0) {
           k = knext;
           ok = (size_t)k * Bp + s0;
           cv = cvn;
           gc = gcn;
 #pragma unroll
-          for (int x = 0; x < 4; ++x)
-            comp(om, x) = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+          for (int x = 0; x < V; ++x) om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
           X = zero;
         }
       }
@@ -218,7 +264,7 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
   }
   if (gq_prev) {
     if (jp == root) gqacc = zero;
-    st4(gq_prev + (size_t)jp * Bp + s0, gqacc);
+    stv<V>(gq_prev + (size_t)jp * Bp + s0, gqacc);
   }
 }
 
@@ -226,16 +272,23 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
   float* out = write_gq_prev ? gq_prev : nullptr;
-#define SM_REV(HI, HC)                                                                         \
-  k_sweep_reverse<LPR, HI, HC><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>( \
+  const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
+  const dim3 grid((sh.M + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
+#define SM_REV2(VV, HI, HC)                                                                    \
+  k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
       sh.M, sh.Bp, sh.root, g.class_ptr, g.pad_child_ptr, g.pad_child, g.pad_batch_node, a.wI,  \
       a.wC, cp, q_prev, gq, pi, am, gcp, out)
-  SM_DISPATCH_LPR(sh.Bp, {
-    if (a.wI != 0.f && a.wC != 0.f) SM_REV(true, true);
-    else if (a.wI != 0.f) SM_REV(true, false);
-    else SM_REV(false, true);
-  });
+#define SM_REV(VV)                                                                             \
+  do {                                                                                         \
+    if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \
+    else if (a.wI != 0.f) SM_REV2(VV, true, false);                                            \
+    else SM_REV2(VV, false, true);                                                             \
+  } while (0)
+  if (V == 4) SM_REV(4);
+  else if (V == 2) SM_REV(2);
+  else SM_REV(1);
 #undef SM_REV
+#undef SM_REV2
   SM_LAUNCH_CHECK();
 }
 
