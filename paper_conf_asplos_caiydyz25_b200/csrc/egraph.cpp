@@ -331,14 +331,57 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     const int32_t n = g.child_ptr[i + 1] - g.child_ptr[i];
     g.pad_child_ptr[i + 1] = g.pad_child_ptr[i] + ((n + 3) & ~3);
   }
-  g.pad_child.assign(g.pad_child_ptr[N], root);
+  g.pad_child.assign(g.pad_child_ptr[N], 0);
   g.pad_batch_node.resize(g.pad_child_ptr[N] / 4);
   for (int32_t i = 0; i < N; ++i) {
     std::copy(g.child_class.begin() + g.child_ptr[i], g.child_class.begin() + g.child_ptr[i + 1],
               g.pad_child.begin() + g.pad_child_ptr[i]);
+    for (int32_t s = g.pad_child_ptr[i] + (g.child_ptr[i + 1] - g.child_ptr[i]);
+         s < g.pad_child_ptr[i + 1]; ++s)
+      g.pad_child[s] = ~g.child_class[g.child_ptr[i]];
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
+  // reverse-sweep work items: runs of <= kRevChunk batches of one class, cut at
+  // e-node boundaries; an e-node with more batches is cut into pieces of its own
+  g.rev_item.clear();
+  g.rev_class_item_ptr.assign(M + 1, 0);
+  g.rev_num_slots = 0;
+  for (int32_t j = 0; j < M; ++j) {
+    const int32_t cb0 = g.pad_child_ptr[g.class_ptr[j]] / 4, cb1 = g.pad_child_ptr[g.class_ptr[j + 1]] / 4;
+    const size_t first = g.rev_item.size();
+    auto emit = [&](int32_t b0, int32_t b1, int32_t piece) {
+      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece});
+    };
+    if (cb1 - cb0 <= kRevChunk) {
+      emit(cb0, cb1, 0);
+    } else {
+      int32_t cur = cb0;
+      for (int32_t k = g.class_ptr[j]; k < g.class_ptr[j + 1]; ++k) {
+        const int32_t nb0 = g.pad_child_ptr[k] / 4, nb1 = g.pad_child_ptr[k + 1] / 4;
+        if (nb1 - nb0 > kRevChunk) {
+          if (cur < nb0) emit(cur, nb0, 0);
+          for (int32_t b = nb0; b < nb1; b += kRevChunk) emit(b, std::min(nb1, b + kRevChunk), 1);
+          cur = nb1;
+        } else if (nb1 - cur > kRevChunk) {
+          emit(cur, nb0, 0);
+          cur = nb0;
+        }
+      }
+      if (cur < cb1) emit(cur, cb1, 0);
+    }
+    const int32_t n = (int32_t)((g.rev_item.size() - first) / 4);
+    if (n == 1) {
+      g.rev_item[first + 3] = -1;  // single item: writes its class's outputs directly
+    } else {
+      for (int32_t t = 0; t < n; ++t) {
+        int32_t& info = g.rev_item[first + 4 * t + 3];
+        info = (g.rev_num_slots++ << 1) | info;
+      }
+    }
+    g.rev_class_item_ptr[j + 1] = g.rev_class_item_ptr[j] + n;
+  }
+
   g.pad_par_ptr.assign(M + 1, 0);
   for (int32_t j = 0; j < M; ++j) {
     const int32_t n = g.par_ptr[j + 1] - g.par_ptr[j];
@@ -348,8 +391,9 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   for (int32_t j = 0; j < M; ++j)
     for (int32_t s = g.pad_par_ptr[j], e = g.par_ptr[j]; s < g.pad_par_ptr[j + 1]; ++s, ++e) {
       const bool real = e < g.par_ptr[j + 1];
-      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
-      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
+      const int32_t f = g.par_ptr[j];
+      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : g.par_node[f];
+      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : ~g.par_class[f];
     }
 }
 

@@ -37,6 +37,8 @@ struct Failure {
 // ---------------------------------------------------------------------------
 // E-graph: host analysis (egraph.cpp) and its device mirror
 // ---------------------------------------------------------------------------
+constexpr int32_t kRevChunk = 16;  // max batches of 4 children per reverse-sweep item
+
 struct HostGraph {
   int32_t M = 0, N = 0, root = 0;
   int64_t E = 0;
@@ -63,12 +65,24 @@ struct HostGraph {
   int32_t K_auto = 0, max_class_size = 0, max_in_degree = 0;
   // Sweep layouts padded to multiples of 4 entries per list (aligned vector
   // index loads, 4 row gathers in flight):
-  //   pad_child_ptr [N+1], pad_child [.]   child classes of e-node i; padding = root
-  //                                        (g_q of the root is 0: inert)
+  //   pad_child_ptr [N+1], pad_child [.]   child classes of e-node i; padding = ~(first
+  //                                        child): the kernels mask it out
   //   pad_par_ptr [M+1],  pad_par [.][2]   (parent e-node, its class) of class j;
-  //                                        padding = (N, root): row N of cp is 0: p = 0
+  //                                        padding = (first node, ~first class), masked
+  // Padding repeats a row the list already gathers (an L1/L2 hit) rather than
+  // one shared inert row: a single row hit by every padded slot of every warp
+  // serialises on one L2 slice (measured: C3 reverse sweep 17x its forward).
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
+  // Reverse-sweep work items (one warp each), [n][4] = (class j, first batch,
+  // end batch, info): a class's batches split into runs of <= kRevChunk cut at
+  // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
+  // info = -1: the class's only item; else (slot << 1) | piece, slot = its
+  // partial-sum row (the class's last item to finish combines them in order).
+  // Without the split one warp walks the largest class serially and sets the
+  // sweep time (C3: one e-node with 1507 children, 4x the rest of the sweep).
+  std::vector<int32_t> rev_item, rev_class_item_ptr;  // rev_class_item_ptr [M+1]
+  int32_t rev_num_slots = 0;
   // Decode schedule: levels of the SCC condensation reachable from the root
   // (level = longest path from the root's component).  Level L holds the
   // classes lvl_class[lvl_cptr[L] .. lvl_cptr[L+1]) and the non-trivial SCCs
@@ -89,6 +103,8 @@ struct DevGraph {
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t *pad_batch_node = nullptr;
+  int32_t *rev_item = nullptr, *rev_class_item_ptr = nullptr;
+  int32_t num_rev_items = 0, rev_num_slots = 0;
   int32_t *lvl_cptr = nullptr, *lvl_class = nullptr, *lvl_sptr = nullptr, *lvl_scc = nullptr;
   int64_t bytes = 0;
 };
@@ -141,7 +157,8 @@ void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, 
                              double* out, double* scratch);
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
-                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev);
+                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
+                          float* rev_part, int32_t* rev_cnt);
 void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
                     int32_t G, double lambda, const float* cp, double* h_part, float* pen);
 void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,

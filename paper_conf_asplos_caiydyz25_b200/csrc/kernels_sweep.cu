@@ -40,8 +40,8 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
   if (j >= M || j == root) return;
   const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
-  // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
-  // row N of cp, so p = 0: factor 1 and never a new max
+  // (node, class) pairs in batches of 4; padding pairs (k, ~c) repeat the first
+  // real pair and are masked to p = 0: factor 1 and never a new max
   const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
@@ -54,7 +54,9 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   }
   for (int e = e0; e < e1; e += 4) {
     const int kk[4] = {n01.x, n01.z, n23.x, n23.z};
-    const int cc[4] = {n01.y, n01.w, n23.y, n23.w};
+    const int cr[4] = {n01.y, n01.w, n23.y, n23.w};
+    const int cc[4] = {cr[0] < 0 ? ~cr[0] : cr[0], cr[1] < 0 ? ~cr[1] : cr[1],
+                       cr[2] < 0 ? ~cr[2] : cr[2], cr[3] < 0 ? ~cr[3] : cr[3]};
     if (e + 4 < e1) {  // next batch's pairs, one step ahead
       n01 = ld4i(pad_par + 2 * (size_t)e + 8);
       n23 = ld4i(pad_par + 2 * (size_t)e + 12);
@@ -69,7 +71,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
     for (int u = 0; u < 4; ++u) {
 #pragma unroll
       for (int x = 0; x < 4; ++x) {
-        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
+        const float p = cr[u] < 0 ? 0.f : __fmul_rn(comp(cv[u], x), comp(qv[u], x));
         const float f = __fsub_rn(1.f, p);
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
@@ -169,55 +171,79 @@ __device__ __forceinline__ void stv_cs(float* p, const Vec<V>& x) {
   else __stcs(p, x.v[0]);
 }
 
+template <int V>
+__device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows other SMs wrote
+  Vec<V> r;
+  if (V == 4) *reinterpret_cast<float4*>(r.v) = __ldcg(reinterpret_cast<const float4*>(p));
+  else if (V == 2) *reinterpret_cast<float2*>(r.v) = __ldcg(reinterpret_cast<const float2*>(p));
+  else r.v[0] = __ldcg(p);
+  return r;
+}
+
+// One warp per work item (HostGraph::rev_item): a run of batches of class j'.
+// Items holding whole e-nodes finalise them; a "piece" of a long e-node only
+// accumulates its part of X.  A class with several items has each write one
+// partial row (its g_q sum, or a piece's X); the last item to finish (a
+// per-class counter) adds them in item order, finalises the pieced e-nodes and
+// writes g_q^{t-1}_{j'} -- a fixed summation order, so the sweep stays
+// deterministic.
 template <int V, bool HI, bool HC>
 __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
-    int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
-    const int32_t* __restrict__ pad_child_ptr, const int32_t* __restrict__ pad_child,
+    int n_items, int Bp, int root, const int4* __restrict__ items,
+    const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
-    const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev) {
-  const int jp = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
-  if (jp >= M) return;
-  const int s0 = blockIdx.y * (32 * V) + (threadIdx.x % 32) * V;
+    const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
+    float* __restrict__ part, int32_t* __restrict__ cnt) {
+  const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
+  if (it >= n_items) return;
+  const int lane = threadIdx.x % 32;
+  const int4 item = items[it];
+  const int jp = item.x, bb = item.y, be = item.z, info = item.w;
+  const bool piece = info >= 0 && (info & 1);
+  const int s0 = blockIdx.y * (32 * V) + lane * V;
   Vec<V> zero;
 #pragma unroll
   for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
   const Vec<V> qp = ldv<V>(q_prev + (size_t)jp * Bp + s0);
-  Vec<V> gqacc = zero;
-  const int bb = pad_child_ptr[class_ptr[jp]] >> 2, be = pad_child_ptr[class_ptr[jp + 1]] >> 2;
+  Vec<V> gqacc = zero, X = zero;
   if (bb < be) {
     int k = pad_batch_node[bb];
     size_t ok = (size_t)k * Bp + s0;
-    Vec<V> cv = ldv_cs<V>(cp + ok), gc = ldv_cs<V>(gcp + ok);
+    Vec<V> cv = ldv_cs<V>(cp + ok), gc = piece ? zero : ldv_cs<V>(gcp + ok);
     Vec<V> cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
     // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
     // three terms: X = sum_j g_j (wI max(s pi_j, 0) + wC [a_j = k] r) with
     // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
     // (then g_p = X).
-    Vec<V> om, X = zero;
+    Vec<V> om;
 #pragma unroll
     for (int x = 0; x < V; ++x) om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
     // batch b's rows are in (g, P, a); batch b+1's are requested before batch b
     // is consumed (double buffering), indices two batches ahead
     Vec<V> g[4], P[4], g1[4], P1[4];
     IVec<V> a[4], a1[4];
-    auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) {
+    // padding slots hold ~(first child): they re-read a row of the same batch
+    // (no warp touches a row outside its own lists) and are masked out
+    auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) -> int {
       const int jj[4] = {j.x, j.y, j.z, j.w};
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const size_t oj = (size_t)jj[u] * Bp + s0;
+        const size_t oj = (size_t)(jj[u] < 0 ? ~jj[u] : jj[u]) * Bp + s0;
         gg[u] = ldv<V>(gq + oj);
         if (HI) PP[u] = ldv<V>(pi + oj);
         if (HC) aa[u] = ldiv<V>(am + oj);
       }
+      // bit u set: slot u is real
+      return (j.x >= 0 ? 1 : 0) | (j.y >= 0 ? 2 : 0) | (j.z >= 0 ? 4 : 0) | (j.w >= 0 ? 8 : 0);
     };
-    fetch(ld4i(pad_child + 4 * (size_t)bb), g, P, a);
-    int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(root, root, root, root);
+    int real = fetch(ld4i(pad_child + 4 * (size_t)bb), g, P, a), real1 = 0;
+    int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(~0, ~0, ~0, ~0);
     int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
     for (int b = bb; b < be; ++b) {
       const int knext = kn;  // e-node of batch b+1 (-1: none)
       if (b + 1 < be) {
-        fetch(j4, g1, P1, a1);
+        real1 = fetch(j4, g1, P1, a1);
         if (b + 2 < be) j4 = ld4i(pad_child + 4 * (size_t)(b + 2));
         kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
       }
@@ -233,7 +259,7 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
           float w = 0.f;
           if (HI) w = wI * fmaxf(nz ? P[u].v[x] : -P[u].v[x], 0.f);
           if (HC) w += a[u].v[x] == k ? (HI && nz ? wC * om.v[x] : wC) : 0.f;
-          X.v[x] = fmaf(g[u].v[x], w, X.v[x]);
+          X.v[x] = (real >> u) & 1 ? fmaf(g[u].v[x], w, X.v[x]) : X.v[x];
         }
       }
 #pragma unroll
@@ -242,7 +268,8 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
         if (HI) P[u] = P1[u];
         if (HC) a[u] = a1[u];
       }
-      if (knext != k) {  // finalise e-node k
+      real = real1;
+      if (knext != k && !piece) {  // finalise e-node k (a piece hands X to the combine)
 #pragma unroll
         for (int x = 0; x < V; ++x) {
           const float gp = HI && om.v[x] != 0.f ? __fdividef(X.v[x], om.v[x]) : X.v[x];
@@ -262,22 +289,67 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
       }
     }
   }
-  if (gq_prev) {
-    if (jp == root) gqacc = zero;
-    stv<V>(gq_prev + (size_t)jp * Bp + s0, gqacc);
+  if (info < 0) {  // the class's only item
+    if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : gqacc);
+    return;
   }
+  stv<V>(part + (size_t)(info >> 1) * Bp + s0, piece ? X : gqacc);
+  __threadfence();
+  __syncwarp();
+  const int i0 = class_item_ptr[jp], i1 = class_item_ptr[jp + 1];
+  int last = 0;
+  int32_t* c = cnt + (size_t)jp * gridDim.y + blockIdx.y;  // one counter per seed slice
+  if (lane == 0) last = atomicAdd(c, 1) == i1 - i0 - 1;
+  if (!__shfl_sync(0xffffffffu, last, 0)) return;
+  __threadfence();
+  if (lane == 0) *c = 0;  // ready for the next launch
+  Vec<V> acc = zero;
+  for (int t = i0; t < i1;) {
+    const int4 itm = items[t];
+    Vec<V> r = ldv_cg<V>(part + (size_t)(itm.w >> 1) * Bp + s0);
+    ++t;
+    if (!(itm.w & 1)) {
+#pragma unroll
+      for (int x = 0; x < V; ++x) acc.v[x] += r.v[x];
+      continue;
+    }
+    const int k = pad_batch_node[itm.y];  // pieces of e-node k: add up X, finalise
+    while (t < i1) {
+      const int4 nx = items[t];
+      if (!(nx.w & 1) || pad_batch_node[nx.y] != k) break;
+      const Vec<V> r2 = ldv_cg<V>(part + (size_t)(nx.w >> 1) * Bp + s0);
+#pragma unroll
+      for (int x = 0; x < V; ++x) r.v[x] += r2.v[x];
+      ++t;
+    }
+    const size_t ok = (size_t)k * Bp + s0;
+    const Vec<V> cv = ldv<V>(cp + ok);
+    Vec<V> gc = ldv<V>(gcp + ok);
+#pragma unroll
+    for (int x = 0; x < V; ++x) {
+      const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+      const float gp = HI && om != 0.f ? __fdividef(r.v[x], om) : r.v[x];
+      gc.v[x] += gp * qp.v[x];
+      acc.v[x] += gp * cv.v[x];
+    }
+    stv<V>(gcp + ok, gc);
+  }
+  if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : acc);
 }
 
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
-                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev) {
+                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
+                          float* rev_part, int32_t* rev_cnt) {
   float* out = write_gq_prev ? gq_prev : nullptr;
   const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
-  const dim3 grid((sh.M + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
+  const int n = g.num_rev_items;
+  const dim3 grid((n + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
 #define SM_REV2(VV, HI, HC)                                                                    \
   k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
-      sh.M, sh.Bp, sh.root, g.class_ptr, g.pad_child_ptr, g.pad_child, g.pad_batch_node, a.wI,  \
-      a.wC, cp, q_prev, gq, pi, am, gcp, out)
+      n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
+      g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out, rev_part,   \
+      rev_cnt)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \

@@ -98,6 +98,8 @@ struct smoothe_run {
   int32_t *best_flag = nullptr, *best_choice = nullptr, *counter = nullptr;
   double* scal = nullptr;
   double* red_scratch = nullptr;  // 128 x Bp, reductions
+  float* rev_part = nullptr;       // reverse sweep partial rows [rev_num_slots][Bp]
+  int32_t* rev_cnt = nullptr;      // [M][seed slices] items finished (self-resetting)
   // cost model
   float* u_f = nullptr;
   double* u_d = nullptr;
@@ -242,7 +244,8 @@ void enqueue_step(smoothe_run* r) {
   for (int t = K; t >= 1; --t)
     launch_sweep_reverse(s, sh, g, r->agg, r->cp, r->qstack + (size_t)(t - 1) * MB, r->gq[t & 1],
                          r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
-                         r->astack + (size_t)(t - 1) * MB, r->gcp, r->gq[(t - 1) & 1], t > 1);
+                         r->astack + (size_t)(t - 1) * MB, r->gcp, r->gq[(t - 1) & 1], t > 1,
+                         r->rev_part, r->rev_cnt);
 
   pm.mark(SMOOTHE_PHASE_UPDATE);
   launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
@@ -324,7 +327,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->theta = dalloc<float>(o, NB);
   r->m = dalloc<float>(o, NB);
   r->v = dalloc<float>(o, NB);
-  r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row: the padding parent of the sweeps
+  r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row (guard)
   r->gcp = dalloc<float>(o, NB);
   r->qstack = dalloc<float>(o, (size_t)(r->K + 1) * MB);
   if (r->agg.wI != 0.f) r->pistack = dalloc<float>(o, std::max<size_t>(1, (size_t)r->K * MB));
@@ -362,6 +365,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->counter = dalloc<int32_t>(o, 1);
   r->scal = dalloc<double>(o, 2);
   r->red_scratch = dalloc<double>(o, (size_t)128 * sh.Bp);
+  r->rev_part = dalloc<float>(o, (size_t)std::max(1, r->g->dev.rev_num_slots) * sh.Bp);
+  r->rev_cnt = dalloc<int32_t>(o, (size_t)sh.M * std::max(1, sh.Bp / 128));
   r->dbg_p = nullptr;
 
   // cost model
@@ -428,6 +433,7 @@ void init_state(smoothe_run* r) {
   SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
   SM_CUDA(cudaMemsetAsync(r->fextra, 0, sizeof(double) * sh.Bp, s));
   SM_CUDA(cudaMemsetAsync(r->counter, 0, sizeof(int32_t), s));
+  SM_CUDA(cudaMemsetAsync(r->rev_cnt, 0, sizeof(int32_t) * sh.M * std::max(1, sh.Bp / 128), s));
   const double init_best[4] = {INFINITY, -1.0, -1.0, 0.0};
   SM_CUDA(cudaMemcpyAsync(r->best, init_best, sizeof(init_best), cudaMemcpyHostToDevice, s));
   SM_CUDA(cudaMemsetAsync(r->best_choice, 0xff, sizeof(int32_t) * sh.M, s));
@@ -512,6 +518,10 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
       d.pad_par = upload(o, h.pad_par, &b);
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
+      d.rev_item = upload(o, h.rev_item, &b);
+      d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
+      d.num_rev_items = (int32_t)(h.rev_item.size() / 4);
+      d.rev_num_slots = h.rev_num_slots;
       d.lvl_cptr = upload(o, h.lvl_cptr, &b);
       d.lvl_class = upload(o, h.lvl_class, &b);
       d.lvl_sptr = upload(o, h.lvl_sptr, &b);

@@ -139,6 +139,18 @@ def test_tiny_families(sm, orc, agg, kind):
         compare_step(sm, orc, eg, 33, 3, agg, lam=0.7, seed=s, K=3 + s % 4)
 
 
+@pytest.mark.parametrize("B,agg,K", [(32, "hybrid", -1), (64, "independent", 12),
+                                     (64, "correlated", 12), (256, "hybrid", 12)])
+def test_long_lists_split_items(sm, orc, B, agg, K):
+    """Classes of > 16 batches of 4 children and e-nodes of > 64 children: the
+    reverse sweep splits them over several warps (HostGraph::rev_item) and
+    combines the partial sums; every width V = 1, 2, 4 (two seed slices at
+    256) and aggregator."""
+    eg = random_tiny(3300, "dag", num_classes=200, max_class_size=40, max_children=150)
+    assert np.diff(eg.child_ptr).max() > 64
+    compare_step(sm, orc, eg, B, 8, agg, K=K)
+
+
 def test_tiny_second_adam_step(sm, orc):
     eg = random_tiny(3100, "cyclic")
     rng = np.random.default_rng(2)
