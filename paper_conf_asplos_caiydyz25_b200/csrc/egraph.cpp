@@ -331,19 +331,25 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     const int32_t n = g.child_ptr[i + 1] - g.child_ptr[i];
     g.pad_child_ptr[i + 1] = g.pad_child_ptr[i] + ((n + 3) & ~3);
   }
-  g.pad_child.assign(g.pad_child_ptr[N], 0);
+  g.pad_child.assign(g.pad_child_ptr[N], root);
   g.pad_batch_node.resize(g.pad_child_ptr[N] / 4);
   for (int32_t i = 0; i < N; ++i) {
     std::copy(g.child_class.begin() + g.child_ptr[i], g.child_class.begin() + g.child_ptr[i + 1],
               g.pad_child.begin() + g.pad_child_ptr[i]);
-    for (int32_t s = g.pad_child_ptr[i] + (g.child_ptr[i + 1] - g.child_ptr[i]);
-         s < g.pad_child_ptr[i + 1]; ++s)
-      g.pad_child[s] = ~g.child_class[g.child_ptr[i]];
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
   // reverse-sweep work items: runs of <= kRevChunk batches of one class, cut at
   // e-node boundaries; an e-node with more batches is cut into pieces of its own
+  {
+    // measured (C2-C5): 8 batches when the whole sweep is a few batches per
+    // resident warp, 32 on the large graphs; ~8K warps are resident on a B200
+    const int64_t total = g.pad_child_ptr[N] / 4;
+    int32_t c = SMOOTHE_REV_CHUNK;
+    if (c <= 0) c = total >= 32 * 8192 ? 32 : total >= 16 * 8192 ? 16 : 8;
+    g.rev_chunk = c;
+  }
+  const int32_t kRevChunk = g.rev_chunk;
   g.rev_item.clear();
   g.rev_class_item_ptr.assign(M + 1, 0);
   g.rev_num_slots = 0;
@@ -391,9 +397,8 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   for (int32_t j = 0; j < M; ++j)
     for (int32_t s = g.pad_par_ptr[j], e = g.par_ptr[j]; s < g.pad_par_ptr[j + 1]; ++s, ++e) {
       const bool real = e < g.par_ptr[j + 1];
-      const int32_t f = g.par_ptr[j];
-      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : g.par_node[f];
-      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : ~g.par_class[f];
+      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
+      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
     }
 }
 

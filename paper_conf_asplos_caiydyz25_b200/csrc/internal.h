@@ -37,7 +37,12 @@ struct Failure {
 // ---------------------------------------------------------------------------
 // E-graph: host analysis (egraph.cpp) and its device mirror
 // ---------------------------------------------------------------------------
-constexpr int32_t kRevChunk = 16;  // max batches of 4 children per reverse-sweep item
+// Max batches of 4 children per reverse-sweep item: 0 = from the graph's size
+// (HostGraph::rev_chunk: small graphs need short items to fill the GPU, large ones pay
+// for every split); a positive value fixes it (A/B experiments).
+#ifndef SMOOTHE_REV_CHUNK
+#define SMOOTHE_REV_CHUNK 0
+#endif
 
 struct HostGraph {
   int32_t M = 0, N = 0, root = 0;
@@ -65,24 +70,23 @@ struct HostGraph {
   int32_t K_auto = 0, max_class_size = 0, max_in_degree = 0;
   // Sweep layouts padded to multiples of 4 entries per list (aligned vector
   // index loads, 4 row gathers in flight):
-  //   pad_child_ptr [N+1], pad_child [.]   child classes of e-node i; padding = ~(first
-  //                                        child): the kernels mask it out
+  //   pad_child_ptr [N+1], pad_child [.]   child classes of e-node i; padding = root
+  //                                        (g_q of the root is 0: inert, no mask)
   //   pad_par_ptr [M+1],  pad_par [.][2]   (parent e-node, its class) of class j;
-  //                                        padding = (first node, ~first class), masked
-  // Padding repeats a row the list already gathers (an L1/L2 hit) rather than
-  // one shared inert row: a single row hit by every padded slot of every warp
-  // serialises on one L2 slice (measured: C3 reverse sweep 17x its forward).
+  //                                        padding = (N, root): row N of cp is 0: p = 0
+  // (Padding with masked copies of a list's first entry instead measured no
+  // faster: the shared inert rows stay L1-resident.)
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
   // Reverse-sweep work items (one warp each), [n][4] = (class j, first batch,
-  // end batch, info): a class's batches split into runs of <= kRevChunk cut at
+  // end batch, info): a class's batches split into runs of <= rev_chunk cut at
   // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
   // info = -1: the class's only item; else (slot << 1) | piece, slot = its
   // partial-sum row (the class's last item to finish combines them in order).
   // Without the split one warp walks the largest class serially and sets the
   // sweep time (C3: one e-node with 1507 children, 4x the rest of the sweep).
   std::vector<int32_t> rev_item, rev_class_item_ptr;  // rev_class_item_ptr [M+1]
-  int32_t rev_num_slots = 0;
+  int32_t rev_num_slots = 0, rev_chunk = 0;
   // Decode schedule: levels of the SCC condensation reachable from the root
   // (level = longest path from the root's component).  Level L holds the
   // classes lvl_class[lvl_cptr[L] .. lvl_cptr[L+1]) and the non-trivial SCCs

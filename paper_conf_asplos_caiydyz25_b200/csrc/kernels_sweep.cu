@@ -40,8 +40,8 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
   if (j >= M || j == root) return;
   const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
-  // (node, class) pairs in batches of 4; padding pairs (k, ~c) repeat the first
-  // real pair and are masked to p = 0: factor 1 and never a new max
+  // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
+  // row N of cp, so p = 0: factor 1 and never a new max
   const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
@@ -54,9 +54,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   }
   for (int e = e0; e < e1; e += 4) {
     const int kk[4] = {n01.x, n01.z, n23.x, n23.z};
-    const int cr[4] = {n01.y, n01.w, n23.y, n23.w};
-    const int cc[4] = {cr[0] < 0 ? ~cr[0] : cr[0], cr[1] < 0 ? ~cr[1] : cr[1],
-                       cr[2] < 0 ? ~cr[2] : cr[2], cr[3] < 0 ? ~cr[3] : cr[3]};
+    const int cc[4] = {n01.y, n01.w, n23.y, n23.w};
     if (e + 4 < e1) {  // next batch's pairs, one step ahead
       n01 = ld4i(pad_par + 2 * (size_t)e + 8);
       n23 = ld4i(pad_par + 2 * (size_t)e + 12);
@@ -71,7 +69,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
     for (int u = 0; u < 4; ++u) {
 #pragma unroll
       for (int x = 0; x < 4; ++x) {
-        const float p = cr[u] < 0 ? 0.f : __fmul_rn(comp(cv[u], x), comp(qv[u], x));
+        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
         const float f = __fsub_rn(1.f, p);
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
@@ -188,7 +186,7 @@ __device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows oth
 // writes g_q^{t-1}_{j'} -- a fixed summation order, so the sweep stays
 // deterministic.
 template <int V, bool HI, bool HC>
-__global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
+__global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
@@ -213,62 +211,59 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
     Vec<V> cv = ldv_cs<V>(cp + ok), gc = piece ? zero : ldv_cs<V>(gcp + ok);
     Vec<V> cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
     // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
-    // three terms: X = sum_j g_j (wI max(s pi_j, 0) + wC [a_j = k] r) with
+    // three terms: X = sum_j g_j (wI max(s pi_j, 0) + [a_j = k] wC r) with
     // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
-    // (then g_p = X).
-    Vec<V> om;
+    // (then g_p = X).  Per e-node constants: sI = s wI, cC = wC r.
+    Vec<V> om, sI, cC;
+    auto node_consts = [&]() {
 #pragma unroll
-    for (int x = 0; x < V; ++x) om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
-    // batch b's rows are in (g, P, a); batch b+1's are requested before batch b
-    // is consumed (double buffering), indices two batches ahead
-    Vec<V> g[4], P[4], g1[4], P1[4];
-    IVec<V> a[4], a1[4];
-    // padding slots hold ~(first child): they re-read a row of the same batch
-    // (no warp touches a row outside its own lists) and are masked out
-    auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) -> int {
+      for (int x = 0; x < V; ++x) {
+        om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+        const bool nz = om.v[x] != 0.f;
+        sI.v[x] = nz ? wI : -wI;
+        cC.v[x] = nz ? wC * om.v[x] : wC;
+      }
+    };
+    node_consts();
+    // Double-buffered rows: batch b+1's are requested before batch b is
+    // consumed; indices two batches ahead.  (Unrolling by two to drop the
+    // buffer copies measured 10-25% slower.)  Padding slots point at the
+    // root, whose g_q row is 0: no mask.
+    Vec<V> gA[4], PA[4], gB[4], PB[4];
+    IVec<V> aA[4], aB[4];
+    auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) {
       const int jj[4] = {j.x, j.y, j.z, j.w};
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const size_t oj = (size_t)(jj[u] < 0 ? ~jj[u] : jj[u]) * Bp + s0;
+        const size_t oj = (size_t)jj[u] * Bp + s0;
         gg[u] = ldv<V>(gq + oj);
         if (HI) PP[u] = ldv<V>(pi + oj);
         if (HC) aa[u] = ldiv<V>(am + oj);
       }
-      // bit u set: slot u is real
-      return (j.x >= 0 ? 1 : 0) | (j.y >= 0 ? 2 : 0) | (j.z >= 0 ? 4 : 0) | (j.w >= 0 ? 8 : 0);
     };
-    int real = fetch(ld4i(pad_child + 4 * (size_t)bb), g, P, a), real1 = 0;
-    int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(~0, ~0, ~0, ~0);
+    fetch(ld4i(pad_child + 4 * (size_t)bb), gA, PA, aA);
+    int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(root, root, root, root);
     int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
-    for (int b = bb; b < be; ++b) {
+    // consume batch b from (g, P, a) while batch b+1 is fetched into (gn, Pn, an)
+    auto step = [&](int b, Vec<V>* g, Vec<V>* P, IVec<V>* a, Vec<V>* gn, Vec<V>* Pn, IVec<V>* an) {
       const int knext = kn;  // e-node of batch b+1 (-1: none)
       if (b + 1 < be) {
-        real1 = fetch(j4, g1, P1, a1);
+        fetch(j4, gn, Pn, an);
         if (b + 2 < be) j4 = ld4i(pad_child + 4 * (size_t)(b + 2));
         kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
       }
       if (knext >= 0 && knext != k) {
         cvn = ldv_cs<V>(cp + (size_t)knext * Bp + s0);
-        gcn = ldv_cs<V>(gcp + (size_t)knext * Bp + s0);
+        if (!piece) gcn = ldv_cs<V>(gcp + (size_t)knext * Bp + s0);
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
 #pragma unroll
         for (int x = 0; x < V; ++x) {
-          const bool nz = om.v[x] != 0.f;
-          float w = 0.f;
-          if (HI) w = wI * fmaxf(nz ? P[u].v[x] : -P[u].v[x], 0.f);
-          if (HC) w += a[u].v[x] == k ? (HI && nz ? wC * om.v[x] : wC) : 0.f;
-          X.v[x] = (real >> u) & 1 ? fmaf(g[u].v[x], w, X.v[x]) : X.v[x];
+          if (HI) X.v[x] = fmaf(g[u].v[x], fmaxf(sI.v[x] * P[u].v[x], 0.f), X.v[x]);
+          if (HC && a[u].v[x] == k) X.v[x] = fmaf(g[u].v[x], cC.v[x], X.v[x]);
         }
       }
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        g[u] = g1[u];
-        if (HI) P[u] = P1[u];
-        if (HC) a[u] = a1[u];
-      }
-      real = real1;
       if (knext != k && !piece) {  // finalise e-node k (a piece hands X to the combine)
 #pragma unroll
         for (int x = 0; x < V; ++x) {
@@ -282,11 +277,15 @@ __global__ void __launch_bounds__(kSweepBlock, 7) k_sweep_reverse(
           ok = (size_t)k * Bp + s0;
           cv = cvn;
           gc = gcn;
-#pragma unroll
-          for (int x = 0; x < V; ++x) om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+          node_consts();
           X = zero;
         }
       }
+    };
+    for (int b = bb; b < be; ++b) {
+      step(b, gA, PA, aA, gB, PB, aB);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) { gA[u] = gB[u]; if (HI) PA[u] = PB[u]; if (HC) aA[u] = aB[u]; }
     }
   }
   if (info < 0) {  // the class's only item
@@ -342,7 +341,10 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
                           float* rev_part, int32_t* rev_cnt) {
   float* out = write_gq_prev ? gq_prev : nullptr;
-  const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
+#ifndef SMOOTHE_REV_VMAX
+#define SMOOTHE_REV_VMAX 4
+#endif
+  const int V = std::min(SMOOTHE_REV_VMAX, sh.Bp >= 128 ? 4 : sh.Bp / 32);
   const int n = g.num_rev_items;
   const dim3 grid((n + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
 #define SM_REV2(VV, HI, HC)                                                                    \

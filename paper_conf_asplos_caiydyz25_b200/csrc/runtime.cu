@@ -327,7 +327,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->theta = dalloc<float>(o, NB);
   r->m = dalloc<float>(o, NB);
   r->v = dalloc<float>(o, NB);
-  r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row (guard)
+  r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row: the padding parent of the sweeps
   r->gcp = dalloc<float>(o, NB);
   r->qstack = dalloc<float>(o, (size_t)(r->K + 1) * MB);
   if (r->agg.wI != 0.f) r->pistack = dalloc<float>(o, std::max<size_t>(1, (size_t)r->K * MB));
@@ -427,7 +427,9 @@ void init_state(smoothe_run* r) {
     SM_CUDA(cudaMemsetAsync(r->pistack, 0, sizeof(float) * (size_t)r->K * MB, s));
     launch_fill_rows(s, r->pistack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K, sh.Bp, 1.0f);
   }
-  SM_CUDA(cudaMemsetAsync(r->astack, 0, sizeof(int32_t) * std::max<size_t>(1, (size_t)r->K * MB), s));
+  // -1: the root rows (never written) match no e-node, so padding slots, which
+  // point at the root, take no correlated term
+  SM_CUDA(cudaMemsetAsync(r->astack, 0xff, sizeof(int32_t) * std::max<size_t>(1, (size_t)r->K * MB), s));
   SM_CUDA(cudaMemsetAsync(r->gq[0], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->gq[1], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
