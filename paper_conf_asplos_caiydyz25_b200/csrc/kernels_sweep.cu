@@ -221,7 +221,7 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
         om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
         const bool nz = om.v[x] != 0.f;
         sI.v[x] = nz ? wI : -wI;
-        cC.v[x] = nz ? wC * om.v[x] : wC;
+        cC.v[x] = HI && nz ? wC * om.v[x] : wC;  // without HI, g_p = X (no division)
       }
     };
     node_consts();
