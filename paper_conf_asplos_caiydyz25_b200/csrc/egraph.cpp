@@ -357,7 +357,9 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     const int32_t cb0 = g.pad_child_ptr[g.class_ptr[j]] / 4, cb1 = g.pad_child_ptr[g.class_ptr[j + 1]] / 4;
     const size_t first = g.rev_item.size();
     auto emit = [&](int32_t b0, int32_t b1, int32_t piece) {
-      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece});
+      const int32_t k0 = b0 < b1 ? g.pad_batch_node[b0] : -1;
+      const int32_t k1 = b0 < b1 ? g.pad_batch_node[b1 - 1] : -1;
+      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece, k0, k1, 0, 0});
     };
     if (cb1 - cb0 <= kRevChunk) {
       emit(cb0, cb1, 0);
@@ -376,12 +378,12 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       }
       if (cur < cb1) emit(cur, cb1, 0);
     }
-    const int32_t n = (int32_t)((g.rev_item.size() - first) / 4);
+    const int32_t n = (int32_t)((g.rev_item.size() - first) / 8);
     if (n == 1) {
       g.rev_item[first + 3] = -1;  // single item: writes its class's outputs directly
     } else {
       for (int32_t t = 0; t < n; ++t) {
-        int32_t& info = g.rev_item[first + 4 * t + 3];
+        int32_t& info = g.rev_item[first + 8 * t + 3];
         info = (g.rev_num_slots++ << 1) | info;
       }
     }

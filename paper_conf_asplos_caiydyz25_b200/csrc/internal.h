@@ -78,8 +78,8 @@ struct HostGraph {
   // faster: the shared inert rows stay L1-resident.)
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
-  // Reverse-sweep work items (one warp each), [n][4] = (class j, first batch,
-  // end batch, info): a class's batches split into runs of <= rev_chunk cut at
+  // Reverse-sweep work items, [n][8] = (class j, first batch, end batch, info,
+  // first e-node, last e-node, 0, 0): a class's batches split into runs of <= rev_chunk cut at
   // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
   // info = -1: the class's only item; else (slot << 1) | piece, slot = its
   // partial-sum row (the class's last item to finish combines them in order).

@@ -178,13 +178,75 @@ __device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows oth
   return r;
 }
 
+// Outputs of one reverse-sweep item: g_q^{t-1}_{j'} directly (the class's only
+// item), else its partial row, and the class's last item to finish combines.
+template <int V, bool HI>
+__device__ __forceinline__ void reverse_epilogue(
+    int lane, int jp, int info, bool piece, int Bp, int root, int s0, const Vec<V>& qp,
+    const Vec<V>& gqacc, const Vec<V>& X, const int4* __restrict__ items,
+    const int32_t* __restrict__ class_item_ptr, const float* __restrict__ cp,
+    float* __restrict__ gcp, float* __restrict__ gq_prev, float* __restrict__ part,
+    int32_t* __restrict__ cnt) {
+  Vec<V> zero;
+#pragma unroll
+  for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
+  if (info < 0) {  // the class's only item
+    if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : gqacc);
+    return;
+  }
+  stv<V>(part + (size_t)(info >> 1) * Bp + s0, piece ? X : gqacc);
+  __threadfence();
+  __syncwarp();
+  const int i0 = class_item_ptr[jp], i1 = class_item_ptr[jp + 1];
+  int last = 0;
+  int32_t* c = cnt + (size_t)jp * gridDim.y + blockIdx.y;  // one counter per seed slice
+  if (lane == 0) last = atomicAdd(c, 1) == i1 - i0 - 1;
+  if (!__shfl_sync(0xffffffffu, last, 0)) return;
+  __threadfence();
+  if (lane == 0) *c = 0;  // ready for the next launch
+  Vec<V> acc = zero;
+  for (int t = i0; t < i1;) {
+    const int4 itm = items[2 * t];
+    Vec<V> r = ldv_cg<V>(part + (size_t)(itm.w >> 1) * Bp + s0);
+    if (!(itm.w & 1)) {
+      ++t;
+#pragma unroll
+      for (int x = 0; x < V; ++x) acc.v[x] += r.v[x];
+      continue;
+    }
+    const int k = items[2 * t + 1].x;  // pieces of e-node k: add up X, finalise
+    for (++t; t < i1; ++t) {
+      const int4 nx = items[2 * t];
+      if (!(nx.w & 1) || items[2 * t + 1].x != k) break;
+      const Vec<V> r2 = ldv_cg<V>(part + (size_t)(nx.w >> 1) * Bp + s0);
+#pragma unroll
+      for (int x = 0; x < V; ++x) r.v[x] += r2.v[x];
+    }
+    const size_t ok = (size_t)k * Bp + s0;
+    const Vec<V> cv = ldv<V>(cp + ok);
+    Vec<V> gc = ldv<V>(gcp + ok);
+#pragma unroll
+    for (int x = 0; x < V; ++x) {
+      const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+      const float gp = HI && om != 0.f ? __fdividef(r.v[x], om) : r.v[x];
+      gc.v[x] += gp * qp.v[x];
+      acc.v[x] += gp * cv.v[x];
+    }
+    stv<V>(gcp + ok, gc);
+  }
+  if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : acc);
+}
+
 // One warp per work item (HostGraph::rev_item): a run of batches of class j'.
 // Items holding whole e-nodes finalise them; a "piece" of a long e-node only
 // accumulates its part of X.  A class with several items has each write one
 // partial row (its g_q sum, or a piece's X); the last item to finish (a
 // per-class counter) adds them in item order, finalises the pieced e-nodes and
 // writes g_q^{t-1}_{j'} -- a fixed summation order, so the sweep stays
-// deterministic.
+// deterministic.  The item header carries its first / last e-node, so the
+// first rows are requested right after the header arrives.  (Persistent warps
+// striding over items, with the next item staged by cp.async, measured 2.3x
+// slower on C4: the in-flight window of classes spreads and L2 reuse drops.)
 template <int V, bool HI, bool HC>
 __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
@@ -192,12 +254,12 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
-    float* __restrict__ part, int32_t* __restrict__ cnt) {
+    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch) {
   const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
-  const int4 item = items[it];
-  const int jp = item.x, bb = item.y, be = item.z, info = item.w;
+  const int4 c0 = items[2 * it], c1 = items[2 * it + 1];
+  const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
   const bool piece = info >= 0 && (info & 1);
   const int s0 = blockIdx.y * (32 * V) + lane * V;
   Vec<V> zero;
@@ -206,7 +268,19 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
   const Vec<V> qp = ldv<V>(q_prev + (size_t)jp * Bp + s0);
   Vec<V> gqacc = zero, X = zero;
   if (bb < be) {
-    int k = pad_batch_node[bb];
+    int k = c1.x;
+    if (l2_prefetch) {
+      // The item's e-nodes are consecutive ids; their cp / g_cp rows stream
+      // from HBM once per sweep (no reuse): pull them into L2 now.
+      const int nn = c1.y - k + 1;
+      const int lines = 2 * nn * V;  // 128-byte lines: V per row
+      for (int l = lane; l < lines; l += 32) {
+        const int arr = l / (nn * V), r = l % (nn * V);
+        const float* base = arr ? gcp : cp;
+        const float* a = base + (size_t)(k + r / V) * Bp + blockIdx.y * (32 * V) + (r % V) * 32;
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+      }
+    }
     size_t ok = (size_t)k * Bp + s0;
     Vec<V> cv = ldv_cs<V>(cp + ok), gc = piece ? zero : ldv_cs<V>(gcp + ok);
     Vec<V> cvn = zero, gcn = zero;  // next e-node's cp / g_cp rows, requested one batch early
@@ -244,11 +318,10 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
     fetch(ld4i(pad_child + 4 * (size_t)bb), gA, PA, aA);
     int4 j4 = bb + 1 < be ? ld4i(pad_child + 4 * (size_t)(bb + 1)) : make_int4(root, root, root, root);
     int kn = bb + 1 < be ? pad_batch_node[bb + 1] : -1;
-    // consume batch b from (g, P, a) while batch b+1 is fetched into (gn, Pn, an)
-    auto step = [&](int b, Vec<V>* g, Vec<V>* P, IVec<V>* a, Vec<V>* gn, Vec<V>* Pn, IVec<V>* an) {
+    for (int b = bb; b < be; ++b) {
       const int knext = kn;  // e-node of batch b+1 (-1: none)
       if (b + 1 < be) {
-        fetch(j4, gn, Pn, an);
+        fetch(j4, gB, PB, aB);
         if (b + 2 < be) j4 = ld4i(pad_child + 4 * (size_t)(b + 2));
         kn = b + 2 < be ? pad_batch_node[b + 2] : -1;
       }
@@ -260,8 +333,8 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
       for (int u = 0; u < 4; ++u) {
 #pragma unroll
         for (int x = 0; x < V; ++x) {
-          if (HI) X.v[x] = fmaf(g[u].v[x], fmaxf(sI.v[x] * P[u].v[x], 0.f), X.v[x]);
-          if (HC && a[u].v[x] == k) X.v[x] = fmaf(g[u].v[x], cC.v[x], X.v[x]);
+          if (HI) X.v[x] = fmaf(gA[u].v[x], fmaxf(sI.v[x] * PA[u].v[x], 0.f), X.v[x]);
+          if (HC && aA[u].v[x] == k) X.v[x] = fmaf(gA[u].v[x], cC.v[x], X.v[x]);
         }
       }
       if (knext != k && !piece) {  // finalise e-node k (a piece hands X to the combine)
@@ -281,59 +354,16 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
           X = zero;
         }
       }
-    };
-    for (int b = bb; b < be; ++b) {
-      step(b, gA, PA, aA, gB, PB, aB);
 #pragma unroll
-      for (int u = 0; u < 4; ++u) { gA[u] = gB[u]; if (HI) PA[u] = PB[u]; if (HC) aA[u] = aB[u]; }
+      for (int u = 0; u < 4; ++u) {
+        gA[u] = gB[u];
+        if (HI) PA[u] = PB[u];
+        if (HC) aA[u] = aB[u];
+      }
     }
   }
-  if (info < 0) {  // the class's only item
-    if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : gqacc);
-    return;
-  }
-  stv<V>(part + (size_t)(info >> 1) * Bp + s0, piece ? X : gqacc);
-  __threadfence();
-  __syncwarp();
-  const int i0 = class_item_ptr[jp], i1 = class_item_ptr[jp + 1];
-  int last = 0;
-  int32_t* c = cnt + (size_t)jp * gridDim.y + blockIdx.y;  // one counter per seed slice
-  if (lane == 0) last = atomicAdd(c, 1) == i1 - i0 - 1;
-  if (!__shfl_sync(0xffffffffu, last, 0)) return;
-  __threadfence();
-  if (lane == 0) *c = 0;  // ready for the next launch
-  Vec<V> acc = zero;
-  for (int t = i0; t < i1;) {
-    const int4 itm = items[t];
-    Vec<V> r = ldv_cg<V>(part + (size_t)(itm.w >> 1) * Bp + s0);
-    ++t;
-    if (!(itm.w & 1)) {
-#pragma unroll
-      for (int x = 0; x < V; ++x) acc.v[x] += r.v[x];
-      continue;
-    }
-    const int k = pad_batch_node[itm.y];  // pieces of e-node k: add up X, finalise
-    while (t < i1) {
-      const int4 nx = items[t];
-      if (!(nx.w & 1) || pad_batch_node[nx.y] != k) break;
-      const Vec<V> r2 = ldv_cg<V>(part + (size_t)(nx.w >> 1) * Bp + s0);
-#pragma unroll
-      for (int x = 0; x < V; ++x) r.v[x] += r2.v[x];
-      ++t;
-    }
-    const size_t ok = (size_t)k * Bp + s0;
-    const Vec<V> cv = ldv<V>(cp + ok);
-    Vec<V> gc = ldv<V>(gcp + ok);
-#pragma unroll
-    for (int x = 0; x < V; ++x) {
-      const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
-      const float gp = HI && om != 0.f ? __fdividef(r.v[x], om) : r.v[x];
-      gc.v[x] += gp * qp.v[x];
-      acc.v[x] += gp * cv.v[x];
-    }
-    stv<V>(gcp + ok, gc);
-  }
-  if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : acc);
+  reverse_epilogue<V, HI>(lane, jp, info, piece, Bp, root, s0, qp, gqacc, X, items, class_item_ptr,
+                          cp, gcp, gq_prev, part, cnt);
 }
 
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
@@ -341,17 +371,17 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
                           float* rev_part, int32_t* rev_cnt) {
   float* out = write_gq_prev ? gq_prev : nullptr;
-#ifndef SMOOTHE_REV_VMAX
-#define SMOOTHE_REV_VMAX 4
-#endif
-  const int V = std::min(SMOOTHE_REV_VMAX, sh.Bp >= 128 ? 4 : sh.Bp / 32);
+  const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
   const int n = g.num_rev_items;
+  // cp / g_cp rows are L2-prefetched per item only when they cannot stay
+  // L2-resident (measured: +7% on C4 at 512 MB, -9% on C3 at 13 MB)
+  const bool l2_prefetch = (double)sh.N * sh.Bp * sizeof(float) > 64e6;
   const dim3 grid((n + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
 #define SM_REV2(VV, HI, HC)                                                                    \
   k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out, rev_part,   \
-      rev_cnt)
+      rev_cnt, l2_prefetch)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \

@@ -522,7 +522,7 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
       d.rev_item = upload(o, h.rev_item, &b);
       d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
-      d.num_rev_items = (int32_t)(h.rev_item.size() / 4);
+      d.num_rev_items = (int32_t)(h.rev_item.size() / 8);
       d.rev_num_slots = h.rev_num_slots;
       d.lvl_cptr = upload(o, h.lvl_cptr, &b);
       d.lvl_class = upload(o, h.lvl_class, &b);
