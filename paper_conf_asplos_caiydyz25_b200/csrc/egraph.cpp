@@ -339,6 +339,13 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
+  g.big_class.clear();
+  for (int32_t j = 0; j < M; ++j)
+    if (g.class_ptr[j + 1] - g.class_ptr[j] > kBigClass) g.big_class.push_back(j);
+  std::stable_sort(g.big_class.begin(), g.big_class.end(), [&](int32_t a, int32_t b) {
+    return g.class_ptr[a + 1] - g.class_ptr[a] > g.class_ptr[b + 1] - g.class_ptr[b];
+  });
+
   // reverse-sweep work items: runs of <= kRevChunk batches of one class, cut at
   // e-node boundaries; an e-node with more batches is cut into pieces of its own
   {

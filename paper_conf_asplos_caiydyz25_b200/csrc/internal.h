@@ -37,6 +37,8 @@ struct Failure {
 // ---------------------------------------------------------------------------
 // E-graph: host analysis (egraph.cpp) and its device mirror
 // ---------------------------------------------------------------------------
+constexpr int32_t kBigClass = 32;  // e-nodes above which a class gets a block (kernels_step.cu)
+
 // Max batches of 4 children per reverse-sweep item: 0 = from the graph's size
 // (HostGraph::rev_chunk: small graphs need short items to fill the GPU, large ones pay
 // for every split); a positive value fixes it (A/B experiments).
@@ -78,6 +80,9 @@ struct HostGraph {
   // faster: the shared inert rows stay L1-resident.)
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
+  // classes with more than kBigClass e-nodes, largest first: the per-class
+  // kernels (softmax, cost, update) give each a whole block
+  std::vector<int32_t> big_class;
   // Reverse-sweep work items, [n][8] = (class j, first batch, end batch, info,
   // first e-node, last e-node, 0, 0): a class's batches split into runs of <= rev_chunk cut at
   // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
@@ -107,6 +112,8 @@ struct DevGraph {
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t *pad_batch_node = nullptr;
+  int32_t* big_class = nullptr;
+  int32_t num_big = 0;
   int32_t *rev_item = nullptr, *rev_class_item_ptr = nullptr;
   int32_t num_rev_items = 0, rev_num_slots = 0;
   int32_t *lvl_cptr = nullptr, *lvl_class = nullptr, *lvl_sptr = nullptr, *lvl_scc = nullptr;

@@ -36,6 +36,68 @@ inline dim3 row_grid(int rows, int Bp, int LPR, int block = kBlock) {
   return dim3((rows + block / LPR - 1) / (block / LPR), num_chunks(Bp));
 }
 
+// Class kernels (softmax, cost, update): blocks [0, num_big) each take one
+// class with more than kBigClass e-nodes (its row groups stride over the
+// class's e-nodes and reduce through shared memory, so no row group walks a
+// 900-node class alone); later blocks hold one row group per class and skip
+// the big ones.
+inline dim3 class_grid(int rows, int Bp, int LPR, int num_big, int block = kBlock) {
+  return dim3(num_big + (rows + block / LPR - 1) / (block / LPR), num_chunks(Bp));
+}
+
+// Sum of a float4 over the R = kBlock / LPR row groups of a block, in row
+// group order (deterministic); every thread receives the total for its lane.
+template <int LPR>
+__device__ __forceinline__ float4 block_sum_rows(float4 (*red)[LPR], float4 v) {
+  const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  red[sub][lane] = v;
+  __syncthreads();
+  float4 acc = red[0][lane];
+  for (int r = 1; r < kBlock / LPR; ++r) {
+    const float4 w = red[r][lane];
+    acc.x += w.x; acc.y += w.y; acc.z += w.z; acc.w += w.w;
+  }
+  __syncthreads();
+  return acc;
+}
+
+// Per-class sums in a big-class block that do not depend on Bp: e-node
+// k0 + i belongs to part i mod 32, each part is summed in e-node order by one
+// row group (row group sub owns parts sub, sub + R, ...), and the 32 part sums
+// are added in part order.  So a seed's result is the same bits whatever the
+// batch it runs in (seed sharding stays bit-identical).
+constexpr int kClassParts = 32;
+template <int LPR>
+struct PartSums {
+  static constexpr int R = kBlock / LPR, PP = kClassParts / R;
+  float4 acc[PP];
+  __device__ PartSums() {
+#pragma unroll
+    for (int q = 0; q < PP; ++q) acc[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  // f(i, acc) for every e-node i of [k0, k1) this thread's parts own
+  template <typename F>
+  __device__ void run(int k0, int k1, F f) {
+    const int sub = threadIdx.x / LPR;
+#pragma unroll
+    for (int q = 0; q < PP; ++q)
+      for (int i = k0 + sub + q * R; i < k1; i += kClassParts) f(i, acc[q]);
+  }
+  __device__ float4 total(float4 (*red)[LPR]) const {  // red: [kClassParts][LPR]
+    const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+#pragma unroll
+    for (int q = 0; q < PP; ++q) red[sub + q * R][lane] = acc[q];
+    __syncthreads();
+    float4 t = red[0][lane];
+    for (int r = 1; r < kClassParts; ++r) {
+      const float4 w = red[r][lane];
+      t.x += w.x; t.y += w.y; t.z += w.z; t.w += w.w;
+    }
+    __syncthreads();
+    return t;
+  }
+};
+
 __device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
 __device__ __forceinline__ int4 ld4i(const int32_t* p) { return *reinterpret_cast<const int4*>(p); }
 __device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }

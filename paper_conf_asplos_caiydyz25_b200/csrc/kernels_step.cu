@@ -69,20 +69,39 @@ void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t se
 // c_j = argmax_{k in m_j} theta_k (lowest id on ties, reading S17) and the
 // selection masks sel[k][w] (bit l = seed 32w+l chose e-node k).
 // One warp per (class, <=4 words of 32 seeds); lane l owns seed 32w+l so a
-// ballot yields the mask word directly.
+// ballot yields the mask word directly.  Classes with more than kBigClass
+// e-nodes get a block of 8 warps striding over the e-nodes (max / arg-max and
+// sum combined through shared memory in warp order).
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(kBlock) k_softmax_argmax(int M, int Bp, int W, int nw,
                                                            const int32_t* __restrict__ class_ptr,
+                                                           const int32_t* __restrict__ big,
+                                                           int nbig,
                                                            const float* __restrict__ theta,
                                                            float* __restrict__ cp,
                                                            int32_t* __restrict__ choice,
                                                            uint32_t* __restrict__ sel) {
-  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
+  constexpr int NWARP = kBlock / 32;
+  __shared__ float smx[NWARP][4][32];
+  __shared__ int sam[NWARP][4][32];
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   const int nwc = W / nw;
-  const int j = warp / nwc;
-  if (j >= M) return;
-  const int w0 = (warp % nwc) * nw;
+  int j, w0, kstart, kstep;
+  const bool is_big = blockIdx.x < nbig * nwc;
+  if (is_big) {
+    j = big[blockIdx.x / nwc];
+    w0 = (blockIdx.x % nwc) * nw;
+    kstart = wi;
+    kstep = NWARP;
+  } else {
+    const int warp = (blockIdx.x - nbig * nwc) * NWARP + wi;
+    j = warp / nwc;
+    if (j >= M) return;
+    if (class_ptr[j + 1] - class_ptr[j] > kBigClass) return;  // a big-class block does it
+    w0 = (warp % nwc) * nw;
+    kstart = 0;
+    kstep = 1;
+  }
   const int k0 = class_ptr[j], k1 = class_ptr[j + 1];
   float mx[4], sum[4];
   int am[4];
@@ -90,26 +109,61 @@ __global__ void __launch_bounds__(kBlock) k_softmax_argmax(int M, int Bp, int W,
   for (int s = 0; s < 4; ++s) {
     mx[s] = -FLT_MAX;
     sum[s] = 0.f;
-    am[s] = k0;
+    am[s] = k1;
   }
-  for (int k = k0; k < k1; ++k) {
+  for (int k = k0 + kstart; k < k1; k += kstep) {
 #pragma unroll
     for (int s = 0; s < 4; ++s) {
       if (s < nw) {
         const float t = theta[(size_t)k * Bp + 32 * (w0 + s) + lane];
-        if (t > mx[s]) {
+        if (t > mx[s] || am[s] == k1) {
           mx[s] = t;
           am[s] = k;
         }
       }
     }
   }
-  for (int k = k0; k < k1; ++k) {
+  if (is_big) {  // combine the warps' (max, lowest arg-max)
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+      smx[wi][s][lane] = mx[s];
+      sam[wi][s][lane] = am[s];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+      float m = smx[0][s][lane];
+      int a = sam[0][s][lane];
+      for (int w = 1; w < NWARP; ++w) {
+        const float m2 = smx[w][s][lane];
+        const int a2 = sam[w][s][lane];
+        if (a2 < k1 && (a == k1 || m2 > m || (m2 == m && a2 < a))) {
+          m = m2;
+          a = a2;
+        }
+      }
+      mx[s] = m;
+      am[s] = a;
+    }
+    __syncthreads();
+  }
+  for (int k = k0 + kstart; k < k1; k += kstep) {
 #pragma unroll
     for (int s = 0; s < 4; ++s)
       if (s < nw) sum[s] += expf(theta[(size_t)k * Bp + 32 * (w0 + s) + lane] - mx[s]);
   }
-  for (int k = k0; k < k1; ++k) {
+  if (is_big) {  // total in warp order
+#pragma unroll
+    for (int s = 0; s < 4; ++s) smx[wi][s][lane] = sum[s];
+    __syncthreads();
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+      float t = smx[0][s][lane];
+      for (int w = 1; w < NWARP; ++w) t += smx[w][s][lane];
+      sum[s] = t;
+    }
+  }
+  for (int k = k0 + kstart; k < k1; k += kstep) {
 #pragma unroll
     for (int s = 0; s < 4; ++s) {
       if (s < nw) {
@@ -120,6 +174,7 @@ __global__ void __launch_bounds__(kBlock) k_softmax_argmax(int M, int Bp, int W,
       }
     }
   }
+  if (is_big && wi != 0) return;
 #pragma unroll
   for (int s = 0; s < 4; ++s)
     if (s < nw) choice[(size_t)j * Bp + 32 * (w0 + s) + lane] = am[s];
@@ -128,9 +183,11 @@ __global__ void __launch_bounds__(kBlock) k_softmax_argmax(int M, int Bp, int W,
 void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
                            float* cp, int32_t* choice, uint32_t* sel) {
   const int nw = sh.W < 4 ? sh.W : 4;
-  const int64_t warps = (int64_t)sh.M * (sh.W / nw);
-  const int grid = (int)((warps * 32 + kBlock - 1) / kBlock);
-  k_softmax_argmax<<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, sh.W, nw, g.class_ptr, theta, cp, choice, sel);
+  const int nwc = sh.W / nw;
+  const int64_t warps = (int64_t)sh.M * nwc;
+  const int grid = g.num_big * nwc + (int)((warps * 32 + kBlock - 1) / kBlock);
+  k_softmax_argmax<<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, sh.W, nw, g.class_ptr, g.big_class,
+                                           g.num_big, theta, cp, choice, sel);
   SM_LAUNCH_CHECK();
 }
 
@@ -142,52 +199,60 @@ void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, c
 // ---------------------------------------------------------------------------
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_cost_linear(
-    int M, int Bp, int root, const int32_t* __restrict__ class_ptr, const float* __restrict__ u,
+    int M, int Bp, int root, const int32_t* __restrict__ class_ptr,
+    const int32_t* __restrict__ big, int nbig, const float* __restrict__ u,
     const float* __restrict__ cp, const float* __restrict__ qK, float* __restrict__ gcp,
     float* __restrict__ gqK, float* __restrict__ f_part, float* __restrict__ p_out) {
   __shared__ float4 red[kBlock / LPR][LPR];
-  const RowGroup<LPR> rg;
+  constexpr int R = kBlock / LPR;
+  const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  const int s0 = blockIdx.y * (4 * LPR) + lane * 4;
   float4 facc = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (rg.row < M) {
-    const int j = rg.row;
-    const float4 qv = ld4(qK + (size_t)j * Bp + rg.s0);
-    float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) {
-      const float ui = __ldg(u + i);
-      const size_t o = (size_t)i * Bp + rg.s0;
-      const float4 cv = ld4(cp + o);
-      float4 p, gc;
+  auto node = [&](int i, const float4& qv, float4& gq) {
+    const float ui = __ldg(u + i);
+    const size_t o = (size_t)i * Bp + s0;
+    const float4 cv = ld4(cp + o);
+    float4 p, gc;
 #pragma unroll
-      for (int x = 0; x < 4; ++x) {
-        comp(p, x) = __fmul_rn(comp(cv, x), comp(qv, x));
-        comp(facc, x) += ui * comp(p, x);
-        comp(gc, x) = ui * comp(qv, x);
-        comp(gq, x) += ui * comp(cv, x);
-      }
-      st4(gcp + o, gc);
-      if (p_out) st4(p_out + o, p);
+    for (int x = 0; x < 4; ++x) {
+      comp(p, x) = __fmul_rn(comp(cv, x), comp(qv, x));
+      comp(facc, x) += ui * comp(p, x);
+      comp(gc, x) = ui * comp(qv, x);
+      comp(gq, x) += ui * comp(cv, x);
     }
+    st4(gcp + o, gc);
+    if (p_out) st4(p_out + o, p);
+  };
+  if (blockIdx.x < nbig) {
+    __shared__ float4 part[kClassParts][LPR];
+    const int j = big[blockIdx.x];
+    const float4 qv = ld4(qK + (size_t)j * Bp + s0);
+    PartSums<LPR> ps;
+    ps.run(class_ptr[j], class_ptr[j + 1], [&](int i, float4& gq) { node(i, qv, gq); });
+    float4 gq = ps.total(part);
     if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
-    st4(gqK + (size_t)j * Bp + rg.s0, gq);
-  }
-  red[rg.sub][threadIdx.x % LPR] = facc;
-  __syncthreads();
-  if (threadIdx.x < LPR) {
-    float4 acc = red[0][threadIdx.x];
-    for (int r = 1; r < kBlock / LPR; ++r) {
-      const float4 v = red[r][threadIdx.x];
-      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    if (sub == 0) st4(gqK + (size_t)j * Bp + s0, gq);
+  } else {
+    const int j = (blockIdx.x - nbig) * R + sub;
+    if (j < M && class_ptr[j + 1] - class_ptr[j] <= kBigClass) {
+      const float4 qv = ld4(qK + (size_t)j * Bp + s0);
+      float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) node(i, qv, gq);
+      if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
+      st4(gqK + (size_t)j * Bp + s0, gq);
     }
-    st4(f_part + (size_t)blockIdx.x * Bp + rg.s0, acc);
   }
+  const float4 ft = block_sum_rows<LPR>(red, facc);
+  if (sub == 0) st4(f_part + (size_t)blockIdx.x * Bp + s0, ft);
 }
 
 void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
                         const float* cp, const float* qK, float* gcp, float* gqK, float* f_part,
                         float* p_out, int32_t) {
   SM_DISPATCH_LPR(sh.Bp, {
-    k_cost_linear<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, g.class_ptr, u, cp, qK, gcp, gqK, f_part, p_out);
+    k_cost_linear<LPR><<<class_grid(sh.M, sh.Bp, LPR, g.num_big), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.class_ptr, g.big_class, g.num_big, u, cp, qK, gcp, gqK, f_part,
+        p_out);
   });
   SM_LAUNCH_CHECK();
 }
@@ -197,18 +262,30 @@ void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, cons
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_materialize_p(int M, int Bp,
                                                           const int32_t* __restrict__ class_ptr,
+                                                          const int32_t* __restrict__ big, int nbig,
                                                           const float* __restrict__ u,
                                                           const float* __restrict__ cp,
                                                           const float* __restrict__ qK,
                                                           float* __restrict__ p,
                                                           float* __restrict__ f_part) {
   __shared__ float4 red[kBlock / LPR][LPR];
-  const RowGroup<LPR> rg;
+  constexpr int R = kBlock / LPR;
+  const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  const int s0 = blockIdx.y * (4 * LPR) + lane * 4;
   float4 facc = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (rg.row < M) {
-    const float4 qv = ld4(qK + (size_t)rg.row * Bp + rg.s0);
-    for (int i = class_ptr[rg.row]; i < class_ptr[rg.row + 1]; ++i) {
-      const size_t o = (size_t)i * Bp + rg.s0;
+  int j = -1, kstart = 0, kstep = 1;
+  if (blockIdx.x < nbig) {
+    j = big[blockIdx.x];
+    kstart = sub;
+    kstep = R;
+  } else {
+    const int row = (blockIdx.x - nbig) * R + sub;
+    if (row < M && class_ptr[row + 1] - class_ptr[row] <= kBigClass) j = row;
+  }
+  if (j >= 0) {
+    const float4 qv = ld4(qK + (size_t)j * Bp + s0);
+    for (int i = class_ptr[j] + kstart; i < class_ptr[j + 1]; i += kstep) {
+      const size_t o = (size_t)i * Bp + s0;
       const float4 cv = ld4(cp + o);
       const float ui = u ? __ldg(u + i) : 0.f;
       float4 pv;
@@ -221,23 +298,15 @@ __global__ void __launch_bounds__(kBlock) k_materialize_p(int M, int Bp,
     }
   }
   if (!f_part) return;
-  red[rg.sub][threadIdx.x % LPR] = facc;
-  __syncthreads();
-  if (threadIdx.x < LPR) {
-    float4 acc = red[0][threadIdx.x];
-    for (int r = 1; r < kBlock / LPR; ++r) {
-      const float4 v = red[r][threadIdx.x];
-      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-    }
-    st4(f_part + (size_t)blockIdx.x * Bp + rg.s0, acc);
-  }
+  const float4 ft = block_sum_rows<LPR>(red, facc);
+  if (sub == 0) st4(f_part + (size_t)blockIdx.x * Bp + s0, ft);
 }
 
 void launch_materialize_p_f(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
                             const float* cp, const float* qK, float* p, float* f_part) {
   SM_DISPATCH_LPR(sh.Bp, {
-    k_materialize_p<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, g.class_ptr, u,
-                                                                      cp, qK, p, f_part);
+    k_materialize_p<LPR><<<class_grid(sh.M, sh.Bp, LPR, g.num_big), kBlock, 0, s>>>(
+        sh.M, sh.Bp, g.class_ptr, g.big_class, g.num_big, u, cp, qK, p, f_part);
   });
   SM_LAUNCH_CHECK();
 }
@@ -280,17 +349,16 @@ void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_cost_gp(int M, int Bp, int root,
                                                     const int32_t* __restrict__ class_ptr,
+                                                    const int32_t* __restrict__ big, int nbig,
                                                     const float* __restrict__ gp,
                                                     const float* __restrict__ cp,
                                                     const float* __restrict__ qK,
                                                     float* __restrict__ gcp, float* __restrict__ gqK) {
-  const RowGroup<LPR> rg;
-  if (rg.row >= M) return;
-  const int j = rg.row;
-  const float4 qv = ld4(qK + (size_t)j * Bp + rg.s0);
-  float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) {
-    const size_t o = (size_t)i * Bp + rg.s0;
+  constexpr int R = kBlock / LPR;
+  const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  const int s0 = blockIdx.y * (4 * LPR) + lane * 4;
+  auto node = [&](int i, const float4& qv, float4& gq) {
+    const size_t o = (size_t)i * Bp + s0;
     const float4 gv = ld4(gp + o), cv = ld4(cp + o);
     float4 gc;
 #pragma unroll
@@ -299,16 +367,32 @@ __global__ void __launch_bounds__(kBlock) k_cost_gp(int M, int Bp, int root,
       comp(gq, x) += comp(gv, x) * comp(cv, x);
     }
     st4(gcp + o, gc);
+  };
+  if (blockIdx.x < nbig) {
+    __shared__ float4 part[kClassParts][LPR];
+    const int j = big[blockIdx.x];
+    const float4 qv = ld4(qK + (size_t)j * Bp + s0);
+    PartSums<LPR> ps;
+    ps.run(class_ptr[j], class_ptr[j + 1], [&](int i, float4& gq) { node(i, qv, gq); });
+    float4 gq = ps.total(part);
+    if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (sub == 0) st4(gqK + (size_t)j * Bp + s0, gq);
+    return;
   }
+  const int j = (blockIdx.x - nbig) * R + sub;
+  if (j >= M || class_ptr[j + 1] - class_ptr[j] > kBigClass) return;
+  const float4 qv = ld4(qK + (size_t)j * Bp + s0);
+  float4 gq = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int i = class_ptr[j]; i < class_ptr[j + 1]; ++i) node(i, qv, gq);
   if (j == root) gq = make_float4(0.f, 0.f, 0.f, 0.f);
-  st4(gqK + (size_t)j * Bp + rg.s0, gq);
+  st4(gqK + (size_t)j * Bp + s0, gq);
 }
 
 void launch_cost_gp(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* gp,
                     const float* cp, const float* qK, float* gcp, float* gqK) {
   SM_DISPATCH_LPR(sh.Bp, {
-    k_cost_gp<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, sh.root, g.class_ptr,
-                                                                gp, cp, qK, gcp, gqK);
+    k_cost_gp<LPR><<<class_grid(sh.M, sh.Bp, LPR, g.num_big), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.class_ptr, g.big_class, g.num_big, gp, cp, qK, gcp, gqK);
   });
   SM_LAUNCH_CHECK();
 }
@@ -449,18 +533,30 @@ void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_sc
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_update(
     int M, int Bp, int G, int ngroups, const int32_t* __restrict__ class_ptr,
-    const int32_t* __restrict__ node_slot, const float* __restrict__ cp,
-    const float* __restrict__ gcp, const float* __restrict__ pen, float* __restrict__ theta,
-    float* __restrict__ m, float* __restrict__ v, const double* __restrict__ scal, int optimizer,
-    float lr, float beta1, float beta2, float eps, float* __restrict__ gth_out,
-    float* __restrict__ gcp_out) {
-  const RowGroup<LPR> rg;
-  if (rg.row >= M) return;
-  const int j = rg.row;
-  const int k0 = class_ptr[j], k1 = class_ptr[j + 1];
+    const int32_t* __restrict__ big, int nbig, const int32_t* __restrict__ node_slot,
+    const float* __restrict__ cp, const float* __restrict__ gcp, const float* __restrict__ pen,
+    float* __restrict__ theta, float* __restrict__ m, float* __restrict__ v,
+    const double* __restrict__ scal, int optimizer, float lr, float beta1, float beta2, float eps,
+    float* __restrict__ gth_out, float* __restrict__ gcp_out) {
+  constexpr int R = kBlock / LPR;
+  const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  const int s0 = blockIdx.y * (4 * LPR) + lane * 4;
+  int j, kstart, kstep;
+  const bool is_big = blockIdx.x < nbig;
+  if (is_big) {
+    j = big[blockIdx.x];
+    kstart = sub;
+    kstep = R;
+  } else {
+    j = (blockIdx.x - nbig) * R + sub;
+    if (j >= M || class_ptr[j + 1] - class_ptr[j] > kBigClass) return;
+    kstart = 0;
+    kstep = 1;
+  }
+  const int k0 = class_ptr[j] + kstart, k1 = class_ptr[j + 1];
   int grp[4];
 #pragma unroll
-  for (int x = 0; x < 4; ++x) grp[x] = min((rg.s0 + x) / G, ngroups - 1);
+  for (int x = 0; x < 4; ++x) grp[x] = min((s0 + x) / G, ngroups - 1);
   auto gtot = [&](int k, float4 gc) {
     const int slot = node_slot ? __ldg(node_slot + k) : -1;
     if (slot >= 0) {
@@ -469,17 +565,25 @@ __global__ void __launch_bounds__(kBlock) k_update(
     }
     return gc;
   };
-  float4 ssum = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (int k = k0; k < k1; ++k) {
-    const size_t o = (size_t)k * Bp + rg.s0;
+  auto dot = [&](int k, float4& acc) {
+    const size_t o = (size_t)k * Bp + s0;
     const float4 cv = ld4(cp + o);
     const float4 gt = gtot(k, ld4(gcp + o));
 #pragma unroll
-    for (int x = 0; x < 4; ++x) comp(ssum, x) += comp(cv, x) * comp(gt, x);
+    for (int x = 0; x < 4; ++x) comp(acc, x) += comp(cv, x) * comp(gt, x);
+  };
+  float4 ssum = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (is_big) {
+    __shared__ float4 part[kClassParts][LPR];
+    PartSums<LPR> ps;
+    ps.run(class_ptr[j], k1, dot);
+    ssum = ps.total(part);
+  } else {
+    for (int k = k0; k < k1; ++k) dot(k, ssum);
   }
   const float c1 = (float)scal[0], c2 = (float)scal[1];
-  for (int k = k0; k < k1; ++k) {
-    const size_t o = (size_t)k * Bp + rg.s0;
+  for (int k = k0; k < k1; k += kstep) {
+    const size_t o = (size_t)k * Bp + s0;
     const float4 cv = ld4(cp + o);
     const float4 gt = gtot(k, ld4(gcp + o));
     float4 th = ld4(theta + o), mv = ld4(m + o), vv = ld4(v + o), gth;
@@ -511,8 +615,9 @@ void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G
                    float beta2, float eps, float* grad_theta_out, float* grad_cp_out) {
   const int ngroups = (sh.B + G - 1) / G;
   SM_DISPATCH_LPR(sh.Bp, {
-    k_update<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, G, ngroups, g.class_ptr, pen ? g.node_slot : nullptr, cp, gcp, pen, theta, m,
+    k_update<LPR><<<class_grid(sh.M, sh.Bp, LPR, g.num_big), kBlock, 0, s>>>(
+        sh.M, sh.Bp, G, ngroups, g.class_ptr, g.big_class, g.num_big, pen ? g.node_slot : nullptr,
+        cp, gcp, pen, theta, m,
         v, step_scalars, optimizer, lr, beta1, beta2, eps, grad_theta_out, grad_cp_out);
   });
   SM_LAUNCH_CHECK();

@@ -335,10 +335,11 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->gq[0] = dalloc<float>(o, MB);
   r->gq[1] = dalloc<float>(o, MB);
   const int rows_per_block_min = 256 / 32;  // kBlock / LPR(32): fewest rows per block
-  r->f_rows = (std::max(sh.M, sh.N) + rows_per_block_min - 1) / rows_per_block_min + 1;
+  const int nbig = r->g->dev.num_big;
+  r->f_rows = (std::max(sh.M, sh.N) + rows_per_block_min - 1) / rows_per_block_min + 1 + nbig;
   {  // rows of partial sums each row-group kernel writes (its grid.x)
     const int per = 256 / (sh.Bp >= 128 ? 32 : sh.Bp / 4);
-    r->rows_M = (sh.M + per - 1) / per;
+    r->rows_M = nbig + (sh.M + per - 1) / per;  // class kernels: one block per big class first
     r->rows_N = (sh.N + per - 1) / per;
   }
   r->f_part = dalloc<float>(o, (size_t)r->f_rows * sh.Bp);
@@ -520,6 +521,8 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
       d.pad_par = upload(o, h.pad_par, &b);
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
+      d.big_class = upload(o, h.big_class, &b);
+      d.num_big = (int32_t)h.big_class.size();
       d.rev_item = upload(o, h.rev_item, &b);
       d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
       d.num_rev_items = (int32_t)(h.rev_item.size() / 8);
