@@ -201,10 +201,13 @@ void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice
                           int64_t seed_begin, int32_t* best_choice);
 // MLP (kernels_mlp.cu): f_mlp[b] (fp64) and gz1 = df/dz1 (may be NULL);
 // gp = u + W1^T gz1.
+// z1_part: [nsplit][128][Bp] split-K partials of the tensor-core layer 1
+// (nsplit = mlp_nsplit(device) CTAs per seed chunk); z1: [H1][Bp]
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
                     const float* b1, const float* W2, const float* b2, const float* W3,
-                    const float* b3, const float* p, float* z1_part, double* f_mlp, float* gz1,
-                    int32_t nsplit);
+                    const float* b3, const float* p, float* z1_part, float* z1, double* f_mlp,
+                    float* gz1, int32_t nsplit);
+int mlp_nsplit(int device);
 void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* u,
                     const float* gz1, float* gp);
 

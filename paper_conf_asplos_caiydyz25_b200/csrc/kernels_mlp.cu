@@ -1,79 +1,266 @@
 // MLP cost model f_mlp(p) = W3 relu(W2 relu(W1 p + b1) + b2) + b3 (
-// reading S22: N -> 64 -> 8 -> 1) and its gradient, CUDA-core version.
+// reading S22: N -> 64 -> 8 -> 1) and its gradient.
 //
 // Layer 1 is the only large contraction: z1[h][b] = sum_k W1[h][k] p[k][b]
-// (2*H1*N*B flop) and g_p[k][b] += sum_h W1[h][k] gz1[h][b] (same).  Split-K
-// partial sums are reduced in a fixed order, so results are deterministic.
+// (2*H1*N*B flop, tensor cores below) and g_p[k][b] += sum_h W1[h][k] gz1[h][b]
+// (same, CUDA cores).  Split-K partial sums are reduced in a fixed order, so
+// results are deterministic.
 #include "kcommon.cuh"
 
 namespace smoothe {
 
-constexpr int kMlpTK = 32;     // nodes per tile
+constexpr int kMlpTK = 32;     // nodes per tile (CUDA-core backward)
 constexpr int kMlpMaxH1 = 64;
 constexpr int kMlpMaxH2 = 16;
 
-// z1_part[split][h][b] over the split's node range; block = 256 threads,
-// seed chunk Bc = min(Bp, 128), each thread owns one seed and H1*Bc/256 hidden units.
-__global__ void __launch_bounds__(256) k_mlp_l1(int N, int Bp, int H1, int nsplit,
-                                                const float* __restrict__ W1,
-                                                const float* __restrict__ p,
-                                                float* __restrict__ z1_part) {
-  __shared__ float sW[kMlpMaxH1][kMlpTK + 1];
-  __shared__ float sP[kMlpTK][128];
-  const int Bc = Bp < 128 ? Bp : 128;
-  const int b = threadIdx.x % Bc;
-  const int hg = threadIdx.x / Bc;
-  const int ngroups = 256 / Bc;
-  const int hper = (H1 + ngroups - 1) / ngroups;
-  const int h0 = hg * hper;
-  const int seed0 = blockIdx.y * Bc;
-  const int split = blockIdx.x;
-  const int64_t per = ((int64_t)N + nsplit - 1) / nsplit;
-  const int64_t kb = (int64_t)split * per, ke = (int64_t)(split + 1) * per;
-  const int k_begin = (int)(kb < N ? kb : N);
-  const int k_end = (int)(ke < N ? ke : N);
-  float acc[kMlpMaxH1];
-#pragma unroll
-  for (int h = 0; h < kMlpMaxH1; ++h) acc[h] = 0.f;
-  for (int kt = k_begin; kt < k_end; kt += kMlpTK) {
-    const int nk = min(kMlpTK, k_end - kt);
-    for (int idx = threadIdx.x; idx < H1 * kMlpTK; idx += 256) {
-      const int h = idx / kMlpTK, kk = idx % kMlpTK;
-      sW[h][kk] = kk < nk ? W1[(size_t)h * N + kt + kk] : 0.f;
-    }
-    for (int idx = threadIdx.x; idx < kMlpTK * Bc; idx += 256) {
-      const int kk = idx / Bc, bb = idx % Bc;
-      sP[kk][bb] = kk < nk ? p[(size_t)(kt + kk) * Bp + seed0 + bb] : 0.f;
-    }
-    __syncthreads();
-    for (int kk = 0; kk < kMlpTK; ++kk) {
-      const float pv = sP[kk][b];
-#pragma unroll
-      for (int h = 0; h < kMlpMaxH1; ++h)
-        if (h < hper && h0 + h < H1) acc[h] += sW[h0 + h][kk] * pv;
-    }
-    __syncthreads();
-  }
-#pragma unroll
-  for (int h = 0; h < kMlpMaxH1; ++h)
-    if (h < hper && h0 + h < H1)
-      z1_part[((size_t)split * H1 + h0 + h) * Bp + seed0 + b] = acc[h];
+// ---------------------------------------------------------------------------
+// Layer 1 on the 5th-generation tensor cores (tcgen05, kind::tf32, fp32
+// accumulation in TMEM), split-K over the e-nodes.
+//
+// TF32 keeps 10 mantissa bits, too few for the 1e-4 parity bar, so both
+// operands are split x = hi + lo (hi = x with the low 13 mantissa bits
+// cleared, lo = x - hi exactly) and one M=128 x N=2Bc x K=8 MMA per K step
+// computes all four products at once:
+//   A = [W1_hi ; W1_lo]  (128 x K, K-major: W1 rows are K-contiguous)
+//   B = [p_hi | p_lo]    (K x 2Bc, staged K-major: 4 x 4 blocks of p are
+//                          transposed in registers; MN-major tf32 operands
+//                          without swizzle read as zeros on sm_100a, measured)
+//   D = A B,   z1 = D[h][b] + D[h][Bc+b] + D[64+h][b] + D[64+h][Bc+b]
+// (the lo*lo term is ~2^-22 relative and harmless).  Each CTA owns one seed
+// chunk of Bc <= 128 seeds and a contiguous e-node range, streams W1 and p
+// once (register loads one K block ahead, hi/lo split on the way into the
+// canonical no-swizzle UMMA layouts in shared memory), one thread issues the
+// MMAs, tcgen05.commit releases each stage, and the 4 warps read their 32 TMEM
+// lanes back at the end: z1_part[cta][128][Bp] (rows 64.. hold the W1_lo
+// products), reduced in a fixed order by k_mlp_reduce.
+// ---------------------------------------------------------------------------
+constexpr int kTcKB = 32;       // e-nodes (K) per stage
+constexpr int kTcStages = 3;
+constexpr int kTcThreads = 128;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+// no-swizzle UMMA shared-memory descriptor (sm_100 version 1)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+         ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity));
+}
+__device__ __forceinline__ float4 tf32_hi(float4 v) {
+  auto h = [](float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); };
+  return make_float4(h(v.x), h(v.y), h(v.z), h(v.w));
+}
+__device__ __forceinline__ float4 sub4(float4 a, float4 b) {
+  return make_float4(a.x - b.x, a.y - b.y, a.z - b.z, a.w - b.w);
 }
 
-// Per seed: reduce splits, layers 2-3, f_mlp, and gz1 = d f_mlp / d z1.
-__global__ void k_mlp_head(int Bp, int H1, int H2, int nsplit, const float* __restrict__ b1,
+template <int BC>
+__global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int H1, int nsplit,
+                                                            const float* __restrict__ W1,
+                                                            const float* __restrict__ p,
+                                                            float* __restrict__ z1_part) {
+  constexpr int NM = 2 * BC;                       // MMA N
+  constexpr int A_BYTES = 128 * kTcKB * 4;         // [W1_hi; W1_lo]
+  constexpr int B_BYTES = kTcKB * NM * 4;          // [p_hi | p_lo]
+  constexpr int STAGE = A_BYTES + B_BYTES;
+  constexpr int A_LBO = 16 * 128;                  // K-chunk (4 elements) stride
+  constexpr int B_LBO = (NM / 8) * 128;            // K-chunk (4 elements) stride
+  constexpr int AV = 64 * kTcKB / 4 / kTcThreads;  // float4 of W1 per thread per stage
+  constexpr int BBLK = (kTcKB / 4) * (BC / 4);     // 4 x 4 blocks of p per stage
+  constexpr int BV = (BBLK + kTcThreads - 1) / kTcThreads;
+  constexpr uint32_t TMEM_COLS = NM <= 32 ? 32 : NM <= 64 ? 64 : NM <= 128 ? 128 : 256;
+  // kind::tf32, D f32, A and B K-major, M = 128, N = NM
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
+                             ((uint32_t)(128 >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t tc_smem[];
+  __shared__ uint64_t bar[kTcStages + 1];
+  __shared__ uint32_t tmem_base_sh;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int seed0 = blockIdx.y * BC;
+  const int64_t per = (((int64_t)N + nsplit - 1) / nsplit + kTcKB - 1) / kTcKB * kTcKB;
+  const int64_t kb64 = (int64_t)blockIdx.x * per;
+  const int k_begin = (int)(kb64 < N ? kb64 : N);
+  const int k_end = (int)(k_begin + per < N ? k_begin + per : N);
+  const int nkb = (k_end - k_begin + kTcKB - 1) / kTcKB;
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&tmem_base_sh)),
+                 "n"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int i = 0; i <= kTcStages; ++i) mbar_init(&bar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem = tmem_base_sh;
+
+  float4 ra[AV], rb[BV][4];
+  auto load = [&](int kb) {
+    const int k0 = k_begin + kb * kTcKB;
+#pragma unroll
+    for (int i = 0; i < AV; ++i) {
+      const int idx = tid + i * kTcThreads, h = idx / (kTcKB / 4), k = k0 + (idx % (kTcKB / 4)) * 4;
+      ra[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (h < H1) {
+        const float* src = W1 + (size_t)h * N + k;
+        if (k + 3 < k_end && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+          ra[i] = __ldcs(reinterpret_cast<const float4*>(src));
+        } else {
+          float t[4];
+#pragma unroll
+          for (int x = 0; x < 4; ++x) t[x] = k + x < k_end ? src[x] : 0.f;
+          ra[i] = make_float4(t[0], t[1], t[2], t[3]);
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < BV; ++i) {
+      const int idx = tid + i * kTcThreads;
+      const int k = k0 + (idx / (BC / 4)) * 4, n = (idx % (BC / 4)) * 4;
+#pragma unroll
+      for (int r = 0; r < 4; ++r)
+        rb[i][r] = idx < BBLK && k + r < k_end
+                       ? __ldcs(reinterpret_cast<const float4*>(p + (size_t)(k + r) * Bp + seed0 + n))
+                       : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+  };
+  auto store = [&](int st) {
+    uint8_t* sa = tc_smem + st * STAGE;
+    uint8_t* sb = sa + A_BYTES;
+#pragma unroll
+    for (int i = 0; i < AV; ++i) {
+      const int idx = tid + i * kTcThreads, h = idx / (kTcKB / 4), kc = idx % (kTcKB / 4);
+      const float4 hi = tf32_hi(ra[i]), lo = sub4(ra[i], hi);
+      // element (r, k): core (k/4, r/8) at (kc * 16 + r/8) * 128, + (r%8) * 16
+      *reinterpret_cast<float4*>(sa + (kc * 16 + h / 8) * 128 + (h % 8) * 16) = hi;
+      *reinterpret_cast<float4*>(sa + (kc * 16 + 8 + h / 8) * 128 + (h % 8) * 16) = lo;
+    }
+#pragma unroll
+    for (int i = 0; i < BV; ++i) {
+      const int idx = tid + i * kTcThreads;
+      if (idx >= BBLK) continue;
+      const int kc = idx / (BC / 4), n = (idx % (BC / 4)) * 4;  // K chunk, first seed
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {  // seed n + x: its 4 K values, transposed
+        const float4 col = make_float4(comp(rb[i][0], x), comp(rb[i][1], x), comp(rb[i][2], x),
+                                       comp(rb[i][3], x));
+        const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+        // element (k, m) (m = output column): core (k/4, m/8) at
+        // ((k/4) * NM/8 + m/8) * 128, + (m%8) * 16 + (k%4) * 4
+        const int m = n + x;
+        *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + m / 8) * 128 + (m % 8) * 16) = hi;
+        *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + (BC + m) / 8) * 128 + (m % 8) * 16) = lo;
+      }
+    }
+  };
+
+  if (nkb > 0) load(0);
+  for (int kb = 0; kb < nkb; ++kb) {
+    const int st = kb % kTcStages;
+    if (kb >= kTcStages) mbar_wait(&bar[st], (uint32_t)((kb / kTcStages - 1) & 1));
+    store(st);
+    if (kb + 1 < nkb) load(kb + 1);  // next block in flight while this one multiplies
+    asm volatile("fence.proxy.async.shared::cta;");
+    __syncthreads();
+    if (tid == 0) {
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const uint32_t sa = smem_u32(tc_smem + st * STAGE), sb = sa + A_BYTES;
+#pragma unroll
+      for (int ks = 0; ks < kTcKB / 8; ++ks) {
+        const uint64_t da = umma_desc(sa + ks * 2 * A_LBO, A_LBO, 128);
+        const uint64_t db = umma_desc(sb + ks * 2 * B_LBO, B_LBO, 128);
+        const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(da), "l"(db), "r"(IDESC), "r"(acc));
+      }
+      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+          smem_u32(&bar[st])));
+    }
+  }
+  // all MMAs done -> accumulator readable
+  if (tid == 0) {
+    if (nkb > 0)
+      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+          smem_u32(&bar[kTcStages])));
+    else
+      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&bar[kTcStages])));
+  }
+  mbar_wait(&bar[kTcStages], 0);
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  // warp w reads TMEM lanes 32w..32w+31 = D rows; thread = one row
+  const int row = warp * 32 + lane;
+  float* out = z1_part + ((size_t)blockIdx.x * 128 + row) * Bp + seed0;
+#pragma unroll
+  for (int c = 0; c < BC; c += 16) {
+    uint32_t v[16], w[16];
+    const uint32_t ta = tmem + ((uint32_t)(warp * 32) << 16) + c;
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+          "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+          "=r"(v[14]), "=r"(v[15])
+        : "r"(ta));
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]),
+          "=r"(w[7]), "=r"(w[8]), "=r"(w[9]), "=r"(w[10]), "=r"(w[11]), "=r"(w[12]), "=r"(w[13]),
+          "=r"(w[14]), "=r"(w[15])
+        : "r"(ta + BC));
+    asm volatile("tcgen05.wait::ld.sync.aligned;");
+#pragma unroll
+    for (int x = 0; x < 16; x += 4)
+      *reinterpret_cast<float4*>(out + c + x) =
+          make_float4(__uint_as_float(v[x]) + __uint_as_float(w[x]),
+                      __uint_as_float(v[x + 1]) + __uint_as_float(w[x + 1]),
+                      __uint_as_float(v[x + 2]) + __uint_as_float(w[x + 2]),
+                      __uint_as_float(v[x + 3]) + __uint_as_float(w[x + 3]));
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+}
+
+// z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h
+__global__ void k_mlp_reduce(int Bp, int H1, int nsplit, const float* __restrict__ b1,
+                             const float* __restrict__ z1_part, float* __restrict__ z1) {
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= H1 * Bp) return;
+  const int h = idx / Bp, b = idx % Bp;
+  float acc = 0.f;
+  for (int c = 0; c < nsplit; ++c) {
+    const float* q = z1_part + (size_t)c * 128 * Bp;
+    acc += q[(size_t)h * Bp + b] + q[(size_t)(64 + h) * Bp + b];
+  }
+  z1[idx] = b1[h] + acc;
+}
+
+// Per seed: layers 2-3, f_mlp, and gz1 = d f_mlp / d z1.
+__global__ void k_mlp_head(int Bp, int H1, int H2, const float* __restrict__ z1g,
                            const float* __restrict__ W2, const float* __restrict__ b2,
                            const float* __restrict__ W3, const float* __restrict__ b3,
-                           const float* __restrict__ z1_part, double* __restrict__ f_mlp,
-                           float* __restrict__ gz1) {
+                           double* __restrict__ f_mlp, float* __restrict__ gz1) {
   const int b = blockIdx.x * blockDim.x + threadIdx.x;
   if (b >= Bp) return;
   float z1[kMlpMaxH1], z2[kMlpMaxH2];
-  for (int h = 0; h < H1; ++h) {
-    float acc = b1[h];
-    for (int sp = 0; sp < nsplit; ++sp) acc += z1_part[((size_t)sp * H1 + h) * Bp + b];
-    z1[h] = acc;
-  }
+  for (int h = 0; h < H1; ++h) z1[h] = z1g[(size_t)h * Bp + b];
   float y = b3[0];
   for (int h2 = 0; h2 < H2; ++h2) {
     float acc = b2[h2];
@@ -119,15 +306,33 @@ __global__ void __launch_bounds__(256) k_mlp_l1_back(int N, int Bp, int H1,
   }
 }
 
+int mlp_nsplit(int device) { return num_sms(device); }
+
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
                     const float* b1, const float* W2, const float* b2, const float* W3,
-                    const float* b3, const float* p, float* z1_part, double* f_mlp, float* gz1,
-                    int32_t nsplit) {
+                    const float* b3, const float* p, float* z1_part, float* z1, double* f_mlp,
+                    float* gz1, int32_t nsplit) {
   const int Bc = sh.Bp < 128 ? sh.Bp : 128;
-  k_mlp_l1<<<dim3(nsplit, sh.Bp / Bc), 256, 0, s>>>(sh.N, sh.Bp, H1, nsplit, W1, p, z1_part);
+  const dim3 grid(nsplit, sh.Bp / Bc);
+#define SM_L1(BCV)                                                                              \
+  do {                                                                                          \
+    constexpr int smem = kTcStages * (128 * kTcKB * 4 + kTcKB * 2 * BCV * 4) + 1024;            \
+    static bool attr = false;                                                                   \
+    if (!attr) {                                                                                \
+      SM_CUDA(cudaFuncSetAttribute(k_mlp_l1_tc<BCV>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                   smem));                                                      \
+      attr = true;                                                                              \
+    }                                                                                           \
+    k_mlp_l1_tc<BCV><<<grid, kTcThreads, smem, s>>>(sh.N, sh.Bp, H1, nsplit, W1, p, z1_part);   \
+  } while (0)
+  if (Bc == 128) SM_L1(128);
+  else if (Bc == 64) SM_L1(64);
+  else SM_L1(32);
+#undef SM_L1
   SM_LAUNCH_CHECK();
-  k_mlp_head<<<(sh.Bp + 127) / 128, 128, 0, s>>>(sh.Bp, H1, H2, nsplit, b1, W2, b2, W3, b3, z1_part,
-                                                 f_mlp, gz1);
+  k_mlp_reduce<<<(H1 * sh.Bp + 255) / 256, 256, 0, s>>>(sh.Bp, H1, nsplit, b1, z1_part, z1);
+  SM_LAUNCH_CHECK();
+  k_mlp_head<<<(sh.Bp + 127) / 128, 128, 0, s>>>(sh.Bp, H1, H2, z1, W2, b2, W3, b3, f_mlp, gz1);
   SM_LAUNCH_CHECK();
 }
 

@@ -106,7 +106,8 @@ struct smoothe_run {
   int32_t *q_ptr = nullptr, *q_nbr = nullptr;
   float* q_w = nullptr;
   float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr, *W3 = nullptr, *b3 = nullptr;
-  float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *gz1 = nullptr;
+  float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *z1 = nullptr,
+        *gz1 = nullptr;
   double* fmlp_s = nullptr;
   // debug outputs (set only during smoothe_debug_step)
   float *dbg_p = nullptr, *dbg_gth = nullptr, *dbg_gcp = nullptr;
@@ -226,7 +227,7 @@ void enqueue_step(smoothe_run* r) {
     launch_materialize_p_f(s, sh, g, r->u_f, r->cp, qK, r->p, r->f_part);
     launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0, r->red_scratch);
     launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
-                   r->z1_part, r->fextra, r->gz1, r->nsplit);
+                   r->z1_part, r->z1, r->fextra, r->gz1, r->nsplit);
     launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
     launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
   }
@@ -267,7 +268,7 @@ void enqueue_step(smoothe_run* r) {
   } else if (r->cost_kind == SMOOTHE_COST_MLP) {
     launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
     launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
-                   r->z1_part, r->dextra, nullptr, r->nsplit);
+                   r->z1_part, r->z1, r->dextra, nullptr, r->nsplit);
     dextra = r->dextra;
   }
 
@@ -410,8 +411,9 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     r->b2 = upload(o, std::vector<float>(cost->b2, cost->b2 + H2));
     r->W3 = upload(o, std::vector<float>(cost->W3, cost->W3 + H2));
     r->b3 = upload(o, std::vector<float>(cost->b3, cost->b3 + 1));
-    r->nsplit = std::max(1, std::min(2 * num_sms(r->device), (sh.N + 255) / 256));
-    r->z1_part = dalloc<float>(o, (size_t)r->nsplit * H1 * sh.Bp);
+    r->nsplit = mlp_nsplit(r->device);
+    r->z1_part = dalloc<float>(o, (size_t)r->nsplit * 128 * sh.Bp);
+    r->z1 = dalloc<float>(o, (size_t)H1 * sh.Bp);
     r->gz1 = dalloc<float>(o, (size_t)H1 * sh.Bp);
   }
 }
