@@ -2,14 +2,13 @@
 // reading S22: N -> 64 -> 8 -> 1) and its gradient.
 //
 // Layer 1 is the only large contraction: z1[h][b] = sum_k W1[h][k] p[k][b]
-// (2*H1*N*B flop, tensor cores below) and g_p[k][b] += sum_h W1[h][k] gz1[h][b]
-// (same, CUDA cores).  Split-K partial sums are reduced in a fixed order, so
+// (2*H1*N*B flop) and g_p[k][b] += sum_h W1[h][k] gz1[h][b] (same); both run
+// on the tensor cores.  Split-K partial sums are reduced in a fixed order, so
 // results are deterministic.
 #include "kcommon.cuh"
 
 namespace smoothe {
 
-constexpr int kMlpTK = 32;     // nodes per tile (CUDA-core backward)
 constexpr int kMlpMaxH1 = 64;
 constexpr int kMlpMaxH2 = 16;
 
@@ -279,31 +278,150 @@ __global__ void k_mlp_head(int Bp, int H1, int H2, const float* __restrict__ z1g
   }
 }
 
-// gp[k][b] = u[k] + sum_h W1[h][k] gz1[h][b]
-__global__ void __launch_bounds__(256) k_mlp_l1_back(int N, int Bp, int H1,
-                                                     const float* __restrict__ W1,
-                                                     const float* __restrict__ u,
-                                                     const float* __restrict__ gz1,
-                                                     float* __restrict__ gp) {
-  __shared__ float sG[kMlpMaxH1][128];
-  __shared__ float sW[kMlpMaxH1][kMlpTK + 1];
-  const int Bc = Bp < 128 ? Bp : 128;
-  const int seed0 = blockIdx.y * Bc;
-  for (int idx = threadIdx.x; idx < H1 * Bc; idx += 256)
-    sG[idx / Bc][idx % Bc] = gz1[(size_t)(idx / Bc) * Bp + seed0 + idx % Bc];
-  const int kt = blockIdx.x * kMlpTK;
-  const int nk = min(kMlpTK, N - kt);
-  for (int idx = threadIdx.x; idx < H1 * kMlpTK; idx += 256) {
-    const int h = idx / kMlpTK, kk = idx % kMlpTK;
-    sW[h][kk] = kk < nk ? W1[(size_t)h * N + kt + kk] : 0.f;
+// ---------------------------------------------------------------------------
+// Backward of layer 1 on the tensor cores: g_p[k][b] = u[k] + sum_h W1[h][k] gz1[h][b].
+// One CTA per tile of 128 e-nodes (M) and seed chunk: A = W1^T tile (128 x H1,
+// staged K-major: 4 x 4 blocks transposed in registers) split hi / lo into two
+// tiles, B = [gz1_hi | gz1_lo] (H1 x 2Bc, K-major), two MMAs per K step:
+//   D = A_hi B + A_lo B,   g_p = u + D[m][b] + D[m][Bc + b].
+// ---------------------------------------------------------------------------
+template <int BC>
+__global__ void __launch_bounds__(kTcThreads) k_mlp_l1_back_tc(int N, int Bp, int H1,
+                                                              const float* __restrict__ W1,
+                                                              const float* __restrict__ u,
+                                                              const float* __restrict__ gz1,
+                                                              float* __restrict__ gp) {
+  constexpr int NM = 2 * BC;
+  constexpr int KH = kMlpMaxH1;                 // K = 64 (H1 padded with zeros)
+  constexpr int A_BYTES = 128 * KH * 4;         // one of A_hi / A_lo
+  constexpr int A_LBO = 16 * 128;               // K chunk stride (16 row groups of 8)
+  constexpr int B_LBO = (NM / 8) * 128;
+  constexpr uint32_t TMEM_COLS = NM <= 32 ? 32 : NM <= 64 ? 64 : NM <= 128 ? 128 : 256;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
+                             ((uint32_t)(128 >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t tc_smem[];
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tmem_base_sh;
+  uint8_t* sAh = tc_smem;
+  uint8_t* sAl = tc_smem + A_BYTES;
+  uint8_t* sB = tc_smem + 2 * A_BYTES;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int k0 = blockIdx.x * 128, seed0 = blockIdx.y * BC;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&tmem_base_sh)),
+                 "n"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
+  if (tid == 0) {
+    mbar_init(&bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  // A: node m, hidden h -> core (h/4, m/8) at ((h/4) * 16 + m/8) * 128 + (m%8) * 16 + (h%4) * 4
+  for (int blk = tid; blk < (KH / 4) * (128 / 4); blk += kTcThreads) {
+    const int hc = blk / 32, m0 = (blk % 32) * 4;  // 4 hidden units x 4 nodes
+    float4 r[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int h = hc * 4 + i;
+      const float* src = W1 + (size_t)h * N + k0 + m0;
+      if (h < H1 && k0 + m0 + 3 < N && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+        r[i] = __ldcs(reinterpret_cast<const float4*>(src));
+      } else {
+        float t[4];
+#pragma unroll
+        for (int x = 0; x < 4; ++x) t[x] = h < H1 && k0 + m0 + x < N ? src[x] : 0.f;
+        r[i] = make_float4(t[0], t[1], t[2], t[3]);
+      }
+    }
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const int m = m0 + x;
+      const float4 col = make_float4(comp(r[0], x), comp(r[1], x), comp(r[2], x), comp(r[3], x));
+      const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+      const int off = (hc * 16 + m / 8) * 128 + (m % 8) * 16;
+      *reinterpret_cast<float4*>(sAh + off) = hi;
+      *reinterpret_cast<float4*>(sAl + off) = lo;
+    }
+  }
+  // B: hidden h (K), column c (N) -> core (h/4, c/8) at ((h/4) * NM/8 + c/8) * 128 + (c%8) * 16 + (h%4) * 4
+  for (int blk = tid; blk < (KH / 4) * (BC / 4); blk += kTcThreads) {
+    const int hc = blk / (BC / 4), n0 = (blk % (BC / 4)) * 4;
+    float4 r[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int h = hc * 4 + i;
+      r[i] = h < H1 ? *reinterpret_cast<const float4*>(gz1 + (size_t)h * Bp + seed0 + n0)
+                    : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const int c = n0 + x;
+      const float4 col = make_float4(comp(r[0], x), comp(r[1], x), comp(r[2], x), comp(r[3], x));
+      const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+      *reinterpret_cast<float4*>(sB + (hc * (NM / 8) + c / 8) * 128 + (c % 8) * 16) = hi;
+      *reinterpret_cast<float4*>(sB + (hc * (NM / 8) + (BC + c) / 8) * 128 + (c % 8) * 16) = lo;
+    }
+  }
+  asm volatile("fence.proxy.async.shared::cta;");
+  asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  for (int idx = threadIdx.x; idx < nk * Bc; idx += 256) {
-    const int kk = idx / Bc, b = idx % Bc;
-    float acc = u[kt + kk];
-    for (int h = 0; h < H1; ++h) acc += sW[h][kk] * sG[h][b];
-    gp[(size_t)(kt + kk) * Bp + seed0 + b] = acc;
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem = tmem_base_sh;
+  if (tid == 0) {
+    const uint32_t ah = smem_u32(sAh), al = smem_u32(sAl), bb = smem_u32(sB);
+#pragma unroll
+    for (int ks = 0; ks < KH / 8; ++ks) {
+      const uint64_t db = umma_desc(bb + ks * 2 * B_LBO, B_LBO, 128);
+#pragma unroll
+      for (int part = 0; part < 2; ++part) {
+        const uint64_t da = umma_desc((part ? al : ah) + ks * 2 * A_LBO, A_LBO, 128);
+        const uint32_t acc = (ks > 0 || part > 0) ? 1u : 0u;
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(da), "l"(db), "r"(IDESC), "r"(acc));
+      }
+    }
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+        smem_u32(&bar)));
   }
+  mbar_wait(&bar, 0);
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const int m = warp * 32 + lane, k = k0 + m;
+  const float uk = k < N ? __ldg(u + k) : 0.f;
+  float* out = gp + (size_t)k * Bp + seed0;
+#pragma unroll
+  for (int c = 0; c < BC; c += 16) {
+    uint32_t v[16], w[16];
+    const uint32_t ta = tmem + ((uint32_t)(warp * 32) << 16) + c;
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+          "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+          "=r"(v[14]), "=r"(v[15])
+        : "r"(ta));
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]),
+          "=r"(w[7]), "=r"(w[8]), "=r"(w[9]), "=r"(w[10]), "=r"(w[11]), "=r"(w[12]), "=r"(w[13]),
+          "=r"(w[14]), "=r"(w[15])
+        : "r"(ta + BC));
+    asm volatile("tcgen05.wait::ld.sync.aligned;");
+    if (k < N) {
+#pragma unroll
+      for (int x = 0; x < 16; x += 4)
+        __stcs(reinterpret_cast<float4*>(out + c + x),
+               make_float4(uk + (__uint_as_float(v[x]) + __uint_as_float(w[x])),
+                           uk + (__uint_as_float(v[x + 1]) + __uint_as_float(w[x + 1])),
+                           uk + (__uint_as_float(v[x + 2]) + __uint_as_float(w[x + 2])),
+                           uk + (__uint_as_float(v[x + 3]) + __uint_as_float(w[x + 3]))));
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
 }
 
 int mlp_nsplit(int device) { return num_sms(device); }
@@ -339,8 +457,22 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
 void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* u,
                     const float* gz1, float* gp) {
   const int Bc = sh.Bp < 128 ? sh.Bp : 128;
-  k_mlp_l1_back<<<dim3((sh.N + kMlpTK - 1) / kMlpTK, sh.Bp / Bc), 256, 0, s>>>(sh.N, sh.Bp, H1, W1,
-                                                                              u, gz1, gp);
+  const dim3 grid((sh.N + 127) / 128, sh.Bp / Bc);
+#define SM_L1B(BCV)                                                                              \
+  do {                                                                                           \
+    constexpr int smem = 2 * 128 * kMlpMaxH1 * 4 + kMlpMaxH1 * 2 * BCV * 4 + 1024;               \
+    static bool attr = false;                                                                    \
+    if (!attr) {                                                                                 \
+      SM_CUDA(cudaFuncSetAttribute(k_mlp_l1_back_tc<BCV>,                                        \
+                                   cudaFuncAttributeMaxDynamicSharedMemorySize, smem));          \
+      attr = true;                                                                               \
+    }                                                                                            \
+    k_mlp_l1_back_tc<BCV><<<grid, kTcThreads, smem, s>>>(sh.N, sh.Bp, H1, W1, u, gz1, gp);        \
+  } while (0)
+  if (Bc == 128) SM_L1B(128);
+  else if (Bc == 64) SM_L1B(64);
+  else SM_L1B(32);
+#undef SM_L1B
   SM_LAUNCH_CHECK();
 }
 
