@@ -183,8 +183,8 @@ void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const
                  const double* fextra, const double* h, double* ftot, double* loss);
 // reached sets and validity masks (kernels_decode.cu); valid_out[W]
 void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
-                   const uint32_t* sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out,
-                   int32_t grid);
+                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* invalid,
+                   uint32_t* valid_out, int32_t grid);
 void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g,
                                const double* u, const int32_t* choice, const uint32_t* reach,
                                double* cost_part);

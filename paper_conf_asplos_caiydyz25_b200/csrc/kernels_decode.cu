@@ -28,19 +28,20 @@ namespace smoothe {
 //  * a class in a trivial component has all its parents at lower levels, so
 //    reach_j = OR_{k in pa_j} (reach_{ec(k)} AND sel_k) is final in one pass
 //    (one warp per (class, 32-seed word), lanes over the parents);
-//  * a non-trivial SCC (one warp per (SCC, word)) ORs in its external parents
-//    once, then iterates its internal edges to the local fixpoint in shared
-//    memory (|S| <= 64);
+//  * a non-trivial SCC S (|S| <= 64) is one block job per (SCC, word): its
+//    classes' external reach comes from phase A; then, per seed (lane), the
+//    chosen e-node of each class of S gives a 64-bit mask of its children
+//    inside S, and the local reach closure R and settle closure
+//    settle_j = !reach_j OR (children of c_j in S all settled) run in
+//    registers on those masks;
 //  * every cycle of a selection lies inside one SCC, so the selection is valid
-//    iff, in every SCC, the reached classes settle bottom-up within the SCC:
-//    settle_j = !reach_j OR OR_{k in m_j} (sel_k AND AND_{c in ch_k cap S} settle_c).
-//    Unsettled reached classes mark their seeds invalid (bit-OR atomics:
-//    order-independent, deterministic).
-// One grid barrier per level; each class is evaluated once per level pass.
+//    iff, in every SCC, every reached class settles.  Unsettled reached classes
+//    mark their seeds invalid (bit-OR atomics: order-independent, deterministic).
+// One grid barrier per phase and level; each class is evaluated once per level.
+// (The previous per-warp version walked every e-node of every class of S in
+// each fixpoint pass: on C5, with 900-node classes, the slowest SCC set the
+// pace of every level, 3.6 ms per decode.)
 constexpr int kDecodeWarps = 8;
-constexpr int kDecodeMaxEnt = 192;    // intra-SCC edge entries cached in shared memory
-constexpr int kDecodeMaxNodes = 384;  // SCC e-nodes staged in shared memory
-constexpr int kDecodeMaxChild = 512;  // their internal child entries
 
 __global__ void __launch_bounds__(256) k_decode_levels(
     int W, int root, int num_levels, const int32_t* __restrict__ lvl_cptr,
@@ -54,13 +55,10 @@ __global__ void __launch_bounds__(256) k_decode_levels(
     const int32_t* __restrict__ ent_node, const int32_t* __restrict__ node_slot,
     const int32_t* __restrict__ slot_ptr, const int32_t* __restrict__ slot_node,
     const int32_t* __restrict__ slot_jptr, const int32_t* __restrict__ slot_jloc,
-    const uint32_t* __restrict__ sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out) {
-  __shared__ uint32_t rs[kDecodeWarps][64];            // reach words of the SCC's classes
-  __shared__ uint32_t st[kDecodeWarps][64];            // settle words
-  __shared__ uint32_t es[kDecodeWarps][kDecodeMaxEnt]; // OR of sel over each intra-SCC entry
-  __shared__ uint32_t qs[kDecodeWarps][kDecodeMaxNodes];     // sel word of each SCC e-node
-  __shared__ uint16_t qp[kDecodeWarps][kDecodeMaxNodes + 1]; // its internal children: offsets
-  __shared__ uint8_t qc[kDecodeWarps][kDecodeMaxChild];      //   ... and local class ids
+    const uint32_t* __restrict__ sel, int Bp, const int32_t* __restrict__ choice, uint32_t* reach,
+    uint32_t* invalid, uint32_t* valid_out) {
+  __shared__ uint64_t cm[64][32];  // phase B: children in S of the chosen e-node, per (class, seed)
+  __shared__ uint32_t rs0[64];     // phase B: reach words after phase A
   cg::grid_group grid = cg::this_grid();
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -77,110 +75,69 @@ __global__ void __launch_bounds__(256) k_decode_levels(
       if (j == root) continue;
       const int sj = scc_of_class[j];
       uint32_t v = 0;
-      for (int e = par_ptr[j] + lane; e < par_ptr[j + 1]; e += 32) {
-        const int pc = par_class[e];
-        if (sj < 0 || scc_of_class[pc] != sj)
-          v |= __ldcg(reach + (size_t)pc * W + w) & sel[(size_t)par_node[e] * W + w];
+      const int e1 = par_ptr[j + 1];
+      for (int e = par_ptr[j] + lane; e < e1; e += 4 * 32) {  // 4 parents per lane in flight
+        int pc[4], pn[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int eu = e + 32 * u;
+          pc[u] = eu < e1 ? par_class[eu] : -1;
+          pn[u] = eu < e1 ? par_node[eu] : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (pc[u] >= 0 && (sj < 0 || scc_of_class[pc[u]] != sj))
+            v |= __ldcg(reach + (size_t)pc[u] * W + w) & sel[(size_t)pn[u] * W + w];
       }
       v = __reduce_or_sync(0xffffffffu, v);
       if (lane == 0) __stcg(reach + (size_t)j * W + w, v);
     }
     const int s0l = lvl_sptr[L];
     const int64_t nB = (int64_t)(lvl_sptr[L + 1] - s0l) * W;
-    if (nB == 0) {
-      grid.sync();
-      continue;
-    }
     grid.sync();
-    // phase B: non-trivial SCCs, one warp per (SCC, word): internal edges to
-    // the local reach fixpoint, then the local settle (acyclicity) check
-    for (int64_t it = gwarp; it < nB; it += nwarps) {
+    if (nB == 0) continue;
+    // phase B: non-trivial SCCs, one block per (SCC, word)
+    for (int64_t it = blockIdx.x; it < nB; it += gridDim.x) {
       const int s = lvl_scc[s0l + it / W];
       const int w = (int)(it % W);
       const int c0 = scc_class_ptr[s], n = scc_class_ptr[s + 1] - c0;
-      for (int l = lane; l < n; l += 32) {
+      for (int l = wib; l < n; l += kDecodeWarps) {
         const int j = scc_class[c0 + l];
-        rs[wib][l] = j == root ? 0xffffffffu : __ldcg(reach + (size_t)j * W + w);
+        const int c = choice[(size_t)j * Bp + 32 * w + lane];
+        const int q = node_slot[c];
+        uint64_t m = 0;
+        if (q >= 0)
+          for (int e = slot_jptr[q]; e < slot_jptr[q + 1]; ++e) m |= 1ull << slot_jloc[e];
+        cm[l][lane] = m;
+        if (lane == 0) rs0[l] = j == root ? 0xffffffffu : __ldcg(reach + (size_t)j * W + w);
       }
-      const int e0 = ent_ptr[s], ne = ent_ptr[s + 1] - e0;
-      for (int e = lane; e < ne && e < kDecodeMaxEnt; e += 32) {
-        uint32_t m = 0;
-        for (int a = ent_node_ptr[e0 + e]; a < ent_node_ptr[e0 + e + 1]; ++a)
-          m |= sel[(size_t)ent_node[a] * W + w];
-        es[wib][e] = m;
-      }
-      __syncwarp();
-      bool changed = true;
-      while (__any_sync(0xffffffffu, changed)) {  // r_j |= r_i & sel(i -> j), monotone
-        changed = false;
-        for (int e = lane; e < ne; e += 32) {
-          uint32_t m;
-          if (e < kDecodeMaxEnt) {
-            m = es[wib][e];
-          } else {
-            m = 0;
-            for (int a = ent_node_ptr[e0 + e]; a < ent_node_ptr[e0 + e + 1]; ++a)
-              m |= sel[(size_t)ent_node[a] * W + w];
-          }
-          const int ji = ent_j[e0 + e];
-          const uint32_t add = rs[wib][ent_i[e0 + e]] & m & ~rs[wib][ji];
-          if (add) {
-            atomicOr(&rs[wib][ji], add);
-            changed = true;
-          }
+      __syncthreads();
+      if (wib == 0) {
+        uint64_t R = 0;
+        for (int l = 0; l < n; ++l)
+          if ((rs0[l] >> lane) & 1u) R |= 1ull << l;
+        for (;;) {  // reach closure inside S for this seed
+          const uint64_t o = R;
+          for (int l = 0; l < n; ++l)
+            if ((R >> l) & 1ull) R |= cm[l][lane];
+          if (R == o) break;
         }
-        __syncwarp();
-      }
-      for (int l = lane; l < n; l += 32) {
-        __stcg(reach + (size_t)scc_class[c0 + l] * W + w, rs[wib][l]);
-        st[wib][l] = ~rs[wib][l];  // unreached classes count as settled
-      }
-      // stage the SCC's e-nodes (selection word, internal children) in shared
-      // memory when they fit, so the settle passes touch no global memory
-      const int q_begin = slot_ptr[s], nq = slot_ptr[s + 1] - q_begin;
-      const int ch_begin = slot_jptr[q_begin], nch = slot_jptr[q_begin + nq] - ch_begin;
-      const bool staged = nq <= kDecodeMaxNodes && nch <= kDecodeMaxChild;
-      if (staged) {
-        for (int q = lane; q < nq; q += 32) {
-          qs[wib][q] = sel[(size_t)slot_node[q_begin + q] * W + w];
-          qp[wib][q + 1] = (uint16_t)(slot_jptr[q_begin + q + 1] - ch_begin);
+        const uint64_t all = n == 64 ? ~0ull : (1ull << n) - 1ull;
+        uint64_t S = ~R & all;
+        for (;;) {  // settle closure: a reached class settles once its children in S have
+          const uint64_t o = S;
+          for (int l = 0; l < n; ++l)
+            if (!((S >> l) & 1ull) && (cm[l][lane] & ~S) == 0) S |= 1ull << l;
+          if (S == o) break;
         }
-        if (lane == 0) qp[wib][0] = 0;
-        for (int e = lane; e < nch; e += 32) qc[wib][e] = (uint8_t)slot_jloc[ch_begin + e];
-      }
-      __syncwarp();
-      changed = true;
-      while (__any_sync(0xffffffffu, changed)) {  // local settle fixpoint (monotone)
-        changed = false;
-        for (int l = lane; l < n; l += 32) {
-          const int j = scc_class[c0 + l];
-          uint32_t v = st[wib][l];
-          const int q0 = node_slot[class_ptr[j]] - q_begin, nk = class_ptr[j + 1] - class_ptr[j];
-          for (int t = 0; t < nk && v != 0xffffffffu; ++t) {
-            const int q = q0 + t;
-            uint32_t acc;
-            if (staged) {
-              acc = qs[wib][q] & ~v;
-              for (int e = qp[wib][q]; acc && e < qp[wib][q + 1]; ++e) acc &= st[wib][qc[wib][e]];
-            } else {
-              acc = sel[(size_t)slot_node[q_begin + q] * W + w] & ~v;
-              for (int e = slot_jptr[q_begin + q]; acc && e < slot_jptr[q_begin + q + 1]; ++e)
-                acc &= st[wib][slot_jloc[e]];
-            }
-            v |= acc;
-          }
-          if (v != st[wib][l]) {
-            st[wib][l] = v;
-            changed = true;
-          }
+        for (int l = 0; l < n; ++l) {
+          const uint32_t word = __ballot_sync(0xffffffffu, (R >> l) & 1ull);
+          if (lane == 0) __stcg(reach + (size_t)scc_class[c0 + l] * W + w, word);
         }
-        __syncwarp();
+        const uint32_t bad = __ballot_sync(0xffffffffu, (R & ~S) != 0);
+        if (lane == 0 && bad) atomicOr(invalid + w, bad);
       }
-      uint32_t bad = 0;
-      for (int l = lane; l < n; l += 32) bad |= rs[wib][l] & ~st[wib][l];
-      bad = __reduce_or_sync(0xffffffffu, bad);
-      if (lane == 0 && bad) atomicOr(invalid + w, bad);
-      __syncwarp();
+      __syncthreads();
     }
     grid.sync();
   }
@@ -194,12 +151,12 @@ static void coop_launch(const void* fn, int grid, void** args, cudaStream_t s) {
 }
 
 void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
-                   const uint32_t* sel, uint32_t* reach, uint32_t* invalid, uint32_t* valid_out,
-                   int32_t grid) {
+                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* invalid,
+                   uint32_t* valid_out, int32_t grid) {
   SM_CUDA(cudaMemsetAsync(invalid, 0, sizeof(uint32_t) * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach + (size_t)sh.root * sh.W, 0xff, sizeof(uint32_t) * sh.W, s));
-  int W = sh.W, root = sh.root, L = hg.num_levels;
+  int W = sh.W, root = sh.root, L = hg.num_levels, Bp = sh.Bp;
   void* args[] = {&W, &root, &L, (void*)&g.lvl_cptr, (void*)&g.lvl_class, (void*)&g.lvl_sptr,
                   (void*)&g.lvl_scc, (void*)&g.par_ptr,
                   (void*)&g.par_node, (void*)&g.par_class, (void*)&g.class_ptr,
@@ -207,7 +164,8 @@ void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const D
                   (void*)&g.ent_ptr, (void*)&g.ent_i, (void*)&g.ent_j, (void*)&g.ent_node_ptr,
                   (void*)&g.ent_node, (void*)&g.node_slot, (void*)&g.slot_ptr,
                   (void*)&g.slot_node, (void*)&g.slot_jptr,
-                  (void*)&g.slot_jloc, (void*)&sel, &reach, &invalid, &valid_out};
+                  (void*)&g.slot_jloc, (void*)&sel, &Bp, (void*)&choice, &reach, &invalid,
+                  &valid_out};
   coop_launch((const void*)k_decode_levels, grid, args, s);
 }
 

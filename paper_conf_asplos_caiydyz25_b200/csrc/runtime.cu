@@ -255,7 +255,7 @@ void enqueue_step(smoothe_run* r) {
                 r->debug ? r->dbg_gcp : nullptr);
 
   pm.mark(SMOOTHE_PHASE_DECODE);
-  launch_decode(s, sh, hg, g, r->sel, r->reach, r->invalid, r->settle + (size_t)sh.root * sh.W,
+  launch_decode(s, sh, hg, g, r->sel, r->choice, r->reach, r->invalid, r->settle + (size_t)sh.root * sh.W,
                 r->coop_grid);
   launch_decode_cost_linear(s, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
   launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost, r->red_scratch);
