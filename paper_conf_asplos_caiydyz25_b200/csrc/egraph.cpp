@@ -339,6 +339,29 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
+  // dmin_j: BFS depth of class j from the root over class -> child-class
+  // edges (unreachable: INT32_MAX).  q^t_j is exactly 0 for t < dmin_j (q^0 =
+  // e_root and each sweep extends the support by one edge), so the sweeps skip
+  // such classes (activity windows).
+  g.dmin.assign(M, INT32_MAX);
+  {
+    std::vector<int32_t> frontier{root}, next;
+    g.dmin[root] = 0;
+    for (int32_t d = 1; !frontier.empty(); ++d) {
+      next.clear();
+      for (int32_t j : frontier)
+        for (int32_t k = g.class_ptr[j]; k < g.class_ptr[j + 1]; ++k)
+          for (int32_t e = g.child_ptr[k]; e < g.child_ptr[k + 1]; ++e) {
+            const int32_t c = g.child_class[e];
+            if (g.dmin[c] == INT32_MAX) {
+              g.dmin[c] = d;
+              next.push_back(c);
+            }
+          }
+      frontier.swap(next);
+    }
+  }
+
   g.big_class.clear();
   for (int32_t j = 0; j < M; ++j)
     if (g.class_ptr[j + 1] - g.class_ptr[j] > kBigClass) g.big_class.push_back(j);
@@ -366,7 +389,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     auto emit = [&](int32_t b0, int32_t b1, int32_t piece) {
       const int32_t k0 = b0 < b1 ? g.pad_batch_node[b0] : -1;
       const int32_t k1 = b0 < b1 ? g.pad_batch_node[b1 - 1] : -1;
-      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece, k0, k1, 0, 0});
+      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece, k0, k1, g.dmin[j], 0});
     };
     if (cb1 - cb0 <= kRevChunk) {
       emit(cb0, cb1, 0);

@@ -83,8 +83,9 @@ struct HostGraph {
   // classes with more than kBigClass e-nodes, largest first: the per-class
   // kernels (softmax, cost, update) give each a whole block
   std::vector<int32_t> big_class;
+  std::vector<int32_t> dmin;  // [M] BFS depth from the root (INT32_MAX: unreachable)
   // Reverse-sweep work items, [n][8] = (class j, first batch, end batch, info,
-  // first e-node, last e-node, 0, 0): a class's batches split into runs of <= rev_chunk cut at
+  // first e-node, last e-node, dmin_j, 0): a class's batches split into runs of <= rev_chunk cut at
   // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
   // info = -1: the class's only item; else (slot << 1) | piece, slot = its
   // partial-sum row (the class's last item to finish combines them in order).
@@ -113,6 +114,7 @@ struct DevGraph {
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t *pad_batch_node = nullptr;
   int32_t* big_class = nullptr;
+  int32_t* dmin = nullptr;
   int32_t num_big = 0;
   int32_t *rev_item = nullptr, *rev_class_item_ptr = nullptr;
   int32_t num_rev_items = 0, rev_num_slots = 0;
@@ -148,7 +150,8 @@ void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t se
                        float* theta, float* m, float* v);
 void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
                            float* cp, int32_t* choice, uint32_t* sel);
-void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+// t: sweep index (classes with dmin > t are skipped: their q^t is exactly 0)
+void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const float* cp, const float* q_prev, float* q, float* pi, int32_t* am);
 void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
                         const float* cp, const float* qK, float* gcp, float* gqK, float* f_part,
@@ -166,7 +169,10 @@ void launch_reduce_rows_f64(cudaStream_t s, const float* part, int32_t nrows, in
                             double* out, double scale, double* scratch);
 void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, int32_t Bp,
                              double* out, double* scratch);
-void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+// t: sweep index (items of classes with dmin > t - 1 are skipped: q^{t-1} = 0
+// there, so they contribute nothing to g_cp and no active class reads their
+// g_q^{t-1})
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
                           float* rev_part, int32_t* rev_cnt);

@@ -33,12 +33,12 @@ constexpr int kSweepBlock = 64;
 // ---------------------------------------------------------------------------
 template <int LPR>
 __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
-    int M, int Bp, int root, const int32_t* __restrict__ pad_par_ptr,
-    const int32_t* __restrict__ pad_par, float wI, float wC, const float* __restrict__ cp,
-    const float* __restrict__ q_prev, float* __restrict__ q, float* __restrict__ pi,
-    int32_t* __restrict__ am) {
+    int M, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,
+    float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
+    float* __restrict__ q, float* __restrict__ pi, int32_t* __restrict__ am) {
   const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
-  if (j >= M || j == root) return;
+  if (j >= M || j == root || __ldg(dmin + j) > t) return;  // q^t_j = 0 (rows stay zero)
   const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
   // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
   // row N of cp, so p = 0: factor 1 and never a new max
@@ -93,11 +93,12 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   stcs4i(am + o, arg);
 }
 
-void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
   SM_DISPATCH_LPR(sh.Bp, {
     k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi, am);
+        sh.M, sh.Bp, sh.root, t, g.dmin, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi,
+        am);
   });
   SM_LAUNCH_CHECK();
 }
@@ -254,11 +255,12 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
-    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch) {
+    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t) {
   const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
   const int4 c0 = items[2 * it], c1 = items[2 * it + 1];
+  if (c1.z > t - 1) return;  // q^{t-1}_{j'} = 0: nothing to add, g_q^{t-1}_{j'} never read
   const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
   const bool piece = info >= 0 && (info & 1);
   const int s0 = blockIdx.y * (32 * V) + lane * V;
@@ -366,7 +368,7 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
                           cp, gcp, gq_prev, part, cnt);
 }
 
-void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const float* cp, const float* q_prev, const float* gq, const float* pi,
                           const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
                           float* rev_part, int32_t* rev_cnt) {
@@ -381,7 +383,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out, rev_part,   \
-      rev_cnt, l2_prefetch)
+      rev_cnt, l2_prefetch, t)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \

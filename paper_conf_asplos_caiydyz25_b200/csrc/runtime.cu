@@ -206,7 +206,7 @@ void enqueue_step(smoothe_run* r) {
 
   pm.mark(SMOOTHE_PHASE_FORWARD);
   for (int t = 1; t <= K; ++t)
-    launch_sweep_forward(s, sh, g, r->agg, r->cp, r->qstack + (size_t)(t - 1) * MB,
+    launch_sweep_forward(s, sh, g, r->agg, t, r->cp, r->qstack + (size_t)(t - 1) * MB,
                          r->qstack + (size_t)t * MB,
                          r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
                          r->astack + (size_t)(t - 1) * MB);
@@ -243,7 +243,7 @@ void enqueue_step(smoothe_run* r) {
 
   pm.mark(SMOOTHE_PHASE_REVERSE);
   for (int t = K; t >= 1; --t)
-    launch_sweep_reverse(s, sh, g, r->agg, r->cp, r->qstack + (size_t)(t - 1) * MB, r->gq[t & 1],
+    launch_sweep_reverse(s, sh, g, r->agg, t, r->cp, r->qstack + (size_t)(t - 1) * MB, r->gq[t & 1],
                          r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
                          r->astack + (size_t)(t - 1) * MB, r->gcp, r->gq[(t - 1) & 1], t > 1,
                          r->rev_part, r->rev_cnt);
@@ -524,6 +524,7 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_par = upload(o, h.pad_par, &b);
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
       d.big_class = upload(o, h.big_class, &b);
+      d.dmin = upload(o, h.dmin, &b);
       d.num_big = (int32_t)h.big_class.size();
       d.rev_item = upload(o, h.rev_item, &b);
       d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
@@ -835,9 +836,20 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       for (int j = 0; j < sh.M; ++j)
         for (int b = 0; b < sh.B; ++b)
           dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
-    if (dump->route) {  // the root row is not a decision (q_root = 1, S3)
+    if (dump->route) {
+      // The root row is not a decision (q_root = 1, S3).  Rows the forward
+      // sweep skipped (t < dmin_j: every p is exactly 0, so every parent ties)
+      // report the lowest-id parent, the kernel's tie rule (S7).
+      const HostGraph& hg = run->g->host;
       for (int t = 0; t < run->K; ++t)
-        for (int b = 0; b < sh.B; ++b) dump->route[((size_t)t * sh.M + sh.root) * sh.B + b] = -1;
+        for (int j = 0; j < sh.M; ++j) {
+          int32_t* row = dump->route + ((size_t)t * sh.M + j) * sh.B;
+          if (j == sh.root) {
+            for (int b = 0; b < sh.B; ++b) row[b] = -1;
+          } else if (hg.dmin[j] > t + 1 && hg.par_ptr[j + 1] > hg.par_ptr[j]) {
+            for (int b = 0; b < sh.B; ++b) row[b] = hg.par_node[hg.par_ptr[j]];
+          }
+        }
     }
     if ((size_t)run->steps_run < run->ev_step.size())
       SM_CUDA(cudaEventRecord(run->ev_step[run->steps_run], s));
