@@ -55,6 +55,37 @@ def byte_model(N, M, K, Bl):
             "step": 52 + 12 * r + K * (16 + 20 * r)}
 
 
+def active_fractions(eg, K):
+    """Mean fraction of e-nodes / classes the sweeps touch (activity windows:
+    a class with BFS depth dmin > t from the root has q^t = 0 and is skipped by
+    forward sweep t and, with dmin > t - 1, by reverse sweep t)."""
+    M, N = eg.num_classes, eg.num_nodes
+    ec = eg.ec()
+    src = ec[np.repeat(np.arange(N), np.diff(eg.child_ptr))]
+    order = np.argsort(src, kind="stable")
+    ptr = np.searchsorted(src[order], np.arange(M + 1))
+    dst = np.asarray(eg.child_class)[order]
+    dmin = np.full(M, np.iinfo(np.int64).max)
+    dmin[eg.root] = 0
+    frontier, d = np.array([eg.root]), 0
+    while frontier.size:
+        d += 1
+        nxt = np.unique(np.concatenate([dst[ptr[j]:ptr[j + 1]] for j in frontier]))
+        nxt = nxt[dmin[nxt] > d]
+        dmin[nxt] = d
+        frontier = nxt
+    sizes = np.diff(eg.class_ptr)
+    out = {}
+    for name, lag in (("forward", 0), ("reverse", 1)):
+        nodes = classes = 0.0
+        for t in range(1, K + 1):
+            act = dmin <= t - lag
+            nodes += sizes[act].sum() / N
+            classes += act.sum() / M
+        out[name] = (nodes / K, classes / K)
+    return out
+
+
 class ClockSampler:
     """nvidia-smi clocks + throttle reasons during the timed region."""
 
@@ -250,7 +281,11 @@ def run_ours(args):
     dom = max(("forward", "reverse"), key=lambda k: ph[k])
     per_launch_ms = ph[dom] / max(1, prof["phase_launches"][dom])
     units_launch = Bl * N
-    alg = bm["forward_sweep" if dom == "forward" else "reverse_sweep"] * units_launch
+    # algorithmic bytes of the rows a launch touches (activity windows), on
+    # average over the K launches: per e-node and per class terms of the model
+    fn, fc = active_fractions(eg, K)[dom]
+    per_node, per_class = (4.0, 8.0) if dom == "forward" else (12.0, 12.0)
+    alg = Bl * (per_node * N * fn + per_class * M * fc)
     peak, peak_src = measured_peaks()
     achieved = alg / (per_launch_ms * 1e-3) / 1e9
     traffic = ncu_traffic(args.config, dom)
@@ -260,6 +295,7 @@ def run_ours(args):
             "frac": achieved / peak, "traffic": traffic, "kernel": f"k_sweep_{dom}",
             "alg_bytes_per_unit": bm["forward_sweep" if dom == "forward" else "reverse_sweep"],
             "units_per_launch": units_launch, "avg_launch_ms": per_launch_ms,
+            "alg_bytes_per_launch": alg, "active_node_frac": fn, "active_class_frac": fc,
             "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
             "step_alg_GBps": bm["step"] * Bl * N / (step_ms * 1e-3) / 1e9}
 
