@@ -33,8 +33,15 @@ constexpr int kMlpMaxH2 = 16;
 // lanes back at the end: z1_part[cta][128][Bp] (rows 64.. hold the W1_lo
 // products), reduced in a fixed order by k_mlp_reduce.
 // ---------------------------------------------------------------------------
-constexpr int kTcKB = 32;       // e-nodes (K) per stage
-constexpr int kTcStages = 3;
+#ifndef SMOOTHE_TC_KB
+#define SMOOTHE_TC_KB 64
+#endif
+constexpr int kTcKB = SMOOTHE_TC_KB;  // e-nodes (K) per stage (16 float4 loads in flight per thread)
+template <int BC>
+#ifndef SMOOTHE_TC_S128
+#define SMOOTHE_TC_S128 2
+#endif
+__host__ __device__ constexpr int tc_stages() { return BC >= 128 ? SMOOTHE_TC_S128 : 3; }  // <= 192 KB of shared memory
 constexpr int kTcThreads = 128;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -83,6 +90,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
   constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
                              ((uint32_t)(128 >> 4) << 24);
   extern __shared__ __align__(1024) uint8_t tc_smem[];
+  constexpr int kTcStages = tc_stages<BC>();
   __shared__ uint64_t bar[kTcStages + 1];
   __shared__ uint32_t tmem_base_sh;
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
@@ -206,8 +214,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
   // warp w reads TMEM lanes 32w..32w+31 = D rows; thread = one row
   const int row = warp * 32 + lane;
   float* out = z1_part + ((size_t)blockIdx.x * 128 + row) * Bp + seed0;
+  if (nkb == 0) {  // no e-nodes in this CTA's range: the accumulator was never written
 #pragma unroll
-  for (int c = 0; c < BC; c += 16) {
+    for (int c = 0; c < BC; c += 4) *reinterpret_cast<float4*>(out + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+#pragma unroll
+  for (int c = 0; c < BC && nkb > 0; c += 16) {
     uint32_t v[16], w[16];
     const uint32_t ta = tmem + ((uint32_t)(warp * 32) << 16) + c;
     asm volatile(
@@ -434,7 +446,7 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
   const dim3 grid(nsplit, sh.Bp / Bc);
 #define SM_L1(BCV)                                                                              \
   do {                                                                                          \
-    constexpr int smem = kTcStages * (128 * kTcKB * 4 + kTcKB * 2 * BCV * 4) + 1024;            \
+    constexpr int smem = tc_stages<BCV>() * (128 * kTcKB * 4 + kTcKB * 2 * BCV * 4) + 1024;     \
     static bool attr = false;                                                                   \
     if (!attr) {                                                                                \
       SM_CUDA(cudaFuncSetAttribute(k_mlp_l1_tc<BCV>, cudaFuncAttributeMaxDynamicSharedMemorySize, \

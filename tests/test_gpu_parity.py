@@ -200,6 +200,29 @@ def test_c5_mlp_full(sm, orc):
     compare_step(sm, orc, make_config("C5"), spec["seeds_per_gpu"], spec["group"], seed=4)
 
 
+@pytest.mark.parametrize("B", [32, 64, 128, 256])
+def test_mlp_layer1_tensor_cores(sm, B):
+    """The tcgen05 layer-1 contraction (hi/lo TF32 split) at every seed-chunk
+    width: with u = 0 the step's f is f_mlp alone, checked against the MLP in
+    fp64 applied to the GPU's own p (1e-4 relative; measured ~4e-6).  C5's
+    e-node count leaves the last split-K CTA without e-nodes, which must
+    contribute zeros."""
+    eg = make_config("C5")
+    eg.u = np.zeros_like(eg.u)
+    g = sm.load_egraph_from(eg, device=0)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), B, sm.Options(penalty_group=8, rng_key=3))
+    theta = np.random.default_rng(B).uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
+    d = run.debug_step(theta, None, None, step_index=0)
+    p = d["p"].astype(np.float64)
+    w = {k: v.astype(np.float64) for k, v in eg.mlp.items()}
+    z1 = w["W1"] @ p + w["b1"][:, None]
+    z2 = w["W2"] @ np.maximum(z1, 0) + w["b2"][:, None]
+    f = (w["W3"] @ np.maximum(z2, 0) + w["b3"][:, None])[0]
+    close("f_mlp", d["f"], f, scale=np.abs(f) + (np.abs(w["W3"]) @ np.abs(np.maximum(z2, 0)))[0])
+    run.close()
+    g.close()
+
+
 def test_c4_full_size_first_group(sm, orc):
     """C4 at the bench launch configuration (128 seeds, G = 16): the oracle
     recomputes the first penalty group (16 seeds) exactly."""
