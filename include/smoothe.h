@@ -236,6 +236,10 @@ typedef struct {
   int64_t steps;
   int64_t launches;          /* kernels launched by the library in the window   */
   int32_t num_seeds_padded;  /* seeds rounded up to the kernels' row width      */
+  /* the sweep kernels alone (CUDA events around each launch on the run's
+     stream): [0] k_sweep_forward, [1] k_sweep_reverse                       */
+  double sweep_kernel_ms[2];
+  int64_t sweep_kernel_launches[2];
 } smoothe_profile;
 
 SMOOTHE_API smoothe_status smoothe_run_profile(smoothe_run *run, int32_t enable);

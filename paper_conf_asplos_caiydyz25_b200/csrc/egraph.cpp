@@ -191,6 +191,44 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   // strongly connected components of the class graph
   std::vector<int32_t> sptr, sadj;
   class_successors(g, sptr, sadj);
+  g.cls_child_ptr = sptr;
+  g.cls_child = sadj;
+  // hmax_j: the longest walk from class j in the class graph, i.e. the
+  // largest L with g_q^{K-L}_j possibly non-zero in the reverse sweeps
+  // (INT32_MAX when j can reach a cycle).  Kahn's algorithm on out-degrees:
+  // a class is final once all its child classes are; classes on or above a
+  // cycle never are.
+  {
+    std::vector<int32_t> outdeg(M), pptr(M + 1, 0), padj(sadj.size()), ready;
+    for (int32_t j = 0; j < M; ++j) {
+      outdeg[j] = sptr[j + 1] - sptr[j];
+      for (int32_t e = sptr[j]; e < sptr[j + 1]; ++e) pptr[sadj[e] + 1]++;
+    }
+    for (int32_t j = 0; j < M; ++j) pptr[j + 1] += pptr[j];
+    {
+      std::vector<int32_t> fill(pptr.begin(), pptr.end() - 1);
+      for (int32_t j = 0; j < M; ++j)
+        for (int32_t e = sptr[j]; e < sptr[j + 1]; ++e) padj[fill[sadj[e]]++] = j;
+    }
+    g.hmax.assign(M, INT32_MAX);
+    for (int32_t j = 0; j < M; ++j)
+      if (outdeg[j] == 0) {
+        g.hmax[j] = 0;
+        ready.push_back(j);
+      }
+    for (size_t r = 0; r < ready.size(); ++r) {
+      const int32_t c = ready[r];
+      for (int32_t e = pptr[c]; e < pptr[c + 1]; ++e) {
+        const int32_t j = padj[e];
+        if (--outdeg[j] == 0) {
+          int32_t h = 0;
+          for (int32_t f = sptr[j]; f < sptr[j + 1]; ++f) h = std::max(h, g.hmax[sadj[f]] + 1);
+          g.hmax[j] = h;
+          ready.push_back(j);
+        }
+      }
+    }
+  }
   std::vector<int32_t> comp = kosaraju(M, sptr, sadj);
   int32_t ncomp = 0;
   for (int32_t c : comp) ncomp = std::max(ncomp, c + 1);
@@ -389,7 +427,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     auto emit = [&](int32_t b0, int32_t b1, int32_t piece) {
       const int32_t k0 = b0 < b1 ? g.pad_batch_node[b0] : -1;
       const int32_t k1 = b0 < b1 ? g.pad_batch_node[b1 - 1] : -1;
-      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece, k0, k1, g.dmin[j], 0});
+      g.rev_item.insert(g.rev_item.end(), {j, b0, b1, piece, k0, k1, g.dmin[j], g.hmax[j]});
     };
     if (cb1 - cb0 <= kRevChunk) {
       emit(cb0, cb1, 0);

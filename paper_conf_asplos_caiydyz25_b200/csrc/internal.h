@@ -84,8 +84,12 @@ struct HostGraph {
   // kernels (softmax, cost, update) give each a whole block
   std::vector<int32_t> big_class;
   std::vector<int32_t> dmin;  // [M] BFS depth from the root (INT32_MAX: unreachable)
+  // class -> distinct child classes of its e-nodes (CSR, sorted): the forward
+  // sweep marks these dirty for the next sweep when the class's q row changes
+  std::vector<int32_t> cls_child_ptr, cls_child;
+  std::vector<int32_t> hmax;  // [M] longest walk from the class (INT32_MAX: reaches a cycle)
   // Reverse-sweep work items, [n][8] = (class j, first batch, end batch, info,
-  // first e-node, last e-node, dmin_j, 0): a class's batches split into runs of <= rev_chunk cut at
+  // first e-node, last e-node, dmin_j, hmax_j): a class's batches split into runs of <= rev_chunk cut at
   // e-node boundaries, an e-node with more batches cut into "pieces" of its own.
   // info = -1: the class's only item; else (slot << 1) | piece, slot = its
   // partial-sum row (the class's last item to finish combines them in order).
@@ -112,9 +116,10 @@ struct DevGraph {
   int32_t *slot_ptr = nullptr, *slot_node = nullptr, *slot_iloc = nullptr;
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
-  int32_t *pad_batch_node = nullptr;
+  int32_t* pad_batch_node = nullptr;
   int32_t* big_class = nullptr;
   int32_t* dmin = nullptr;
+  int32_t *cls_child_ptr = nullptr, *cls_child = nullptr;
   int32_t num_big = 0;
   int32_t *rev_item = nullptr, *rev_class_item_ptr = nullptr;
   int32_t num_rev_items = 0, rev_num_slots = 0;
@@ -150,9 +155,29 @@ void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t se
                        float* theta, float* m, float* v);
 void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
                            float* cp, int32_t* choice, uint32_t* sel);
-// t: sweep index (classes with dmin > t are skipped: their q^t is exactly 0)
+// Per-run sweep state (kernels_sweep.cu, "change propagation").  Stacks are
+// indexed by version: slot t holds the rows of the classes recomputed in
+// forward sweep t; ver[t][j] is the version that holds class j's values at
+// sweep t (slot 0: q^0 = e_root, pi = 1, am = first parent).
+struct SweepState {
+  float* qstack = nullptr;    // [K+1][M][Bp]
+  float* pistack = nullptr;   // [K+1][M][Bp] (NULL for the correlated aggregator)
+  int32_t* astack = nullptr;  // [K+1][M][Bp]
+  float* qbuf[2] = {nullptr, nullptr};  // complete q^t rows, buffer t & 1
+  float* cur_pi = nullptr;    // [M][Bp] pi^t of every class during reverse sweep t
+  int32_t* cur_am = nullptr;  // [M][Bp]
+  int32_t* ver = nullptr;     // [K+1][M]
+  int32_t* dirty[2] = {nullptr, nullptr};  // [M] stamp t: recompute in sweep t
+  int32_t* chg[2] = {nullptr, nullptr};    // [M] stamp t: q row changed in sweep t
+  bool all = false;  // recompute every class in every sweep (env SMOOTHE_SWEEP_ALL=1; A/B and tests)
+};
+// Reset the per-step sweep state (stamps, q buffers = q^0).
+void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
+void launch_stack_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, float* pi0,
+                           int32_t* am0);
+// Forward sweep t: q^t (qbuf[t & 1]) from q^{t-1} and versions t of the stacks.
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
-                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am);
+                          const SweepState& st, const float* cp);
 void launch_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* u,
                         const float* cp, const float* qK, float* gcp, float* gqK, float* f_part,
                         float* p_out, int32_t nblocks_hint);
@@ -172,10 +197,12 @@ void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, 
 // t: sweep index (items of classes with dmin > t - 1 are skipped: q^{t-1} = 0
 // there, so they contribute nothing to g_cp and no active class reads their
 // g_q^{t-1})
-void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
-                          const float* cp, const float* q_prev, const float* gq, const float* pi,
-                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
-                          float* rev_part, int32_t* rev_cnt);
+// Bring cur_q / cur_pi / cur_am to reverse sweep t (before each reverse sweep).
+void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
+                           const SweepState& st);
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
+                          const SweepState& st, const float* cp, const float* gq, float* gcp,
+                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt);
 void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
                     int32_t G, double lambda, const float* cp, double* h_part, float* pen);
 void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,

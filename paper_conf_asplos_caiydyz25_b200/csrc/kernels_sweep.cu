@@ -30,16 +30,48 @@ constexpr int kSweepBlock = 64;
 // am = the lowest e-node id attaining the max (reading S7).  Products, the
 // difference 1 - p and the max use explicit round-to-nearest intrinsics so the
 // reverse sweep can recompute 1 - p_k bit for bit.
+//
+// Change propagation ("frozen classes"): q^t_j is a
+// deterministic function of the rows q^{t-1}_c of its parent classes c, so
+// if none of them changed in sweep t-1 (bitwise, any seed), q^t_j, pi^t_j and
+// am^t_j equal their values of sweep t-1 bit for bit and the class is not
+// recomputed.  A class whose q row changes marks its child classes dirty for
+// the next sweep (stamp t+1 in dirty_next); sweep 1 computes the classes
+// adjacent to the root (q^0 = e_root).  In fp32 the iterates of the whole
+// graph freeze long before K (C4: by sweep ~60 of 207), so most sweeps
+// compute almost nothing.  Results are identical to computing every class.
+//
+//   q_prev / q_cur   complete rows q^{t-1} / q^t (ping-pong; a class that
+//                    changed in t-1 but is not recomputed copies its row)
+//   q_slot, pi_slot, am_slot   version t of the stacks, written only by the
+//                    classes computed in this sweep; ver_cur[j] = the sweep
+//                    whose rows hold class j's values at t (0: the all-zero
+//                    input, slot 0)
 // ---------------------------------------------------------------------------
 template <int LPR>
 __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
-    int M, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,
+    const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,
+    const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,
+    const int32_t* __restrict__ ver_prev, int32_t* __restrict__ ver_cur,
+    const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,
     const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,
     float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
-    float* __restrict__ q, float* __restrict__ pi, int32_t* __restrict__ am) {
+    float* __restrict__ q_cur, float* __restrict__ q_slot, float* __restrict__ pi_slot,
+    int32_t* __restrict__ am_slot) {
   const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
-  if (j >= M || j == root || __ldg(dmin + j) > t) return;  // q^t_j = 0 (rows stay zero)
-  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
+  if (j >= M) return;
+  const int gl = threadIdx.x % LPR;
+  const bool leader = gl == 0 && blockIdx.y == 0;
+  const int s0 = blockIdx.y * (4 * LPR) + gl * 4;
+  const size_t o = (size_t)j * Bp + s0;
+  const bool dirty = j != root && (all || (t == 1 ? __ldg(dmin + j) == 1 : dirty_cur[j] == t));
+  if (!dirty) {  // q^t_j = q^{t-1}_j; q_cur already holds it unless j changed in t-1
+    if (leader) ver_cur[j] = ver_prev[j];
+    if (chg_prev[j] == t - 1) st4(q_cur + o, ld4(q_prev + o));
+    return;
+  }
+  const float4 qold = ld4(q_prev + o);
   // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
   // row N of cp, so p = 0: factor 1 and never a new max
   const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
@@ -87,21 +119,115 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
     comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
     comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
-  const size_t o = (size_t)j * Bp + s0;
-  st4(q + o, qo);
-  if (pi) stcs4(pi + o, po);
-  stcs4i(am + o, arg);
+  st4(q_cur + o, qo);
+  stcs4(q_slot + o, qo);
+  if (pi_slot) stcs4(pi_slot + o, po);
+  if (leader) ver_cur[j] = t;
+  stcs4i(am_slot + o, arg);
+  // bitwise change of the row (any seed of this chunk); chunks of a class write
+  // the same stamps, so concurrent stores are benign
+  const bool ne = __float_as_uint(qo.x) != __float_as_uint(qold.x) ||
+                  __float_as_uint(qo.y) != __float_as_uint(qold.y) ||
+                  __float_as_uint(qo.z) != __float_as_uint(qold.z) ||
+                  __float_as_uint(qo.w) != __float_as_uint(qold.w);
+  const unsigned gm = LPR == 32 ? 0xffffffffu : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
+  if (__ballot_sync(gm, ne) == 0u) return;
+  if (gl == 0) chg_cur[j] = t;
+  for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
+    dirty_next[cls_child[c]] = t + 1;
 }
 
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
-                          const float* cp, const float* q_prev, float* q, float* pi, int32_t* am) {
+                          const SweepState& st, const float* cp) {
+  const size_t MB = (size_t)sh.M * sh.Bp;
+  const float* q_prev = t == 1 ? st.qstack : st.qbuf[(t - 1) & 1];
   SM_DISPATCH_LPR(sh.Bp, {
     k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, t, g.dmin, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp, q_prev, q, pi,
-        am);
+        sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
+        st.chg[(t - 1) & 1], st.chg[t & 1], st.ver + (size_t)(t - 1) * sh.M,
+        st.ver + (size_t)t * sh.M, g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI,
+        a.wC, cp, q_prev, st.qbuf[t & 1], st.qstack + (size_t)t * MB,
+        st.pistack ? st.pistack + (size_t)t * MB : nullptr,
+        st.astack + (size_t)t * MB);
   });
   SM_LAUNCH_CHECK();
 }
+
+// Before reverse sweep t: the reverse reads q^{t-1} (its own class) and
+// pi^t / am^t (child classes) from complete rows cur_q / cur_pi / cur_am.
+// Going from sweep t+1 to t, only the classes recomputed in forward sweep t+1
+// (pi, am) or t (q) change version: copy their previous version's rows.
+// t == K fills cur_pi / cur_am from every class's last version (cur_q is the
+// forward's complete q^{K-1} buffer).
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_rev_transition(
+    int M, int Bp, int t, int K, const int32_t* __restrict__ ver, const float* __restrict__ qstack,
+    const float* __restrict__ pistack, const int32_t* __restrict__ astack, float* __restrict__ cur_q,
+    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
+  const RowGroup<LPR> rg;
+  const int j = rg.row;
+  if (j >= M) return;
+  const size_t MB = (size_t)M * Bp, o = (size_t)j * Bp + rg.s0;
+  const int vt = ver[(size_t)t * M + j];
+  if (t == K || ver[(size_t)(t + 1) * M + j] != vt) {
+    if (cur_pi) st4(cur_pi + o, ld4(pistack + (size_t)vt * MB + o));
+    st4i(cur_am + o, ld4i(astack + (size_t)vt * MB + o));
+  }
+  if (t < K) {
+    const int vq = ver[(size_t)(t - 1) * M + j];
+    if (vq != vt) st4(cur_q + o, ld4(qstack + (size_t)vq * MB + o));
+  }
+}
+
+void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
+                           const SweepState& st) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_rev_transition<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, t, K, st.ver, st.qstack, st.pistack, st.astack, st.qbuf[(K - 1) & 1],
+        st.cur_pi, st.cur_am);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+// Version 0 of the stacks (a class never recomputed: every parent's q is 0):
+// pi = +1 (every factor 1 - 0 is non-zero), am = the first (lowest-id) parent,
+// the forward kernel's tie rule; -1 for the root and parentless classes.
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_stack_version0(int M, int Bp, int root,
+                                                           const int32_t* __restrict__ pad_par_ptr,
+                                                           const int32_t* __restrict__ pad_par,
+                                                           float* __restrict__ pi0,
+                                                           int32_t* __restrict__ am0) {
+  const RowGroup<LPR> rg;
+  const int j = rg.row;
+  if (j >= M) return;
+  const size_t o = (size_t)j * Bp + rg.s0;
+  const int e0 = pad_par_ptr[j];
+  const int a = j != root && e0 < pad_par_ptr[j + 1] ? pad_par[2 * (size_t)e0] : -1;
+  if (pi0) st4(pi0 + o, make_float4(1.f, 1.f, 1.f, 1.f));
+  st4i(am0 + o, make_int4(a, a, a, a));
+}
+
+void launch_stack_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, float* pi0,
+                           int32_t* am0) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_stack_version0<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, pi0, am0);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
+  const size_t MB = (size_t)sh.M * sh.Bp;
+  for (int b = 0; b < 2; ++b) {
+    SM_CUDA(cudaMemsetAsync(st.dirty[b], 0xff, sizeof(int32_t) * sh.M, s));
+    SM_CUDA(cudaMemsetAsync(st.chg[b], 0xff, sizeof(int32_t) * sh.M, s));
+    SM_CUDA(cudaMemsetAsync(st.qbuf[b], 0, sizeof(float) * MB, s));
+  }
+  // qbuf[1] = qbuf[0] + M Bp (one allocation)
+  launch_fill_rows(s, st.qbuf[0] + (size_t)sh.root * sh.Bp, (int64_t)MB, 2, sh.Bp, 1.0f);
+}
+
 
 // ---------------------------------------------------------------------------
 // Reverse sweep t, one row group per class j'; for
@@ -248,14 +374,17 @@ __device__ __forceinline__ void reverse_epilogue(
 // first rows are requested right after the header arrives.  (Persistent warps
 // striding over items, with the next item staged by cp.async, measured 2.3x
 // slower on C4: the in-flight window of classes spreads and L2 reuse drops.)
+#ifndef SMOOTHE_REV_MINB4
+#define SMOOTHE_REV_MINB4 6  // min resident 64-thread blocks per SM at V = 4
+#endif
 template <int V, bool HI, bool HC>
-__global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
+__global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
-    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t) {
+    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K) {
   const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
@@ -264,6 +393,20 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
   const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
   const bool piece = info >= 0 && (info & 1);
   const int s0 = blockIdx.y * (32 * V) + lane * V;
+  // Reverse window: the loss reads only q^K, so g_q^t_j is exactly 0 unless a
+  // walk of length K - t leaves class j (t >= K - hmax_j); every child of j'
+  // then has g_q^t = 0 while t <= K - hmax_j', and so has g_q^{t-1}_{j'}.  The
+  // first two such sweeps write that zero row over the stale g_q^{t+1} /
+  // g_q^{t+2} of the ping-pong buffer (parents may still be active).
+  if ((int64_t)t + c1.w <= K) {
+    if ((int64_t)t + c1.w >= K - 1 && gq_prev && (info < 0 || it == class_item_ptr[jp])) {
+      Vec<V> z;
+#pragma unroll
+      for (int x = 0; x < V; ++x) z.v[x] = 0.f;
+      stv<V>(gq_prev + (size_t)jp * Bp + s0, z);
+    }
+    return;
+  }
   Vec<V> zero;
 #pragma unroll
   for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
@@ -368,10 +511,11 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? 6 : 8) k_sweep_reverse(
                           cp, gcp, gq_prev, part, cnt);
 }
 
-void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
-                          const float* cp, const float* q_prev, const float* gq, const float* pi,
-                          const int32_t* am, float* gcp, float* gq_prev, bool write_gq_prev,
-                          float* rev_part, int32_t* rev_cnt) {
+void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
+                          const SweepState& st, const float* cp, const float* gq, float* gcp,
+                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt) {
+  const float* q_prev = st.qbuf[(K - 1) & 1];
+  const float* pi = st.cur_pi;
   float* out = write_gq_prev ? gq_prev : nullptr;
   const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
   const int n = g.num_rev_items;
@@ -382,8 +526,8 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 #define SM_REV2(VV, HI, HC)                                                                    \
   k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
-      g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out, rev_part,   \
-      rev_cnt, l2_prefetch, t)
+      g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, st.cur_am, gcp, out,      \
+      rev_part, rev_cnt, l2_prefetch, t, K)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \

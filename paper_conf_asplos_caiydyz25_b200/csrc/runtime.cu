@@ -17,6 +17,7 @@
 #include <array>
 #include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -83,8 +84,7 @@ struct smoothe_run {
   std::vector<void*> owned;
   // state
   float *theta = nullptr, *m = nullptr, *v = nullptr, *cp = nullptr, *gcp = nullptr;
-  float *qstack = nullptr, *pistack = nullptr;
-  int32_t* astack = nullptr;
+  SweepState sw;  // q / pi / am version stacks, q buffers, change stamps
   float* gq[2] = {nullptr, nullptr};
   float* f_part = nullptr;
   double *f = nullptr, *fextra = nullptr, *ftot = nullptr, *h_part = nullptr, *h = nullptr,
@@ -124,6 +124,7 @@ struct smoothe_run {
   size_t prof_pool_used = 0;
   int64_t prof_launch[SMOOTHE_NUM_PHASES] = {0};
   int64_t prof_launch_total = 0, prof_steps = 0;
+  std::vector<std::array<cudaEvent_t, 2>> prof_kev[2];  // around each sweep kernel
   // graph
   cudaGraphExec_t graph_exec = nullptr;
   bool graph_failed = false;
@@ -205,14 +206,22 @@ void enqueue_step(smoothe_run* r) {
   launch_softmax_argmax(s, sh, g, r->theta, r->cp, r->choice, r->sel);
 
   pm.mark(SMOOTHE_PHASE_FORWARD);
-  for (int t = 1; t <= K; ++t)
-    launch_sweep_forward(s, sh, g, r->agg, t, r->cp, r->qstack + (size_t)(t - 1) * MB,
-                         r->qstack + (size_t)t * MB,
-                         r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
-                         r->astack + (size_t)(t - 1) * MB);
+  launch_sweep_reset(s, sh, r->sw);
+  // (when profiling, events bracket each sweep kernel: bench.py's roofline)
+  auto kmark = [&](int which, int at) {
+    if (!r->profiling) return;
+    if (at == 0) r->prof_kev[which].push_back({pool_event(r), nullptr});
+    else r->prof_kev[which].back()[1] = pool_event(r);
+    SM_CUDA(cudaEventRecord(r->prof_kev[which].back()[at], s));
+  };
+  for (int t = 1; t <= K; ++t) {
+    kmark(0, 0);
+    launch_sweep_forward(s, sh, g, r->agg, t, r->sw, r->cp);
+    kmark(0, 1);
+  }
 
   pm.mark(SMOOTHE_PHASE_COST);
-  const float* qK = r->qstack + (size_t)K * MB;
+  const float* qK = r->sw.qbuf[K & 1];
   float* gqK = r->gq[K & 1];
   if (r->cost_kind == SMOOTHE_COST_LINEAR) {
     launch_cost_linear(s, sh, g, r->u_f, r->cp, qK, r->gcp, gqK, r->f_part,
@@ -242,11 +251,13 @@ void enqueue_step(smoothe_run* r) {
               r->ftot, r->loss);
 
   pm.mark(SMOOTHE_PHASE_REVERSE);
-  for (int t = K; t >= 1; --t)
-    launch_sweep_reverse(s, sh, g, r->agg, t, r->cp, r->qstack + (size_t)(t - 1) * MB, r->gq[t & 1],
-                         r->pistack ? r->pistack + (size_t)(t - 1) * MB : nullptr,
-                         r->astack + (size_t)(t - 1) * MB, r->gcp, r->gq[(t - 1) & 1], t > 1,
-                         r->rev_part, r->rev_cnt);
+  for (int t = K; t >= 1; --t) {
+    launch_rev_transition(s, sh, g, t, K, r->sw);
+    kmark(1, 0);
+    launch_sweep_reverse(s, sh, g, r->agg, t, K, r->sw, r->cp, r->gq[t & 1], r->gcp,
+                         r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt);
+    kmark(1, 1);
+  }
 
   pm.mark(SMOOTHE_PHASE_UPDATE);
   launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
@@ -330,9 +341,27 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->v = dalloc<float>(o, NB);
   r->cp = dalloc<float>(o, NB + sh.Bp);  // + one zero row: the padding parent of the sweeps
   r->gcp = dalloc<float>(o, NB);
-  r->qstack = dalloc<float>(o, (size_t)(r->K + 1) * MB);
-  if (r->agg.wI != 0.f) r->pistack = dalloc<float>(o, std::max<size_t>(1, (size_t)r->K * MB));
-  r->astack = dalloc<int32_t>(o, std::max<size_t>(1, (size_t)r->K * MB));
+  {
+    SweepState& w = r->sw;
+    const char* env = std::getenv("SMOOTHE_SWEEP_ALL");
+    w.all = env && env[0] == '1';
+    const size_t slots = (size_t)r->K + 1;
+    w.qstack = dalloc<float>(o, slots * MB);
+    if (r->agg.wI != 0.f) {
+      w.pistack = dalloc<float>(o, slots * MB);
+      w.cur_pi = dalloc<float>(o, MB);
+    }
+    w.astack = dalloc<int32_t>(o, slots * MB);
+    w.cur_am = dalloc<int32_t>(o, MB);
+    w.qbuf[0] = dalloc<float>(o, 2 * MB);
+    w.qbuf[1] = w.qbuf[0] + MB;
+    w.ver = dalloc<int32_t>(o, slots * sh.M);
+    int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
+    for (int b = 0; b < 2; ++b) {
+      w.dirty[b] = stamps + (size_t)b * sh.M;
+      w.chg[b] = stamps + (size_t)(2 + b) * sh.M;
+    }
+  }
   r->gq[0] = dalloc<float>(o, MB);
   r->gq[1] = dalloc<float>(o, MB);
   const int rows_per_block_min = 256 / 32;  // kBlock / LPR(32): fewest rows per block
@@ -424,15 +453,14 @@ void init_state(smoothe_run* r) {
   const size_t MB = (size_t)sh.M * sh.Bp;
   launch_theta_init(s, sh, r->opt.rng_key, r->opt.seed_begin, r->theta, r->m, r->v);
   SM_CUDA(cudaMemsetAsync(r->cp + (size_t)sh.N * sh.Bp, 0, sizeof(float) * sh.Bp, s));
-  SM_CUDA(cudaMemsetAsync(r->qstack, 0, sizeof(float) * (size_t)(r->K + 1) * MB, s));
-  launch_fill_rows(s, r->qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K + 1, sh.Bp, 1.0f);
-  if (r->pistack) {
-    SM_CUDA(cudaMemsetAsync(r->pistack, 0, sizeof(float) * (size_t)r->K * MB, s));
-    launch_fill_rows(s, r->pistack + (size_t)sh.root * sh.Bp, (int64_t)MB, r->K, sh.Bp, 1.0f);
-  }
-  // -1: the root rows (never written) match no e-node, so padding slots, which
-  // point at the root, take no correlated term
-  SM_CUDA(cudaMemsetAsync(r->astack, 0xff, sizeof(int32_t) * std::max<size_t>(1, (size_t)r->K * MB), s));
+  // version 0 of the stacks (never overwritten: sweeps write slots 1..K):
+  // q^0 = e_root; pi = 1; am = the first parent, -1 for the root, whose rows
+  // therefore match no e-node, so padding slots (which point at the root) take
+  // no correlated term
+  SM_CUDA(cudaMemsetAsync(r->sw.qstack, 0, sizeof(float) * MB, s));
+  launch_fill_rows(s, r->sw.qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, 1, sh.Bp, 1.0f);
+  launch_stack_version0(s, sh, r->g->dev, r->sw.pistack, r->sw.astack);
+  SM_CUDA(cudaMemsetAsync(r->sw.ver, 0, sizeof(int32_t) * sh.M, s));
   SM_CUDA(cudaMemsetAsync(r->gq[0], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->gq[1], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
@@ -525,6 +553,8 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.pad_batch_node = upload(o, h.pad_batch_node, &b);
       d.big_class = upload(o, h.big_class, &b);
       d.dmin = upload(o, h.dmin, &b);
+      d.cls_child_ptr = upload(o, h.cls_child_ptr, &b);
+      d.cls_child = upload(o, h.cls_child, &b);
       d.num_big = (int32_t)h.big_class.size();
       d.rev_item = upload(o, h.rev_item, &b);
       d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
@@ -800,15 +830,22 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     const size_t MB = (size_t)sh.M * sh.Bp;
     const float* pdev = run->cost_kind == SMOOTHE_COST_LINEAR ? run->dbg_p : run->p;
     copy_rows_d2h(dump->cp, run->cp, sh.N, sh.B, sh.Bp, s);
-    copy_rows_d2h(dump->qK, run->qstack + (size_t)run->K * MB, sh.M, sh.B, sh.Bp, s);
+    copy_rows_d2h(dump->qK, run->sw.qbuf[run->K & 1], sh.M, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->p, pdev, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->grad_cp, run->dbg_gcp, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->grad_theta, run->dbg_gth, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->theta_out, run->theta, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->m_out, run->m, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->v_out, run->v, sh.N, sh.B, sh.Bp, s);
+    // version stacks: slot t holds the classes recomputed in sweep t; the rest
+    // of row t is filled from ver on the host below
+    std::vector<int32_t> ver;
+    if (dump->qstack || dump->route) {
+      ver.resize((size_t)(run->K + 1) * sh.M);
+      SM_CUDA(cudaMemcpyAsync(ver.data(), run->sw.ver, sizeof(int32_t) * ver.size(), cudaMemcpyDeviceToHost, s));
+    }
     if (dump->qstack)
-      copy_rows_d2h(dump->qstack, run->qstack, (run->K + 1) * sh.M, sh.B, sh.Bp, s);
+      copy_rows_d2h(dump->qstack, run->sw.qstack, (run->K + 1) * sh.M, sh.B, sh.Bp, s);
     if (dump->f) SM_CUDA(cudaMemcpyAsync(dump->f, run->ftot, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
     if (dump->h) {
       if (run->g->host.num_scc > 0)
@@ -823,9 +860,10 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     if (dump->valid) SM_CUDA(cudaMemcpyAsync(dump->valid, run->dbg_valid, sh.B, cudaMemcpyDeviceToHost, s));
     if (dump->disc_cost)
       SM_CUDA(cudaMemcpyAsync(dump->disc_cost, run->dbg_dcost, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
-    if (dump->route && run->K > 0)
-      SM_CUDA(cudaMemcpy2DAsync(dump->route, sizeof(int32_t) * sh.B, run->astack, sizeof(int32_t) * sh.Bp,
-                                sizeof(int32_t) * sh.B, (size_t)run->K * sh.M, cudaMemcpyDeviceToHost, s));
+    if (dump->route && run->K > 0)  // rows of sweep t + 1 = slot t + 1
+      SM_CUDA(cudaMemcpy2DAsync(dump->route, sizeof(int32_t) * sh.B, run->sw.astack + MB,
+                                sizeof(int32_t) * sh.Bp, sizeof(int32_t) * sh.B,
+                                (size_t)run->K * sh.M, cudaMemcpyDeviceToHost, s));
     std::vector<uint32_t> rbits;
     if (dump->reached) {
       rbits.resize((size_t)sh.M * sh.W);
@@ -836,18 +874,30 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       for (int j = 0; j < sh.M; ++j)
         for (int b = 0; b < sh.B; ++b)
           dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
+    if (dump->qstack)  // row t of a class not recomputed in sweep t = its version's row
+      for (int t = 1; t <= run->K; ++t)
+        for (int j = 0; j < sh.M; ++j) {
+          const int v = ver[(size_t)t * sh.M + j];
+          if (v != t)
+            std::memcpy(dump->qstack + ((size_t)t * sh.M + j) * sh.B,
+                        dump->qstack + ((size_t)v * sh.M + j) * sh.B, sizeof(float) * sh.B);
+        }
     if (dump->route) {
-      // The root row is not a decision (q_root = 1, S3).  Rows the forward
-      // sweep skipped (t < dmin_j: every p is exactly 0, so every parent ties)
-      // report the lowest-id parent, the kernel's tie rule (S7).
+      // Row t = sweep t + 1.  A class not recomputed in that sweep takes the
+      // row of its version; version 0 (every p exactly 0, so every parent
+      // ties) is the lowest-id parent, the kernel's tie rule (S7), and -1 for
+      // the root (q_root = 1 is not a decision, S3) and parentless classes.
       const HostGraph& hg = run->g->host;
       for (int t = 0; t < run->K; ++t)
         for (int j = 0; j < sh.M; ++j) {
+          const int v = ver[(size_t)(t + 1) * sh.M + j];
+          if (v == t + 1) continue;
           int32_t* row = dump->route + ((size_t)t * sh.M + j) * sh.B;
-          if (j == sh.root) {
-            for (int b = 0; b < sh.B; ++b) row[b] = -1;
-          } else if (hg.dmin[j] > t + 1 && hg.par_ptr[j + 1] > hg.par_ptr[j]) {
-            for (int b = 0; b < sh.B; ++b) row[b] = hg.par_node[hg.par_ptr[j]];
+          if (v > 0) {
+            std::memcpy(row, dump->route + ((size_t)(v - 1) * sh.M + j) * sh.B, sizeof(int32_t) * sh.B);
+          } else {
+            const int32_t a = j != sh.root && hg.par_ptr[j + 1] > hg.par_ptr[j] ? hg.par_node[hg.par_ptr[j]] : -1;
+            for (int b = 0; b < sh.B; ++b) row[b] = a;
           }
         }
     }
@@ -876,6 +926,8 @@ smoothe_status smoothe_run_profile(smoothe_run* run, int32_t enable) {
     SM_CUDA(cudaStreamSynchronize(run->stream));
     run->profiling = enable != 0;
     run->prof_ev.clear();
+    run->prof_kev[0].clear();
+    run->prof_kev[1].clear();
     run->prof_pool_used = 0;
     std::memset(run->prof_launch, 0, sizeof(run->prof_launch));
     run->prof_launch_total = 0;
@@ -897,6 +949,14 @@ smoothe_status smoothe_run_get_profile(smoothe_run* run, smoothe_profile* out) {
       }
     }
     for (int ph = 0; ph < SMOOTHE_NUM_PHASES; ++ph) out->phase_launches[ph] = run->prof_launch[ph];
+    for (int w = 0; w < 2; ++w) {
+      for (const auto& ev : run->prof_kev[w]) {
+        float ms = 0.f;
+        SM_CUDA(cudaEventElapsedTime(&ms, ev[0], ev[1]));
+        out->sweep_kernel_ms[w] += ms;
+      }
+      out->sweep_kernel_launches[w] = (int64_t)run->prof_kev[w].size();
+    }
     out->steps = run->prof_steps;
     out->launches = run->prof_launch_total;
     out->num_seeds_padded = run->sh.Bp;

@@ -246,6 +246,33 @@ def test_graphs_and_direct_launches_identical(sm):
     assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
 
 
+@pytest.mark.parametrize("name,B,G,agg", [("C2", 64, 8, "hybrid"), ("C2", 32, 8, "independent"),
+                                          ("C3", 32, 8, "correlated"), ("C5", 256, 8, "hybrid")])
+def test_change_propagation_bit_identical(sm, monkeypatch, name, B, G, agg):
+    """Skipping classes none of whose parent classes changed in the previous
+    sweep (frozen classes) gives the same bits as recomputing
+    every class in every sweep (SMOOTHE_SWEEP_ALL=1): theta after several
+    Adam steps, the best extraction, and the whole q stack and routes of a
+    debug step."""
+    eg = make_config(name)
+    outs = []
+    for env in ("0", "1"):
+        monkeypatch.setenv("SMOOTHE_SWEEP_ALL", env)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=3, assumption=agg))
+        run.steps(6)
+        th = run.theta()
+        dump = run.debug_step(th, qstack=True, route=True)
+        outs.append((run.theta(), run.extract(), dump))
+        run.close()
+    (t0, e0, d0), (t1, e1, d1) = outs
+    assert np.array_equal(t0, t1)
+    assert np.array_equal(e0[0], e1[0]) and e0[1]["best_cost"] == e1[1]["best_cost"]
+    for key in ("qstack", "route", "qK", "grad_cp", "theta_out"):
+        assert np.array_equal(d0[key], d1[key]), key
+
+
 def test_seed_sharding_bit_identical(sm):
     """8(e): a run of 64 seeds equals two runs of 32 seeds (seed_begin 0, 32)
     seed by seed, and the lexicographic best of the shards is the full best."""
