@@ -157,8 +157,8 @@ void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, c
                            float* cp, int32_t* choice, uint32_t* sel);
 // Per-run sweep state (kernels_sweep.cu, "change propagation").  Stacks are
 // indexed by version: slot t holds the rows of the classes recomputed in
-// forward sweep t; ver[t][j] is the version that holds class j's values at
-// sweep t (slot 0: q^0 = e_root, pi = 1, am = first parent).
+// forward sweep t, listed in list[t] with their previous version (slot 0:
+// q^0 = e_root, pi = 1, am = first parent).
 struct SweepState {
   float* qstack = nullptr;    // [K+1][M][Bp]
   float* pistack = nullptr;   // [K+1][M][Bp] (NULL for the correlated aggregator)
@@ -166,7 +166,10 @@ struct SweepState {
   float* qbuf[2] = {nullptr, nullptr};  // complete q^t rows, buffer t & 1
   float* cur_pi = nullptr;    // [M][Bp] pi^t of every class during reverse sweep t
   int32_t* cur_am = nullptr;  // [M][Bp]
-  int32_t* ver = nullptr;     // [K+1][M]
+  int32_t* lastver = nullptr; // [M] last version of each class (during the forward)
+  int2* list = nullptr;       // [K+1][M] (class, previous version) recomputed in sweep t
+  int32_t* list_n = nullptr;  // [K+2] list lengths
+  int K = 0, num_sms = 148;
   int32_t* dirty[2] = {nullptr, nullptr};  // [M] stamp t: recompute in sweep t
   int32_t* chg[2] = {nullptr, nullptr};    // [M] stamp t: q row changed in sweep t
   bool all = false;  // recompute every class in every sweep (env SMOOTHE_SWEEP_ALL=1; A/B and tests)

@@ -44,16 +44,16 @@ constexpr int kSweepBlock = 64;
 //   q_prev / q_cur   complete rows q^{t-1} / q^t (ping-pong; a class that
 //                    changed in t-1 but is not recomputed copies its row)
 //   q_slot, pi_slot, am_slot   version t of the stacks, written only by the
-//                    classes computed in this sweep; ver_cur[j] = the sweep
-//                    whose rows hold class j's values at t (0: the all-zero
-//                    input, slot 0)
+//                    classes recomputed in this sweep; they are appended to
+//                    the list of sweep t with their previous version
+//                    (lastver; 0: the all-zero input, slot 0)
 // ---------------------------------------------------------------------------
 template <int LPR>
 __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
     int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,
     const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,
-    const int32_t* __restrict__ ver_prev, int32_t* __restrict__ ver_cur,
+    int32_t* __restrict__ lastver, int32_t* __restrict__ list_n, int2* __restrict__ list,
     const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,
     const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,
     float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
@@ -67,7 +67,6 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   const size_t o = (size_t)j * Bp + s0;
   const bool dirty = j != root && (all || (t == 1 ? __ldg(dmin + j) == 1 : dirty_cur[j] == t));
   if (!dirty) {  // q^t_j = q^{t-1}_j; q_cur already holds it unless j changed in t-1
-    if (leader) ver_cur[j] = ver_prev[j];
     if (chg_prev[j] == t - 1) st4(q_cur + o, ld4(q_prev + o));
     return;
   }
@@ -122,7 +121,10 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
   st4(q_cur + o, qo);
   stcs4(q_slot + o, qo);
   if (pi_slot) stcs4(pi_slot + o, po);
-  if (leader) ver_cur[j] = t;
+  if (leader) {
+    list[atomicAdd(list_n + t, 1)] = make_int2(j, lastver[j]);
+    lastver[j] = t;
+  }
   stcs4i(am_slot + o, arg);
   // bitwise change of the row (any seed of this chunk); chunks of a class write
   // the same stamps, so concurrent stores are benign
@@ -144,8 +146,8 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   SM_DISPATCH_LPR(sh.Bp, {
     k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>(
         sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
-        st.chg[(t - 1) & 1], st.chg[t & 1], st.ver + (size_t)(t - 1) * sh.M,
-        st.ver + (size_t)t * sh.M, g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI,
+        st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n,
+        st.list + (size_t)t * sh.M, g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI,
         a.wC, cp, q_prev, st.qbuf[t & 1], st.qstack + (size_t)t * MB,
         st.pistack ? st.pistack + (size_t)t * MB : nullptr,
         st.astack + (size_t)t * MB);
@@ -156,35 +158,61 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // Before reverse sweep t: the reverse reads q^{t-1} (its own class) and
 // pi^t / am^t (child classes) from complete rows cur_q / cur_pi / cur_am.
 // Going from sweep t+1 to t, only the classes recomputed in forward sweep t+1
-// (pi, am) or t (q) change version: copy their previous version's rows.
+// (pi, am) or t (q) change version: copy their previous version's rows (the
+// forward's lists, so the work is proportional to the recomputed classes).
 // t == K fills cur_pi / cur_am from every class's last version (cur_q is the
 // forward's complete q^{K-1} buffer).
 template <int LPR>
-__global__ void __launch_bounds__(kBlock) k_rev_transition(
-    int M, int Bp, int t, int K, const int32_t* __restrict__ ver, const float* __restrict__ qstack,
-    const float* __restrict__ pistack, const int32_t* __restrict__ astack, float* __restrict__ cur_q,
-    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
+__global__ void __launch_bounds__(kBlock) k_rev_restore_all(
+    int M, int Bp, const int32_t* __restrict__ lastver, const float* __restrict__ pistack,
+    const int32_t* __restrict__ astack, float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
   const RowGroup<LPR> rg;
   const int j = rg.row;
   if (j >= M) return;
   const size_t MB = (size_t)M * Bp, o = (size_t)j * Bp + rg.s0;
-  const int vt = ver[(size_t)t * M + j];
-  if (t == K || ver[(size_t)(t + 1) * M + j] != vt) {
-    if (cur_pi) st4(cur_pi + o, ld4(pistack + (size_t)vt * MB + o));
-    st4i(cur_am + o, ld4i(astack + (size_t)vt * MB + o));
-  }
-  if (t < K) {
-    const int vq = ver[(size_t)(t - 1) * M + j];
-    if (vq != vt) st4(cur_q + o, ld4(qstack + (size_t)vq * MB + o));
+  const size_t v = (size_t)lastver[j];
+  if (cur_pi) st4(cur_pi + o, ld4(pistack + v * MB + o));
+  st4i(cur_am + o, ld4i(astack + v * MB + o));
+}
+
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_rev_transition(
+    int M, int Bp, const int32_t* __restrict__ n_pa, const int2* __restrict__ l_pa,
+    const int32_t* __restrict__ n_q, const int2* __restrict__ l_q, const float* __restrict__ qstack,
+    const float* __restrict__ pistack, const int32_t* __restrict__ astack, float* __restrict__ cur_q,
+    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
+  const int groups = gridDim.x * (kBlock / LPR);
+  const int n1 = *n_pa, n = n1 + *n_q;
+  const size_t MB = (size_t)M * Bp;
+  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
+  for (int i = blockIdx.x * (kBlock / LPR) + (int)threadIdx.x / LPR; i < n; i += groups) {
+    if (i < n1) {
+      const int2 e = l_pa[i];
+      const size_t o = (size_t)e.x * Bp + s0, src = (size_t)e.y * MB + o;
+      if (cur_pi) st4(cur_pi + o, ld4(pistack + src));
+      st4i(cur_am + o, ld4i(astack + src));
+    } else {
+      const int2 e = l_q[i - n1];
+      const size_t o = (size_t)e.x * Bp + s0;
+      st4(cur_q + o, ld4(qstack + (size_t)e.y * MB + o));
+    }
   }
 }
 
 void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
                            const SweepState& st) {
+  (void)g;
   SM_DISPATCH_LPR(sh.Bp, {
-    k_rev_transition<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, t, K, st.ver, st.qstack, st.pistack, st.astack, st.qbuf[(K - 1) & 1],
-        st.cur_pi, st.cur_am);
+    if (t == K) {
+      k_rev_restore_all<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
+          sh.M, sh.Bp, st.lastver, st.pistack, st.astack, st.cur_pi, st.cur_am);
+    } else {
+      const dim3 grid(2 * st.num_sms, num_chunks(sh.Bp));
+      k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(
+          sh.M, sh.Bp, st.list_n + t + 1, st.list + (size_t)(t + 1) * sh.M, st.list_n + t,
+          st.list + (size_t)t * sh.M, st.qstack, st.pistack, st.astack, st.qbuf[(K - 1) & 1],
+          st.cur_pi, st.cur_am);
+    }
   });
   SM_LAUNCH_CHECK();
 }
@@ -224,6 +252,8 @@ void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
     SM_CUDA(cudaMemsetAsync(st.chg[b], 0xff, sizeof(int32_t) * sh.M, s));
     SM_CUDA(cudaMemsetAsync(st.qbuf[b], 0, sizeof(float) * MB, s));
   }
+  SM_CUDA(cudaMemsetAsync(st.lastver, 0, sizeof(int32_t) * sh.M, s));
+  SM_CUDA(cudaMemsetAsync(st.list_n, 0, sizeof(int32_t) * (st.K + 2), s));
   // qbuf[1] = qbuf[0] + M Bp (one allocation)
   launch_fill_rows(s, st.qbuf[0] + (size_t)sh.root * sh.Bp, (int64_t)MB, 2, sh.Bp, 1.0f);
 }
@@ -432,15 +462,20 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
     // om = 1 - p_k, known at the e-node's start, lets one accumulator carry all
     // three terms: X = sum_j g_j (wI max(s pi_j, 0) + [a_j = k] wC r) with
     // (s, r) = (+1, om) if om != 0 (then g_p = X / om) and (-1, 1) if om = 0
-    // (then g_p = X).  Per e-node constants: sI = s wI, cC = wC r.
-    Vec<V> om, sI, cC;
+    // (then g_p = X).  Per e-node constants: sI = s wI, cC = wC r, and
+    // rom = 1 / om (approximate reciprocal, one MUFU per e-node; om is 0 or at
+    // least 2^-24, so flushing denormals is exact) or 1 when om = 0.
+    Vec<V> rom, sI, cC;
     auto node_consts = [&]() {
 #pragma unroll
       for (int x = 0; x < V; ++x) {
-        om.v[x] = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
-        const bool nz = om.v[x] != 0.f;
+        const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+        const bool nz = om != 0.f;
+        float r;
+        asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
+        rom.v[x] = HI && nz ? r : 1.f;
         sI.v[x] = nz ? wI : -wI;
-        cC.v[x] = HI && nz ? wC * om.v[x] : wC;  // without HI, g_p = X (no division)
+        cC.v[x] = HI && nz ? wC * om : wC;  // without HI, g_p = X (no division)
       }
     };
     node_consts();
@@ -450,14 +485,18 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
     // root, whose g_q row is 0: no mask.
     Vec<V> gA[4], PA[4], gB[4], PB[4];
     IVec<V> aA[4], aB[4];
+    // byte offset of (row, this lane's seeds): one 32 x 32 -> 64-bit
+    // multiply-add per slot (class ids are non-negative)
+    const uint32_t rowb = (uint32_t)Bp * 4u;
+    const uint64_t s0b = (uint64_t)s0 * 4u;
     auto fetch = [&](int4 j, Vec<V>* gg, Vec<V>* PP, IVec<V>* aa) {
-      const int jj[4] = {j.x, j.y, j.z, j.w};
+      const uint32_t jj[4] = {(uint32_t)j.x, (uint32_t)j.y, (uint32_t)j.z, (uint32_t)j.w};
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const size_t oj = (size_t)jj[u] * Bp + s0;
-        gg[u] = ldv<V>(gq + oj);
-        if (HI) PP[u] = ldv<V>(pi + oj);
-        if (HC) aa[u] = ldiv<V>(am + oj);
+        const uint64_t ob = (uint64_t)jj[u] * rowb + s0b;
+        gg[u] = ldv<V>(reinterpret_cast<const float*>(reinterpret_cast<const char*>(gq) + ob));
+        if (HI) PP[u] = ldv<V>(reinterpret_cast<const float*>(reinterpret_cast<const char*>(pi) + ob));
+        if (HC) aa[u] = ldiv<V>(reinterpret_cast<const int32_t*>(reinterpret_cast<const char*>(am) + ob));
       }
     };
     fetch(ld4i(pad_child + 4 * (size_t)bb), gA, PA, aA);
@@ -485,7 +524,7 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
       if (knext != k && !piece) {  // finalise e-node k (a piece hands X to the combine)
 #pragma unroll
         for (int x = 0; x < V; ++x) {
-          const float gp = HI && om.v[x] != 0.f ? __fdividef(X.v[x], om.v[x]) : X.v[x];
+          const float gp = X.v[x] * rom.v[x];
           gc.v[x] += gp * qp.v[x];
           gqacc.v[x] += gp * cv.v[x];
         }
@@ -517,7 +556,10 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   const float* q_prev = st.qbuf[(K - 1) & 1];
   const float* pi = st.cur_pi;
   float* out = write_gq_prev ? gq_prev : nullptr;
-  const int V = sh.Bp >= 128 ? 4 : sh.Bp / 32;
+#ifndef SMOOTHE_REV_VMAX
+#define SMOOTHE_REV_VMAX 4  // seeds per lane at Bp >= 128 (4: one warp per 128-seed slice)
+#endif
+  const int V = sh.Bp >= 32 * SMOOTHE_REV_VMAX ? SMOOTHE_REV_VMAX : sh.Bp / 32;
   const int n = g.num_rev_items;
   // cp / g_cp rows are L2-prefetched per item only when they cannot stay
   // L2-resident (measured: +7% on C4 at 512 MB, -9% on C3 at 13 MB)

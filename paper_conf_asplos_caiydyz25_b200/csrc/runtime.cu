@@ -355,7 +355,11 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     w.cur_am = dalloc<int32_t>(o, MB);
     w.qbuf[0] = dalloc<float>(o, 2 * MB);
     w.qbuf[1] = w.qbuf[0] + MB;
-    w.ver = dalloc<int32_t>(o, slots * sh.M);
+    w.K = r->K;
+    w.num_sms = num_sms(r->device);
+    w.lastver = dalloc<int32_t>(o, sh.M);
+    w.list = dalloc<int2>(o, slots * sh.M);
+    w.list_n = dalloc<int32_t>(o, slots + 1);
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
     for (int b = 0; b < 2; ++b) {
       w.dirty[b] = stamps + (size_t)b * sh.M;
@@ -397,7 +401,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->scal = dalloc<double>(o, 2);
   r->red_scratch = dalloc<double>(o, (size_t)128 * sh.Bp);
   r->rev_part = dalloc<float>(o, (size_t)std::max(1, r->g->dev.rev_num_slots) * sh.Bp);
-  r->rev_cnt = dalloc<int32_t>(o, (size_t)sh.M * std::max(1, sh.Bp / 128));
+  r->rev_cnt = dalloc<int32_t>(o, (size_t)sh.M * std::max(1, sh.Bp / 32));  // per (class, warp seed slice)
   r->dbg_p = nullptr;
 
   // cost model
@@ -460,13 +464,12 @@ void init_state(smoothe_run* r) {
   SM_CUDA(cudaMemsetAsync(r->sw.qstack, 0, sizeof(float) * MB, s));
   launch_fill_rows(s, r->sw.qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, 1, sh.Bp, 1.0f);
   launch_stack_version0(s, sh, r->g->dev, r->sw.pistack, r->sw.astack);
-  SM_CUDA(cudaMemsetAsync(r->sw.ver, 0, sizeof(int32_t) * sh.M, s));
   SM_CUDA(cudaMemsetAsync(r->gq[0], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->gq[1], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
   SM_CUDA(cudaMemsetAsync(r->fextra, 0, sizeof(double) * sh.Bp, s));
   SM_CUDA(cudaMemsetAsync(r->counter, 0, sizeof(int32_t), s));
-  SM_CUDA(cudaMemsetAsync(r->rev_cnt, 0, sizeof(int32_t) * sh.M * std::max(1, sh.Bp / 128), s));
+  SM_CUDA(cudaMemsetAsync(r->rev_cnt, 0, sizeof(int32_t) * sh.M * std::max(1, sh.Bp / 32), s));
   const double init_best[4] = {INFINITY, -1.0, -1.0, 0.0};
   SM_CUDA(cudaMemcpyAsync(r->best, init_best, sizeof(init_best), cudaMemcpyHostToDevice, s));
   SM_CUDA(cudaMemsetAsync(r->best_choice, 0xff, sizeof(int32_t) * sh.M, s));
@@ -839,10 +842,21 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     copy_rows_d2h(dump->v_out, run->v, sh.N, sh.B, sh.Bp, s);
     // version stacks: slot t holds the classes recomputed in sweep t; the rest
     // of row t is filled from ver on the host below
+    // ver[t][j]: the version holding class j's rows at sweep t, rebuilt from
+    // the forward's lists of recomputed classes
     std::vector<int32_t> ver;
     if (dump->qstack || dump->route) {
-      ver.resize((size_t)(run->K + 1) * sh.M);
-      SM_CUDA(cudaMemcpyAsync(ver.data(), run->sw.ver, sizeof(int32_t) * ver.size(), cudaMemcpyDeviceToHost, s));
+      std::vector<int32_t> ln(run->K + 2);
+      std::vector<int2> lst((size_t)(run->K + 1) * sh.M);
+      SM_CUDA(cudaMemcpyAsync(ln.data(), run->sw.list_n, sizeof(int32_t) * ln.size(), cudaMemcpyDeviceToHost, s));
+      SM_CUDA(cudaMemcpyAsync(lst.data(), run->sw.list, sizeof(int2) * lst.size(), cudaMemcpyDeviceToHost, s));
+      SM_CUDA(cudaStreamSynchronize(s));
+      ver.assign((size_t)(run->K + 1) * sh.M, 0);
+      for (int t = 1; t <= run->K; ++t) {
+        std::copy(ver.begin() + (size_t)(t - 1) * sh.M, ver.begin() + (size_t)t * sh.M,
+                  ver.begin() + (size_t)t * sh.M);
+        for (int i = 0; i < ln[t]; ++i) ver[(size_t)t * sh.M + lst[(size_t)t * sh.M + i].x] = t;
+      }
     }
     if (dump->qstack)
       copy_rows_d2h(dump->qstack, run->sw.qstack, (run->K + 1) * sh.M, sh.B, sh.Bp, s);

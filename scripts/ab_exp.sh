@@ -7,7 +7,8 @@ for L in default "$@"; do
   timeout 600 python bench.py --config $C --steps ${STEPS:-4} --warmup 3 --no-e2e --no-cpu --ttb-steps 0 > gpurun_out/ab_${C}_$i.json 2> gpurun_out/ab_${C}_$i.err
   python -c "
 import json,sys; d=json.load(open('gpurun_out/ab_${C}_$i.json')); p=d['phases_ms_per_step']
-print('$C', '$L', round(d['ms_per_step'],2), 'fwd', round(p['forward'],2), 'rev', round(p['reverse'],2), 'decode', round(p['decode'],2))" || tail -3 gpurun_out/ab_${C}_$i.err
+k=d.get('sweep_kernel_ms_per_step',{})
+print('$C', '$L', round(d['ms_per_step'],2), 'fwd', round(p['forward'],2), 'rev', round(p['reverse'],2), 'decode', round(p['decode'],2), 'kernels', {a: round(b,2) for a,b in k.items()})" || tail -3 gpurun_out/ab_${C}_$i.err
   i=$((i+1))
 done
 done
