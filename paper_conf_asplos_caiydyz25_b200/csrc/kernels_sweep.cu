@@ -15,6 +15,8 @@
 //  * no division in the inner loops: the reverse sweep forms one reciprocal per
 //    e-node (an IEEE divide per edge or per node cost ~30% of the sweep);
 //  * deterministic: every output row has exactly one owner, no atomics.
+#include <algorithm>
+
 #include "kcommon.cuh"
 
 namespace smoothe {
@@ -48,8 +50,153 @@ constexpr int kSweepBlock = 64;
 //                    the list of sweep t with their previous version
 //                    (lastver; 0: the all-zero input, slot 0)
 // ---------------------------------------------------------------------------
+// read-only path for the gathers (as the former kernel-parameter version got)
+__device__ __forceinline__ float4 ldg4(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ int4 ldg4i(const int32_t* p) { return __ldg(reinterpret_cast<const int4*>(p)); }
+
+#define SM_FWD_PARAMS                                                                        \
+  int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,                   \
+      const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,                 \
+      const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,                     \
+      int32_t* __restrict__ lastver, int32_t* __restrict__ list_n, int2* __restrict__ list,    \
+      const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,        \
+      const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,  \
+      float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,                \
+      float* __restrict__ q_cur, float* __restrict__ q_slot, float* __restrict__ pi_slot,      \
+      int32_t* __restrict__ am_slot
+#define SM_FWD_ARGS                                                                            \
+  M, Bp, root, t, all, dmin, dirty_cur, dirty_next, chg_prev, chg_cur, lastver, list_n, list,  \
+      cls_child_ptr, cls_child, pad_par_ptr, pad_par, wI, wC, cp, q_prev, q_cur, q_slot,       \
+      pi_slot, am_slot
+
+// Recompute class j (its row group: LPR lanes, this lane's 4 seeds from s0).
 template <int LPR>
-__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
+__device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int s0, bool leader,
+                                              unsigned gm) {
+  const size_t o = (size_t)j * Bp + s0;
+  const float4 qold = ldg4(q_prev + o);
+  // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
+  // row N of cp, so p = 0: factor 1 and never a new max
+  const int e0 = __ldg(pad_par_ptr + j), e1 = __ldg(pad_par_ptr + j + 1);
+  float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
+  float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
+  int4 arg = make_int4(-1, -1, -1, -1);
+  int4 zc = make_int4(0, 0, 0, 0);
+  int4 n01 = make_int4(0, 0, 0, 0), n23 = n01;
+  if (e0 < e1) {
+    n01 = ldg4i(pad_par + 2 * (size_t)e0);
+    n23 = ldg4i(pad_par + 2 * (size_t)e0 + 4);
+  }
+  for (int e = e0; e < e1; e += 4) {
+    const int kk[4] = {n01.x, n01.z, n23.x, n23.z};
+    const int cc[4] = {n01.y, n01.w, n23.y, n23.w};
+    if (e + 4 < e1) {  // next batch's pairs, one step ahead
+      n01 = ldg4i(pad_par + 2 * (size_t)e + 8);
+      n23 = ldg4i(pad_par + 2 * (size_t)e + 12);
+    }
+    float4 cv[4], qv[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      cv[u] = ldg4(cp + (size_t)kk[u] * Bp + s0);
+      qv[u] = ldg4(q_prev + (size_t)cc[u] * Bp + s0);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        const float p = __fmul_rn(comp(cv[u], x), comp(qv[u], x));
+        const float f = __fsub_rn(1.f, p);
+        comp(zc, x) += f == 0.f ? 1 : 0;
+        comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
+        const bool gt = p > comp(mx, x);
+        comp(mx, x) = gt ? p : comp(mx, x);
+        comp(arg, x) = gt ? kk[u] : comp(arg, x);
+      }
+    }
+  }
+  float4 qo, po;
+#pragma unroll
+  for (int x = 0; x < 4; ++x) {
+    const int z = comp(zc, x);
+    const float P = z > 0 ? 0.f : comp(prod, x);
+    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
+    comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
+  }
+  st4(q_cur + o, qo);
+  stcs4(q_slot + o, qo);
+  if (pi_slot) stcs4(pi_slot + o, po);
+  if (leader) {
+    list[atomicAdd(list_n + t, 1)] = make_int2(j, lastver[j]);
+    lastver[j] = t;
+  }
+  stcs4i(am_slot + o, arg);
+  // bitwise change of the row (any seed of this chunk); chunks of a class write
+  // the same stamps, so concurrent stores are benign
+  const bool ne = __float_as_uint(qo.x) != __float_as_uint(qold.x) ||
+                  __float_as_uint(qo.y) != __float_as_uint(qold.y) ||
+                  __float_as_uint(qo.z) != __float_as_uint(qold.z) ||
+                  __float_as_uint(qo.w) != __float_as_uint(qold.w);
+  if (__ballot_sync(gm, ne) == 0u) return;
+  if (gl == 0) chg_cur[j] = t;
+  for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
+    dirty_next[cls_child[c]] = t + 1;
+}
+
+// Persistent row groups over the classes in round-robin order (row group g of
+// G takes classes g, g + G, ...: the classes in flight at any time are a
+// window of consecutive ids, whose parent rows share L2).  Each row group
+// reads the stamps of its next LPR classes at once (one per lane) and visits
+// only those with work: recompute (dirty) or copy the q row (changed in the
+// previous sweep, not dirty now).  A frozen sweep is thus a few loads per row
+// group instead of one thread block per 2 classes.
+template <int LPR>
+__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(SM_FWD_PARAMS) {
+  const int gl = threadIdx.x % LPR;
+  const int G = gridDim.x * (kSweepBlock / LPR);
+  const int g = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
+  const int sh = (int)(threadIdx.x % 32) / LPR * LPR;
+  const unsigned gm = LPR == 32 ? 0xffffffffu : ((1u << LPR) - 1u) << sh;
+  const int s0 = blockIdx.y * (4 * LPR) + gl * 4;
+  const bool lead = gl == 0 && blockIdx.y == 0;
+  // the warp iterates together (row groups of LPR < 32 lanes share it): loop
+  // bounds from the warp's first row group, and the union of the groups' work
+  // bits, so the row groups of a warp run their classes side by side
+  const int gw = g - sh / LPR;
+  for (int64_t r0 = 0; r0 * G + gw < M; r0 += LPR) {
+    const int64_t jl = (r0 + gl) * G + g;
+    bool dirty = false, work = false;
+    if (jl < M && jl != root) {
+      dirty = all || (t == 1 ? __ldg(dmin + jl) == 1 : dirty_cur[jl] == t);
+      work = dirty || chg_prev[jl] == t - 1;
+    }
+    const unsigned wall = __ballot_sync(0xffffffffu, work);
+    const unsigned dall = __ballot_sync(0xffffffffu, dirty);
+    const unsigned wb = wall >> sh, db = dall >> sh;  // this group's bits (low LPR)
+    unsigned un = wall;
+#pragma unroll
+    for (int k = LPR; k < 32; k += LPR) un |= wall >> k;
+    if (LPR < 32) un &= (1u << (LPR & 31)) - 1u;
+    for (; un; un &= un - 1) {
+      const int i = __ffs(un) - 1;
+      if (!((wb >> i) & 1u)) continue;
+      const int j = (int)((r0 + i) * G + g);
+      if ((db >> i) & 1u) {
+        forward_class<LPR>(SM_FWD_ARGS, j, gl, s0, lead, gm);
+      } else {  // q^t_j = q^{t-1}_j, which q_cur (written two sweeps ago) lacks
+        const size_t o = (size_t)j * Bp + s0;
+        st4(q_cur + o, ld4(q_prev + o));
+      }
+    }
+  }
+}
+
+// One row group per class (graphs up to a few waves of resident blocks): the
+// hardware block scheduler balances big classes.  The per-class code is the
+// same as forward_class; kept as a kernel of its own because the inlined
+// version schedules its loads worse (measured 15% slower on C5, same
+// instruction and sector counts, more long-scoreboard stalls).
+template <int LPR>
+__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
     int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,
     const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,
@@ -139,18 +286,44 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(
     dirty_next[cls_child[c]] = t + 1;
 }
 
+template <int LPR>
+static int forward_grid(int device) {
+  static int blocks[64] = {0};
+  int& b = blocks[device & 63];
+  if (!b) {
+    SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_sweep_forward<LPR>, kSweepBlock, 0));
+    // 4 waves of resident blocks: graphs up to that size keep one class per
+    // row group (hardware block scheduling balances the big classes); larger
+    // ones loop (C4: ~10 classes per row group)
+    b = 4 * std::max(1, b) * num_sms(device);
+  }
+  return b;
+}
+
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const SweepState& st, const float* cp) {
   const size_t MB = (size_t)sh.M * sh.Bp;
-  const float* q_prev = t == 1 ? st.qstack : st.qbuf[(t - 1) & 1];
+  int dev = 0;
+  SM_CUDA(cudaGetDevice(&dev));
   SM_DISPATCH_LPR(sh.Bp, {
-    k_sweep_forward<LPR><<<row_grid(sh.M, sh.Bp, LPR, kSweepBlock), kSweepBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
-        st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n,
-        st.list + (size_t)t * sh.M, g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI,
-        a.wC, cp, q_prev, st.qbuf[t & 1], st.qstack + (size_t)t * MB,
-        st.pistack ? st.pistack + (size_t)t * MB : nullptr,
-        st.astack + (size_t)t * MB);
+    const int rows_per_block = kSweepBlock / LPR;
+    const int need = (sh.M + rows_per_block - 1) / rows_per_block;
+    const int cap = forward_grid<LPR>(dev);
+    const dim3 grid(need <= cap ? need : cap, num_chunks(sh.Bp));
+    if (need <= cap)
+      k_sweep_forward_direct<LPR><<<grid, kSweepBlock, 0, s>>>(
+          sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
+          st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n, st.list + (size_t)t * sh.M,
+          g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp,
+          t == 1 ? st.qstack : st.qbuf[(t - 1) & 1], st.qbuf[t & 1], st.qstack + (size_t)t * MB,
+          st.pistack ? st.pistack + (size_t)t * MB : nullptr, st.astack + (size_t)t * MB);
+    else
+      k_sweep_forward<LPR><<<grid, kSweepBlock, 0, s>>>(
+          sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
+          st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n, st.list + (size_t)t * sh.M,
+          g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp,
+          t == 1 ? st.qstack : st.qbuf[(t - 1) & 1], st.qbuf[t & 1], st.qstack + (size_t)t * MB,
+          st.pistack ? st.pistack + (size_t)t * MB : nullptr, st.astack + (size_t)t * MB);
   });
   SM_LAUNCH_CHECK();
 }
