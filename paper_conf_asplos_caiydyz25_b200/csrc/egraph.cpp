@@ -304,6 +304,15 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       a = b;
     }
     g.ent_ptr.push_back((int32_t)g.ent_i.size());
+    if (g.scc_class_ptr[s + 1] - g.scc_class_ptr[s] > kSmallScc) {
+      int32_t mx = 1;
+      for (int32_t l = g.slot_ptr[s]; l < g.slot_ptr[s + 1]; ++l)
+        mx = std::max(mx, g.slot_jptr[l + 1] - g.slot_jptr[l]);
+      int32_t sq = 1;  // ceil(log2 mx) + 1
+      while ((1 << (sq - 1)) < mx) ++sq;
+      g.big_scc.push_back(s);
+      g.big_scc_sq.push_back(sq);
+    }
   }
   g.K_auto = k_auto(g, sptr, sadj, comp);
 

@@ -38,6 +38,10 @@ struct Failure {
 // E-graph: host analysis (egraph.cpp) and its device mirror
 // ---------------------------------------------------------------------------
 constexpr int32_t kBigClass = 32;  // e-nodes above which a class gets a block (kernels_step.cu)
+// Components up to this many classes keep Abar / e^Abar in shared memory and
+// their decode closures in 64-bit registers; larger ones take the global-memory
+// paths (batched fp64 GEMMs for the penalty, block-wide fixpoints for decode).
+constexpr int32_t kSmallScc = 64;
 
 // Max batches of 4 children per reverse-sweep item: 0 = from the graph's size
 // (HostGraph::rev_chunk: small graphs need short items to fill the GPU, large ones pay
@@ -69,6 +73,11 @@ struct HostGraph {
   std::vector<int32_t> slot_node, slot_iloc;       // [num_slots]
   std::vector<int32_t> slot_jptr, slot_jloc;       // children in the component (local)
   std::vector<int32_t> node_slot;                  // [N] slot id or -1
+  // components with more than kSmallScc classes and, per component, the number
+  // of squarings s of its matrix exponential: the row sums of Abar are
+  // sum_{k in m_i} cp_k |ch_k cap S| <= max_k |ch_k cap S| (cp sums to 1 over
+  // a class), so 2^-s Abar has inf-norm <= 1/2 with s = ceil(log2 max) + 1
+  std::vector<int32_t> big_scc, big_scc_sq;
   int32_t K_auto = 0, max_class_size = 0, max_in_degree = 0;
   // Sweep layouts padded to multiples of 4 entries per list (aligned vector
   // index loads, 4 row gathers in flight):
@@ -207,7 +216,11 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const SweepState& st, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt);
 void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
-                    int32_t G, double lambda, const float* cp, double* h_part, float* pen);
+                    int32_t G, double lambda, const float* cp, double* h_part, float* pen,
+                    double* big_scratch, int big_groups_per_batch);
+// bytes of fp64 scratch the large-component path needs, and how many penalty
+// groups it processes per batch (0 when every component is small)
+size_t notears_big_scratch(const HostGraph& hg, int ngroups, int* groups_per_batch);
 void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,
                    const float* gcp, const float* pen, float* theta, float* m, float* v,
                    const double* step_scalars, int32_t optimizer, float lr, float beta1,
@@ -219,8 +232,8 @@ void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const
                  const double* fextra, const double* h, double* ftot, double* loss);
 // reached sets and validity masks (kernels_decode.cu); valid_out[W]
 void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
-                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* invalid,
-                   uint32_t* valid_out, int32_t grid);
+                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* settle,
+                   uint32_t* invalid, uint32_t* valid_out, int32_t grid);
 void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& g,
                                const double* u, const int32_t* choice, const uint32_t* reach,
                                double* cost_part);

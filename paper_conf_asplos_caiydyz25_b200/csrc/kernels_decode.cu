@@ -34,6 +34,11 @@ namespace smoothe {
 //    inside S, and the local reach closure R and settle closure
 //    settle_j = !reach_j OR (children of c_j in S all settled) run in
 //    registers on those masks;
+//  * a component with more than 64 classes (kSmallScc) runs the same two
+//    closures block-wide in place: reach words in `reach`, settle words in
+//    `settle`, bit-OR atomics per seed (lane), passes repeated until one
+//    changes nothing (__syncthreads_or).  The closures are monotone, so the
+//    order of the updates inside a pass does not change the fixpoint;
 //  * every cycle of a selection lies inside one SCC, so the selection is valid
 //    iff, in every SCC, every reached class settles.  Unsettled reached classes
 //    mark their seeds invalid (bit-OR atomics: order-independent, deterministic).
@@ -42,6 +47,68 @@ namespace smoothe {
 // each fixpoint pass: on C5, with 900-node classes, the slowest SCC set the
 // pace of every level, 3.6 ms per decode.)
 constexpr int kDecodeWarps = 8;
+
+// Phase B for one (large component, 32-seed word), the whole block: lane =
+// seed, warps over the component's classes.
+__device__ void decode_big_scc(int n, int c0, int w, int W, int Bp, int root,
+                               const int32_t* __restrict__ scc_class,
+                               const int32_t* __restrict__ node_slot,
+                               const int32_t* __restrict__ slot_jptr,
+                               const int32_t* __restrict__ slot_jloc,
+                               const int32_t* __restrict__ choice, uint32_t* reach,
+                               uint32_t* settle, uint32_t* invalid) {
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t bit = 1u << lane;
+  // reach closure: a reached class's chosen e-node reaches its children in S
+  for (;;) {
+    int chg = 0;
+    for (int l = wib; l < n; l += kDecodeWarps) {
+      const int j = scc_class[c0 + l];
+      if (!(__ldcg(reach + (size_t)j * W + w) & bit)) continue;
+      const int q = node_slot[choice[(size_t)j * Bp + 32 * w + lane]];
+      if (q < 0) continue;
+      for (int e = slot_jptr[q]; e < slot_jptr[q + 1]; ++e) {
+        uint32_t* dst = reach + (size_t)scc_class[c0 + slot_jloc[e]] * W + w;
+        if (!(__ldcg(dst) & bit)) {
+          atomicOr(dst, bit);
+          chg = 1;
+        }
+      }
+    }
+    if (!__syncthreads_or(chg)) break;
+  }
+  (void)root;  // the root's reach word is all ones (launch_decode)
+  for (int l = wib; l < n; l += kDecodeWarps) {
+    const size_t o = (size_t)scc_class[c0 + l] * W + w;
+    if (lane == 0) __stcg(settle + o, ~__ldcg(reach + o));
+  }
+  __syncthreads();
+  // settle closure: a reached class settles once every child of its chosen
+  // e-node inside S has settled (children outside S settled at lower levels)
+  for (;;) {
+    int chg = 0;
+    for (int l = wib; l < n; l += kDecodeWarps) {
+      const int j = scc_class[c0 + l];
+      uint32_t* sj = settle + (size_t)j * W + w;
+      if (__ldcg(sj) & bit) continue;
+      const int q = node_slot[choice[(size_t)j * Bp + 32 * w + lane]];
+      bool ok = true;
+      if (q >= 0)
+        for (int e = slot_jptr[q]; e < slot_jptr[q + 1] && ok; ++e)
+          ok = (__ldcg(settle + (size_t)scc_class[c0 + slot_jloc[e]] * W + w) & bit) != 0;
+      if (ok) {
+        atomicOr(sj, bit);
+        chg = 1;
+      }
+    }
+    if (!__syncthreads_or(chg)) break;
+  }
+  for (int l = wib; l < n; l += kDecodeWarps) {
+    const size_t o = (size_t)scc_class[c0 + l] * W + w;
+    const uint32_t bad = __ldcg(reach + o) & ~__ldcg(settle + o);
+    if (lane == 0 && bad) atomicOr(invalid + w, bad);
+  }
+}
 
 __global__ void __launch_bounds__(256) k_decode_levels(
     int W, int root, int num_levels, const int32_t* __restrict__ lvl_cptr,
@@ -56,7 +123,7 @@ __global__ void __launch_bounds__(256) k_decode_levels(
     const int32_t* __restrict__ slot_ptr, const int32_t* __restrict__ slot_node,
     const int32_t* __restrict__ slot_jptr, const int32_t* __restrict__ slot_jloc,
     const uint32_t* __restrict__ sel, int Bp, const int32_t* __restrict__ choice, uint32_t* reach,
-    uint32_t* invalid, uint32_t* valid_out) {
+    uint32_t* settle, uint32_t* invalid, uint32_t* valid_out) {
   __shared__ uint64_t cm[64][32];  // phase B: children in S of the chosen e-node, per (class, seed)
   __shared__ uint32_t rs0[64];     // phase B: reach words after phase A
   cg::grid_group grid = cg::this_grid();
@@ -101,6 +168,11 @@ __global__ void __launch_bounds__(256) k_decode_levels(
       const int s = lvl_scc[s0l + it / W];
       const int w = (int)(it % W);
       const int c0 = scc_class_ptr[s], n = scc_class_ptr[s + 1] - c0;
+      if (n > kSmallScc) {
+        decode_big_scc(n, c0, w, W, Bp, root, scc_class, node_slot, slot_jptr, slot_jloc, choice,
+                       reach, settle, invalid);
+        continue;
+      }
       for (int l = wib; l < n; l += kDecodeWarps) {
         const int j = scc_class[c0 + l];
         const int c = choice[(size_t)j * Bp + 32 * w + lane];
@@ -151,8 +223,8 @@ static void coop_launch(const void* fn, int grid, void** args, cudaStream_t s) {
 }
 
 void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
-                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* invalid,
-                   uint32_t* valid_out, int32_t grid) {
+                   const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* settle,
+                   uint32_t* invalid, uint32_t* valid_out, int32_t grid) {
   SM_CUDA(cudaMemsetAsync(invalid, 0, sizeof(uint32_t) * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach, 0, sizeof(uint32_t) * (size_t)sh.M * sh.W, s));
   SM_CUDA(cudaMemsetAsync(reach + (size_t)sh.root * sh.W, 0xff, sizeof(uint32_t) * sh.W, s));
@@ -164,7 +236,7 @@ void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const D
                   (void*)&g.ent_ptr, (void*)&g.ent_i, (void*)&g.ent_j, (void*)&g.ent_node_ptr,
                   (void*)&g.ent_node, (void*)&g.node_slot, (void*)&g.slot_ptr,
                   (void*)&g.slot_node, (void*)&g.slot_jptr,
-                  (void*)&g.slot_jloc, (void*)&sel, &Bp, (void*)&choice, &reach, &invalid,
+                  (void*)&g.slot_jloc, (void*)&sel, &Bp, (void*)&choice, &reach, &settle, &invalid,
                   &valid_out};
   coop_launch((const void*)k_decode_levels, grid, args, s);
 }

@@ -29,7 +29,11 @@ constexpr int kSweepBlock = 64;
 //   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
 // and, for the reverse sweep, pi = the product over the non-zero factors signed
 // by the number of zero factors (+: none, -: exactly one, 0: two or more), and
-// am = the lowest e-node id attaining the max (reading S7).  Products, the
+// am = the lowest e-node id attaining the max (reading S7).  The independent
+// term 1 - prod(1 - p) is accumulated as the union u <- u + p (1 - u), which
+// keeps its relative accuracy when every p is small (1 - prod of factors
+// rounded near 1 loses it: q ~ 1e-4 came out 5e-4 off in fp32); a zero factor
+// (p = 1) gives exactly 1.  Products, the
 // difference 1 - p and the max use explicit round-to-nearest intrinsics so the
 // reverse sweep can recompute 1 - p_k bit for bit.
 //
@@ -79,6 +83,7 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
   // row N of cp, so p = 0: factor 1 and never a new max
   const int e0 = __ldg(pad_par_ptr + j), e1 = __ldg(pad_par_ptr + j + 1);
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
+  float4 un = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
   int4 arg = make_int4(-1, -1, -1, -1);
   int4 zc = make_int4(0, 0, 0, 0);
@@ -108,6 +113,7 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
         const float f = __fsub_rn(1.f, p);
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
+        comp(un, x) = __fmaf_rn(p, __fsub_rn(1.f, comp(un, x)), comp(un, x));
         const bool gt = p > comp(mx, x);
         comp(mx, x) = gt ? p : comp(mx, x);
         comp(arg, x) = gt ? kk[u] : comp(arg, x);
@@ -118,8 +124,8 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
 #pragma unroll
   for (int x = 0; x < 4; ++x) {
     const int z = comp(zc, x);
-    const float P = z > 0 ? 0.f : comp(prod, x);
-    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
+    const float U = z > 0 ? 1.f : comp(un, x);
+    comp(qo, x) = __fadd_rn(__fmul_rn(wI, U), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
     comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
   st4(q_cur + o, qo);
@@ -222,6 +228,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
   // row N of cp, so p = 0: factor 1 and never a new max
   const int e0 = pad_par_ptr[j], e1 = pad_par_ptr[j + 1];
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
+  float4 un = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
   int4 arg = make_int4(-1, -1, -1, -1);
   int4 zc = make_int4(0, 0, 0, 0);
@@ -251,6 +258,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
         const float f = __fsub_rn(1.f, p);
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
+        comp(un, x) = __fmaf_rn(p, __fsub_rn(1.f, comp(un, x)), comp(un, x));
         const bool gt = p > comp(mx, x);
         comp(mx, x) = gt ? p : comp(mx, x);
         comp(arg, x) = gt ? kk[u] : comp(arg, x);
@@ -261,8 +269,8 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
 #pragma unroll
   for (int x = 0; x < 4; ++x) {
     const int z = comp(zc, x);
-    const float P = z > 0 ? 0.f : comp(prod, x);
-    comp(qo, x) = __fadd_rn(__fmul_rn(wI, __fsub_rn(1.f, P)), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
+    const float U = z > 0 ? 1.f : comp(un, x);
+    comp(qo, x) = __fadd_rn(__fmul_rn(wI, U), __fmul_rn(wC, fmaxf(comp(mx, x), 0.f)));
     comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
   st4(q_cur + o, qo);

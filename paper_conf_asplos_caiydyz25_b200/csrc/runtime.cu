@@ -90,6 +90,8 @@ struct smoothe_run {
   double *f = nullptr, *fextra = nullptr, *ftot = nullptr, *h_part = nullptr, *h = nullptr,
          *loss = nullptr;
   float* pen = nullptr;
+  double* big_scratch = nullptr;  // large-component penalty matrices
+  int big_gpb = 0;
   int32_t* choice = nullptr;
   uint32_t *sel = nullptr, *reach = nullptr, *settle = nullptr, *invalid = nullptr;
   int32_t* flags = nullptr;
@@ -243,7 +245,8 @@ void enqueue_step(smoothe_run* r) {
 
   pm.mark(SMOOTHE_PHASE_PENALTY);
   if (hg.num_scc > 0) {
-    launch_notears(s, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen);
+    launch_notears(s, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen, r->big_scratch,
+                   r->big_gpb);
     launch_reduce_rows_f64d(s, r->h_part, hg.num_scc, r->ngroups, r->h, r->red_scratch);
   }
   launch_loss(s, sh.B, r->G, r->ngroups, r->opt.lambda, r->f,
@@ -266,8 +269,8 @@ void enqueue_step(smoothe_run* r) {
                 r->debug ? r->dbg_gcp : nullptr);
 
   pm.mark(SMOOTHE_PHASE_DECODE);
-  launch_decode(s, sh, hg, g, r->sel, r->choice, r->reach, r->invalid, r->settle + (size_t)sh.root * sh.W,
-                r->coop_grid);
+  launch_decode(s, sh, hg, g, r->sel, r->choice, r->reach, r->settle, r->invalid,
+                r->settle + (size_t)sh.root * sh.W, r->coop_grid);
   launch_decode_cost_linear(s, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
   launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost, r->red_scratch);
   const double* dextra = nullptr;
@@ -384,6 +387,10 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->h = dalloc<double>(o, r->ngroups);
   r->loss = dalloc<double>(o, 1);
   r->pen = dalloc<float>(o, std::max<size_t>(1, hg.slot_node.size() * (size_t)r->ngroups));
+  {
+    const size_t bytes = notears_big_scratch(hg, r->ngroups, &r->big_gpb);
+    if (bytes) r->big_scratch = dalloc<double>(o, bytes / sizeof(double));
+  }
   r->choice = dalloc<int32_t>(o, MB);
   r->sel = dalloc<uint32_t>(o, (size_t)sh.N * sh.W);
   r->reach = dalloc<uint32_t>(o, (size_t)sh.M * sh.W);
@@ -650,8 +657,6 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
     SM_REQUIRE(opt->assumption >= 0 && opt->assumption <= 2, SMOOTHE_E_INVALID_ARG, "bad assumption");
     SM_REQUIRE(opt->optimizer == 0 || opt->optimizer == 1, SMOOTHE_E_INVALID_ARG, "bad optimizer");
     SM_REQUIRE(cost->kind >= 0 && cost->kind <= 2, SMOOTHE_E_INVALID_ARG, "bad cost kind");
-    SM_REQUIRE(g->host.scc_max <= 64, SMOOTHE_E_INVALID_ARG,
-               "strongly connected components larger than 64 classes are not supported yet");
     r->g = g;
     r->opt = *opt;
     r->device = g->device;

@@ -190,6 +190,27 @@ def test_c2_aggregators(sm, orc, agg):
     compare_step(sm, orc, make_config("C2"), 64, 8, agg, seed=5)
 
 
+@pytest.mark.parametrize("p_back,G", [(0.06, 8), (0.1, 8), (0.15, 16), (0.06, 1)])
+def test_large_scc(sm, orc, p_back, G):
+    """Components larger than 64 classes (217 / 702 / 1112 classes): the
+    global-memory penalty path (batched fp64 GEMMs) and the block-wide decode
+    closures.  The first half of the seeds favour the anchor e-nodes (children
+    strictly deeper: a valid extraction), so both verdicts occur.  G = 1 is the
+    exact per-seed penalty (no Eq. 11 averaging)."""
+    eg = make_config("C2", scc_max=10**9, p_back=p_back)
+    assert eg.meta["scc_max"] > 64
+    B = 64
+    rng = np.random.default_rng(11)
+    theta = rng.uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
+    # anchors just above every other logit (U(-2, 2)): the arg-max without
+    # pushing cp towards 1, where 1 - p in fp32 loses the relative accuracy
+    # the parity bar asks of the independence derivatives
+    theta[eg.class_ptr[:-1], : B // 2] = 2.05
+    d, o = compare_step(sm, orc, eg, B, G, theta=theta)
+    assert o["valid"][: B // 2].all() and not o["valid"].all()
+    assert np.all(o["h"] > 0)
+
+
 def test_c3_quadratic_full(sm, orc):
     spec = CONFIGS["C3"]
     compare_step(sm, orc, make_config("C3"), spec["seeds_per_gpu"], spec["group"], seed=3)

@@ -71,6 +71,17 @@ def test_loader_matches_oracle_analysis(sm, orc, name):
     assert len(pairs) == len({x for x, _ in pairs}) == len({y for _, y in pairs})
 
 
+@pytest.mark.parametrize("p_back", [0.06, 0.15])
+def test_loader_large_components(sm, orc, p_back):
+    # components above 64 classes (the global-memory penalty / decode paths)
+    eg = make_config("C2", scc_max=10**9, p_back=p_back)
+    g = _host_graph(sm, eg)
+    o = orc.Graph(eg)
+    assert g.info["scc_max"] == o.scc_max > 64
+    assert (g.info["num_scc"], g.info["scc_classes"], g.info["K_auto"]) == \
+        (o.num_scc, o.scc_classes, o.K_auto)
+
+
 def test_loader_tiny_families(sm, orc):
     for s in range(60):
         eg = random_tiny(2000 + s, ["tree", "dag", "cyclic"][s % 3])
