@@ -209,6 +209,40 @@ typedef struct {
 SMOOTHE_API smoothe_status smoothe_debug_step(smoothe_run *run, const float *theta_in, const float *m_in,
                                   const float *v_in, int32_t step_index, smoothe_debug_out *dump);
 
+/* ---------------------------------------------------------------------------
+ * Greedy worklist extraction, the paper's "heuristic method" (PAPER.md:133,
+ * Sec. 2), on the e-graph's device: e-class costs start
+ * at infinity; an e-node's aggregated cost is u_i plus the costs of its child
+ * e-classes; an e-class takes the best aggregated cost of its e-nodes; the
+ * extraction is read top-down from the root.  Ties (reading G1):
+ * (cost, height, e-node id) lexicographically, height = 1 + max child height
+ * (0 for a leaf), so the selection is acyclic and independent of the order of
+ * evaluation.  Linear cost only (the heuristic's own model).
+ *   u           [N] e-node costs (copied)
+ *   choice      [M] caller-owned or NULL: selected e-node of every class in the
+ *               extraction, -1 elsewhere
+ *   class_cost  [M] caller-owned or NULL: the heuristic's class cost (its tree
+ *               estimate, shared subterms counted once per use); +inf for
+ *               classes without a finite derivation or unreachable from the root
+ * Errors: E_INVALID_ARG (NULL g / u / out), E_STATE (host-only e-graph), E_CUDA.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  double dag_cost;          /* f_b(s) of the extraction: sum of u over the selected
+                               e-node of each reached class, once (P100, S19); +inf if none */
+  double root_cost;         /* the heuristic's estimate for the root (tree cost)          */
+  int32_t valid;            /* 1 iff the root has a finite derivation                     */
+  int32_t selected_classes; /* classes in the extraction                                  */
+} smoothe_greedy_result;
+
+SMOOTHE_API smoothe_status smoothe_greedy(smoothe_egraph *g, const double *u, int32_t *choice,
+                              double *class_cost, smoothe_greedy_result *out);
+
+/* Warm start: theta_k += bias for k = choice[j] (every class j with choice[j] >= 0,
+ * every seed of the run), e.g. from smoothe_greedy.  Call after smoothe_run_create,
+ * before the first step.  choice [M] host, copied; E_INVALID_ARG if choice[j] is
+ * not an e-node of class j. */
+SMOOTHE_API smoothe_status smoothe_run_warm_start(smoothe_run *run, const int32_t *choice, float bias);
+
 /* theta [N][B] of the run as it stands (host copy). */
 SMOOTHE_API smoothe_status smoothe_get_theta(smoothe_run *run, float *theta);
 

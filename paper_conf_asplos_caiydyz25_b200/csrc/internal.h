@@ -240,6 +240,14 @@ void launch_decode_cost_linear(cudaStream_t s, const Shape& sh, const DevGraph& 
 void launch_decode_s(cudaStream_t s, const Shape& sh, const DevGraph& g, const uint32_t* sel,
                      const uint32_t* reach, float* s_out);
 int decode_grid(int device);
+// greedy worklist extraction (kernels_greedy.cu)
+int greedy_grid(int device);
+void launch_greedy(cudaStream_t s, const HostGraph& hg, const DevGraph& g, int grid,
+                   const double* u, double* cost, int32_t* height, int32_t* sel, int32_t* reach,
+                   int32_t* frontier, int32_t* counts, double* part, int32_t* npart,
+                   int32_t* choice_out, double* result);
+void launch_warm_start(cudaStream_t s, int M, int Bp, const int32_t* choice, float bias,
+                       float* theta);
 int decode_cost_rows(const Shape& sh);
 void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
                         const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,

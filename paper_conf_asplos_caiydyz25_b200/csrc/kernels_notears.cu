@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(256) k_notears(
 // The scaling uses the loader's structural bound (HostGraph::big_scc_sq), so
 // the launch sequence is fixed and the step stays capturable in a CUDA graph.
 // fp64 because e^A - I is squared s times (relative errors double per
-// squaring) and h is compared with the fp64 oracle; tcgen05 has no fp64 kind,
+// squaring) and h must match an fp64 reference; tcgen05 has no fp64 kind,
 // and the CUDA-core DFMA rate of B200 makes |S| in the thousands cost
 // milliseconds.
 // ---------------------------------------------------------------------------

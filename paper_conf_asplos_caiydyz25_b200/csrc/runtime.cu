@@ -619,6 +619,77 @@ smoothe_status smoothe_egraph_get_scc(const smoothe_egraph* g, int32_t* scc_of_c
   return SMOOTHE_OK;
 }
 
+smoothe_status smoothe_greedy(smoothe_egraph* g, const double* u, int32_t* choice,
+                             double* class_cost, smoothe_greedy_result* out) {
+  return guarded(nullptr, [&] {
+    SM_REQUIRE(g && u && out, SMOOTHE_E_INVALID_ARG, "NULL argument");
+    SM_REQUIRE(g->device >= 0, SMOOTHE_E_STATE, "host-only e-graph (device_ordinal = -1)");
+    SM_CUDA(cudaSetDevice(g->device));
+    const HostGraph& hg = g->host;
+    const int M = hg.M, grid = greedy_grid(g->device);
+    std::vector<void*> o;
+    struct Free {
+      std::vector<void*>& o;
+      cudaStream_t s = nullptr;
+      ~Free() {
+        if (s) cudaStreamDestroy(s);
+        for (void* p : o) cudaFree(p);
+      }
+    } fr{o};
+    SM_CUDA(cudaStreamCreateWithFlags(&fr.s, cudaStreamNonBlocking));
+    std::vector<double> uh(u, u + hg.N);
+    double* ud = upload(o, uh);
+    double* cost = dalloc<double>(o, M);
+    int32_t* ints = dalloc<int32_t>(o, (size_t)6 * M + 3 + grid);
+    int32_t *height = ints, *sel = ints + M, *reach = ints + 2 * (size_t)M,
+            *frontier = ints + 3 * (size_t)M, *chout = ints + 5 * (size_t)M,
+            *counts = ints + 6 * (size_t)M, *npart = counts + 3;
+    double* part = dalloc<double>(o, (size_t)grid + 4);
+    double* result = part + grid;
+    SM_CUDA(cudaMemsetAsync(cost, 0, sizeof(double) * M, fr.s));
+    SM_CUDA(cudaMemsetAsync(ints, 0, sizeof(int32_t) * ((size_t)6 * M + 3 + grid), fr.s));
+    launch_greedy(fr.s, hg, g->dev, grid, ud, cost, height, sel, reach, frontier, counts, part,
+                  npart, chout, result);
+    double res[4];
+    SM_CUDA(cudaMemcpyAsync(res, result, sizeof(res), cudaMemcpyDeviceToHost, fr.s));
+    if (choice)
+      SM_CUDA(cudaMemcpyAsync(choice, chout, sizeof(int32_t) * M, cudaMemcpyDeviceToHost, fr.s));
+    if (class_cost)
+      SM_CUDA(cudaMemcpyAsync(class_cost, cost, sizeof(double) * M, cudaMemcpyDeviceToHost, fr.s));
+    SM_CUDA(cudaStreamSynchronize(fr.s));
+    if (class_cost)  // classes the root cannot reach are not evaluated
+      for (int j = 0; j < M; ++j)
+        if (hg.dmin[j] == INT32_MAX) class_cost[j] = INFINITY;
+    out->dag_cost = res[0];
+    out->root_cost = res[1];
+    out->valid = (int32_t)res[2];
+    out->selected_classes = (int32_t)res[3];
+  });
+}
+
+smoothe_status smoothe_run_warm_start(smoothe_run* run, const int32_t* choice, float bias) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(choice, SMOOTHE_E_INVALID_ARG, "NULL choice");
+    const Shape& sh = run->sh;
+    for (int j = 0; j < sh.M; ++j)
+      SM_REQUIRE(choice[j] < 0 || (choice[j] >= run->g->host.class_ptr[j] &&
+                                   choice[j] < run->g->host.class_ptr[j + 1]),
+                 SMOOTHE_E_INVALID_ARG, "choice[j] is not an e-node of class j");
+    struct Tmp {
+      std::vector<void*> o;
+      ~Tmp() {
+        for (void* p : o) cudaFree(p);
+      }
+    } tmp;
+    int32_t* d = dalloc<int32_t>(tmp.o, sh.M);
+    SM_CUDA(cudaMemcpyAsync(d, choice, sizeof(int32_t) * sh.M, cudaMemcpyHostToDevice,
+                            run->stream));
+    launch_warm_start(run->stream, sh.M, sh.Bp, d, bias, run->theta);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+  });
+}
+
 smoothe_status smoothe_options_default(smoothe_options* opt) {
   if (!opt) {
     set_error("NULL options");

@@ -66,6 +66,11 @@ class _Dump(C.Structure):
                  "loss", "choice", "reached", "valid", "disc_cost", "qstack", "route")]
 
 
+class _Greedy(C.Structure):
+    _fields_ = [("dag_cost", C.c_double), ("root_cost", C.c_double), ("valid", C.c_int32),
+                ("selected_classes", C.c_int32)]
+
+
 class _Profile(C.Structure):
     _fields_ = [("phase_ms", C.c_double * 8), ("phase_launches", C.c_int64 * 8),
                 ("steps", C.c_int64), ("launches", C.c_int64), ("num_seeds_padded", C.c_int32),
@@ -91,6 +96,9 @@ _SIGS = {
     "smoothe_debug_step": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32,
                                      C.POINTER(_Dump)]),
     "smoothe_get_theta": (C.c_int, [C.c_void_p, C.c_void_p]),
+    "smoothe_greedy": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
+                                 C.POINTER(_Greedy)]),
+    "smoothe_run_warm_start": (C.c_int, [C.c_void_p, C.c_void_p, C.c_float]),
     "smoothe_run_profile": (C.c_int, [C.c_void_p, C.c_int32]),
     "smoothe_run_get_profile": (C.c_int, [C.c_void_p, C.POINTER(_Profile)]),
     "smoothe_last_error": (C.c_char_p, []),
@@ -148,6 +156,18 @@ class EGraph:
         self.info = {n: getattr(info, n) for n, _ in _Info._fields_}
         self.M, self.N = info.num_classes, info.num_nodes
         self.K_auto = info.K_auto
+
+    def greedy(self, u):
+        """smoothe_greedy: the paper's worklist heuristic on the
+        device.  Returns (choice [M] int32, -1 outside the extraction,
+        class_cost [M], result dict)."""
+        ud = _c(u, np.float64)
+        assert ud.shape == (self.N,)
+        choice = np.zeros(self.M, np.int32)
+        cost = np.zeros(self.M)
+        r = _Greedy()
+        _check(lib().smoothe_greedy(self._h, _p(ud), _p(choice), _p(cost), C.byref(r)))
+        return choice, cost, {n: getattr(r, n) for n, _ in _Greedy._fields_}
 
     def scc(self):
         out = np.zeros(self.M, np.int32)
@@ -274,6 +294,12 @@ class Run:
         if st not in (OK, E_NO_VALID):
             _check(st)
         return choice, {n: getattr(s, n) for n, _ in _Summary._fields_}
+
+    def warm_start(self, choice, bias: float):
+        """smoothe_run_warm_start: theta_k += bias at the chosen e-nodes."""
+        ch = _c(choice, np.int32)
+        assert ch.shape == (self.egraph.M,)
+        _check(lib().smoothe_run_warm_start(self._h, _p(ch), float(bias)))
 
     def theta(self):
         out = np.zeros((self.egraph.N, self.B), np.float32)

@@ -1,0 +1,77 @@
+"""smoothe_greedy (the paper's worklist heuristic on the GPU)
+against the oracle's worklist (oracle/greedy.py): bit-exact selections,
+class costs (integer u: exact in any summation order), extraction cost and
+verdict; and the theta warm start from it."""
+import numpy as np
+import pytest
+
+from gen import fig1c_fixture, make_config, random_tiny
+from oracle.greedy import greedy
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sm():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_asplos_caiydyz25_b200 as pkg
+    pkg.lib()
+    return pkg
+
+
+def compare(sm, eg):
+    g = sm.load_egraph_from(eg)
+    choice, cost, r = g.greedy(eg.u)
+    o = greedy(eg)
+    assert r["valid"] == int(o["valid"])
+    assert np.array_equal(choice, o["choice"])
+    # classes the root cannot reach are reported +inf by the library
+    fin = np.isfinite(cost)
+    assert np.array_equal(cost[fin], o["class_cost"][fin])
+    assert r["root_cost"] == o["root_cost"]
+    assert r["dag_cost"] == o["dag_cost"]
+    assert r["selected_classes"] == int((o["choice"] >= 0).sum())
+    g.close()
+    return choice, r
+
+
+def test_fig1c(sm):
+    choice, r = compare(sm, fig1c_fixture())
+    assert r["dag_cost"] == 27  # PAPER.md:166, Fig. 2b
+
+
+@pytest.mark.parametrize("kind", ["tree", "dag", "cyclic"])
+def test_tiny(sm, kind):
+    for s in range(20):
+        compare(sm, random_tiny(5000 + s, kind))
+
+
+@pytest.mark.parametrize("name,kw", [("C2", {}), ("C3", {}), ("C5", {}),
+                                     ("C2", dict(scc_max=10**9, p_back=0.1))])
+def test_configs(sm, name, kw):
+    compare(sm, make_config(name, **kw))
+
+
+def test_warm_start(sm, orc):
+    eg = make_config("C2")
+    g = sm.load_egraph_from(eg)
+    choice, _, r = g.greedy(eg.u)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), 64,
+                        sm.Options(penalty_group=8, rng_key=21))
+    run.warm_start(choice, 2.5)
+    th = run.theta().astype(np.float64)
+    ref = orc.theta_init(21, 0, 64, eg.num_nodes)
+    bias = np.zeros(eg.num_nodes)
+    bias[choice[choice >= 0]] = 2.5
+    assert np.array_equal(th, (ref + bias[:, None]).astype(np.float32))
+    # step 0 decodes theta_0: every seed extracts the greedy term (bias 2.5
+    # beats any U(-1, 1) difference), so the best is the greedy cost or better
+    run.steps(1)
+    _, s = run.extract()
+    assert s["valid"] == 1 and s["best_cost"] == r["dag_cost"]
+    run.steps(30)
+    _, s = run.extract()
+    assert s["best_cost"] <= r["dag_cost"]
+    run.close()
+    g.close()
