@@ -311,6 +311,15 @@ def run_ours(args):
            "best_cost": best["best_cost"], "best_step": best["best_step"],
            "best_seed": best["best_seed"],
            "note": "wall time on the GPU from run creation to the end of the best step"}
+    # quality context: the paper's greedy worklist heuristic on
+    # the same graph and u (smoothe_greedy, on the GPU; its own objective is
+    # the linear cost, so for MLP / quadratic configs it ignores those terms)
+    if rank == 0:
+        tg = time.time()
+        _, _, gr = g.greedy(eg.u)
+        ttb["greedy"] = {"dag_cost": gr["dag_cost"], "wall_ms": (time.time() - tg) * 1e3,
+                         "valid": gr["valid"], "linear_cost_only": eg.mlp is not None
+                         or eg.quad is not None}
 
     # roofline for the dominant phase
     bm = byte_model(N, M, K, Bl)

@@ -1,0 +1,46 @@
+"""Set cover -> e-graph extraction (gen/adversarial.py):
+the conversion is pinned by brute force (the optimum extraction is the
+minimum-weight set cover, enumerated over subsets of sets), and the planted
+instance reproduces the paper's point that the heuristic misses shared
+subterms (P135)."""
+import itertools
+
+import numpy as np
+import pytest
+
+from gen.adversarial import planted_cover, random_set_cover
+from oracle import brute
+from oracle.greedy import greedy
+
+
+def min_cover(eg):
+    """minimum-weight set cover by enumerating subsets of the sets."""
+    n, m = eg.meta["elements"], eg.meta["sets"]
+    members = []
+    for j in range(m):
+        members.append({e for e in range(n)
+                        if 1 + n + j in [int(c) for k in range(int(eg.class_ptr[1 + e]),
+                                                             int(eg.class_ptr[2 + e]))
+                                         for c in eg.children(k)]})
+    w = eg.u[-m:]
+    best = np.inf
+    for r in range(1, m + 1):
+        for sub in itertools.combinations(range(m), r):
+            if set().union(*(members[j] for j in sub)) == set(range(n)):
+                best = min(best, float(sum(w[j] for j in sub)))
+    return best
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_optimum_extraction_is_min_cover(seed):
+    eg = random_set_cover(7, 6, 0.35, seed)
+    assert brute.exhaustive_optimum(eg) == min_cover(eg)
+    g = greedy(eg)
+    assert g["valid"] and g["dag_cost"] >= min_cover(eg)
+
+
+def test_planted_heuristic_gap():
+    eg = planted_cover(4, seed=1)
+    assert min_cover(eg) == 8.0
+    g = greedy(eg)
+    assert g["dag_cost"] == 12.0 and g["root_cost"] == 12.0
