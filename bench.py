@@ -327,29 +327,49 @@ def run_ours(args):
     # the dominant sweep kernel, timed alone (CUDA events around each launch on
     # the library's stream, inside the timed region)
     kms, kn = prof["sweep_kernel_ms"], prof["sweep_kernel_launches"]
-    dom = max(("forward", "reverse"), key=lambda k: kms[k])
-    per_launch_ms = kms[dom] / max(1, kn[dom])
+    dom = max(("forward", "reverse", "frozen"), key=lambda k: kms.get(k, 0.0))
     units_launch = Bl * N
-    # algorithmic bytes of the rows a launch touches (activity windows), on
-    # average over the K launches: per e-node and per class terms of the model
-    # (the forward kernel recomputes only classes whose parents changed in the
-    # previous sweep, a data-dependent set; it is far from dominant)
-    fn, fc = active_fractions(eg, K) if dom == "reverse" else (1.0, 1.0)
-    per_node, per_class = (4.0, 8.0) if dom == "forward" else (12.0, 12.0)
-    alg = Bl * (per_node * N * fn + per_class * M * fc)
     peak, peak_src = measured_peaks()
+    if dom == "frozen":
+        # k_wspmv (frozen reverse sweeps): per working
+        # launch it streams one W row per class edge and gathers one g_q row
+        # per class edge (counted once per class row in the streaming model,
+        # like the reverse sweep's gathers), reads g_q^t_i, updates S_i and
+        # writes g_q^{t-1}_i: Bl (4 C + 16 M) bytes, C = distinct class edges.
+        # Launches in sweeps with no frozen seed exit at once; the time of all
+        # launches is charged to the working ones.
+        C_edges = len(class_graph(eg)[0])
+        nwork = max(1, prof.get("frozen_sweeps", 0))
+        per_launch_ms = kms[dom] / nwork
+        alg = Bl * (4.0 * C_edges + 16.0 * M)
+        fn = fc = 1.0
+        alg_unit = alg / units_launch
+        kname = "k_wspmv"
+    else:
+        per_launch_ms = kms[dom] / max(1, kn[dom])
+        # algorithmic bytes of the rows a launch touches (activity windows), on
+        # average over the K launches: per e-node and per class terms of the
+        # model (the forward kernel recomputes only classes whose parents
+        # changed in the previous sweep, a data-dependent set)
+        fn, fc = active_fractions(eg, K) if dom == "reverse" else (1.0, 1.0)
+        per_node, per_class = (4.0, 8.0) if dom == "forward" else (12.0, 12.0)
+        alg = Bl * (per_node * N * fn + per_class * M * fc)
+        alg_unit = bm["forward_sweep" if dom == "forward" else "reverse_sweep"]
+        kname = f"k_sweep_{dom}"
     achieved = alg / (per_launch_ms * 1e-3) / 1e9
     traffic = ncu_traffic(args.config, dom)
     # fwd+bwd share of the profiled step, applied to the graph-timed step
     fwdbwd_ms = (ms / args.steps) * sum(ph[k] for k in ("softmax", "forward", "cost", "penalty",
                                                         "reverse", "update")) / max(1e-9, sum(ph.values()))
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": traffic, "kernel": f"k_sweep_{dom}",
-            "alg_bytes_per_unit": bm["forward_sweep" if dom == "forward" else "reverse_sweep"],
+            "frac": achieved / peak, "traffic": traffic, "kernel": kname,
+            "alg_bytes_per_unit": alg_unit,
             "units_per_launch": units_launch, "avg_launch_ms": per_launch_ms,
             "kernel_share_of_step": kms[dom] / max(1e-9, sum(ph.values())),
             "alg_bytes_per_launch": alg, "active_node_frac": fn, "active_class_frac": fc,
             "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)"}
+    if dom == "frozen":
+        roof["working_launches_per_step"] = nwork / max(1, prof["steps"])
 
     run.close()
     g.close()

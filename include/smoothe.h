@@ -271,9 +271,11 @@ typedef struct {
   int64_t launches;          /* kernels launched by the library in the window   */
   int32_t num_seeds_padded;  /* seeds rounded up to the kernels' row width      */
   /* the sweep kernels alone (CUDA events around each launch on the run's
-     stream): [0] k_sweep_forward, [1] k_sweep_reverse                       */
-  double sweep_kernel_ms[2];
-  int64_t sweep_kernel_launches[2];
+     stream): [0] k_sweep_forward, [1] k_sweep_reverse, [2] k_wspmv (frozen
+     reverse sweeps)                                    */
+  double sweep_kernel_ms[3];
+  int64_t sweep_kernel_launches[3];
+  int64_t frozen_sweeps;     /* k_wspmv launches with at least one frozen seed */
 } smoothe_profile;
 
 SMOOTHE_API smoothe_status smoothe_run_profile(smoothe_run *run, int32_t enable);

@@ -386,6 +386,35 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
+  // class-edge index of every padded child slot (W rows of the frozen sweeps)
+  g.pad_cedge.assign(g.pad_child_ptr[N], -1);
+  for (int32_t i = 0; i < N; ++i) {
+    const int32_t c = g.ec[i];
+    const auto b = g.cls_child.begin() + g.cls_child_ptr[c];
+    const auto e = g.cls_child.begin() + g.cls_child_ptr[c + 1];
+    for (int32_t q = g.child_ptr[i]; q < g.child_ptr[i + 1]; ++q) {
+      const auto it = std::lower_bound(b, e, g.child_class[q]);
+      SM_REQUIRE(it != e && *it == g.child_class[q], SMOOTHE_E_BAD_GRAPH,
+                 "internal: class successor list misses a child");
+      g.pad_cedge[g.pad_child_ptr[i] + (q - g.child_ptr[i])] = (int32_t)(it - g.cls_child.begin());
+    }
+  }
+  {
+    const size_t nce = g.cls_child.size();
+    g.cedge_class.assign(nce, 0);
+    for (int32_t c = 0; c < M; ++c)
+      for (int32_t e = g.cls_child_ptr[c]; e < g.cls_child_ptr[c + 1]; ++e) g.cedge_class[e] = c;
+    g.cedge_ptr.assign(nce + 1, 0);
+    for (int32_t i = 0; i < N; ++i)
+      for (int32_t q = g.pad_child_ptr[i]; q < g.pad_child_ptr[i + 1]; ++q)
+        if (g.pad_cedge[q] >= 0) g.cedge_ptr[g.pad_cedge[q] + 1]++;
+    for (size_t e = 0; e < nce; ++e) g.cedge_ptr[e + 1] += g.cedge_ptr[e];
+    g.cedge_node.assign(g.cedge_ptr[nce], 0);
+    std::vector<int32_t> fill(g.cedge_ptr.begin(), g.cedge_ptr.end() - 1);
+    for (int32_t i = 0; i < N; ++i)  // ascending e-node ids per class edge
+      for (int32_t q = g.pad_child_ptr[i]; q < g.pad_child_ptr[i + 1]; ++q)
+        if (g.pad_cedge[q] >= 0) g.cedge_node[fill[g.pad_cedge[q]]++] = i;
+  }
   // dmin_j: BFS depth of class j from the root over class -> child-class
   // edges (unreachable: INT32_MAX).  q^t_j is exactly 0 for t < dmin_j (q^0 =
   // e_root and each sweep extends the support by one edge), so the sweeps skip

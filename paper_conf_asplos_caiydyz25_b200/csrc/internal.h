@@ -89,6 +89,12 @@ struct HostGraph {
   // faster: the shared inert rows stay L1-resident.)
   std::vector<int32_t> pad_child_ptr, pad_child, pad_par_ptr, pad_par;
   std::vector<int32_t> pad_batch_node;  // [pad_child_ptr[N] / 4] e-node owning each batch of 4
+  // [pad_child_ptr[N]] index of (ec(i), child) in cls_child for each padded
+  // child slot of e-node i; -1 for padding (frozen-sweep matrix W, section 7)
+  std::vector<int32_t> pad_cedge;
+  // per class edge (i, j): its class i and the e-nodes k of m_i with j in ch_k
+  // (ascending), CSR -- the rows of W are built one class edge at a time
+  std::vector<int32_t> cedge_class, cedge_ptr, cedge_node;
   // classes with more than kBigClass e-nodes, largest first: the per-class
   // kernels (softmax, cost, update) give each a whole block
   std::vector<int32_t> big_class;
@@ -126,6 +132,9 @@ struct DevGraph {
   int32_t *slot_jptr = nullptr, *slot_jloc = nullptr, *node_slot = nullptr;
   int32_t *pad_child_ptr = nullptr, *pad_child = nullptr, *pad_par_ptr = nullptr, *pad_par = nullptr;
   int32_t* pad_batch_node = nullptr;
+  int32_t* pad_cedge = nullptr;
+  int32_t *cedge_class = nullptr, *cedge_ptr = nullptr, *cedge_node = nullptr;
+  int64_t num_cedge = 0;
   int32_t* big_class = nullptr;
   int32_t* dmin = nullptr;
   int32_t *cls_child_ptr = nullptr, *cls_child = nullptr;
@@ -182,6 +191,13 @@ struct SweepState {
   int32_t* dirty[2] = {nullptr, nullptr};  // [M] stamp t: recompute in sweep t
   int32_t* chg[2] = {nullptr, nullptr};    // [M] stamp t: q row changed in sweep t
   bool all = false;  // recompute every class in every sweep (env SMOOTHE_SWEEP_ALL=1; A/B and tests)
+  // Frozen reverse sweeps: W [num_cedge][Bp] class-level
+  // reverse coefficients of the K-state, S [M][Bp] the sums of g_q over a
+  // seed's frozen sweeps, the K-state rows kq / kpi / kam, wm [Bp] 1 while the
+  // seed's rows still equal the K-state (env SMOOTHE_REV_W=0 disables).
+  bool wmode = false;
+  float *W = nullptr, *S = nullptr, *kq = nullptr, *kpi = nullptr;
+  int32_t *kam = nullptr, *wm = nullptr;
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).
 void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
@@ -212,9 +228,18 @@ void launch_reduce_rows_f64d(cudaStream_t s, const double* part, int32_t nrows, 
 // Bring cur_q / cur_pi / cur_am to reverse sweep t (before each reverse sweep).
 void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
                            const SweepState& st);
+// Reverse sweep t over the rows q_prev (q^{t-1}), pi / am (pi^t, am^t); seeds
+// with wm[s] != 0 are left to the frozen-sweep kernels (wm may be NULL).
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
-                          const SweepState& st, const float* cp, const float* gq, float* gcp,
+                          const float* q_prev, const float* pi, const int32_t* am,
+                          const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt);
+// W from the K-state rows (before reverse sweep K)
+void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                   const SweepState& st, const float* cp);
+// frozen reverse sweep t for the seeds with wm set: g_q^{t-1} = W g_q^t, S += g_q^t
+void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
+                  const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count);
 void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
                     int32_t G, double lambda, const float* cp, double* h_part, float* pen,
                     double* big_scratch, int big_groups_per_batch);

@@ -361,7 +361,7 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(
     int M, int Bp, const int32_t* __restrict__ n_pa, const int2* __restrict__ l_pa,
     const int32_t* __restrict__ n_q, const int2* __restrict__ l_q, const float* __restrict__ qstack,
     const float* __restrict__ pistack, const int32_t* __restrict__ astack, float* __restrict__ cur_q,
-    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
+    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am, int32_t* __restrict__ wm) {
   const int groups = gridDim.x * (kBlock / LPR);
   const int n1 = *n_pa, n = n1 + *n_q;
   const size_t MB = (size_t)M * Bp;
@@ -375,7 +375,16 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(
     } else {
       const int2 e = l_q[i - n1];
       const size_t o = (size_t)e.x * Bp + s0;
-      st4(cur_q + o, ld4(qstack + (size_t)e.y * MB + o));
+      const float4 prev = ld4(qstack + (size_t)e.y * MB + o);
+      if (wm) {  // a seed whose q row changed in forward sweep t leaves the K-state
+        const float4 now = ld4(cur_q + o);
+#pragma unroll
+        for (int x = 0; x < 4; ++x)
+          if (__float_as_uint(comp(prev, x)) != __float_as_uint(comp(now, x)) &&
+              __ldcg(wm + s0 + x))
+            __stcg(wm + s0 + x, 0);
+      }
+      st4(cur_q + o, prev);
     }
   }
 }
@@ -392,7 +401,7 @@ void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, i
       k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(
           sh.M, sh.Bp, st.list_n + t + 1, st.list + (size_t)(t + 1) * sh.M, st.list_n + t,
           st.list + (size_t)t * sh.M, st.qstack, st.pistack, st.astack, st.qbuf[(K - 1) & 1],
-          st.cur_pi, st.cur_am);
+          st.cur_pi, st.cur_am, st.wmode ? st.wm : nullptr);
     }
   });
   SM_LAUNCH_CHECK();
@@ -520,7 +529,8 @@ __device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows oth
 // item), else its partial row, and the class's last item to finish combines.
 template <int V, bool HI>
 __device__ __forceinline__ void reverse_epilogue(
-    int lane, int jp, int info, bool piece, int Bp, int root, int s0, const Vec<V>& qp,
+    int lane, int jp, int info, bool piece, int Bp, int root, int s0, const Vec<V>& keep,
+    const Vec<V>& qp,
     const Vec<V>& gqacc, const Vec<V>& X, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const float* __restrict__ cp,
     float* __restrict__ gcp, float* __restrict__ gq_prev, float* __restrict__ part,
@@ -566,7 +576,7 @@ __device__ __forceinline__ void reverse_epilogue(
 #pragma unroll
     for (int x = 0; x < V; ++x) {
       const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
-      const float gp = HI && om != 0.f ? __fdividef(r.v[x], om) : r.v[x];
+      const float gp = (HI && om != 0.f ? __fdividef(r.v[x], om) : r.v[x]) * keep.v[x];
       gc.v[x] += gp * qp.v[x];
       acc.v[x] += gp * cv.v[x];
     }
@@ -595,10 +605,24 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
-    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K) {
+    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
+    const int32_t* __restrict__ wm) {
   const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
+  // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
+  Vec<V> keep;
+  {
+    const int sw = blockIdx.y * (32 * V) + lane * V;
+    bool allw = true;
+#pragma unroll
+    for (int x = 0; x < V; ++x) {
+      const bool w = wm && __ldg(wm + sw + x) != 0;
+      keep.v[x] = w ? 0.f : 1.f;
+      allw = allw && w;
+    }
+    if (__all_sync(0xffffffffu, allw)) return;
+  }
   const int4 c0 = items[2 * it], c1 = items[2 * it + 1];
   if (c1.z > t - 1) return;  // q^{t-1}_{j'} = 0: nothing to add, g_q^{t-1}_{j'} never read
   const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
@@ -654,7 +678,7 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
         const bool nz = om != 0.f;
         float r;
         asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
-        rom.v[x] = HI && nz ? r : 1.f;
+        rom.v[x] = (HI && nz ? r : 1.f) * keep.v[x];
         sI.v[x] = nz ? wI : -wI;
         cC.v[x] = HI && nz ? wC * om : wC;  // without HI, g_p = X (no division)
       }
@@ -727,15 +751,14 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
       }
     }
   }
-  reverse_epilogue<V, HI>(lane, jp, info, piece, Bp, root, s0, qp, gqacc, X, items, class_item_ptr,
+  reverse_epilogue<V, HI>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X, items, class_item_ptr,
                           cp, gcp, gq_prev, part, cnt);
 }
 
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
-                          const SweepState& st, const float* cp, const float* gq, float* gcp,
+                          const float* q_prev, const float* pi, const int32_t* am,
+                          const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt) {
-  const float* q_prev = st.qbuf[(K - 1) & 1];
-  const float* pi = st.cur_pi;
   float* out = write_gq_prev ? gq_prev : nullptr;
 #ifndef SMOOTHE_REV_VMAX
 #define SMOOTHE_REV_VMAX 4  // seeds per lane at Bp >= 128 (4: one warp per 128-seed slice)
@@ -749,8 +772,8 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 #define SM_REV2(VV, HI, HC)                                                                    \
   k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
-      g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, st.cur_am, gcp, out,      \
-      rev_part, rev_cnt, l2_prefetch, t, K)
+      g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,             \
+      rev_part, rev_cnt, l2_prefetch, t, K, wm)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \
@@ -762,6 +785,162 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   else SM_REV(1);
 #undef SM_REV
 #undef SM_REV2
+  SM_LAUNCH_CHECK();
+}
+
+
+// ---------------------------------------------------------------------------
+// Frozen reverse sweeps.  In fp32 the forward iterates
+// freeze: from some sweep on, a seed's q^{t-1}, pi^t and am^t rows equal the
+// K-state (q^{K-1}, pi^K, am^K) bit for bit.  Reverse sweep t is then linear
+// in g_q^t with coefficients that no longer depend on t:
+//   g_p^t_k = sum_{j in ch_k} c_kj g_q^t_j,
+//   c_kj = (wI max(s pi_j, 0) + [am_j = k] wC r) * rom    (the reverse kernel's
+//          per-e-node constants s, r, rom of the K-state),
+//   g_q^{t-1}_i = sum_{k in m_i} cp_k g_p^t_k = sum_j W_ij g_q^t_j,
+//   W_ij = sum_{k in m_i, j in ch_k} cp_k c_kj        (one row per class edge),
+// and its g_cp contribution q_i g_p^t_k sums over the frozen sweeps to
+// q_i sum_j c_kj S_j with S_j = sum_t g_q^t_j: one more reverse-kernel pass
+// over the K-state with g = S at the end of the step.  A frozen sweep is thus
+// one streamed W row and one gathered g_q row per class edge (C4: 3.5M class
+// edges against 5.5M child slots x three gathered rows).  A seed is frozen in
+// reverse sweep t while none of its q rows changed in forward sweeps t..K-1:
+// every seed is at t = K, and the transition into sweep t (which restores the
+// rows forward sweep t recomputed) clears wm[s] when a restored row differs
+// in seed s.  Decisions are per seed, so results do not depend on the batch.
+// ---------------------------------------------------------------------------
+// One row group per class edge (i, j): W_ij = sum over its e-nodes k (ascending)
+// of cp_k c_kj, with pi_j / am_j / q_i loaded once.
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_wbuild(
+    int64_t n_cedge, int Bp, float wI, float wC, const int32_t* __restrict__ cedge_class,
+    const int32_t* __restrict__ cedge_ptr, const int32_t* __restrict__ cedge_node,
+    const int32_t* __restrict__ cls_child, const float* __restrict__ cp,
+    const float* __restrict__ kq, const float* __restrict__ kpi, const int32_t* __restrict__ kam,
+    float* __restrict__ W) {
+  const RowGroup<LPR> rg;
+  const int64_t ce = (int64_t)blockIdx.x * (kBlock / LPR) + rg.sub;
+  if (ce >= n_cedge) return;
+  const bool HI = wI != 0.f, HC = wC != 0.f;
+  const int i = cedge_class[ce], j = cls_child[ce];
+  const float4 qp = ld4(kq + (size_t)i * Bp + rg.s0);
+  const float4 P = HI ? ld4(kpi + (size_t)j * Bp + rg.s0) : make_float4(0.f, 0.f, 0.f, 0.f);
+  const int4 A = ld4i(kam + (size_t)j * Bp + rg.s0);
+  float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int a = cedge_ptr[ce]; a < cedge_ptr[ce + 1]; ++a) {
+    const int k = cedge_node[a];
+    const float4 cv = ld4(cp + (size_t)k * Bp + rg.s0);
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {  // node_consts of k_sweep_reverse, then c_kj
+      const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
+      const bool nz = om != 0.f;
+      float r;
+      asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
+      const float rom = HI && nz ? r : 1.f;
+      const float cC = HI && nz ? wC * om : wC;
+      float c = HI ? wI * fmaxf((nz ? 1.f : -1.f) * comp(P, x), 0.f) : 0.f;
+      if (HC && comp(A, x) == k) c += cC;
+      comp(w, x) = fmaf(comp(cv, x), c * rom, comp(w, x));
+    }
+  }
+  st4(W + (size_t)ce * Bp + rg.s0, w);
+}
+
+void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
+                   const SweepState& st, const float* cp) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_wbuild<LPR><<<row_grid((int)g.num_cedge, sh.Bp, LPR), kBlock, 0, s>>>(
+        g.num_cedge, sh.Bp, a.wI, a.wC, g.cedge_class, g.cedge_ptr, g.cedge_node, g.cls_child,
+        cp, st.kq, st.kpi, st.kam, st.W);
+  });
+  SM_LAUNCH_CHECK();
+}
+
+constexpr int kWBlock = 64;
+// min resident blocks: 14 (<= 73 registers) for 128-seed rows (C4: 124.6 vs
+// 137.9 ms per step with 125 registers), none for narrower rows (C5: slower)
+#ifndef SMOOTHE_WSPMV_MINB
+#define SMOOTHE_WSPMV_MINB 14
+#endif
+template <int LPR>
+__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k_wspmv(
+    int M, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,
+    const float* __restrict__ W, const int32_t* __restrict__ wm, const float* __restrict__ gq,
+    float* __restrict__ S, float* __restrict__ gq_prev, int64_t* __restrict__ frozen_count) {
+  const RowGroup<LPR, kWBlock> rg;
+  const int i = rg.row;
+  if (frozen_count && blockIdx.x == 0 && threadIdx.x == 0) {  // profiling: a working launch?
+    bool any = false;
+    for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
+    if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
+  }
+  if (i >= M) return;
+  const int4 w4 = ld4i(wm + rg.s0);
+  const unsigned gm = LPR == 32 ? 0xffffffffu
+                                : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
+  if (!__any_sync(gm, (w4.x | w4.y | w4.z | w4.w) != 0)) return;  // row-group uniform
+  const int d = __ldg(dmin + i);
+  const size_t oi = (size_t)i * Bp + rg.s0;
+  if (d <= t) {  // g_q^t_i is a valid row: S_i += g_q^t_i for the frozen seeds
+    const float4 gi = ld4(gq + oi);
+    float4 si = ld4(S + oi);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (comp(w4, x)) comp(si, x) += comp(gi, x);
+    st4(S + oi, si);
+  }
+  if (d > t - 1 || !gq_prev) return;  // q^{t-1}_i = 0: the row is never read
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  const int e0 = cls_child_ptr[i], e1 = cls_child_ptr[i + 1];
+  // the row group loads LPR child indices at once (one per lane, coalesced)
+  // and broadcasts them, so the W rows (streamed) and g_q rows (gathered) of
+  // 8 edges are in flight together without a dependent index load each
+  const int gl = threadIdx.x % LPR;
+  for (int c0 = e0; c0 < e1; c0 += LPR) {
+    const int n = min(LPR, e1 - c0);
+    const int myj = gl < n ? __ldg(cls_child + c0 + gl) : 0;
+    const float* wrow = W + (size_t)c0 * Bp + rg.s0;
+    for (int u = 0; u < n; u += 8) {  // 8 edges in flight; the last batch predicated
+      float4 wv[8], gv[8];
+#pragma unroll
+      for (int v = 0; v < 8; ++v) {
+        const int j = __shfl_sync(gm, myj, (u + v) & (LPR - 1), LPR);
+        if (u + v < n) {
+          wv[v] = ldcs4(wrow + (size_t)(u + v) * Bp);
+          gv[v] = ld4(gq + (size_t)j * Bp + rg.s0);
+        } else {
+          wv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+          gv[v] = wv[v];
+        }
+      }
+#pragma unroll
+      for (int v = 0; v < 8; ++v) {
+        acc.x = fmaf(wv[v].x, gv[v].x, acc.x);
+        acc.y = fmaf(wv[v].y, gv[v].y, acc.y);
+        acc.z = fmaf(wv[v].z, gv[v].z, acc.z);
+        acc.w = fmaf(wv[v].w, gv[v].w, acc.w);
+      }
+    }
+  }
+  if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  float4 o = acc;
+  if (!(w4.x && w4.y && w4.z && w4.w)) {  // mixed: keep the reverse kernel's seeds
+    const float4 cur = ld4(gq_prev + oi);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (!comp(w4, x)) comp(o, x) = comp(cur, x);
+  }
+  st4(gq_prev + oi, o);
+}
+
+void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
+                  const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count) {
+  SM_DISPATCH_LPR(sh.Bp, {
+    k_wspmv<LPR><<<row_grid(sh.M, sh.Bp, LPR, kWBlock), kWBlock, 0, s>>>(
+        sh.M, sh.Bp, sh.root, t, g.dmin, g.cls_child_ptr, g.cls_child, st.W, st.wm, gq, st.S,
+        gq_prev, frozen_count);
+  });
   SM_LAUNCH_CHECK();
 }
 

@@ -18,6 +18,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdlib>
+#include <cstdio>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -126,7 +127,8 @@ struct smoothe_run {
   size_t prof_pool_used = 0;
   int64_t prof_launch[SMOOTHE_NUM_PHASES] = {0};
   int64_t prof_launch_total = 0, prof_steps = 0;
-  std::vector<std::array<cudaEvent_t, 2>> prof_kev[2];  // around each sweep kernel
+  std::vector<std::array<cudaEvent_t, 2>> prof_kev[3];  // around each sweep kernel
+  int64_t* frozen_count = nullptr;  // device: k_wspmv launches with frozen seeds (profiling)
   // graph
   cudaGraphExec_t graph_exec = nullptr;
   bool graph_failed = false;
@@ -254,13 +256,48 @@ void enqueue_step(smoothe_run* r) {
               r->ftot, r->loss);
 
   pm.mark(SMOOTHE_PHASE_REVERSE);
+  SweepState& sw = r->sw;
+  const float* cur_q = sw.qbuf[(K - 1) & 1];
   for (int t = K; t >= 1; --t) {
-    launch_rev_transition(s, sh, g, t, K, r->sw);
+    launch_rev_transition(s, sh, g, t, K, sw);
+    if (sw.wmode && t == K) {  // K-state rows, W, every seed frozen at t = K
+      SM_CUDA(cudaMemcpyAsync(sw.kq, cur_q, sizeof(float) * MB, cudaMemcpyDeviceToDevice, s));
+      if (sw.kpi)
+        SM_CUDA(cudaMemcpyAsync(sw.kpi, sw.cur_pi, sizeof(float) * MB, cudaMemcpyDeviceToDevice, s));
+      SM_CUDA(cudaMemcpyAsync(sw.kam, sw.cur_am, sizeof(int32_t) * MB, cudaMemcpyDeviceToDevice, s));
+      SM_CUDA(cudaMemsetAsync(sw.wm, 1, sizeof(int32_t) * sh.Bp, s));
+      SM_CUDA(cudaMemsetAsync(sw.S, 0, sizeof(float) * MB, s));
+      launch_wbuild(s, sh, g, r->agg, sw, r->cp);
+    }
+    if (sw.wmode && r->profiling && std::getenv("SMOOTHE_REV_W_STATS")) {
+      // diagnostic: seeds still frozen before reverse sweep t (stderr, one line per sweep)
+      std::vector<int32_t> h(sh.Bp);
+      SM_CUDA(cudaMemcpyAsync(h.data(), sw.wm, sizeof(int32_t) * sh.Bp, cudaMemcpyDeviceToHost, s));
+      SM_CUDA(cudaStreamSynchronize(s));
+      int n = 0, slices = 0;
+      for (int b = 0; b < sh.B; ++b) n += h[b] != 0;
+      for (int c = 0; c * 128 < sh.Bp; ++c) {
+        bool all = true;
+        for (int b = c * 128; b < std::min(sh.Bp, (c + 1) * 128); ++b) all = all && h[b] != 0;
+        slices += all;
+      }
+      fprintf(stderr, "[wstats] t=%d frozen_seeds=%d full_slices=%d\n", t, n, slices);
+    }
     kmark(1, 0);
-    launch_sweep_reverse(s, sh, g, r->agg, t, K, r->sw, r->cp, r->gq[t & 1], r->gcp,
+    launch_sweep_reverse(s, sh, g, r->agg, t, K, cur_q, sw.cur_pi, sw.cur_am,
+                         sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
                          r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt);
     kmark(1, 1);
+    if (sw.wmode) {
+      kmark(2, 0);
+      launch_wspmv(s, sh, g, t, sw, r->gq[t & 1], t > 1 ? r->gq[(t - 1) & 1] : nullptr,
+                   r->profiling ? r->frozen_count : nullptr);
+      kmark(2, 1);
+    }
   }
+  if (sw.wmode)  // the frozen sweeps' g_cp: one pass over the K-state with g = S
+    launch_sweep_reverse(s, sh, g, r->agg, K, K, sw.kq, sw.kpi, sw.kam, nullptr, r->cp, sw.S,
+                         r->gcp, nullptr, false, r->rev_part, r->rev_cnt);
 
   pm.mark(SMOOTHE_PHASE_UPDATE);
   launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
@@ -367,6 +404,20 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     for (int b = 0; b < 2; ++b) {
       w.dirty[b] = stamps + (size_t)b * sh.M;
       w.chg[b] = stamps + (size_t)(2 + b) * sh.M;
+    }
+    // frozen-sweep path: on for K >= 48 (enough sweeps to freeze and pay for
+    // the W build and the final pass), SMOOTHE_REV_W=0 / 1 forces it
+    const char* wenv = std::getenv("SMOOTHE_REV_W");
+    w.wmode = (wenv ? wenv[0] == '1' : r->K >= 48) && r->g->dev.num_cedge > 0;
+    if (w.wmode) {
+      w.W = dalloc<float>(o, (size_t)r->g->dev.num_cedge * sh.Bp);
+      w.S = dalloc<float>(o, MB);
+      w.kq = dalloc<float>(o, MB);
+      if (w.pistack) w.kpi = dalloc<float>(o, MB);
+      w.kam = dalloc<int32_t>(o, MB);
+      w.wm = dalloc<int32_t>(o, sh.Bp);
+      r->frozen_count = dalloc<int64_t>(o, 1);
+      SM_CUDA(cudaMemset(r->frozen_count, 0, sizeof(int64_t)));
     }
   }
   r->gq[0] = dalloc<float>(o, MB);
@@ -565,6 +616,11 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.dmin = upload(o, h.dmin, &b);
       d.cls_child_ptr = upload(o, h.cls_child_ptr, &b);
       d.cls_child = upload(o, h.cls_child, &b);
+      d.pad_cedge = upload(o, h.pad_cedge, &b);
+      d.cedge_class = upload(o, h.cedge_class, &b);
+      d.cedge_ptr = upload(o, h.cedge_ptr, &b);
+      d.cedge_node = upload(o, h.cedge_node, &b);
+      d.num_cedge = (int64_t)h.cls_child.size();
       d.num_big = (int32_t)h.big_class.size();
       d.rev_item = upload(o, h.rev_item, &b);
       d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
@@ -1016,8 +1072,8 @@ smoothe_status smoothe_run_profile(smoothe_run* run, int32_t enable) {
     SM_CUDA(cudaStreamSynchronize(run->stream));
     run->profiling = enable != 0;
     run->prof_ev.clear();
-    run->prof_kev[0].clear();
-    run->prof_kev[1].clear();
+    for (auto& v : run->prof_kev) v.clear();
+    if (run->frozen_count) SM_CUDA(cudaMemsetAsync(run->frozen_count, 0, sizeof(int64_t), run->stream));
     run->prof_pool_used = 0;
     std::memset(run->prof_launch, 0, sizeof(run->prof_launch));
     run->prof_launch_total = 0;
@@ -1039,7 +1095,10 @@ smoothe_status smoothe_run_get_profile(smoothe_run* run, smoothe_profile* out) {
       }
     }
     for (int ph = 0; ph < SMOOTHE_NUM_PHASES; ++ph) out->phase_launches[ph] = run->prof_launch[ph];
-    for (int w = 0; w < 2; ++w) {
+    if (run->frozen_count)
+      SM_CUDA(cudaMemcpy(&out->frozen_sweeps, run->frozen_count, sizeof(int64_t),
+                         cudaMemcpyDeviceToHost));
+    for (int w = 0; w < 3; ++w) {
       for (const auto& ev : run->prof_kev[w]) {
         float ms = 0.f;
         SM_CUDA(cudaEventElapsedTime(&ms, ev[0], ev[1]));

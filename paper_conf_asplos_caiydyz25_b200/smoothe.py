@@ -74,7 +74,8 @@ class _Greedy(C.Structure):
 class _Profile(C.Structure):
     _fields_ = [("phase_ms", C.c_double * 8), ("phase_launches", C.c_int64 * 8),
                 ("steps", C.c_int64), ("launches", C.c_int64), ("num_seeds_padded", C.c_int32),
-                ("sweep_kernel_ms", C.c_double * 2), ("sweep_kernel_launches", C.c_int64 * 2)]
+                ("sweep_kernel_ms", C.c_double * 3), ("sweep_kernel_launches", C.c_int64 * 3),
+                ("frozen_sweeps", C.c_int64)]
 
 
 _lib = None
@@ -334,9 +335,12 @@ class Run:
         return {"phase_ms": dict(zip(PHASES, list(p.phase_ms))),
                 "phase_launches": dict(zip(PHASES, list(p.phase_launches))),
                 "steps": p.steps, "launches": p.launches, "num_seeds_padded": p.num_seeds_padded,
-                "sweep_kernel_ms": {"forward": p.sweep_kernel_ms[0], "reverse": p.sweep_kernel_ms[1]},
+                "sweep_kernel_ms": {"forward": p.sweep_kernel_ms[0], "reverse": p.sweep_kernel_ms[1],
+                                    "frozen": p.sweep_kernel_ms[2]},
                 "sweep_kernel_launches": {"forward": p.sweep_kernel_launches[0],
-                                          "reverse": p.sweep_kernel_launches[1]}}
+                                          "reverse": p.sweep_kernel_launches[1],
+                                          "frozen": p.sweep_kernel_launches[2]},
+                "frozen_sweeps": p.frozen_sweeps}
 
     def close(self):
         if self._h:

@@ -103,7 +103,8 @@ def main():
                     lines.append(f"| {label} | {d[label][0]} {d[label][1]} |")
             if "DRAM read" in d and "DRAM write" in d:
                 b = to_bytes(d["DRAM read"]) + to_bytes(d["DRAM write"])
-                kind = "reverse" if "reverse" in d["kernel"] else "forward" if "forward" in d["kernel"] else d["kernel"]
+                kind = ("frozen" if "wspmv" in d["kernel"] else "reverse" if "reverse" in d["kernel"]
+                        else "forward" if "forward" in d["kernel"] else d["kernel"])
                 traffic.setdefault(cfg, {})[kind] = b
                 lines.append(f"| traffic (read + write) per launch | {b / 1e9:.3f} GB |")
     with open(os.path.join(ROOT, "profiles", f"{tag}_{cfg}.md"), "w") as fh:

@@ -211,6 +211,18 @@ def test_large_scc(sm, orc, p_back, G):
     assert np.all(o["h"] > 0)
 
 
+@pytest.mark.parametrize("name,B,G,K,agg", [("C2", 64, 8, 80, "hybrid"),
+                                             ("C2", 64, 8, 80, "independent"),
+                                             ("C2", 64, 8, 80, "correlated"),
+                                             ("C3", 32, 8, 60, "hybrid")])
+def test_frozen_sweeps_parity(sm, orc, monkeypatch, name, B, G, K, agg):
+    """The frozen reverse sweeps (W = class-level coefficients of the K-state,
+    deferred g_cp pass) forced on with K beyond the
+    freezing point: the step still matches the fp64 oracle."""
+    monkeypatch.setenv("SMOOTHE_REV_W", "1")
+    compare_step(sm, orc, make_config(name), B, G, agg, K=K, seed=B + K)
+
+
 def test_c3_quadratic_full(sm, orc):
     spec = CONFIGS["C3"]
     compare_step(sm, orc, make_config("C3"), spec["seeds_per_gpu"], spec["group"], seed=3)
@@ -298,19 +310,24 @@ def test_change_propagation_bit_identical(sm, monkeypatch, name, B, G, agg, step
             assert np.array_equal(d0[key], d1[key]), key
 
 
-def test_seed_sharding_bit_identical(sm):
+@pytest.mark.parametrize("wmode,K", [("0", -1), ("1", 80)])
+def test_seed_sharding_bit_identical(sm, monkeypatch, wmode, K):
     """8(e): a run of 64 seeds equals two runs of 32 seeds (seed_begin 0, 32)
-    seed by seed, and the lexicographic best of the shards is the full best."""
+    seed by seed, and the lexicographic best of the shards is the full best.
+    With the frozen-sweep path (SMOOTHE_REV_W=1, K = 80: most sweeps frozen)
+    the per-seed decisions keep this exact."""
+    monkeypatch.setenv("SMOOTHE_REV_W", wmode)
     eg = make_config("C2")
     g = sm.load_egraph_from(eg)
     cost = sm.CostModel.from_input(eg)
-    full = sm.run_create(g, cost, 64, sm.Options(penalty_group=8, rng_key=5))
+    full = sm.run_create(g, cost, 64, sm.Options(penalty_group=8, rng_key=5, prop_iters=K))
     full.steps(15)
     tf = full.theta()
     cf, sf = full.extract()
     halves = []
     for sb in (0, 32):
-        r = sm.run_create(g, cost, 32, sm.Options(penalty_group=8, rng_key=5, seed_begin=sb))
+        r = sm.run_create(g, cost, 32, sm.Options(penalty_group=8, rng_key=5, seed_begin=sb,
+                                                  prop_iters=K))
         r.steps(15)
         halves.append((r.theta(), r.extract()))
     assert np.array_equal(np.concatenate([halves[0][0], halves[1][0]], axis=1), tf)
