@@ -415,6 +415,21 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       for (int32_t q = g.pad_child_ptr[i]; q < g.pad_child_ptr[i + 1]; ++q)
         if (g.pad_cedge[q] >= 0) g.cedge_node[fill[g.pad_cedge[q]]++] = i;
   }
+  g.witem.clear();
+  g.wmulti.clear();
+  g.wmulti_ptr.assign(1, 0);
+  g.w_num_slots = 0;
+  for (int32_t c = 0; c < M; ++c) {
+    const int32_t e0 = g.cls_child_ptr[c], e1 = g.cls_child_ptr[c + 1];
+    if (e1 - e0 <= kWChunk) {
+      g.witem.insert(g.witem.end(), {c, e0, e1, -1});
+      continue;
+    }
+    for (int32_t e = e0; e < e1; e += kWChunk)
+      g.witem.insert(g.witem.end(), {c, e, std::min(e1, e + kWChunk), g.w_num_slots++});
+    g.wmulti.push_back(c);
+    g.wmulti_ptr.push_back(g.w_num_slots);
+  }
   // dmin_j: BFS depth of class j from the root over class -> child-class
   // edges (unreachable: INT32_MAX).  q^t_j is exactly 0 for t < dmin_j (q^0 =
   // e_root and each sweep extends the support by one edge), so the sweeps skip

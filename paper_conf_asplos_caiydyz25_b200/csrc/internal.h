@@ -42,6 +42,7 @@ constexpr int32_t kBigClass = 32;  // e-nodes above which a class gets a block (
 // their decode closures in 64-bit registers; larger ones take the global-memory
 // paths (batched fp64 GEMMs for the penalty, block-wide fixpoints for decode).
 constexpr int32_t kSmallScc = 64;
+constexpr int32_t kWChunk = 64;  // class edges per frozen-sweep work item
 
 // Max batches of 4 children per reverse-sweep item: 0 = from the graph's size
 // (HostGraph::rev_chunk: small graphs need short items to fill the GPU, large ones pay
@@ -95,6 +96,12 @@ struct HostGraph {
   // per class edge (i, j): its class i and the e-nodes k of m_i with j in ch_k
   // (ascending), CSR -- the rows of W are built one class edge at a time
   std::vector<int32_t> cedge_class, cedge_ptr, cedge_node;
+  // frozen-sweep work items [n][4] = (class, first edge, end edge, partial
+  // slot or -1): a class's edges in chunks of <= kWChunk (every class has at
+  // least one item; the first carries the S update), and the classes with
+  // several chunks, whose partial rows k_wcombine adds in item order
+  std::vector<int32_t> witem, wmulti, wmulti_ptr;
+  int32_t w_num_slots = 0;
   // classes with more than kBigClass e-nodes, largest first: the per-class
   // kernels (softmax, cost, update) give each a whole block
   std::vector<int32_t> big_class;
@@ -135,6 +142,8 @@ struct DevGraph {
   int32_t* pad_cedge = nullptr;
   int32_t *cedge_class = nullptr, *cedge_ptr = nullptr, *cedge_node = nullptr;
   int64_t num_cedge = 0;
+  int32_t *witem = nullptr, *wmulti = nullptr, *wmulti_ptr = nullptr;
+  int32_t num_witems = 0, num_wmulti = 0, w_num_slots = 0;
   int32_t* big_class = nullptr;
   int32_t* dmin = nullptr;
   int32_t *cls_child_ptr = nullptr, *cls_child = nullptr;
@@ -196,7 +205,7 @@ struct SweepState {
   // seed's frozen sweeps, the K-state rows kq / kpi / kam, wm [Bp] 1 while the
   // seed's rows still equal the K-state (env SMOOTHE_REV_W=0 disables).
   bool wmode = false;
-  float *W = nullptr, *S = nullptr, *kq = nullptr, *kpi = nullptr;
+  float *W = nullptr, *S = nullptr, *kq = nullptr, *kpi = nullptr, *wpart = nullptr;
   int32_t *kam = nullptr, *wm = nullptr;
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).

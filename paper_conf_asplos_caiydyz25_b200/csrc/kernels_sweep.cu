@@ -857,32 +857,41 @@ void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
 }
 
 constexpr int kWBlock = 64;
-// min resident blocks: 14 (<= 73 registers) for 128-seed rows (C4: 124.6 vs
-// 137.9 ms per step with 125 registers), none for narrower rows (C5: slower)
+// min resident blocks for 128-seed rows: 12 (<= 85 registers, no spills);
+// measured on C4 (ms per step): 10 -> 135.7, 12 -> 120.2, 14 -> 128.5, 16 ->
+// 147.4.  None for narrower rows (C5: slower).  DEPTH edges in flight per row group.
 #ifndef SMOOTHE_WSPMV_MINB
-#define SMOOTHE_WSPMV_MINB 14
+#define SMOOTHE_WSPMV_MINB 20
 #endif
-template <int LPR>
+#ifndef SMOOTHE_WSPMV_DEPTH
+#define SMOOTHE_WSPMV_DEPTH 6
+#endif
+#ifndef SMOOTHE_WSPMV_DEPTH32
+#define SMOOTHE_WSPMV_DEPTH32 4
+#endif
+template <int LPR, bool STREAM>
 __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k_wspmv(
-    int M, int Bp, int root, int t, const int32_t* __restrict__ dmin,
-    const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,
-    const float* __restrict__ W, const int32_t* __restrict__ wm, const float* __restrict__ gq,
-    float* __restrict__ S, float* __restrict__ gq_prev, int64_t* __restrict__ frozen_count) {
+    int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
+    const int32_t* __restrict__ cls_child, const float* __restrict__ W,
+    const int32_t* __restrict__ wm, const float* __restrict__ gq, float* __restrict__ S,
+    float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count) {
   const RowGroup<LPR, kWBlock> rg;
-  const int i = rg.row;
   if (frozen_count && blockIdx.x == 0 && threadIdx.x == 0) {  // profiling: a working launch?
     bool any = false;
     for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
     if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
   }
-  if (i >= M) return;
+  if (rg.row >= n_items) return;
   const int4 w4 = ld4i(wm + rg.s0);
   const unsigned gm = LPR == 32 ? 0xffffffffu
                                 : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
   if (!__any_sync(gm, (w4.x | w4.y | w4.z | w4.w) != 0)) return;  // row-group uniform
+  const int4 itm = items[rg.row];
+  const int i = itm.x, e0 = itm.y, e1 = itm.z, slot = itm.w;
   const int d = __ldg(dmin + i);
   const size_t oi = (size_t)i * Bp + rg.s0;
-  if (d <= t) {  // g_q^t_i is a valid row: S_i += g_q^t_i for the frozen seeds
+  if (d <= t && e0 == cls_child_ptr[i]) {  // first item: S_i += g_q^t_i (a valid row)
     const float4 gi = ld4(gq + oi);
     float4 si = ld4(S + oi);
 #pragma unroll
@@ -892,7 +901,6 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k
   }
   if (d > t - 1 || !gq_prev) return;  // q^{t-1}_i = 0: the row is never read
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-  const int e0 = cls_child_ptr[i], e1 = cls_child_ptr[i + 1];
   // the row group loads LPR child indices at once (one per lane, coalesced)
   // and broadcasts them, so the W rows (streamed) and g_q rows (gathered) of
   // 8 edges are in flight together without a dependent index load each
@@ -901,13 +909,14 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k
     const int n = min(LPR, e1 - c0);
     const int myj = gl < n ? __ldg(cls_child + c0 + gl) : 0;
     const float* wrow = W + (size_t)c0 * Bp + rg.s0;
-    for (int u = 0; u < n; u += 8) {  // 8 edges in flight; the last batch predicated
-      float4 wv[8], gv[8];
+    constexpr int DP = LPR == 32 ? SMOOTHE_WSPMV_DEPTH32 : SMOOTHE_WSPMV_DEPTH;
+    for (int u = 0; u < n; u += DP) {  // DP edges in flight; the last batch predicated
+      float4 wv[DP], gv[DP];
 #pragma unroll
-      for (int v = 0; v < 8; ++v) {
+      for (int v = 0; v < DP; ++v) {
         const int j = __shfl_sync(gm, myj, (u + v) & (LPR - 1), LPR);
         if (u + v < n) {
-          wv[v] = ldcs4(wrow + (size_t)(u + v) * Bp);
+          wv[v] = STREAM ? ldcs4(wrow + (size_t)(u + v) * Bp) : ld4(wrow + (size_t)(u + v) * Bp);
           gv[v] = ld4(gq + (size_t)j * Bp + rg.s0);
         } else {
           wv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -915,13 +924,17 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k
         }
       }
 #pragma unroll
-      for (int v = 0; v < 8; ++v) {
+      for (int v = 0; v < DP; ++v) {
         acc.x = fmaf(wv[v].x, gv[v].x, acc.x);
         acc.y = fmaf(wv[v].y, gv[v].y, acc.y);
         acc.z = fmaf(wv[v].z, gv[v].z, acc.z);
         acc.w = fmaf(wv[v].w, gv[v].w, acc.w);
       }
     }
+  }
+  if (slot >= 0) {  // one chunk of a long class: k_wcombine adds the chunks
+    st4(part + (size_t)slot * Bp + rg.s0, acc);
+    return;
   }
   if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 o = acc;
@@ -934,12 +947,61 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k
   st4(gq_prev + oi, o);
 }
 
+// g_q^{t-1}_i of the classes split into several chunks: their partial rows in
+// item order (deterministic)
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_wcombine(
+    int n_multi, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    const int32_t* __restrict__ wmulti, const int32_t* __restrict__ wmulti_ptr,
+    const int32_t* __restrict__ wm, const float* __restrict__ part, float* __restrict__ gq_prev) {
+  const RowGroup<LPR> rg;
+  if (rg.row >= n_multi) return;
+  const int4 w4 = ld4i(wm + rg.s0);
+  if (!(w4.x | w4.y | w4.z | w4.w)) return;
+  const int i = wmulti[rg.row];
+  if (__ldg(dmin + i) > t - 1) return;
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int sl = wmulti_ptr[rg.row]; sl < wmulti_ptr[rg.row + 1]; ++sl) {
+    const float4 p = ld4(part + (size_t)sl * Bp + rg.s0);
+    acc.x += p.x;
+    acc.y += p.y;
+    acc.z += p.z;
+    acc.w += p.w;
+  }
+  if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  const size_t oi = (size_t)i * Bp + rg.s0;
+  float4 o = acc;
+  if (!(w4.x && w4.y && w4.z && w4.w)) {
+    const float4 cur = ld4(gq_prev + oi);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (!comp(w4, x)) comp(o, x) = comp(cur, x);
+  }
+  st4(gq_prev + oi, o);
+}
+
 void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
                   const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count) {
+  // W streams from HBM once per sweep (evict-first) unless it fits in L2 with
+  // room to spare, where it stays resident across the frozen sweeps (C5: 69 MB)
+  const bool stream = (double)g.num_cedge * sh.Bp * sizeof(float) > 96e6;
+  const int4* items = reinterpret_cast<const int4*>(g.witem);
   SM_DISPATCH_LPR(sh.Bp, {
-    k_wspmv<LPR><<<row_grid(sh.M, sh.Bp, LPR, kWBlock), kWBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, t, g.dmin, g.cls_child_ptr, g.cls_child, st.W, st.wm, gq, st.S,
-        gq_prev, frozen_count);
+    const dim3 grid = row_grid(g.num_witems, sh.Bp, LPR, kWBlock);
+    if (stream)
+      k_wspmv<LPR, true><<<grid, kWBlock, 0, s>>>(
+          g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,
+          st.wm, gq, st.S, gq_prev, st.wpart, frozen_count);
+    else
+      k_wspmv<LPR, false><<<grid, kWBlock, 0, s>>>(
+          g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,
+          st.wm, gq, st.S, gq_prev, st.wpart, frozen_count);
+    if (g.num_wmulti > 0 && gq_prev) {
+      SM_LAUNCH_CHECK();
+      k_wcombine<LPR><<<row_grid(g.num_wmulti, sh.Bp, LPR), kBlock, 0, s>>>(
+          g.num_wmulti, sh.Bp, sh.root, t, g.dmin, g.wmulti, g.wmulti_ptr, st.wm, st.wpart,
+          gq_prev);
+    }
   });
   SM_LAUNCH_CHECK();
 }

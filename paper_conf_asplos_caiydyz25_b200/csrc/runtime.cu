@@ -416,6 +416,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       if (w.pistack) w.kpi = dalloc<float>(o, MB);
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
+      w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
       r->frozen_count = dalloc<int64_t>(o, 1);
       SM_CUDA(cudaMemset(r->frozen_count, 0, sizeof(int64_t)));
     }
@@ -620,6 +621,12 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       d.cedge_class = upload(o, h.cedge_class, &b);
       d.cedge_ptr = upload(o, h.cedge_ptr, &b);
       d.cedge_node = upload(o, h.cedge_node, &b);
+      d.witem = upload(o, h.witem, &b);
+      d.wmulti = upload(o, h.wmulti, &b);
+      d.wmulti_ptr = upload(o, h.wmulti_ptr, &b);
+      d.num_witems = (int32_t)(h.witem.size() / 4);
+      d.num_wmulti = (int32_t)h.wmulti.size();
+      d.w_num_slots = h.w_num_slots;
       d.num_cedge = (int64_t)h.cls_child.size();
       d.num_big = (int32_t)h.big_class.size();
       d.rev_item = upload(o, h.rev_item, &b);
