@@ -1,3 +1,6 @@
+#include <cstdlib>
+#include <cstdio>
+#include <chrono>
 // E-graph loader: validation, CSR/CSC, strongly connected components, K_auto.
 //
 // Problem statement: PAPER.md:91-101 (classes m_j, nodes n_i, ch_i, pa_j, ec(i)).
@@ -9,14 +12,31 @@
 
 #include "internal.h"
 
+namespace {
+// SMOOTHE_LOAD_TIMING=1: seconds per loader phase on stderr (diagnostic)
+struct LoadTimer {
+  bool on = std::getenv("SMOOTHE_LOAD_TIMING") != nullptr;
+  std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+  void operator()(const char* what) {
+    if (!on) return;
+    const auto n = std::chrono::steady_clock::now();
+    std::fprintf(stderr, "[load] %-22s %.4f s\n", what, std::chrono::duration<double>(n - t).count());
+    t = n;
+  }
+};
+}  // namespace
+
 namespace smoothe {
 
 namespace {
 
 // Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
+// Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
+// (A parallel two-pass version over ranges of classes measured slower here.)
 void class_successors(const HostGraph& g, std::vector<int32_t>& ptr, std::vector<int32_t>& adj) {
   ptr.assign(g.M + 1, 0);
   adj.clear();
+  adj.reserve(g.child_class.size());
   std::vector<int32_t> buf;
   for (int32_t j = 0; j < g.M; ++j) {
     buf.clear();
@@ -129,6 +149,7 @@ int32_t k_auto(const HostGraph& g, const std::vector<int32_t>& ptr, const std::v
 
 void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
                       const int32_t* child_class, int32_t root, HostGraph& g) {
+  LoadTimer lt;
   SM_REQUIRE(class_ptr && child_ptr && (child_class || child_ptr[N] == 0), SMOOTHE_E_INVALID_ARG,
              "NULL e-graph array");
   SM_REQUIRE(M > 0 && N > 0, SMOOTHE_E_INVALID_ARG, "num_classes and num_nodes must be > 0");
@@ -157,6 +178,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     for (int32_t i = class_ptr[j]; i < class_ptr[j + 1]; ++i) g.ec[i] = j;
     g.max_class_size = std::max(g.max_class_size, class_ptr[j + 1] - class_ptr[j]);
   }
+  lt("validate");
   // CSR children as sets
   g.child_ptr.assign(N + 1, 0);
   g.child_class.reserve(child_ptr[N]);
@@ -169,6 +191,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     g.child_ptr[i + 1] = (int32_t)g.child_class.size();
   }
   g.E = (int64_t)g.child_class.size();
+  lt("csr children");
   // CSC parents, by increasing e-node id
   g.par_ptr.assign(M + 1, 0);
   for (int32_t c : g.child_class) g.par_ptr[c + 1]++;
@@ -188,11 +211,13 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       }
   }
 
+  lt("csc parents");
   // strongly connected components of the class graph
   std::vector<int32_t> sptr, sadj;
   class_successors(g, sptr, sadj);
   g.cls_child_ptr = sptr;
   g.cls_child = sadj;
+  lt("scc");
   // hmax_j: the longest walk from class j in the class graph, i.e. the
   // largest L with g_q^{K-L}_j possibly non-zero in the reverse sweeps
   // (INT32_MAX when j can reach a cycle).  Kahn's algorithm on out-degrees:
@@ -265,6 +290,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       g.scc_class[fill[s]++] = j;
     }
   }
+  lt("hmax+scc lists");
   // Abar entries and penalty slots per component
   g.ent_ptr.assign(1, 0);
   g.ent_node_ptr.assign(1, 0);
@@ -316,6 +342,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   }
   g.K_auto = k_auto(g, sptr, sadj, comp);
 
+  lt("abar slots+k_auto");
   // decode schedule: condensation levels reachable from the root (Kahn order)
   {
     std::vector<std::vector<int32_t>> cadj(ncomp);
@@ -372,6 +399,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     }
   }
 
+  lt("decode levels");
   // padded sweep layouts (multiples of 4 entries per list)
   g.pad_child_ptr.assign(N + 1, 0);
   for (int32_t i = 0; i < N; ++i) {
@@ -386,17 +414,22 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     for (int32_t b = g.pad_child_ptr[i] / 4; b < g.pad_child_ptr[i + 1] / 4; ++b)
       g.pad_batch_node[b] = i;
   }
-  // class-edge index of every padded child slot (W rows of the frozen sweeps)
+  lt("padded layouts");
+  // class-edge index of every padded child slot (W rows of the frozen sweeps):
+  // per class, pos[child class] = its index in the class's successor list
   g.pad_cedge.assign(g.pad_child_ptr[N], -1);
-  for (int32_t i = 0; i < N; ++i) {
-    const int32_t c = g.ec[i];
-    const auto b = g.cls_child.begin() + g.cls_child_ptr[c];
-    const auto e = g.cls_child.begin() + g.cls_child_ptr[c + 1];
-    for (int32_t q = g.child_ptr[i]; q < g.child_ptr[i + 1]; ++q) {
-      const auto it = std::lower_bound(b, e, g.child_class[q]);
-      SM_REQUIRE(it != e && *it == g.child_class[q], SMOOTHE_E_BAD_GRAPH,
-                 "internal: class successor list misses a child");
-      g.pad_cedge[g.pad_child_ptr[i] + (q - g.child_ptr[i])] = (int32_t)(it - g.cls_child.begin());
+  {
+    std::vector<int32_t> pos(M, -1);
+    for (int32_t c = 0; c < M; ++c) {
+      for (int32_t e = g.cls_child_ptr[c]; e < g.cls_child_ptr[c + 1]; ++e) pos[g.cls_child[e]] = e;
+      for (int32_t i = g.class_ptr[c]; i < g.class_ptr[c + 1]; ++i)
+        for (int32_t q = g.child_ptr[i]; q < g.child_ptr[i + 1]; ++q) {
+          const int32_t e = pos[g.child_class[q]];
+          SM_REQUIRE(e >= g.cls_child_ptr[c] && e < g.cls_child_ptr[c + 1] &&
+                         g.cls_child[e] == g.child_class[q],
+                     SMOOTHE_E_BAD_GRAPH, "internal: class successor list misses a child");
+          g.pad_cedge[g.pad_child_ptr[i] + (q - g.child_ptr[i])] = e;
+        }
     }
   }
   {
@@ -430,6 +463,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     g.wmulti.push_back(c);
     g.wmulti_ptr.push_back(g.w_num_slots);
   }
+  lt("cedges+witems");
   // dmin_j: BFS depth of class j from the root over class -> child-class
   // edges (unreachable: INT32_MAX).  q^t_j is exactly 0 for t < dmin_j (q^0 =
   // e_root and each sweep extends the support by one edge), so the sweeps skip
@@ -460,6 +494,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     return g.class_ptr[a + 1] - g.class_ptr[a] > g.class_ptr[b + 1] - g.class_ptr[b];
   });
 
+  lt("dmin");
   // reverse-sweep work items: runs of <= kRevChunk batches of one class, cut at
   // e-node boundaries; an e-node with more batches is cut into pieces of its own
   {
@@ -523,6 +558,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
       g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
     }
+  lt("rev items+pad parents");
 }
 
 }  // namespace smoothe

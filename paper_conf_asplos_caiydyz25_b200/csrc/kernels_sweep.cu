@@ -595,11 +595,15 @@ __device__ __forceinline__ void reverse_epilogue(
 // first rows are requested right after the header arrives.  (Persistent warps
 // striding over items, with the next item staged by cp.async, measured 2.3x
 // slower on C4: the in-flight window of classes spreads and L2 reuse drops.)
+#ifndef SMOOTHE_REV_BLOCK
+#define SMOOTHE_REV_BLOCK 64  // threads per block (one item per warp)
+#endif
+constexpr int kRevBlock = SMOOTHE_REV_BLOCK;
 #ifndef SMOOTHE_REV_MINB4
-#define SMOOTHE_REV_MINB4 6  // min resident 64-thread blocks per SM at V = 4
+#define SMOOTHE_REV_MINB4 (6 * 64 / SMOOTHE_REV_BLOCK)  // min resident blocks per SM at V = 4
 #endif
 template <int V, bool HI, bool HC>
-__global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k_sweep_reverse(
+__global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64 / kRevBlock) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
     const int32_t* __restrict__ pad_batch_node, float wI, float wC, const float* __restrict__ cp,
@@ -607,7 +611,7 @@ __global__ void __launch_bounds__(kSweepBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8) k
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
     float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
     const int32_t* __restrict__ wm) {
-  const int it = blockIdx.x * (kSweepBlock / 32) + (int)threadIdx.x / 32;
+  const int it = blockIdx.x * (kRevBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
   // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
@@ -768,9 +772,9 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   // cp / g_cp rows are L2-prefetched per item only when they cannot stay
   // L2-resident (measured: +7% on C4 at 512 MB, -9% on C3 at 13 MB)
   const bool l2_prefetch = (double)sh.N * sh.Bp * sizeof(float) > 64e6;
-  const dim3 grid((n + kSweepBlock / 32 - 1) / (kSweepBlock / 32), sh.Bp / (32 * V));
+  const dim3 grid((n + kRevBlock / 32 - 1) / (kRevBlock / 32), sh.Bp / (32 * V));
 #define SM_REV2(VV, HI, HC)                                                                    \
-  k_sweep_reverse<VV, HI, HC><<<grid, kSweepBlock, 0, s>>>(                                   \
+  k_sweep_reverse<VV, HI, HC><<<grid, kRevBlock, 0, s>>>(                                   \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,             \
       rev_part, rev_cnt, l2_prefetch, t, K, wm)
@@ -856,7 +860,10 @@ void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
   SM_LAUNCH_CHECK();
 }
 
-constexpr int kWBlock = 64;
+#ifndef SMOOTHE_WSPMV_BLOCK
+#define SMOOTHE_WSPMV_BLOCK 64
+#endif
+constexpr int kWBlock = SMOOTHE_WSPMV_BLOCK;
 // min resident blocks for 128-seed rows: 12 (<= 85 registers, no spills);
 // measured on C4 (ms per step): 10 -> 135.7, 12 -> 120.2, 14 -> 128.5, 16 ->
 // 147.4.  None for narrower rows (C5: slower).  DEPTH edges in flight per row group.
@@ -870,7 +877,7 @@ constexpr int kWBlock = 64;
 #define SMOOTHE_WSPMV_DEPTH32 4
 #endif
 template <int LPR, bool STREAM>
-__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB : 1) k_wspmv(
+__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : 1) k_wspmv(
     int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
     const int32_t* __restrict__ cls_child, const float* __restrict__ W,
