@@ -212,6 +212,8 @@ def test_large_scc(sm, orc, p_back, G):
 
 
 @pytest.mark.parametrize("name,B,G,K,agg", [("C2", 64, 8, 80, "hybrid"),
+                                             ("C2", 100, 10, 80, "hybrid"),
+                                             ("C2", 200, 8, 70, "hybrid"),
                                              ("C2", 64, 8, 80, "independent"),
                                              ("C2", 64, 8, 80, "correlated"),
                                              ("C3", 32, 8, 60, "hybrid")])
