@@ -16,6 +16,8 @@
 // class, each class once, accumulated in fp64 (exact for integer-valued u).
 #include <cooperative_groups.h>
 
+#include <cstdlib>
+
 #include "kcommon.cuh"
 
 namespace cg = cooperative_groups;
@@ -244,7 +246,9 @@ void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const D
 int decode_grid(int device) {
   int per_sm = 0;
   SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decode_levels, 256, 0));
-  return std::max(1, std::min(per_sm, 4)) * num_sms(device);
+  const char* e = std::getenv("SMOOTHE_DECODE_BPS");  // blocks per SM (A/B)
+  const int want = e ? std::max(1, std::atoi(e)) : 2;  // 2: measured best with the decode overlapped
+  return std::max(1, std::min(per_sm, want)) * num_sms(device);
 }
 
 // Discrete linear cost per seed: part[blockIdx.x][b] = sum over the block's

@@ -82,6 +82,13 @@ struct smoothe_run {
   int coop_grid = 0, f_rows = 0, dcost_rows = 0, rows_M = 0, rows_N = 0;
   Agg agg{0.f, 0.f};
   cudaStream_t stream = nullptr;
+  // decode / keep-best run on a second stream, concurrently with the sweeps of
+  // the same step (they only need the step's choices), joined at the step end
+  cudaStream_t stream2 = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  bool overlap = false;
+  double* red_scratch_d = nullptr;  // the decode stream's own reduction / cost scratch
+  float *f_part_d = nullptr, *z1_part_d = nullptr, *z1_d = nullptr;
   std::vector<void*> owned;
   // state
   float *theta = nullptr, *m = nullptr, *v = nullptr, *cp = nullptr, *gcp = nullptr;
@@ -195,6 +202,41 @@ struct PhaseMarks {
   }
 };
 
+// Decode (P279, P103-111), its discrete cost and keep-best (P297) on stream ds.
+// With the decode stream (overlap), it uses its own scratch buffers.
+void enqueue_decode(smoothe_run* r, cudaStream_t ds, PhaseMarks* pm) {
+  const Shape& sh = r->sh;
+  const DevGraph& g = r->g->dev;
+  const HostGraph& hg = r->g->host;
+  const bool side = ds != r->stream;
+  double* red = side ? r->red_scratch_d : r->red_scratch;
+  float* fpart = side ? r->f_part_d : r->f_part;
+  float* z1p = side ? r->z1_part_d : r->z1_part;
+  float* z1 = side ? r->z1_d : r->z1;
+  launch_decode(ds, sh, hg, g, r->sel, r->choice, r->reach, r->settle, r->invalid,
+                r->settle + (size_t)sh.root * sh.W, r->coop_grid);
+  launch_decode_cost_linear(ds, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
+  launch_reduce_rows_f64d(ds, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost, red);
+  const double* dextra = nullptr;
+  if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
+    launch_decode_s(ds, sh, g, r->sel, r->reach, r->sbin);
+    launch_quadratic(ds, sh, r->q_ptr, r->q_nbr, r->q_w, nullptr, r->sbin, nullptr, fpart);
+    launch_reduce_rows_f64(ds, fpart, r->rows_N, sh.Bp, r->dextra, 1.0, red);
+    dextra = r->dextra;
+  } else if (r->cost_kind == SMOOTHE_COST_MLP) {
+    launch_decode_s(ds, sh, g, r->sel, r->reach, r->sbin);
+    launch_mlp_fwd(ds, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
+                   z1p, z1, r->dextra, nullptr, r->nsplit);
+    dextra = r->dextra;
+  }
+  if (pm) pm->mark(SMOOTHE_PHASE_BEST);
+  launch_best_update(ds, sh, r->settle, r->dcost, dextra, r->opt.seed_begin, r->counter, r->best,
+                     r->best_flag, r->debug ? r->dbg_dcost : nullptr,
+                     r->debug ? r->dbg_valid : nullptr);
+  launch_best_snapshot(ds, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
+                       r->best_choice);
+}
+
 void enqueue_step(smoothe_run* r) {
   const Shape& sh = r->sh;
   const DevGraph& g = r->g->dev;
@@ -208,6 +250,13 @@ void enqueue_step(smoothe_run* r) {
   pm.mark(SMOOTHE_PHASE_SOFTMAX);
   launch_step_prologue(s, r->counter, r->scal, r->opt.beta1, r->opt.beta2, nullptr);
   launch_softmax_argmax(s, sh, g, r->theta, r->cp, r->choice, r->sel);
+  const bool overlap_now = r->overlap && !r->profiling && !r->debug;
+  if (overlap_now) {  // decode this step's choices alongside the sweeps
+    SM_CUDA(cudaEventRecord(r->ev_fork, s));
+    SM_CUDA(cudaStreamWaitEvent(r->stream2, r->ev_fork, 0));
+    enqueue_decode(r, r->stream2, nullptr);
+    SM_CUDA(cudaEventRecord(r->ev_join, r->stream2));
+  }
 
   pm.mark(SMOOTHE_PHASE_FORWARD);
   launch_sweep_reset(s, sh, r->sw);
@@ -305,30 +354,12 @@ void enqueue_step(smoothe_run* r) {
                 (float)r->opt.beta2, (float)r->opt.eps, r->debug ? r->dbg_gth : nullptr,
                 r->debug ? r->dbg_gcp : nullptr);
 
-  pm.mark(SMOOTHE_PHASE_DECODE);
-  launch_decode(s, sh, hg, g, r->sel, r->choice, r->reach, r->settle, r->invalid,
-                r->settle + (size_t)sh.root * sh.W, r->coop_grid);
-  launch_decode_cost_linear(s, sh, g, r->u_d, r->choice, r->reach, r->dcost_part);
-  launch_reduce_rows_f64d(s, r->dcost_part, r->dcost_rows, sh.Bp, r->dcost, r->red_scratch);
-  const double* dextra = nullptr;
-  if (r->cost_kind == SMOOTHE_COST_QUADRATIC) {
-    launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
-    launch_quadratic(s, sh, r->q_ptr, r->q_nbr, r->q_w, nullptr, r->sbin, nullptr, r->f_part);
-    launch_reduce_rows_f64(s, r->f_part, r->rows_N, sh.Bp, r->dextra, 1.0, r->red_scratch);
-    dextra = r->dextra;
-  } else if (r->cost_kind == SMOOTHE_COST_MLP) {
-    launch_decode_s(s, sh, g, r->sel, r->reach, r->sbin);
-    launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
-                   r->z1_part, r->z1, r->dextra, nullptr, r->nsplit);
-    dextra = r->dextra;
+  if (!overlap_now) {
+    pm.mark(SMOOTHE_PHASE_DECODE);
+    enqueue_decode(r, s, &pm);
+  } else {
+    SM_CUDA(cudaStreamWaitEvent(s, r->ev_join, 0));
   }
-
-  pm.mark(SMOOTHE_PHASE_BEST);
-  launch_best_update(s, sh, r->settle, r->dcost, dextra, r->opt.seed_begin, r->counter, r->best,
-                     r->best_flag, r->debug ? r->dbg_dcost : nullptr,
-                     r->debug ? r->dbg_valid : nullptr);
-  launch_best_snapshot(s, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
-                       r->best_choice);
   pm.finish();
   if (r->profiling) {
     r->prof_launch_total += launch_counter() - l0;
@@ -432,6 +463,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     r->rows_N = (sh.N + per - 1) / per;
   }
   r->f_part = dalloc<float>(o, (size_t)r->f_rows * sh.Bp);
+  if (r->overlap) r->f_part_d = dalloc<float>(o, (size_t)r->f_rows * sh.Bp);
   r->f = dalloc<double>(o, sh.Bp);
   r->fextra = dalloc<double>(o, sh.Bp);
   r->ftot = dalloc<double>(o, sh.Bp);
@@ -459,6 +491,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->counter = dalloc<int32_t>(o, 1);
   r->scal = dalloc<double>(o, 2);
   r->red_scratch = dalloc<double>(o, (size_t)128 * sh.Bp);
+  if (r->overlap) r->red_scratch_d = dalloc<double>(o, (size_t)128 * sh.Bp);
   r->rev_part = dalloc<float>(o, (size_t)std::max(1, r->g->dev.rev_num_slots) * sh.Bp);
   r->rev_cnt = dalloc<int32_t>(o, (size_t)sh.M * std::max(1, sh.Bp / 32));  // per (class, warp seed slice)
   r->dbg_p = nullptr;
@@ -506,6 +539,10 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     r->nsplit = mlp_nsplit(r->device);
     r->z1_part = dalloc<float>(o, (size_t)r->nsplit * 128 * sh.Bp);
     r->z1 = dalloc<float>(o, (size_t)H1 * sh.Bp);
+    if (r->overlap) {
+      r->z1_part_d = dalloc<float>(o, (size_t)r->nsplit * 128 * sh.Bp);
+      r->z1_d = dalloc<float>(o, (size_t)H1 * sh.Bp);
+    }
     r->gz1 = dalloc<float>(o, (size_t)H1 * sh.Bp);
   }
 }
@@ -828,6 +865,15 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
       r->H2 = cost->mlp_hidden2;
     }
     SM_CUDA(cudaStreamCreateWithFlags(&r->stream, cudaStreamNonBlocking));
+    {
+      const char* ov = std::getenv("SMOOTHE_DECODE_OVERLAP");
+      r->overlap = !(ov && ov[0] == '0');
+    }
+    if (r->overlap) {
+      SM_CUDA(cudaStreamCreateWithFlags(&r->stream2, cudaStreamNonBlocking));
+      SM_CUDA(cudaEventCreateWithFlags(&r->ev_fork, cudaEventDisableTiming));
+      SM_CUDA(cudaEventCreateWithFlags(&r->ev_join, cudaEventDisableTiming));
+    }
     r->coop_grid = decode_grid(r->device);
     alloc_state(r, cost);
     SM_CUDA(cudaEventCreate(&r->ev_start));
@@ -1129,6 +1175,9 @@ void smoothe_free_run(smoothe_run* run) {
   for (auto e : run->prof_pool) cudaEventDestroy(e);
   if (run->ev_start) cudaEventDestroy(run->ev_start);
   if (run->stream) cudaStreamDestroy(run->stream);
+  if (run->stream2) cudaStreamDestroy(run->stream2);
+  if (run->ev_fork) cudaEventDestroy(run->ev_fork);
+  if (run->ev_join) cudaEventDestroy(run->ev_join);
   if (run->g) {
     run->g->refcount--;
     if (run->g->freed && run->g->refcount == 0) smoothe_free_egraph(run->g);
