@@ -85,7 +85,7 @@ struct smoothe_run {
   // decode / keep-best run on a second stream, concurrently with the sweeps of
   // the same step (they only need the step's choices), joined at the step end
   cudaStream_t stream2 = nullptr;
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_pen = nullptr;
   bool overlap = false;
   double* red_scratch_d = nullptr;  // the decode stream's own reduction / cost scratch
   float *f_part_d = nullptr, *z1_part_d = nullptr, *z1_d = nullptr;
@@ -251,9 +251,16 @@ void enqueue_step(smoothe_run* r) {
   launch_step_prologue(s, r->counter, r->scal, r->opt.beta1, r->opt.beta2, nullptr);
   launch_softmax_argmax(s, sh, g, r->theta, r->cp, r->choice, r->sel);
   const bool overlap_now = r->overlap && !r->profiling && !r->debug;
-  if (overlap_now) {  // decode this step's choices alongside the sweeps
+  if (overlap_now) {  // penalty and decode of this step alongside the sweeps
     SM_CUDA(cudaEventRecord(r->ev_fork, s));
     SM_CUDA(cudaStreamWaitEvent(r->stream2, r->ev_fork, 0));
+    if (hg.num_scc > 0) {  // needs cp only; joined before the loss
+      launch_notears(r->stream2, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen,
+                     r->big_scratch, r->big_gpb);
+      launch_reduce_rows_f64d(r->stream2, r->h_part, hg.num_scc, r->ngroups, r->h,
+                              r->red_scratch_d);
+      SM_CUDA(cudaEventRecord(r->ev_pen, r->stream2));
+    }
     enqueue_decode(r, r->stream2, nullptr);
     SM_CUDA(cudaEventRecord(r->ev_join, r->stream2));
   }
@@ -295,7 +302,9 @@ void enqueue_step(smoothe_run* r) {
   }
 
   pm.mark(SMOOTHE_PHASE_PENALTY);
-  if (hg.num_scc > 0) {
+  if (overlap_now && hg.num_scc > 0) {
+    SM_CUDA(cudaStreamWaitEvent(s, r->ev_pen, 0));  // computed on the second stream
+  } else if (hg.num_scc > 0) {
     launch_notears(s, sh, hg, g, r->G, r->opt.lambda, r->cp, r->h_part, r->pen, r->big_scratch,
                    r->big_gpb);
     launch_reduce_rows_f64d(s, r->h_part, hg.num_scc, r->ngroups, r->h, r->red_scratch);
@@ -873,6 +882,7 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
       SM_CUDA(cudaStreamCreateWithFlags(&r->stream2, cudaStreamNonBlocking));
       SM_CUDA(cudaEventCreateWithFlags(&r->ev_fork, cudaEventDisableTiming));
       SM_CUDA(cudaEventCreateWithFlags(&r->ev_join, cudaEventDisableTiming));
+      SM_CUDA(cudaEventCreateWithFlags(&r->ev_pen, cudaEventDisableTiming));
     }
     r->coop_grid = decode_grid(r->device);
     alloc_state(r, cost);
@@ -1178,6 +1188,7 @@ void smoothe_free_run(smoothe_run* run) {
   if (run->stream2) cudaStreamDestroy(run->stream2);
   if (run->ev_fork) cudaEventDestroy(run->ev_fork);
   if (run->ev_join) cudaEventDestroy(run->ev_join);
+  if (run->ev_pen) cudaEventDestroy(run->ev_pen);
   if (run->g) {
     run->g->refcount--;
     if (run->g->freed && run->g->refcount == 0) smoothe_free_egraph(run->g);
