@@ -281,6 +281,28 @@ def test_graphs_and_direct_launches_identical(sm):
     assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
 
 
+@pytest.mark.parametrize("name,B,G", [("C2", 64, 8), ("C3", 32, 8), ("C5", 64, 8)])
+def test_decode_overlap_identical(sm, monkeypatch, name, B, G):
+    """Penalty and decode on the second stream give the
+    same bits as the sequential step: theta, the best extraction and its
+    step / seed (quadratic and MLP configs use the decode stream's own
+    scratch buffers)."""
+    eg = make_config(name)
+    outs = []
+    for ov in ("1", "0"):
+        monkeypatch.setenv("SMOOTHE_DECODE_OVERLAP", ov)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=13))
+        run.steps(8)
+        outs.append((run.theta(), run.extract()))
+        run.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][1][0], outs[1][1][0])
+    for k in ("best_cost", "best_step", "best_seed", "last_loss"):
+        assert outs[0][1][1][k] == outs[1][1][1][k], k
+
+
 @pytest.mark.parametrize("name,B,G,agg,steps", [
     ("C2", 64, 8, "hybrid", 6), ("C2", 32, 8, "independent", 6), ("C3", 32, 8, "correlated", 6),
     ("C5", 256, 8, "hybrid", 6), ("C4", 32, 16, "hybrid", 3)])
