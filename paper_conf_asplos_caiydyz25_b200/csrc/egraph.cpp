@@ -31,23 +31,43 @@ namespace smoothe {
 namespace {
 
 // Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
-// Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
-// (A parallel two-pass version over ranges of classes measured slower here.)
+// Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique):
+// duplicates dropped with a per-class stamp, then the (short) unique list sorted.
 void class_successors(const HostGraph& g, std::vector<int32_t>& ptr, std::vector<int32_t>& adj) {
   ptr.assign(g.M + 1, 0);
   adj.clear();
   adj.reserve(g.child_class.size());
-  std::vector<int32_t> buf;
+  std::vector<int32_t> stamp(g.M, -1);
   for (int32_t j = 0; j < g.M; ++j) {
-    buf.clear();
+    const size_t b = adj.size();
     for (int32_t k = g.class_ptr[j]; k < g.class_ptr[j + 1]; ++k)
-      buf.insert(buf.end(), g.child_class.begin() + g.child_ptr[k],
-                 g.child_class.begin() + g.child_ptr[k + 1]);
-    std::sort(buf.begin(), buf.end());
-    buf.erase(std::unique(buf.begin(), buf.end()), buf.end());
-    adj.insert(adj.end(), buf.begin(), buf.end());
+      for (int32_t e = g.child_ptr[k]; e < g.child_ptr[k + 1]; ++e) {
+        const int32_t c = g.child_class[e];
+        if (stamp[c] != j) {
+          stamp[c] = j;
+          adj.push_back(c);
+        }
+      }
+    std::sort(adj.begin() + b, adj.end());
     ptr[j + 1] = (int32_t)adj.size();
   }
+}
+
+// Condensation adjacency as CSR (component -> components of its classes'
+// successors, duplicates kept: harmless for longest paths and Kahn's order).
+void condensation_csr(int32_t M, int32_t nc, const std::vector<int32_t>& ptr,
+                      const std::vector<int32_t>& adj, const std::vector<int32_t>& comp,
+                      std::vector<int32_t>& cptr, std::vector<int32_t>& cadj) {
+  cptr.assign(nc + 1, 0);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t e = ptr[j]; e < ptr[j + 1]; ++e)
+      if (comp[adj[e]] != comp[j]) cptr[comp[j] + 1]++;
+  for (int32_t a = 0; a < nc; ++a) cptr[a + 1] += cptr[a];
+  cadj.assign(cptr[nc], 0);
+  std::vector<int32_t> fill(cptr.begin(), cptr.end() - 1);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t e = ptr[j]; e < ptr[j + 1]; ++e)
+      if (comp[adj[e]] != comp[j]) cadj[fill[comp[j]]++] = comp[adj[e]];
 }
 
 // Kosaraju: finish order on the graph, then components on the transpose.
@@ -111,15 +131,8 @@ int32_t k_auto(const HostGraph& g, const std::vector<int32_t>& ptr, const std::v
   int32_t nc = 0;
   for (int32_t c : comp) nc = std::max(nc, c + 1);
   // condensation adjacency (duplicates are harmless for a longest path)
-  std::vector<int32_t> cptr(nc + 1, 0), cadj;
-  std::vector<std::vector<int32_t>> tmp(nc);
-  for (int32_t j = 0; j < g.M; ++j)
-    for (int32_t e = ptr[j]; e < ptr[j + 1]; ++e)
-      if (comp[adj[e]] != comp[j]) tmp[comp[j]].push_back(comp[adj[e]]);
-  for (int32_t a = 0; a < nc; ++a) {
-    cadj.insert(cadj.end(), tmp[a].begin(), tmp[a].end());
-    cptr[a + 1] = (int32_t)cadj.size();
-  }
+  std::vector<int32_t> cptr, cadj;
+  condensation_csr(g.M, nc, ptr, adj, comp, cptr, cadj);
   // height(a) = longest path starting at a; the answer is height(root component)
   std::vector<int32_t> height(nc, -1);
   std::vector<std::pair<int32_t, int32_t>> st;
@@ -345,31 +358,30 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   lt("abar slots+k_auto");
   // decode schedule: condensation levels reachable from the root (Kahn order)
   {
-    std::vector<std::vector<int32_t>> cadj(ncomp);
-    for (int32_t j = 0; j < M; ++j)
-      for (int32_t e = sptr[j]; e < sptr[j + 1]; ++e)
-        if (comp[sadj[e]] != comp[j]) cadj[comp[j]].push_back(comp[sadj[e]]);
+    std::vector<int32_t> cptr, cadj;
+    condensation_csr(M, ncomp, sptr, sadj, comp, cptr, cadj);
     std::vector<uint8_t> seen(ncomp, 0);
     std::vector<int32_t> stack{comp[root]};
     seen[comp[root]] = 1;
     while (!stack.empty()) {
       const int32_t a = stack.back();
       stack.pop_back();
-      for (int32_t b : cadj[a])
-        if (!seen[b]) {
-          seen[b] = 1;
-          stack.push_back(b);
+      for (int32_t e = cptr[a]; e < cptr[a + 1]; ++e)
+        if (!seen[cadj[e]]) {
+          seen[cadj[e]] = 1;
+          stack.push_back(cadj[e]);
         }
     }
     std::vector<int32_t> indeg(ncomp, 0), depth(ncomp, -1), order;
     for (int32_t a = 0; a < ncomp; ++a)
       if (seen[a])
-        for (int32_t b : cadj[a]) indeg[b]++;
+        for (int32_t e = cptr[a]; e < cptr[a + 1]; ++e) indeg[cadj[e]]++;
     order.push_back(comp[root]);
     depth[comp[root]] = 0;
     for (size_t i = 0; i < order.size(); ++i) {
       const int32_t a = order[i];
-      for (int32_t b : cadj[a]) {
+      for (int32_t e = cptr[a]; e < cptr[a + 1]; ++e) {
+        const int32_t b = cadj[e];
         depth[b] = std::max(depth[b], depth[a] + 1);
         if (--indeg[b] == 0) order.push_back(b);
       }
