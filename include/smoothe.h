@@ -284,6 +284,11 @@ SMOOTHE_API smoothe_status smoothe_run_get_profile(smoothe_run *run, smoothe_pro
 SMOOTHE_API const char *smoothe_last_error(void);
 SMOOTHE_API const char *smoothe_version(void);
 SMOOTHE_API void smoothe_free_run(smoothe_run *run);
+/* smoothe_free_run keeps the freed run's device blocks (per device, the last
+ * freed run's only) for the next run of the same shape; this returns them to
+ * the driver.  device_ordinal -1: every device.  (Allocation failures release
+ * the cache of the device by themselves.) */
+SMOOTHE_API void smoothe_release_cached_memory(int device_ordinal);
 SMOOTHE_API void smoothe_free_egraph(smoothe_egraph *g);
 
 #ifdef __cplusplus

@@ -4,4 +4,5 @@ The product is libsmoothe.so (C ABI: include/smoothe.h); this package is its
 thin Python binding plus the multi-GPU driver (torch.distributed).
 """
 from .smoothe import (CostModel, EGraph, Options, Run, SmootheError, extract, lib,  # noqa: F401
-                      load_egraph, load_egraph_from, optimize, run_create, torch_stream, version)
+                      load_egraph, load_egraph_from, optimize, release_cached_memory, run_create,
+                      torch_stream, version)

@@ -159,6 +159,7 @@ struct DevGraph {
 struct smoothe_egraph {
   smoothe::HostGraph host;
   smoothe::DevGraph dev;
+  std::vector<void*> owned;  // device allocations (one arena)
   int device = -1;
   int refcount = 1;  // the handle itself + one per live run
   bool freed = false;

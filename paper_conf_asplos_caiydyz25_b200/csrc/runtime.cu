@@ -22,6 +22,7 @@
 #include <cstring>
 #include <mutex>
 #include <new>
+#include <map>
 
 #include "internal.h"
 
@@ -66,6 +67,111 @@ static T* upload(std::vector<void*>& owned, const std::vector<T>& v, int64_t* by
   return d;
 }
 
+// One device allocation for all arrays of an e-graph: run the upload sequence
+// once to measure (base == nullptr), allocate, run it again to copy.
+struct Arena {
+  char* base = nullptr;
+  size_t used = 0;
+};
+
+template <typename T>
+static T* upload(Arena& A, const std::vector<T>& v, int64_t* bytes = nullptr) {
+  const size_t off = (A.used + 255) & ~(size_t)255;
+  A.used = off + std::max<size_t>(1, v.size()) * sizeof(T);
+  if (!A.base) return nullptr;
+  T* d = reinterpret_cast<T*>(A.base + off);
+  if (!v.empty()) SM_CUDA(cudaMemcpy(d, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
+  if (bytes) *bytes += (int64_t)(v.size() * sizeof(T));
+  return d;
+}
+
+// Caching allocator for run state: a freed run's device blocks are kept (per
+// device, the last freed run only) and handed to the next run that asks for
+// blocks of the same sizes, so back-to-back runs of one configuration do not
+// pay for unmapping and mapping tens of GB.  On an allocation failure the cache
+// of the device is released and the allocation retried.
+struct DevCache {
+  std::mutex mu;
+  std::multimap<std::pair<int, size_t>, void*> blocks;
+};
+DevCache& dev_cache() {
+  static DevCache c;
+  return c;
+}
+void cache_release(int device) {
+  DevCache& c = dev_cache();
+  std::lock_guard<std::mutex> lk(c.mu);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  for (auto it = c.blocks.begin(); it != c.blocks.end();) {
+    if (device < 0 || it->first.first == device) {
+      cudaSetDevice(it->first.first);
+      cudaFree(it->second);
+      it = c.blocks.erase(it);
+    } else {
+      ++it;
+    }
+  }
+  cudaSetDevice(cur);
+}
+
+struct RunMem {
+  std::vector<void*> p;
+  std::vector<size_t> n;
+  int device = 0;
+};
+
+template <typename T>
+static T* dalloc(RunMem& m, size_t count) {
+  if (count == 0) count = 1;
+  const size_t bytes = count * sizeof(T);
+  {
+    DevCache& c = dev_cache();
+    std::lock_guard<std::mutex> lk(c.mu);
+    auto it = c.blocks.find({m.device, bytes});
+    if (it != c.blocks.end()) {
+      void* q = it->second;
+      c.blocks.erase(it);
+      m.p.push_back(q);
+      m.n.push_back(bytes);
+      return static_cast<T*>(q);
+    }
+  }
+  void* q = nullptr;
+  cudaError_t e = cudaMalloc(&q, bytes);
+  if (e == cudaErrorMemoryAllocation) {
+    (void)cudaGetLastError();
+    cache_release(m.device);
+    e = cudaMalloc(&q, bytes);
+  }
+  if (e == cudaErrorMemoryAllocation) {
+    (void)cudaGetLastError();
+    throw Failure{SMOOTHE_E_OOM, "cudaMalloc of " + std::to_string(bytes) + " bytes failed"};
+  }
+  SM_CUDA(e);
+  m.p.push_back(q);
+  m.n.push_back(bytes);
+  return static_cast<T*>(q);
+}
+
+template <typename T>
+static T* upload(RunMem& m, const std::vector<T>& v, int64_t* bytes = nullptr) {
+  T* d = dalloc<T>(m, v.size());
+  if (!v.empty()) SM_CUDA(cudaMemcpy(d, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice));
+  if (bytes) *bytes += (int64_t)(v.size() * sizeof(T));
+  return d;
+}
+
+// a freed run's blocks replace the device's cache
+void runmem_recycle(RunMem& m) {
+  cache_release(m.device);
+  DevCache& c = dev_cache();
+  std::lock_guard<std::mutex> lk(c.mu);
+  for (size_t i = 0; i < m.p.size(); ++i) c.blocks.insert({{m.device, m.n[i]}, m.p[i]});
+  m.p.clear();
+  m.n.clear();
+}
+
 }  // namespace smoothe
 
 using namespace smoothe;
@@ -89,7 +195,7 @@ struct smoothe_run {
   bool overlap = false;
   double* red_scratch_d = nullptr;  // the decode stream's own reduction / cost scratch
   float *f_part_d = nullptr, *z1_part_d = nullptr, *z1_d = nullptr;
-  std::vector<void*> owned;
+  RunMem owned;  // device state (recycled through the caching allocator)
   // state
   float *theta = nullptr, *m = nullptr, *v = nullptr, *cp = nullptr, *gcp = nullptr;
   SweepState sw;  // q / pi / am version stacks, q buffers, change stamps
@@ -612,9 +718,18 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
   *out = nullptr;
   smoothe_egraph* g = nullptr;
   auto owner = new (std::nothrow) smoothe_egraph_dev_owner();
+  const bool timing = std::getenv("SMOOTHE_LOAD_TIMING") != nullptr;
+  auto t0 = std::chrono::steady_clock::now();
+  auto lap = [&](const char* what) {
+    if (!timing) return;
+    const auto t1 = std::chrono::steady_clock::now();
+    std::fprintf(stderr, "[load] %-22s %.4f s\n", what, std::chrono::duration<double>(t1 - t0).count());
+    t0 = t1;
+  };
   smoothe_status st = guarded(nullptr, [&] {
     g = new smoothe_egraph();
     build_host_graph(num_classes, num_nodes, class_ptr, child_ptr, child_class, root_class, g->host);
+    lap("host analysis (total)");
     g->device = device_ordinal;
     if (device_ordinal >= 0) {
       int ndev = 0;
@@ -626,63 +741,73 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       SM_REQUIRE(prop.major == 10, SMOOTHE_E_CUDA,
                  "libsmoothe is built for sm_100a; device has sm_" + std::to_string(prop.major) +
                      std::to_string(prop.minor));
-      auto& o = owner->owned;
+      lap("device query");
       const HostGraph& h = g->host;
       DevGraph& d = g->dev;
       int64_t& b = d.bytes;
-      d.class_ptr = upload(o, h.class_ptr, &b);
-      d.child_ptr = upload(o, h.child_ptr, &b);
-      {  // padded with the root id so batched kernels may read up to 8 past E
-        std::vector<int32_t> padded(h.child_class);
-        padded.resize(h.child_class.size() + 8, h.root);
-        d.child_class = upload(o, padded, &b);
-      }
-      d.par_ptr = upload(o, h.par_ptr, &b);
-      d.par_node = upload(o, h.par_node, &b);
-      d.par_class = upload(o, h.par_class, &b);
-      d.scc_class_ptr = upload(o, h.scc_class_ptr, &b);
-      d.scc_class = upload(o, h.scc_class, &b);
-      d.scc_of_class = upload(o, h.scc_of_class, &b);
-      d.ent_ptr = upload(o, h.ent_ptr, &b);
-      d.ent_i = upload(o, h.ent_i, &b);
-      d.ent_j = upload(o, h.ent_j, &b);
-      d.ent_node_ptr = upload(o, h.ent_node_ptr, &b);
-      d.ent_node = upload(o, h.ent_node, &b);
-      d.slot_ptr = upload(o, h.slot_ptr, &b);
-      d.slot_node = upload(o, h.slot_node, &b);
-      d.slot_iloc = upload(o, h.slot_iloc, &b);
-      d.slot_jptr = upload(o, h.slot_jptr, &b);
-      d.slot_jloc = upload(o, h.slot_jloc, &b);
-      d.node_slot = upload(o, h.node_slot, &b);
-      d.pad_child_ptr = upload(o, h.pad_child_ptr, &b);
-      d.pad_child = upload(o, h.pad_child, &b);
-      d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
-      d.pad_par = upload(o, h.pad_par, &b);
-      d.pad_batch_node = upload(o, h.pad_batch_node, &b);
-      d.big_class = upload(o, h.big_class, &b);
-      d.dmin = upload(o, h.dmin, &b);
-      d.cls_child_ptr = upload(o, h.cls_child_ptr, &b);
-      d.cls_child = upload(o, h.cls_child, &b);
-      d.pad_cedge = upload(o, h.pad_cedge, &b);
-      d.cedge_class = upload(o, h.cedge_class, &b);
-      d.cedge_ptr = upload(o, h.cedge_ptr, &b);
-      d.cedge_node = upload(o, h.cedge_node, &b);
-      d.witem = upload(o, h.witem, &b);
-      d.wmulti = upload(o, h.wmulti, &b);
-      d.wmulti_ptr = upload(o, h.wmulti_ptr, &b);
-      d.num_witems = (int32_t)(h.witem.size() / 4);
-      d.num_wmulti = (int32_t)h.wmulti.size();
-      d.w_num_slots = h.w_num_slots;
-      d.num_cedge = (int64_t)h.cls_child.size();
-      d.num_big = (int32_t)h.big_class.size();
-      d.rev_item = upload(o, h.rev_item, &b);
-      d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
-      d.num_rev_items = (int32_t)(h.rev_item.size() / 8);
-      d.rev_num_slots = h.rev_num_slots;
-      d.lvl_cptr = upload(o, h.lvl_cptr, &b);
-      d.lvl_class = upload(o, h.lvl_class, &b);
-      d.lvl_sptr = upload(o, h.lvl_sptr, &b);
-      d.lvl_scc = upload(o, h.lvl_scc, &b);
+      auto uploads = [&](Arena& o) {
+        d.class_ptr = upload(o, h.class_ptr, &b);
+        d.child_ptr = upload(o, h.child_ptr, &b);
+        {  // padded with the root id so batched kernels may read up to 8 past E
+          std::vector<int32_t> padded(h.child_class);
+          padded.resize(h.child_class.size() + 8, h.root);
+          d.child_class = upload(o, padded, &b);
+        }
+        d.par_ptr = upload(o, h.par_ptr, &b);
+        d.par_node = upload(o, h.par_node, &b);
+        d.par_class = upload(o, h.par_class, &b);
+        d.scc_class_ptr = upload(o, h.scc_class_ptr, &b);
+        d.scc_class = upload(o, h.scc_class, &b);
+        d.scc_of_class = upload(o, h.scc_of_class, &b);
+        d.ent_ptr = upload(o, h.ent_ptr, &b);
+        d.ent_i = upload(o, h.ent_i, &b);
+        d.ent_j = upload(o, h.ent_j, &b);
+        d.ent_node_ptr = upload(o, h.ent_node_ptr, &b);
+        d.ent_node = upload(o, h.ent_node, &b);
+        d.slot_ptr = upload(o, h.slot_ptr, &b);
+        d.slot_node = upload(o, h.slot_node, &b);
+        d.slot_iloc = upload(o, h.slot_iloc, &b);
+        d.slot_jptr = upload(o, h.slot_jptr, &b);
+        d.slot_jloc = upload(o, h.slot_jloc, &b);
+        d.node_slot = upload(o, h.node_slot, &b);
+        d.pad_child_ptr = upload(o, h.pad_child_ptr, &b);
+        d.pad_child = upload(o, h.pad_child, &b);
+        d.pad_par_ptr = upload(o, h.pad_par_ptr, &b);
+        d.pad_par = upload(o, h.pad_par, &b);
+        d.pad_batch_node = upload(o, h.pad_batch_node, &b);
+        d.big_class = upload(o, h.big_class, &b);
+        d.dmin = upload(o, h.dmin, &b);
+        d.cls_child_ptr = upload(o, h.cls_child_ptr, &b);
+        d.cls_child = upload(o, h.cls_child, &b);
+        d.pad_cedge = upload(o, h.pad_cedge, &b);
+        d.cedge_class = upload(o, h.cedge_class, &b);
+        d.cedge_ptr = upload(o, h.cedge_ptr, &b);
+        d.cedge_node = upload(o, h.cedge_node, &b);
+        d.witem = upload(o, h.witem, &b);
+        d.wmulti = upload(o, h.wmulti, &b);
+        d.wmulti_ptr = upload(o, h.wmulti_ptr, &b);
+        d.num_witems = (int32_t)(h.witem.size() / 4);
+        d.num_wmulti = (int32_t)h.wmulti.size();
+        d.w_num_slots = h.w_num_slots;
+        d.num_cedge = (int64_t)h.cls_child.size();
+        d.num_big = (int32_t)h.big_class.size();
+        d.rev_item = upload(o, h.rev_item, &b);
+        d.rev_class_item_ptr = upload(o, h.rev_class_item_ptr, &b);
+        d.num_rev_items = (int32_t)(h.rev_item.size() / 8);
+        d.rev_num_slots = h.rev_num_slots;
+        d.lvl_cptr = upload(o, h.lvl_cptr, &b);
+        d.lvl_class = upload(o, h.lvl_class, &b);
+        d.lvl_sptr = upload(o, h.lvl_sptr, &b);
+        d.lvl_scc = upload(o, h.lvl_scc, &b);
+      };
+      Arena measure;
+      uploads(measure);
+      Arena arena;
+      SM_CUDA(cudaMalloc(&arena.base, measure.used));
+      owner->owned.push_back(arena.base);
+      b = 0;
+      uploads(arena);
+      lap("device upload");
     }
   });
   if (st != SMOOTHE_OK) {
@@ -693,7 +818,8 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
     delete g;
     return st;
   }
-  delete owner;  // the allocations now belong to g->dev (freed by smoothe_free_egraph)
+  g->owned = std::move(owner->owned);  // freed by smoothe_free_egraph
+  delete owner;
   *out = g;
   return SMOOTHE_OK;
 }
@@ -840,6 +966,7 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
     r->g = g;
     r->opt = *opt;
     r->device = g->device;
+    r->owned.device = g->device;
     SM_CUDA(cudaSetDevice(r->device));
     const HostGraph& hg = g->host;
     Shape& sh = r->sh;
@@ -895,7 +1022,7 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
     g->refcount++;
   });
   if (st != SMOOTHE_OK) {
-    for (void* p : r->owned) cudaFree(p);
+    runmem_recycle(r->owned);
     if (r->stream) cudaStreamDestroy(r->stream);
     delete r;
     return st;
@@ -1175,12 +1302,14 @@ smoothe_status smoothe_run_get_profile(smoothe_run* run, smoothe_profile* out) {
   });
 }
 
+void smoothe_release_cached_memory(int device_ordinal) { cache_release(device_ordinal); }
+
 void smoothe_free_run(smoothe_run* run) {
   if (!run) return;
   cudaSetDevice(run->device);
   cudaStreamSynchronize(run->stream);
   if (run->graph_exec) cudaGraphExecDestroy(run->graph_exec);
-  for (void* p : run->owned) cudaFree(p);
+  runmem_recycle(run->owned);
   for (auto e : run->ev_step) cudaEventDestroy(e);
   for (auto e : run->prof_pool) cudaEventDestroy(e);
   if (run->ev_start) cudaEventDestroy(run->ev_start);
@@ -1203,16 +1332,9 @@ void smoothe_free_egraph(smoothe_egraph* g) {
     g->refcount--;
     return;
   }
-  // device arrays
-  DevGraph& d = g->dev;
-  if (g->device >= 0) {
+  if (g->device >= 0) {  // the arena holding every device array
     cudaSetDevice(g->device);
-    void* ptrs[] = {d.class_ptr, d.child_ptr, d.child_class, d.par_ptr, d.par_node, d.par_class,
-                    d.scc_class_ptr, d.scc_class, d.scc_of_class, d.ent_ptr, d.ent_i, d.ent_j, d.ent_node_ptr, d.ent_node,
-                    d.slot_ptr, d.slot_node, d.slot_iloc, d.slot_jptr, d.slot_jloc, d.node_slot,
-                    d.pad_child_ptr, d.pad_child, d.pad_par_ptr, d.pad_par, d.pad_batch_node,
-                    d.lvl_cptr, d.lvl_class, d.lvl_sptr, d.lvl_scc};
-    for (void* p : ptrs) cudaFree(p);
+    for (void* p : g->owned) cudaFree(p);
   }
   delete g;
 }

@@ -105,6 +105,7 @@ _SIGS = {
     "smoothe_last_error": (C.c_char_p, []),
     "smoothe_version": (C.c_char_p, []),
     "smoothe_free_run": (None, [C.c_void_p]),
+    "smoothe_release_cached_memory": (None, [C.c_int]),
     "smoothe_free_egraph": (None, [C.c_void_p]),
 }
 
@@ -371,6 +372,11 @@ def optimize(egraph, cost, num_seeds, steps, options=None) -> Run:
 
 def extract(run: Run):
     return run.extract()
+
+
+def release_cached_memory(device: int = -1):
+    """smoothe_release_cached_memory: return the recycled run blocks to the driver."""
+    lib().smoothe_release_cached_memory(int(device))
 
 
 def version() -> str:
