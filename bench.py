@@ -254,7 +254,7 @@ def run_ours(args):
     torch.cuda.set_stream(stream)
     opts = sm.Options(assumption="hybrid", prop_iters=-1, lam=lam, penalty_group=G, lr=0.1,
                       rng_key=key, seed_begin=rank * Bl, cuda_stream=stream.cuda_stream,
-                      use_graphs=True)
+                      use_graphs=True, converge=args.converge)
     t0 = time.time()
     g = sm.load_egraph_from(eg, device=local)
     run = sm.run_create(g, cost, Bl, opts)
@@ -416,6 +416,8 @@ def run_ours(args):
                        "seeds_per_gpu": Bl, "global_seeds": Bl * world, "penalty_group": G,
                        "assumption": "hybrid", "optimizer": "adam lr=0.1",
                        "lambda": lam, "parallelism": f"seed-sharded dp{world}",
+                       "sweeps": ("each seed until convergence, at most K (reading S1b)"
+                                  if args.converge else "K (reading S1)"),
                        "l2": "inputs larger than L2 (cp %.0f MB, q-stack %.1f GB)" %
                              (N * Bl * 4 / 1e6, (K + 1) * M * Bl * 4 / 1e9)},
             "fwd_bwd_units_per_s": units_rank * world / (fwdbwd_ms * 1e-3),
@@ -442,6 +444,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--converge", action="store_true",
+                    help="reading S1b: each seed's sweeps stop at convergence (not the default K)")
     ap.add_argument("--ttb-steps", type=int, default=80,
                     help="step budget of the time-to-best-cost measurement (same run)")
     args = ap.parse_args()

@@ -133,6 +133,10 @@ typedef struct {
   int64_t seed_begin;      /* global index of this rank's first seed (multi-GPU sharding)  */
   void *cuda_stream;       /* cudaStream_t to launch on, or NULL for a private stream      */
   int32_t use_graphs;      /* 1 = replay each step as a captured CUDA graph                */
+  int32_t converge;        /* 1 = "repeat until convergence" (P215, reading S1b): each     */
+                           /* seed's sweeps stop at the first one that changes none of its */
+                           /* q rows (fp32, bitwise), at most K; the reverse mode runs the */
+                           /* sweeps performed.  0 = exactly K sweeps (default)            */
 } smoothe_options;
 
 /* Defaults: HYBRID, K_auto, lambda 1, G = 1, Adam(lr 0.1, 0.9, 0.999, 1e-8),
@@ -204,6 +208,8 @@ typedef struct {
   int32_t *route;      /* [K][M][B] e-node the max of sweep t routed to, i.e.  */
                        /* the lowest id attaining the fp32 max (reading S7);  */
                        /* -1 for classes without parents; NULL = skip         */
+  int32_t *sweeps;     /* [B]     sweeps the seed's step performed (K, or its */
+                       /* convergence sweep with converge = 1); NULL = skip  */
 } smoothe_debug_out;
 
 SMOOTHE_API smoothe_status smoothe_debug_step(smoothe_run *run, const float *theta_in, const float *m_in,

@@ -206,6 +206,11 @@ struct SweepState {
   // seed's frozen sweeps, the K-state rows kq / kpi / kam, wm [Bp] 1 while the
   // seed's rows still equal the K-state (env SMOOTHE_REV_W=0 disables).
   bool wmode = false;
+  // "until convergence" (smoothe_options.converge, reading S1b): lastchg[s] =
+  // the last forward sweep that changed a q row of seed s; the seed's step is
+  // sweeps 1..lastchg+1 (its reverse skips the later, frozen sweeps)
+  bool converge = false;
+  int32_t* lastchg = nullptr;
   float *W = nullptr, *S = nullptr, *kq = nullptr, *kpi = nullptr, *wpart = nullptr;
   int32_t *kam = nullptr, *wm = nullptr;
 };
@@ -250,6 +255,9 @@ void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
 // frozen reverse sweep t for the seeds with wm set: g_q^{t-1} = W g_q^t, S += g_q^t
 void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
                   const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count);
+// converge mode: lastchg[s] from the forward's version lists (per seed, the
+// last sweep whose recomputed q rows differ from their previous versions)
+void launch_last_change(cudaStream_t s, const Shape& sh, const SweepState& st);
 void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
                     int32_t G, double lambda, const float* cp, double* h_part, float* pen,
                     double* big_scratch, int big_groups_per_batch);

@@ -876,13 +876,14 @@ constexpr int kWBlock = SMOOTHE_WSPMV_BLOCK;
 #ifndef SMOOTHE_WSPMV_DEPTH32
 #define SMOOTHE_WSPMV_DEPTH32 4
 #endif
-template <int LPR, bool STREAM>
+template <int LPR, bool STREAM, bool CONV>
 __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : 1) k_wspmv(
     int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
     const int32_t* __restrict__ cls_child, const float* __restrict__ W,
     const int32_t* __restrict__ wm, const float* __restrict__ gq, float* __restrict__ S,
-    float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count) {
+    float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
+    const int32_t* __restrict__ lastchg) {
   const RowGroup<LPR, kWBlock> rg;
   if (frozen_count && blockIdx.x == 0 && threadIdx.x == 0) {  // profiling: a working launch?
     bool any = false;
@@ -898,15 +899,38 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   const int i = itm.x, e0 = itm.y, e1 = itm.z, slot = itm.w;
   const int d = __ldg(dmin + i);
   const size_t oi = (size_t)i * Bp + rg.s0;
+  // converge mode: a frozen seed's sweeps after its convergence sweep
+  // lastchg + 1 were never performed: its g_q passes through unchanged
+  int4 cp4 = make_int4(0, 0, 0, 0);  // copy mode per seed
+  if (CONV) {
+    const int4 lc = ld4i(lastchg + rg.s0);
+    cp4 = make_int4(w4.x && t > lc.x + 1, w4.y && t > lc.y + 1, w4.z && t > lc.z + 1,
+                    w4.w && t > lc.w + 1);
+  }
   if (d <= t && e0 == cls_child_ptr[i]) {  // first item: S_i += g_q^t_i (a valid row)
     const float4 gi = ld4(gq + oi);
     float4 si = ld4(S + oi);
 #pragma unroll
     for (int x = 0; x < 4; ++x)
-      if (comp(w4, x)) comp(si, x) += comp(gi, x);
+      if (comp(w4, x) && !comp(cp4, x)) comp(si, x) += comp(gi, x);
     st4(S + oi, si);
   }
   if (d > t - 1 || !gq_prev) return;  // q^{t-1}_i = 0: the row is never read
+  const bool anyw = !CONV || __any_sync(gm, (comp(w4, 0) && !comp(cp4, 0)) || (comp(w4, 1) && !comp(cp4, 1)) ||
+                                       (comp(w4, 2) && !comp(cp4, 2)) || (comp(w4, 3) && !comp(cp4, 3)));
+  if (!anyw) {  // every frozen seed of the row group is past its convergence sweep
+    if (e0 != cls_child_ptr[i]) return;  // the class's first item copies the row
+    const float4 gi = ld4(gq + oi);
+    float4 o = gi;
+    if (!(w4.x && w4.y && w4.z && w4.w)) {
+      const float4 cur = ld4(gq_prev + oi);
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+        if (!comp(w4, x)) comp(o, x) = comp(cur, x);
+    }
+    st4(gq_prev + oi, o);
+    return;
+  }
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
   // the row group loads LPR child indices at once (one per lane, coalesced)
   // and broadcasts them, so the W rows (streamed) and g_q rows (gathered) of
@@ -945,6 +969,12 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   }
   if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 o = acc;
+  if (CONV) {  // seeds past their convergence sweep pass g_q^t through
+    const float4 gi = ld4(gq + oi);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (comp(cp4, x)) comp(o, x) = comp(gi, x);
+  }
   if (!(w4.x && w4.y && w4.z && w4.w)) {  // mixed: keep the reverse kernel's seeds
     const float4 cur = ld4(gq_prev + oi);
 #pragma unroll
@@ -960,13 +990,22 @@ template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_wcombine(
     int n_multi, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ wmulti, const int32_t* __restrict__ wmulti_ptr,
-    const int32_t* __restrict__ wm, const float* __restrict__ part, float* __restrict__ gq_prev) {
+    const int32_t* __restrict__ wm, const float* __restrict__ part, float* __restrict__ gq_prev,
+    const int32_t* __restrict__ lastchg, const float* __restrict__ gq) {
   const RowGroup<LPR> rg;
   if (rg.row >= n_multi) return;
   const int4 w4 = ld4i(wm + rg.s0);
   if (!(w4.x | w4.y | w4.z | w4.w)) return;
   const int i = wmulti[rg.row];
   if (__ldg(dmin + i) > t - 1) return;
+  int4 cp4 = make_int4(0, 0, 0, 0);
+  if (lastchg) {
+    const int4 lc = ld4i(lastchg + rg.s0);
+    cp4 = make_int4(w4.x && t > lc.x + 1, w4.y && t > lc.y + 1, w4.z && t > lc.z + 1,
+                    w4.w && t > lc.w + 1);
+    // every frozen seed past its convergence sweep: k_wspmv's first item copied the row
+    if ((!w4.x || cp4.x) && (!w4.y || cp4.y) && (!w4.z || cp4.z) && (!w4.w || cp4.w)) return;
+  }
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
   for (int sl = wmulti_ptr[rg.row]; sl < wmulti_ptr[rg.row + 1]; ++sl) {
     const float4 p = ld4(part + (size_t)sl * Bp + rg.s0);
@@ -978,6 +1017,12 @@ __global__ void __launch_bounds__(kBlock) k_wcombine(
   if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
   const size_t oi = (size_t)i * Bp + rg.s0;
   float4 o = acc;
+  if (lastchg) {
+    const float4 gi = ld4(gq + oi);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (comp(cp4, x)) comp(o, x) = comp(gi, x);
+  }
   if (!(w4.x && w4.y && w4.z && w4.w)) {
     const float4 cur = ld4(gq_prev + oi);
 #pragma unroll
@@ -993,22 +1038,70 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
   // room to spare, where it stays resident across the frozen sweeps (C5: 69 MB)
   const bool stream = (double)g.num_cedge * sh.Bp * sizeof(float) > 96e6;
   const int4* items = reinterpret_cast<const int4*>(g.witem);
+#define SM_WSPMV(ST, CV)                                                                       \
+  k_wspmv<LPR, ST, CV><<<grid, kWBlock, 0, s>>>(                                               \
+      g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W, st.wm, \
+      gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg)
   SM_DISPATCH_LPR(sh.Bp, {
     const dim3 grid = row_grid(g.num_witems, sh.Bp, LPR, kWBlock);
-    if (stream)
-      k_wspmv<LPR, true><<<grid, kWBlock, 0, s>>>(
-          g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,
-          st.wm, gq, st.S, gq_prev, st.wpart, frozen_count);
-    else
-      k_wspmv<LPR, false><<<grid, kWBlock, 0, s>>>(
-          g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,
-          st.wm, gq, st.S, gq_prev, st.wpart, frozen_count);
+    if (st.converge) {
+      if (stream) SM_WSPMV(true, true);
+      else SM_WSPMV(false, true);
+    } else {
+      if (stream) SM_WSPMV(true, false);
+      else SM_WSPMV(false, false);
+    }
+
     if (g.num_wmulti > 0 && gq_prev) {
       SM_LAUNCH_CHECK();
       k_wcombine<LPR><<<row_grid(g.num_wmulti, sh.Bp, LPR), kBlock, 0, s>>>(
           g.num_wmulti, sh.Bp, sh.root, t, g.dmin, g.wmulti, g.wmulti_ptr, st.wm, st.wpart,
-          gq_prev);
+          gq_prev, st.converge ? st.lastchg : nullptr, gq);
     }
+  });
+#undef SM_WSPMV
+  SM_LAUNCH_CHECK();
+}
+
+
+// Converge mode: lastchg[s] = max over sweeps t and classes j recomputed in t of
+// t if version t of q_j differs from its previous version in seed s.  Grid
+// (x: entries, y: sweep t - 1, z: seed chunk); per-block flags, one atomicMax
+// per seed and block.
+template <int LPR>
+__global__ void __launch_bounds__(kBlock) k_last_change(int M, int Bp,
+                                                       const int32_t* __restrict__ list_n,
+                                                       const int2* __restrict__ list,
+                                                       const float* __restrict__ qstack,
+                                                       int32_t* __restrict__ lastchg) {
+  __shared__ int flag[4 * LPR];
+  const int t = blockIdx.y + 1;
+  const int gl = threadIdx.x % LPR, sub = threadIdx.x / LPR;
+  const int s0 = blockIdx.z * (4 * LPR) + gl * 4;
+  if (threadIdx.x < 4 * LPR) flag[threadIdx.x] = 0;
+  __syncthreads();
+  const int n = list_n[t];
+  const size_t MB = (size_t)M * Bp;
+  const int2* lt = list + (size_t)t * M;
+  for (int e = blockIdx.x * (kBlock / LPR) + sub; e < n; e += gridDim.x * (kBlock / LPR)) {
+    const int2 en = lt[e];
+    const size_t o = (size_t)en.x * Bp + s0;
+    const float4 a = ld4(qstack + (size_t)t * MB + o), b = ld4(qstack + (size_t)en.y * MB + o);
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+      if (__float_as_uint(comp(a, x)) != __float_as_uint(comp(b, x))) flag[gl * 4 + x] = 1;
+  }
+  __syncthreads();
+  if (threadIdx.x < 4 * LPR && flag[threadIdx.x])
+    atomicMax(lastchg + blockIdx.z * (4 * LPR) + threadIdx.x, t);
+}
+
+void launch_last_change(cudaStream_t s, const Shape& sh, const SweepState& st) {
+  SM_CUDA(cudaMemsetAsync(st.lastchg, 0, sizeof(int32_t) * sh.Bp, s));
+  SM_DISPATCH_LPR(sh.Bp, {
+    const dim3 grid(64, st.K, num_chunks(sh.Bp));
+    k_last_change<LPR><<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, st.list_n, st.list, st.qstack,
+                                                st.lastchg);
   });
   SM_LAUNCH_CHECK();
 }

@@ -432,6 +432,7 @@ void enqueue_step(smoothe_run* r) {
       SM_CUDA(cudaMemsetAsync(sw.wm, 1, sizeof(int32_t) * sh.Bp, s));
       SM_CUDA(cudaMemsetAsync(sw.S, 0, sizeof(float) * MB, s));
       launch_wbuild(s, sh, g, r->agg, sw, r->cp);
+      if (sw.converge) launch_last_change(s, sh, sw);
     }
     if (sw.wmode && r->profiling && std::getenv("SMOOTHE_REV_W_STATS")) {
       // diagnostic: seeds still frozen before reverse sweep t (stderr, one line per sweep)
@@ -448,7 +449,10 @@ void enqueue_step(smoothe_run* r) {
       fprintf(stderr, "[wstats] t=%d frozen_seeds=%d full_slices=%d\n", t, n, slices);
     }
     kmark(1, 0);
-    launch_sweep_reverse(s, sh, g, r->agg, t, K, cur_q, sw.cur_pi, sw.cur_am,
+    // converge mode: a seed's loss reads q^{t*} (t* = its convergence sweep),
+    // so the reverse window (g_q^t_j = 0 while t + hmax_j <= K) does not hold
+    // for K; no window then (the window argument with t* would be per seed)
+    launch_sweep_reverse(s, sh, g, r->agg, t, sw.converge ? -1 : K, cur_q, sw.cur_pi, sw.cur_am,
                          sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
                          r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt);
     kmark(1, 1);
@@ -554,7 +558,10 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     // frozen-sweep path: on for K >= 48 (enough sweeps to freeze and pay for
     // the W build and the final pass), SMOOTHE_REV_W=0 / 1 forces it
     const char* wenv = std::getenv("SMOOTHE_REV_W");
-    w.wmode = (wenv ? wenv[0] == '1' : r->K >= 48) && r->g->dev.num_cedge > 0;
+    w.converge = r->opt.converge != 0;
+    // converge mode runs on the frozen-sweep machinery (its skipped sweeps are frozen ones)
+    w.wmode = (w.converge || (wenv ? wenv[0] == '1' : r->K >= 48)) && r->g->dev.num_cedge > 0;
+    if (w.converge && r->g->dev.num_cedge == 0) w.converge = false;  // no edges: nothing to iterate
     if (w.wmode) {
       w.W = dalloc<float>(o, (size_t)r->g->dev.num_cedge * sh.Bp);
       w.S = dalloc<float>(o, MB);
@@ -562,6 +569,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       if (w.pistack) w.kpi = dalloc<float>(o, MB);
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
+      if (w.converge) w.lastchg = dalloc<int32_t>(o, sh.Bp);
       w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
       r->frozen_count = dalloc<int64_t>(o, 1);
       SM_CUDA(cudaMemset(r->frozen_count, 0, sizeof(int64_t)));
@@ -1196,6 +1204,15 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     if (dump->valid) SM_CUDA(cudaMemcpyAsync(dump->valid, run->dbg_valid, sh.B, cudaMemcpyDeviceToHost, s));
     if (dump->disc_cost)
       SM_CUDA(cudaMemcpyAsync(dump->disc_cost, run->dbg_dcost, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
+    if (dump->sweeps) {
+      std::vector<int32_t> lc(sh.Bp, run->K - 1);
+      if (run->sw.converge) {
+        SM_CUDA(cudaMemcpyAsync(lc.data(), run->sw.lastchg, sizeof(int32_t) * sh.Bp,
+                                cudaMemcpyDeviceToHost, s));
+        SM_CUDA(cudaStreamSynchronize(s));
+      }
+      for (int b = 0; b < sh.B; ++b) dump->sweeps[b] = std::min(run->K, lc[b] + 1);
+    }
     if (dump->route && run->K > 0)  // rows of sweep t + 1 = slot t + 1
       SM_CUDA(cudaMemcpy2DAsync(dump->route, sizeof(int32_t) * sh.B, run->sw.astack + MB,
                                 sizeof(int32_t) * sh.Bp, sizeof(int32_t) * sh.B,

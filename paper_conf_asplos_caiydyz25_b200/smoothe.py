@@ -50,7 +50,8 @@ class _Opts(C.Structure):
                 ("penalty_group", C.c_int32), ("lr", C.c_double), ("beta1", C.c_double),
                 ("beta2", C.c_double), ("eps", C.c_double), ("optimizer", C.c_int32),
                 ("patience", C.c_int32), ("time_limit_s", C.c_double), ("rng_key", C.c_uint64),
-                ("seed_begin", C.c_int64), ("cuda_stream", C.c_void_p), ("use_graphs", C.c_int32)]
+                ("seed_begin", C.c_int64), ("cuda_stream", C.c_void_p), ("use_graphs", C.c_int32),
+                ("converge", C.c_int32)]
 
 
 class _Summary(C.Structure):
@@ -63,7 +64,7 @@ class _Summary(C.Structure):
 class _Dump(C.Structure):
     _fields_ = [(n, C.c_void_p) for n in
                 ("cp", "qK", "p", "grad_cp", "grad_theta", "theta_out", "m_out", "v_out", "f", "h",
-                 "loss", "choice", "reached", "valid", "disc_cost", "qstack", "route")]
+                 "loss", "choice", "reached", "valid", "disc_cost", "qstack", "route", "sweeps")]
 
 
 class _Greedy(C.Structure):
@@ -249,12 +250,13 @@ class Options:
     seed_begin: int = 0
     cuda_stream: int | None = None
     use_graphs: bool = True
+    converge: bool = False
 
     def c(self) -> _Opts:
         return _Opts(ASSUMPTIONS[self.assumption], self.prop_iters, self.lam, self.penalty_group,
                      self.lr, self.beta1, self.beta2, self.eps, 0 if self.optimizer == "adam" else 1,
                      self.patience, self.time_limit_s, self.rng_key, self.seed_begin,
-                     self.cuda_stream, 1 if self.use_graphs else 0)
+                     self.cuda_stream, 1 if self.use_graphs else 0, 1 if self.converge else 0)
 
 
 def torch_stream():
@@ -316,7 +318,7 @@ class Run:
         out.update(qK=np.zeros((M, B), np.float32), f=np.zeros(B), h=np.zeros(B // G),
                    loss=np.zeros(1), choice=np.zeros((M, B), np.int32),
                    reached=np.zeros((M, B), np.uint8), valid=np.zeros(B, np.uint8),
-                   disc_cost=np.zeros(B))
+                   disc_cost=np.zeros(B), sweeps=np.zeros(B, np.int32))
         if qstack:
             out["qstack"] = np.zeros((self.K + 1, M, B), np.float32)
         if route:

@@ -225,6 +225,42 @@ def test_frozen_sweeps_parity(sm, orc, monkeypatch, name, B, G, K, agg):
     compare_step(sm, orc, make_config(name), B, G, agg, K=K, seed=B + K)
 
 
+@pytest.mark.parametrize("name,B,K,agg", [("C2", 64, 80, "hybrid"), ("C2", 32, 80, "independent"),
+                                          ("C5", 64, 57, "hybrid")])
+def test_converge_mode_parity(sm, orc, name, B, K, agg):
+    """Reading S1b ("repeat until convergence", P215): each seed's step stops
+    at its first sweep that changes none of its q rows (an fp32 decision the
+    GPU exports, like the max routing), and the reverse mode runs the sweeps
+    performed.  The oracle, given each seed's sweep count, recomputes the step
+    of that seed with exactly that many sweeps."""
+    eg = make_config(name)
+    g = sm.load_egraph_from(eg)
+    opts = sm.Options(assumption=agg, prop_iters=K, lam=1.0, penalty_group=1, rng_key=3,
+                      converge=True)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), B, opts)
+    theta = np.random.default_rng(K + B).uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
+    d = run.debug_step(theta, route=True)
+    sw = d["sweeps"]
+    assert np.all((sw >= 1) & (sw <= K)) and np.median(sw) < K, sw  # most seeds converged
+    og = orc.Graph(eg)
+    for b in list(range(0, B, max(1, B // 8))):
+        th = theta[:, [b]].astype(np.float64)
+        oo = orc.Options(assumption=agg, K=int(sw[b]), lam=1.0, G=1)
+        o = og.step(th, oo, route=d["route"][: sw[b], :, [b]])
+        assert o["route_invalid"].sum() == 0
+        col = lambda a: a[:, [b]]
+        close(f"cp[{b}]", col(d["cp"]), o["cp"])
+        close(f"p[{b}]", col(d["p"]), o["p"])
+        close(f"f[{b}]", d["f"][[b]], o["f"])
+        gco = o["grad_cp"]
+        close(f"grad_cp[{b}]", col(d["grad_cp"]), gco, scale=np.abs(gco))
+        cpo = o["cp"]
+        gscale = cpo * (np.abs(gco) + class_sums(eg, cpo * np.abs(gco)))
+        close(f"grad_theta[{b}]", col(d["grad_theta"]), o["grad_theta"], scale=gscale)
+    run.close()
+    g.close()
+
+
 def test_c3_quadratic_full(sm, orc):
     spec = CONFIGS["C3"]
     compare_step(sm, orc, make_config("C3"), spec["seeds_per_gpu"], spec["group"], seed=3)
@@ -334,8 +370,8 @@ def test_change_propagation_bit_identical(sm, monkeypatch, name, B, G, agg, step
             assert np.array_equal(d0[key], d1[key]), key
 
 
-@pytest.mark.parametrize("wmode,K", [("0", -1), ("1", 80)])
-def test_seed_sharding_bit_identical(sm, monkeypatch, wmode, K):
+@pytest.mark.parametrize("wmode,K,conv", [("0", -1, False), ("1", 80, False), ("1", 80, True)])
+def test_seed_sharding_bit_identical(sm, monkeypatch, wmode, K, conv):
     """8(e): a run of 64 seeds equals two runs of 32 seeds (seed_begin 0, 32)
     seed by seed, and the lexicographic best of the shards is the full best.
     With the frozen-sweep path (SMOOTHE_REV_W=1, K = 80: most sweeps frozen)
@@ -344,14 +380,15 @@ def test_seed_sharding_bit_identical(sm, monkeypatch, wmode, K):
     eg = make_config("C2")
     g = sm.load_egraph_from(eg)
     cost = sm.CostModel.from_input(eg)
-    full = sm.run_create(g, cost, 64, sm.Options(penalty_group=8, rng_key=5, prop_iters=K))
+    full = sm.run_create(g, cost, 64, sm.Options(penalty_group=8, rng_key=5, prop_iters=K,
+                                                 converge=conv))
     full.steps(15)
     tf = full.theta()
     cf, sf = full.extract()
     halves = []
     for sb in (0, 32):
         r = sm.run_create(g, cost, 32, sm.Options(penalty_group=8, rng_key=5, seed_begin=sb,
-                                                  prop_iters=K))
+                                                  prop_iters=K, converge=conv))
         r.steps(15)
         halves.append((r.theta(), r.extract()))
     assert np.array_equal(np.concatenate([halves[0][0], halves[1][0]], axis=1), tf)
