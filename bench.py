@@ -372,6 +372,28 @@ def run_ours(args):
         roof["working_launches_per_step"] = nwork / max(1, prof["steps"])
 
     run.close()
+
+    # the same workload in convergence mode (reading S1b, an option, not the
+    # headline: the north star fixes the number of iterations): each seed's
+    # sweeps stop at convergence; same graph, seeds and timing rules
+    conv = None
+    if not args.converge and not args.no_converge_leg:
+        copts = sm.Options(assumption="hybrid", prop_iters=-1, lam=lam, penalty_group=G, lr=0.1,
+                           rng_key=key, seed_begin=rank * Bl, cuda_stream=stream.cuda_stream,
+                           use_graphs=True, converge=True)
+        crun = sm.run_create(g, cost, Bl, copts)
+        crun.steps(args.warmup)
+        torch.cuda.synchronize()
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        c0.record(stream)
+        crun.steps(args.steps)
+        c1.record(stream)
+        torch.cuda.synchronize()
+        cms = c0.elapsed_time(c1)
+        crun.close()
+        conv = {"ms_per_step": cms / args.steps, "value": units_rank * world / (cms * 1e-3),
+                "note": "smoothe_options.converge = 1 (reading S1b): each seed's sweeps stop at "
+                        "its first change-free sweep; this rank's device time"}
     g.close()
     torch.cuda.synchronize()
 
@@ -427,6 +449,7 @@ def run_ours(args):
                                          for k, v in prof["sweep_kernel_ms"].items()},
             "gpu_launches": prof["launches"],
             "time_to_best": ttb,
+            "converge_mode": conv,
             "roofline": roof, "e2e": e2e, "cpu_baseline": cb, "clocks": ck,
         }
         print(json.dumps(line), flush=True)
@@ -446,6 +469,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--converge", action="store_true",
                     help="reading S1b: each seed's sweeps stop at convergence (not the default K)")
+    ap.add_argument("--no-converge-leg", action="store_true",
+                    help="skip the extra convergence-mode measurement")
     ap.add_argument("--ttb-steps", type=int, default=80,
                     help="step budget of the time-to-best-cost measurement (same run)")
     args = ap.parse_args()
