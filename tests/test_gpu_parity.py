@@ -139,6 +139,32 @@ def test_tiny_families(sm, orc, agg, kind):
         compare_step(sm, orc, eg, 33, 3, agg, lam=0.7, seed=s, K=3 + s % 4)
 
 
+@pytest.mark.parametrize("agg", AGGS)
+def test_tiny_frozen_and_converge(sm, orc, monkeypatch, agg):
+    """Tiny cyclic graphs with K well past the freezing point: the frozen-sweep
+    path forced on (ragged B = 33, groups of 3), and the convergence mode per
+    seed (G = 1), both against the oracle."""
+    monkeypatch.setenv("SMOOTHE_REV_W", "1")
+    for s in range(6):
+        eg = random_tiny(3100 + s, "cyclic", num_classes=8)
+        compare_step(sm, orc, eg, 33, 3, agg, lam=0.7, seed=s, K=12 + s)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), 16,
+                            sm.Options(assumption=agg, prop_iters=12 + s, lam=0.7,
+                                       penalty_group=1, converge=True))
+        th = np.random.default_rng(s).uniform(-2, 2, (eg.num_nodes, 16)).astype(np.float32)
+        d = run.debug_step(th, route=True)
+        og = orc.Graph(eg)
+        for b in range(16):
+            oo = orc.Options(assumption=agg, K=int(d["sweeps"][b]), lam=0.7, G=1)
+            o = og.step(th[:, [b]].astype(np.float64), oo, route=d["route"][: d["sweeps"][b], :, [b]])
+            close("p", d["p"][:, [b]], o["p"])
+            gco = o["grad_cp"]
+            close("grad_cp", d["grad_cp"][:, [b]], gco, scale=np.abs(gco))
+        run.close()
+        g.close()
+
+
 @pytest.mark.parametrize("B,agg,K", [(32, "hybrid", -1), (64, "independent", 12),
                                      (64, "correlated", 12), (256, "hybrid", 12)])
 def test_long_lists_split_items(sm, orc, B, agg, K):
