@@ -248,7 +248,8 @@ void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, i
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
-                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt);
+                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
+                          const int32_t* lastchg = nullptr);
 // W from the K-state rows (before reverse sweep K)
 void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                    const SweepState& st, const float* cp);

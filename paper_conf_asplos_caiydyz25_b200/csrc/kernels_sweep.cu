@@ -527,19 +527,40 @@ __device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows oth
 
 // Outputs of one reverse-sweep item: g_q^{t-1}_{j'} directly (the class's only
 // item), else its partial row, and the class's last item to finish combines.
-template <int V, bool HI>
+// CONV (convergence mode without the frozen-sweep path): seeds with pass = 1
+// are past their convergence sweep; their g_q^{t-1}_{j'} is g_q^t_{j'}.
+template <int V, bool CONV>
+__device__ __forceinline__ Vec<V> pass_through(const Vec<V>& out, const Vec<V>& pass,
+                                               const float* __restrict__ gq, int jp, int Bp,
+                                               int s0) {
+  if (!CONV) return out;
+  bool any = false;
+#pragma unroll
+  for (int x = 0; x < V; ++x) any = any || pass.v[x] != 0.f;
+  if (!__any_sync(0xffffffffu, any)) return out;
+  const Vec<V> g = ldv_cg<V>(gq + (size_t)jp * Bp + s0);
+  Vec<V> o = out;
+#pragma unroll
+  for (int x = 0; x < V; ++x)
+    if (pass.v[x] != 0.f) o.v[x] = g.v[x];
+  return o;
+}
+
+template <int V, bool HI, bool CONV>
 __device__ __forceinline__ void reverse_epilogue(
     int lane, int jp, int info, bool piece, int Bp, int root, int s0, const Vec<V>& keep,
     const Vec<V>& qp,
     const Vec<V>& gqacc, const Vec<V>& X, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const float* __restrict__ cp,
     float* __restrict__ gcp, float* __restrict__ gq_prev, float* __restrict__ part,
-    int32_t* __restrict__ cnt) {
+    int32_t* __restrict__ cnt, const Vec<V>& pass, const float* __restrict__ gq) {
   Vec<V> zero;
 #pragma unroll
   for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
   if (info < 0) {  // the class's only item
-    if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : gqacc);
+    if (gq_prev)
+      stv<V>(gq_prev + (size_t)jp * Bp + s0,
+             jp == root ? zero : pass_through<V, CONV>(gqacc, pass, gq, jp, Bp, s0));
     return;
   }
   stv<V>(part + (size_t)(info >> 1) * Bp + s0, piece ? X : gqacc);
@@ -582,7 +603,9 @@ __device__ __forceinline__ void reverse_epilogue(
     }
     stv<V>(gcp + ok, gc);
   }
-  if (gq_prev) stv<V>(gq_prev + (size_t)jp * Bp + s0, jp == root ? zero : acc);
+  if (gq_prev)
+    stv<V>(gq_prev + (size_t)jp * Bp + s0,
+           jp == root ? zero : pass_through<V, CONV>(acc, pass, gq, jp, Bp, s0));
 }
 
 // One warp per work item (HostGraph::rev_item): a run of batches of class j'.
@@ -602,7 +625,7 @@ constexpr int kRevBlock = SMOOTHE_REV_BLOCK;
 #ifndef SMOOTHE_REV_MINB4
 #define SMOOTHE_REV_MINB4 (6 * 64 / SMOOTHE_REV_BLOCK)  // min resident blocks per SM at V = 4
 #endif
-template <int V, bool HI, bool HC>
+template <int V, bool HI, bool HC, bool CONV>
 __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64 / kRevBlock) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
@@ -610,19 +633,34 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
     float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
-    const int32_t* __restrict__ wm) {
+    const int32_t* __restrict__ wm, const int32_t* __restrict__ lastchg) {
   const int it = blockIdx.x * (kRevBlock / 32) + (int)threadIdx.x / 32;
   if (it >= n_items) return;
   const int lane = threadIdx.x % 32;
   // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
-  Vec<V> keep;
+  Vec<V> keep, pass;
+  bool allpass = false;
+  if (CONV) {  // convergence mode: seeds past their convergence sweep pass g_q through
+    const int sw = blockIdx.y * (32 * V) + lane * V;
+    bool all = true;
+#pragma unroll
+    for (int x = 0; x < V; ++x) {
+      const bool p = t > __ldg(lastchg + sw + x) + 1;
+      pass.v[x] = p ? 1.f : 0.f;
+      all = all && p;
+    }
+    allpass = __all_sync(0xffffffffu, all);
+  } else {
+#pragma unroll
+    for (int x = 0; x < V; ++x) pass.v[x] = 0.f;
+  }
   {
     const int sw = blockIdx.y * (32 * V) + lane * V;
     bool allw = true;
 #pragma unroll
     for (int x = 0; x < V; ++x) {
       const bool w = wm && __ldg(wm + sw + x) != 0;
-      keep.v[x] = w ? 0.f : 1.f;
+      keep.v[x] = w || pass.v[x] != 0.f ? 0.f : 1.f;
       allw = allw && w;
     }
     if (__all_sync(0xffffffffu, allw)) return;
@@ -632,6 +670,16 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
   const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
   const bool piece = info >= 0 && (info & 1);
   const int s0 = blockIdx.y * (32 * V) + lane * V;
+  if (CONV && allpass) {  // the class's first item copies g_q^t_{j'} (root: 0)
+    if (gq_prev && (info < 0 || it == class_item_ptr[jp])) {
+      Vec<V> g = ldv_cg<V>(gq + (size_t)jp * Bp + s0);
+      if (jp == root)
+#pragma unroll
+        for (int x = 0; x < V; ++x) g.v[x] = 0.f;
+      stv<V>(gq_prev + (size_t)jp * Bp + s0, g);
+    }
+    return;
+  }
   // Reverse window: the loss reads only q^K, so g_q^t_j is exactly 0 unless a
   // walk of length K - t leaves class j (t >= K - hmax_j); every child of j'
   // then has g_q^t = 0 while t <= K - hmax_j', and so has g_q^{t-1}_{j'}.  The
@@ -755,14 +803,15 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
       }
     }
   }
-  reverse_epilogue<V, HI>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X, items, class_item_ptr,
-                          cp, gcp, gq_prev, part, cnt);
+  reverse_epilogue<V, HI, CONV>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X, items,
+                                class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq);
 }
 
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
-                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt) {
+                          float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
+                          const int32_t* lastchg) {
   float* out = write_gq_prev ? gq_prev : nullptr;
 #ifndef SMOOTHE_REV_VMAX
 #define SMOOTHE_REV_VMAX 4  // seeds per lane at Bp >= 128 (4: one warp per 128-seed slice)
@@ -773,11 +822,16 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   // L2-resident (measured: +7% on C4 at 512 MB, -9% on C3 at 13 MB)
   const bool l2_prefetch = (double)sh.N * sh.Bp * sizeof(float) > 64e6;
   const dim3 grid((n + kRevBlock / 32 - 1) / (kRevBlock / 32), sh.Bp / (32 * V));
-#define SM_REV2(VV, HI, HC)                                                                    \
-  k_sweep_reverse<VV, HI, HC><<<grid, kRevBlock, 0, s>>>(                                   \
+#define SM_REV3(VV, HI, HC, CV)                                                                \
+  k_sweep_reverse<VV, HI, HC, CV><<<grid, kRevBlock, 0, s>>>(                                  \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,             \
-      rev_part, rev_cnt, l2_prefetch, t, K, wm)
+      rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg)
+#define SM_REV2(VV, HI, HC)                                                                    \
+  do {                                                                                         \
+    if (lastchg) SM_REV3(VV, HI, HC, true);                                                    \
+    else SM_REV3(VV, HI, HC, false);                                                           \
+  } while (0)
 #define SM_REV(VV)                                                                             \
   do {                                                                                         \
     if (a.wI != 0.f && a.wC != 0.f) SM_REV2(VV, true, true);                                   \
@@ -789,6 +843,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   else SM_REV(1);
 #undef SM_REV
 #undef SM_REV2
+#undef SM_REV3
   SM_LAUNCH_CHECK();
 }
 

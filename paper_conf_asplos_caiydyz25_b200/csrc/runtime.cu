@@ -432,8 +432,8 @@ void enqueue_step(smoothe_run* r) {
       SM_CUDA(cudaMemsetAsync(sw.wm, 1, sizeof(int32_t) * sh.Bp, s));
       SM_CUDA(cudaMemsetAsync(sw.S, 0, sizeof(float) * MB, s));
       launch_wbuild(s, sh, g, r->agg, sw, r->cp);
-      if (sw.converge) launch_last_change(s, sh, sw);
     }
+    if (sw.converge && t == K) launch_last_change(s, sh, sw);
     if (sw.wmode && r->profiling && std::getenv("SMOOTHE_REV_W_STATS")) {
       // diagnostic: seeds still frozen before reverse sweep t (stderr, one line per sweep)
       std::vector<int32_t> h(sh.Bp);
@@ -454,7 +454,8 @@ void enqueue_step(smoothe_run* r) {
     // for K; no window then (the window argument with t* would be per seed)
     launch_sweep_reverse(s, sh, g, r->agg, t, sw.converge ? -1 : K, cur_q, sw.cur_pi, sw.cur_am,
                          sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
-                         r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt);
+                         r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt,
+                         sw.converge && !sw.wmode ? sw.lastchg : nullptr);
     kmark(1, 1);
     if (sw.wmode) {
       kmark(2, 0);
@@ -557,11 +558,12 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     }
     // frozen-sweep path: on for K >= 48 (enough sweeps to freeze and pay for
     // the W build and the final pass), SMOOTHE_REV_W=0 / 1 forces it
+    if (r->opt.converge) w.lastchg = dalloc<int32_t>(o, sh.Bp);
     const char* wenv = std::getenv("SMOOTHE_REV_W");
     w.converge = r->opt.converge != 0;
-    // converge mode runs on the frozen-sweep machinery (its skipped sweeps are frozen ones)
-    w.wmode = (w.converge || (wenv ? wenv[0] == '1' : r->K >= 48)) && r->g->dev.num_cedge > 0;
-    if (w.converge && r->g->dev.num_cedge == 0) w.converge = false;  // no edges: nothing to iterate
+    // convergence mode: with the frozen-sweep path the W kernels pass a
+    // converged seed's g_q through, without it the reverse kernel does
+    w.wmode = (wenv ? wenv[0] == '1' : r->K >= 48) && r->g->dev.num_cedge > 0;
     if (w.wmode) {
       w.W = dalloc<float>(o, (size_t)r->g->dev.num_cedge * sh.Bp);
       w.S = dalloc<float>(o, MB);
@@ -569,7 +571,6 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       if (w.pistack) w.kpi = dalloc<float>(o, MB);
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
-      if (w.converge) w.lastchg = dalloc<int32_t>(o, sh.Bp);
       w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
       r->frozen_count = dalloc<int64_t>(o, 1);
       SM_CUDA(cudaMemset(r->frozen_count, 0, sizeof(int64_t)));

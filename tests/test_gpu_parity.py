@@ -251,14 +251,21 @@ def test_frozen_sweeps_parity(sm, orc, monkeypatch, name, B, G, K, agg):
     compare_step(sm, orc, make_config(name), B, G, agg, K=K, seed=B + K)
 
 
-@pytest.mark.parametrize("name,B,K,agg", [("C2", 64, 80, "hybrid"), ("C2", 32, 80, "independent"),
-                                          ("C5", 64, 57, "hybrid")])
-def test_converge_mode_parity(sm, orc, name, B, K, agg):
+@pytest.mark.parametrize("name,B,K,agg,wpath", [("C2", 64, 80, "hybrid", "1"),
+                                                ("C2", 32, 80, "independent", "1"),
+                                                ("C5", 64, 57, "hybrid", "1"),
+                                                ("C2", 64, 80, "hybrid", "0"),
+                                                ("C2", 100, 40, "correlated", "0"),
+                                                ("C3", 32, 60, "hybrid", "0")])
+def test_converge_mode_parity(sm, orc, monkeypatch, name, B, K, agg, wpath):
     """Reading S1b ("repeat until convergence", P215): each seed's step stops
     at its first sweep that changes none of its q rows (an fp32 decision the
     GPU exports, like the max routing), and the reverse mode runs the sweeps
     performed.  The oracle, given each seed's sweep count, recomputes the step
-    of that seed with exactly that many sweeps."""
+    of that seed with exactly that many sweeps.  wpath: the converged seeds'
+    pass-through runs in the frozen-sweep kernels ("1") or in the reverse
+    kernel ("0")."""
+    monkeypatch.setenv("SMOOTHE_REV_W", wpath)
     eg = make_config(name)
     g = sm.load_egraph_from(eg)
     opts = sm.Options(assumption=agg, prop_iters=K, lam=1.0, penalty_group=1, rng_key=3,
@@ -267,7 +274,9 @@ def test_converge_mode_parity(sm, orc, name, B, K, agg):
     theta = np.random.default_rng(K + B).uniform(-2, 2, (eg.num_nodes, B)).astype(np.float32)
     d = run.debug_step(theta, route=True)
     sw = d["sweeps"]
-    assert np.all((sw >= 1) & (sw <= K)) and np.median(sw) < K, sw  # most seeds converged
+    assert np.all((sw >= 1) & (sw <= K)), sw
+    if name == "C2":
+        assert np.median(sw) < K, sw  # most seeds converged
     og = orc.Graph(eg)
     for b in list(range(0, B, max(1, B // 8))):
         th = theta[:, [b]].astype(np.float64)
@@ -279,7 +288,13 @@ def test_converge_mode_parity(sm, orc, name, B, K, agg):
         close(f"p[{b}]", col(d["p"]), o["p"])
         close(f"f[{b}]", d["f"][[b]], o["f"])
         gco = o["grad_cp"]
-        close(f"grad_cp[{b}]", col(d["grad_cp"]), gco, scale=np.abs(gco))
+        if eg.quad is not None:  # cancellation in g_p: scale by the |w| backward (compare_step)
+            qi, qj, qw = eg.quad
+            eg.quad = (qi, qj, np.abs(qw))
+            oa = orc.Graph(eg).step(th, oo, route=d["route"][: sw[b], :, [b]])
+            eg.quad = (qi, qj, qw)
+            gco = np.maximum(np.abs(gco), np.abs(oa["grad_cp"]))
+        close(f"grad_cp[{b}]", col(d["grad_cp"]), o["grad_cp"], scale=np.abs(gco))
         cpo = o["cp"]
         gscale = cpo * (np.abs(gco) + class_sums(eg, cpo * np.abs(gco)))
         close(f"grad_theta[{b}]", col(d["grad_theta"]), o["grad_theta"], scale=gscale)
