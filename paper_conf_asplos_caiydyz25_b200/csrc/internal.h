@@ -250,6 +250,9 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
                           const int32_t* lastchg = nullptr);
+// sets the conditional handle to 1 iff some seed is not frozen (wm[s] == 0)
+void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
+                         cudaGraphConditionalHandle h);
 // W from the K-state rows (before reverse sweep K)
 void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                    const SweepState& st, const float* cp);

@@ -1161,4 +1161,21 @@ void launch_last_change(cudaStream_t s, const Shape& sh, const SweepState& st) {
   SM_LAUNCH_CHECK();
 }
 
+
+// Conditional graph node of the plain reverse sweep: run it iff some seed is
+// not frozen (the real seeds; padded columns carry nothing anyone reads).
+__global__ void k_any_unfrozen(cudaGraphConditionalHandle h, const int32_t* __restrict__ wm,
+                               int Bp) {
+  int any = 0;
+  for (int b = threadIdx.x; b < Bp; b += blockDim.x) any |= wm[b] == 0;
+  any = __syncthreads_or(any);
+  if (threadIdx.x == 0) cudaGraphSetConditional(h, any ? 1u : 0u);
+}
+
+void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
+                         cudaGraphConditionalHandle h) {
+  k_any_unfrozen<<<1, 256, 0, s>>>(h, wm, sh.B);
+  SM_LAUNCH_CHECK();
+}
+
 }  // namespace smoothe
