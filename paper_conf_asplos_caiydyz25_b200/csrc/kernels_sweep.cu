@@ -928,11 +928,14 @@ constexpr int kWBlock = SMOOTHE_WSPMV_BLOCK;
 #ifndef SMOOTHE_WSPMV_DEPTH
 #define SMOOTHE_WSPMV_DEPTH 6
 #endif
+#ifndef SMOOTHE_WSPMV_MINB16
+#define SMOOTHE_WSPMV_MINB16 1  // min resident blocks for narrower rows (LPR <= 16)
+#endif
 #ifndef SMOOTHE_WSPMV_DEPTH32
 #define SMOOTHE_WSPMV_DEPTH32 4
 #endif
 template <int LPR, bool STREAM, bool CONV>
-__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : 1) k_wspmv(
+__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : SMOOTHE_WSPMV_MINB16) k_wspmv(
     int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
     const int32_t* __restrict__ cls_child, const float* __restrict__ W,
