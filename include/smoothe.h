@@ -176,6 +176,10 @@ typedef struct {
   double time_to_best_s;   /* run creation -> end of best_step, CUDA events                */
   double step_time_s;      /* mean device time per step                                    */
   double last_loss;        /* L of the last step = sum_b f_b + lambda * sum_g G h_g (S12) */
+  int32_t graph_mode;      /* how the steps ran: 1 = replayed from the captured CUDA graph, */
+                           /* 0 = direct launches (use_graphs = 0, profiling or debug),     */
+                           /* -1 = capture failed, fell back to direct launches (warned on  */
+                           /* stderr; results identical, timing not the graph path's)       */
 } smoothe_summary;
 
 /* Copies the best extraction: choice[M] = chosen e-node of each selected class,
@@ -205,8 +209,9 @@ typedef struct {
   uint8_t *valid;      /* [B]                                                  */
   double *disc_cost;   /* [B]     f_b(s), +inf when invalid                    */
   float *qstack;       /* [(K+1)][M][B] or NULL                                */
-  int32_t *route;      /* [K][M][B] e-node the max of sweep t routed to, i.e.  */
-                       /* the lowest id attaining the fp32 max (reading S7);  */
+  int32_t *route;      /* [K][M][B] e-node the max of sweep t routed to: the  */
+                       /* champion of the ascending-id scan with takeover at */
+                       /* p > p_champion (1 + 2^-10), fp32 (reading S7');    */
                        /* -1 for classes without parents; NULL = skip         */
   int32_t *sweeps;     /* [B]     sweeps the seed's step performed (K, or its */
                        /* convergence sweep with converge = 1); NULL = skip  */
@@ -230,7 +235,8 @@ SMOOTHE_API smoothe_status smoothe_debug_step(smoothe_run *run, const float *the
  *   class_cost  [M] caller-owned or NULL: the heuristic's class cost (its tree
  *               estimate, shared subterms counted once per use); +inf for
  *               classes without a finite derivation or unreachable from the root
- * Errors: E_INVALID_ARG (NULL g / u / out), E_STATE (host-only e-graph), E_CUDA.
+ * Errors: E_INVALID_ARG (NULL g / u / out, or a negative or non-finite u: the
+ * worklist's fixpoint needs u >= 0), E_STATE (host-only e-graph), E_CUDA.
  * ------------------------------------------------------------------------- */
 typedef struct {
   double dag_cost;          /* f_b(s) of the extraction: sum of u over the selected
@@ -251,6 +257,13 @@ SMOOTHE_API smoothe_status smoothe_run_warm_start(smoothe_run *run, const int32_
 
 /* theta [N][B] of the run as it stands (host copy). */
 SMOOTHE_API smoothe_status smoothe_get_theta(smoothe_run *run, float *theta);
+
+/* The optimiser state as it stands, host copies [N][B] (any pointer may be
+ * NULL), and the number of steps run: a debug step from this state with
+ * step_index = *steps_run continues the run exactly (tests: parity after
+ * steps replayed from the CUDA graph). */
+SMOOTHE_API smoothe_status smoothe_get_state(smoothe_run *run, float *theta, float *m, float *v,
+                                             int32_t *steps_run);
 
 /* ---------------------------------------------------------------------------
  * Measurement.  With profiling on, every phase of every step is bracketed by

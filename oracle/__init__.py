@@ -47,14 +47,15 @@ class _Cost(C.Structure):
 class _Opts(C.Structure):
     _fields_ = [("assumption", C.c_int32), ("K", C.c_int32), ("lam", C.c_double),
                 ("G", C.c_int32), ("lr", C.c_double), ("beta1", C.c_double),
-                ("beta2", C.c_double), ("eps", C.c_double), ("optimizer", C.c_int32)]
+                ("beta2", C.c_double), ("eps", C.c_double), ("optimizer", C.c_int32),
+                ("route_delta", C.c_double), ("route_alt", C.c_int32)]
 
 
 class _Dump(C.Structure):
     _fields_ = [(n, C.c_void_p) for n in
                 ("cp", "qstack", "p", "f", "h", "loss", "grad_cp", "grad_theta", "theta_out",
                  "m_out", "v_out", "choice", "valid", "disc_cost", "reached", "route",
-                 "route_invalid")]
+                 "route_margin", "route_margin_all", "route_namb", "grad_cp_spread")]
 
 
 def lib():
@@ -118,14 +119,20 @@ def expm(A: np.ndarray) -> np.ndarray:
 
 class Options:
     def __init__(self, assumption="hybrid", K=-1, lam=1.0, G=1, lr=0.1, beta1=0.9,
-                 beta2=0.999, eps=1e-8, optimizer="adam"):
+                 beta2=0.999, eps=1e-8, optimizer="adam", route_delta=1e-5, route_alt=0):
+        """route_delta: relative margin below which a max-routing comparison
+        may go either way (reading S7', smoothe_oracle.cpp backward());
+        route_alt (pins of the spread bound only): 1 / 2 route decisions with
+        several admissible routes to the highest / lowest admissible parent."""
         self.assumption, self.K, self.lam, self.G = assumption, K, lam, G
         self.lr, self.beta1, self.beta2, self.eps = lr, beta1, beta2, eps
         self.optimizer = optimizer
+        self.route_delta, self.route_alt = route_delta, route_alt
 
     def c(self) -> _Opts:
         return _Opts(ASSUMPTIONS[self.assumption], self.K, self.lam, self.G, self.lr, self.beta1,
-                     self.beta2, self.eps, 0 if self.optimizer == "adam" else 1)
+                     self.beta2, self.eps, 0 if self.optimizer == "adam" else 1,
+                     self.route_delta, self.route_alt)
 
 
 def update(theta, grad, opts: Options, m=None, v=None, step_index=0):
@@ -192,11 +199,21 @@ class Graph:
         lib().oracle_graph_scc(self.h, _p(out))
         return out
 
-    def step(self, theta, opts: Options, m=None, v=None, step_index=0, qstack=False, route=None):
+    def step(self, theta, opts: Options, m=None, v=None, step_index=0, qstack=False, route=False,
+             spread=False):
         """One step for B seeds; theta [N][B] (any float dtype; upcast exactly).
 
-        route [K][M][B] int32 (optional): the max-routing decisions of the
-        system under test; the oracle validates and uses them (backward())."""
+        Every decision is the oracle's own (fp64).  Always returned:
+        route_margin / route_margin_all [B], the smallest relative margin of a
+        max-routing decision (reading S7', smoothe_oracle.cpp backward()) that
+        the gradient uses / of any decision, and route_namb [B], the number
+        of decisions (sweep, class) the gradient uses that have several
+        admissible routes (comparisons within opts.route_delta may go either
+        way).  route=True adds the oracle's routes [K][M][B] int32 (-1: root
+        or no parents; -2 - k: fp64 outcome k, other routes admissible).
+        spread=True adds grad_cp_spread [N][B]: an elementwise bound on how
+        far g_cp can move over all admissible routings (0 where none
+        reaches)."""
         theta = np.ascontiguousarray(theta, dtype=np.float64)
         N, B = theta.shape
         assert N == self.N
@@ -213,12 +230,13 @@ class Graph:
         }
         if qstack:
             out["qstack"] = np.zeros((K + 1, self.M, B))
-        out["route_invalid"] = np.zeros(B, dtype=np.int64)
-        keep = None
-        if route is not None:
-            keep = np.ascontiguousarray(route, dtype=np.int32)
-            assert keep.shape == (K, self.M, B)
-            out["route"] = keep
+        out["route_margin"] = np.zeros(B)
+        out["route_margin_all"] = np.zeros(B)
+        out["route_namb"] = np.zeros(B, dtype=np.int32)
+        if spread:
+            out["grad_cp_spread"] = np.zeros((N, B))
+        if route:
+            out["route"] = np.zeros((K, self.M, B), dtype=np.int32)
         d = _Dump(**{k: _p(a) for k, a in out.items()})
         rc = lib().oracle_step(self.h, C.byref(self.cost), C.byref(opts.c()), B, _p(theta), _p(m),
                                _p(v), step_index, C.byref(d))

@@ -263,6 +263,8 @@ struct oracle_opts {
   int32_t G;           // penalty group size (S13)
   double lr, beta1, beta2, eps;
   int32_t optimizer;   // 0 Adam, 1 SGD (S10)
+  double route_delta;  // margin below which a routing comparison may go either way (see backward)
+  int32_t route_alt;   // 0: fp64 champion; 1 / 2: the highest / lowest-id admissible route
 };
 
 // Outputs of one step; every pointer may be NULL.  [row][B] layout.
@@ -282,8 +284,11 @@ struct oracle_dump {
   uint8_t* valid;      // [B]
   double* disc_cost;   // [B]      f_b(s), +inf when invalid
   uint8_t* reached;    // [M][B]
-  const int32_t* route;   // INPUT [K][M][B] or NULL: max-routing decisions to use (see backward)
-  int64_t* route_invalid; // [B] routes that are not near-maximising parents
+  int32_t* route;         // [K][M][B] the oracle's own max routes (reading S7', see backward)
+  double* route_margin;   // [B] smallest relative margin of a routing decision the gradient uses
+  double* route_margin_all; // [B] the same over every routing decision
+  int32_t* route_namb;    // [B] decisions (sweep, class) with several admissible routes, g_q != 0
+  double* grad_cp_spread; // [N][B] bound on |g_cp| deviation over the admissible routings
 };
 
 void* oracle_graph_new(int32_t M, int32_t N, const int32_t* class_ptr, const int64_t* child_ptr,
@@ -456,30 +461,93 @@ double cost_and_grad(const Graph& g, const oracle_cost& c, const double* p, doub
 }
 
 // Reverse mode of the sweeps.  Exclusive products are
-// formed from prefix and suffix products: no division (reading S8); the max
-// routes to the lowest e-node id among the maximisers (reading S7).
+// formed from prefix and suffix products: no division (reading S8).
 //
-// The arg-max of the correlated term is a floating-point DECISION.  When
-// `route` is given ([K][M] with stride `rstride` per class, the e-node each
-// sweep's max routed to, as decided by the system under test in its own
-// precision), the oracle uses it -- after checking that it is a valid
-// subgradient choice: a parent of the class whose p is a maximiser up to the
-// parity tolerance of p (1e-4 relative + 1e-6 absolute: fp32 rounding, which
-// is absolute where 1 - prod cancels); violations are counted in *invalid.
+// Route of the max (reading S7'): the correlated term's
+// subgradient goes to one parent a^t_j of class j, chosen by a scan of pa_j in
+// ascending e-node id: the first parent is the champion c, and a later parent
+// k takes over iff p_k > p_c (1 + tau), tau = 2^-10.  Parents whose p agree to
+// better than tau (structural ties, computed along different rounding paths)
+// therefore route to the lowest id in any precision; the routed parent attains
+// the max within a factor 1 + tau.  The decision is taken here, in fp64, from
+// the oracle's own p; the system under test takes it in its own precision.
+//
+// Where fp32 and fp64 may disagree -- a comparison of the scan within a
+// relative margin delta of its threshold, margin = |p_k - p_c (1+tau)| /
+// max(p_k, p_c (1+tau)) -- the oracle reports it instead of hiding it, and
+// bounds its effect:
+//  * *margin / *margin_all: the smallest margin over the comparisons on the
+//    scan paths of the decisions the gradient uses (g_q^t_j != 0) / of all
+//    decisions (comparisons of two exact zeros -- classes outside the
+//    activity window -- have no margin: zeros agree in every precision);
+//  * the admissible routes adm_j of a decision: the champions the scan can
+//    end with when every comparison within delta may go either way (a
+//    system whose p carry relative errors below delta/2 ends in adm_j);
+//  * spread (optional): an elementwise bound U on |g_cp(rho) - g_cp| over
+//    every routing rho that picks from adm_j at every decision.  The reverse
+//    mode has non-negative coefficients (D_jk >= 0, cp, q >= 0), so the
+//    deviation obeys |e_p^t_k| <= sum_j |e_q^t_j| Dmax_jk + sum_{j: |adm_j|>1,
+//    k in adm_j} wC |g_q^t_j| with Dmax_jk = wI prod_{k' != k}(1 - p_k') +
+//    wC [k in adm_j]; U is that recursion run beside the gradient:
+//      U_p^t_k = sum_j U_q^t_j Dmax_jk + wC sum_{j: |adm_j| > 1, k in adm_j} |g_q^t_j|
+//      U_gcp_k += U_p^t_k q^{t-1}_{ec(k)},  U_q^{t-1}_j = sum_{k in m_j} U_p^t_k cp_k.
+//    It is 0 wherever no near-threshold decision reaches.
+//  * alt (tests): route every decision with several admissible routes to the
+//    highest (1) or lowest (2) admissible parent instead, an admissible
+//    routing whose gradient must stay within the spread.
+// route (optional): the oracle's own routes, [K][M] with stride rstride
+// (-1 for the root and for classes without parents; -2 - k when the
+// decision, whose fp64 outcome is e-node k, has other admissible routes).
+constexpr double kRouteTau = 1.0 / 1024.0;
+
+struct RouteIO {
+  double delta = 0.0;
+  int32_t* route = nullptr;
+  size_t rstride = 1;
+  double* spread = nullptr;               // [N] (stride sstride) or NULL
+  size_t sstride = 1;
+  double margin = std::numeric_limits<double>::infinity();
+  double margin_all = std::numeric_limits<double>::infinity();
+  int64_t namb = 0;                       // decisions with |adm| > 1 and g_q != 0
+  int alt = 0;                            // 1 / 2: route to the highest / lowest admissible
+};
+
+// champions reachable by the scan over pt[pa[0..n)] when comparisons within
+// delta may go either way (positions into pa; depth-first over the branches)
+void admissible(const std::vector<int>& pa, const std::vector<double>& pt, double delta,
+                size_t a, size_t champ, std::vector<char>& adm, int budget, bool& overflow) {
+  for (; a < pa.size(); ++a) {
+    const double pk = pt[pa[a]], thr = pt[pa[champ]] * (1.0 + kRouteTau);
+    const bool take = pk > thr;
+    if (!(pk == 0.0 && thr == 0.0) && std::fabs(pk - thr) / std::max(pk, thr) < delta) {
+      if (budget <= 0) { overflow = true; return; }
+      admissible(pa, pt, delta, a + 1, take ? champ : a, adm, budget - 1, overflow);  // other way
+    }
+    if (take) champ = a;
+  }
+  adm[champ] = 1;
+}
+
 void backward(const Graph& g, int K, Weights w, const double* cp, const double* qstack,
-              const double* gp, double* gcp, const int32_t* route = nullptr,
-              size_t rstride = 1, int64_t* invalid = nullptr) {
+              const double* gp, double* gcp, RouteIO* rio = nullptr) {
   const int M = g.M, N = g.N;
   const double* qK = qstack + (size_t)K * M;
   std::vector<double> gq(M, 0.0), gq_prev(M), gpt(N), pt(N);
   for (int i = 0; i < N; ++i) gcp[i] = gp[i] * qK[g.ec[i]];           // p = cp * q^K[ec]
   for (int i = 0; i < N; ++i) gq[g.ec[i]] += gp[i] * cp[i];
   gq[g.root] = 0.0;                                                    // q_root is constant (S3)
+  const double delta = rio ? rio->delta : 0.0;
+  const bool unc = rio && rio->spread;
+  std::vector<double> uq(unc ? M : 0, 0.0), uq_prev(unc ? M : 0), up(unc ? N : 0), ugcp(unc ? N : 0, 0.0);
   std::vector<double> pre, suf;
+  std::vector<char> adm;
   for (int t = K; t >= 1; --t) {
     const double* qprev = qstack + (size_t)(t - 1) * M;
     for (int k = 0; k < N; ++k) { pt[k] = cp[k] * qprev[g.ec[k]]; gpt[k] = 0.0; }
+    if (unc) std::fill(up.begin(), up.end(), 0.0);
     for (int j = 0; j < M; ++j) {
+      int32_t* rt = rio && rio->route ? rio->route + ((size_t)(t - 1) * M + j) * rio->rstride : nullptr;
+      if (rt) *rt = -1;
       if (j == g.root) continue;
       const auto& pa = g.pa[j];
       const size_t n = pa.size();
@@ -488,25 +556,50 @@ void backward(const Graph& g, int K, Weights w, const double* cp, const double* 
       suf.assign(n + 1, 1.0);
       for (size_t a = 0; a < n; ++a) pre[a + 1] = pre[a] * (1.0 - pt[pa[a]]);
       for (size_t a = n; a > 0; --a) suf[a - 1] = suf[a] * (1.0 - pt[pa[a - 1]]);
+      // the champion scan of reading S7'
       size_t amax = 0;
-      for (size_t a = 1; a < n; ++a)
-        if (pt[pa[a]] > pt[pa[amax]]) amax = a;  // strict: lowest id wins ties
-      if (route && w.wC != 0.0) {
-        const int r = route[((size_t)(t - 1) * M + j) * rstride];
-        const double mx = pt[pa[amax]];
-        size_t pos = n;
-        for (size_t a = 0; a < n; ++a)
-          if (pa[a] == r) pos = a;
-        // valid iff the routed parent attains the max within the parity bar
-        // (1e-4 relative + 1e-6 absolute, the fp32-vs-fp64 tolerance of p)
-        if (pos == n || pt[r] < mx - (1e-4 * mx + 1e-6)) {
-          if (invalid) ++*invalid;
+      for (size_t a = 1; a < n; ++a) {
+        const double pk = pt[pa[a]], thr = pt[pa[amax]] * (1.0 + kRouteTau);
+        if (rio && w.wC != 0.0 && !(pk == 0.0 && thr == 0.0)) {
+          const double dm = std::fabs(pk - thr) / std::max(pk, thr);
+          rio->margin_all = std::min(rio->margin_all, dm);
+          if (gq[j] != 0.0) rio->margin = std::min(rio->margin, dm);
         }
-        if (pos < n) amax = pos;
+        if (pk > thr) amax = a;
       }
+      int nadm = 1;
+      if (rio && w.wC != 0.0 && n > 1) {
+        adm.assign(n, 0);
+        bool overflow = false;
+        admissible(pa, pt, delta, 1, 0, adm, 16, overflow);
+        if (overflow) {  // a superset: every parent within a factor (1+tau)(1+delta)^2 of the max
+          double mx = 0.0;
+          for (size_t a = 0; a < n; ++a) mx = std::max(mx, pt[pa[a]]);
+          for (size_t a = 0; a < n; ++a)
+            adm[a] = pt[pa[a]] * (1.0 + kRouteTau) * (1.0 + delta) * (1.0 + delta) >= mx;
+        }
+        adm[amax] = 1;
+        nadm = 0;
+        for (size_t a = 0; a < n; ++a) nadm += adm[a];
+        if (nadm > 1 && gq[j] != 0.0) rio->namb++;
+        if (nadm > 1 && rio->alt) {  // an alternative admissible routing (tests of the bound)
+          size_t pick = amax;
+          for (size_t a = 0; a < n; ++a)
+            if (adm[a] && (rio->alt == 1 || pick == amax)) pick = a;
+          if (rio->alt == 2) for (size_t a = 0; a < n; ++a) if (adm[a]) { pick = a; break; }
+          amax = pick;
+        }
+      }
+      if (rt) *rt = nadm > 1 ? -2 - pa[amax] : pa[amax];
       for (size_t a = 0; a < n; ++a) {
-        double D = w.wI * (pre[a] * suf[a + 1]) + w.wC * (a == amax ? 1.0 : 0.0);
+        const double excl = pre[a] * suf[a + 1];
+        double D = w.wI * excl + w.wC * (a == amax ? 1.0 : 0.0);
         gpt[pa[a]] += gq[j] * D;
+        if (unc) {
+          const bool in = nadm > 1 ? adm[a] != 0 : a == amax;
+          up[pa[a]] += uq[j] * (w.wI * excl + w.wC * (in ? 1.0 : 0.0));
+          if (nadm > 1 && in) up[pa[a]] += w.wC * std::fabs(gq[j]);
+        }
       }
     }
     for (int k = 0; k < N; ++k) gcp[k] += gpt[k] * qprev[g.ec[k]];
@@ -514,7 +607,16 @@ void backward(const Graph& g, int K, Weights w, const double* cp, const double* 
     for (int k = 0; k < N; ++k) gq_prev[g.ec[k]] += gpt[k] * cp[k];
     gq_prev[g.root] = 0.0;
     gq.swap(gq_prev);
+    if (unc) {
+      for (int k = 0; k < N; ++k) ugcp[k] += up[k] * qprev[g.ec[k]];
+      std::fill(uq_prev.begin(), uq_prev.end(), 0.0);
+      for (int k = 0; k < N; ++k) uq_prev[g.ec[k]] += up[k] * cp[k];
+      uq_prev[g.root] = 0.0;
+      uq.swap(uq_prev);
+    }
   }
+  if (unc)
+    for (int k = 0; k < N; ++k) rio->spread[(size_t)k * rio->sstride] = ugcp[k];
 }
 
 // Optimiser step on one logit (reading S10): Adam with bias correction
@@ -644,10 +746,17 @@ int oracle_step(void* hg, const oracle_cost* cost, const oracle_opts* opt, int32
     std::vector<double> q((size_t)(K + 1) * M), p(N), gp(N), gcp(N), gth(N);
     forward(g, K, w, cp[b].data(), q.data(), p.data());
     fvals[b] = cost_and_grad(g, *cost, p.data(), gp.data());
-    int64_t bad = 0;
-    backward(g, K, w, cp[b].data(), q.data(), gp.data(), gcp.data(),
-             out->route ? out->route + b : nullptr, (size_t)B, &bad);
-    if (out->route_invalid) out->route_invalid[b] = bad;
+    RouteIO rio;
+    rio.delta = opt->route_delta;
+    rio.alt = opt->route_alt;
+    rio.route = out->route ? out->route + b : nullptr;
+    rio.rstride = (size_t)B;
+    rio.spread = out->grad_cp_spread ? out->grad_cp_spread + b : nullptr;
+    rio.sstride = (size_t)B;
+    backward(g, K, w, cp[b].data(), q.data(), gp.data(), gcp.data(), &rio);
+    if (out->route_margin) out->route_margin[b] = rio.margin;
+    if (out->route_margin_all) out->route_margin_all[b] = rio.margin_all;
+    if (out->route_namb) out->route_namb[b] = (int32_t)rio.namb;
     const int gi = b / G;
     for (int k = 0; k < N; ++k) gcp[k] += pen[gi][k];
     // softmax backward: g_theta_i = cp_i (g_cp_i - sum_{k in m_ec(i)} cp_k g_cp_k)

@@ -30,7 +30,6 @@ namespace smoothe {
 
 namespace {
 
-// Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique).
 // Class graph successors: j -> c for every c in ch_k, k in m_j (sorted, unique):
 // duplicates dropped with a per-class stamp, then the (short) unique list sorted.
 void class_successors(const HostGraph& g, std::vector<int32_t>& ptr, std::vector<int32_t>& adj) {

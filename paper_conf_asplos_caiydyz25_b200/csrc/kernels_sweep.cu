@@ -22,6 +22,8 @@
 namespace smoothe {
 
 constexpr int kSweepBlock = 64;
+// 1 + tau of reading S7' (exact in fp32)
+constexpr float kRouteTau1 = 1.0f + 1.0f / 1024.0f;
 
 // ---------------------------------------------------------------------------
 // Forward sweep t (readings S2-S4, S6-S8):
@@ -29,7 +31,11 @@ constexpr int kSweepBlock = 64;
 //   q^t_j = wI (1 - prod_{k in pa_j}(1 - p^t_k)) + wC max_{k in pa_j} p^t_k   (Eqs. 6b, 7)
 // and, for the reverse sweep, pi = the product over the non-zero factors signed
 // by the number of zero factors (+: none, -: exactly one, 0: two or more), and
-// am = the lowest e-node id attaining the max (reading S7).  The independent
+// am = the route of the max (reading S7'): parents are
+// scanned in ascending e-node id, the first is the champion, and a later one
+// takes over iff its p exceeds the champion's by more than a factor 1 + tau
+// (tau = 2^-10), so parents tied up to rounding route to the lowest id.  The
+// max itself (the correlated term) is the exact fp32 max.  The independent
 // term 1 - prod(1 - p) is accumulated as the union u <- u + p (1 - u), which
 // keeps its relative accuracy when every p is small (1 - prod of factors
 // rounded near 1 loses it: q ~ 1e-4 came out 5e-4 off in fp32); a zero factor
@@ -85,6 +91,7 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
   float4 un = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
+  float4 pc = mx;  // the routing champion's p (reading S7')
   int4 arg = make_int4(-1, -1, -1, -1);
   int4 zc = make_int4(0, 0, 0, 0);
   int4 n01 = make_int4(0, 0, 0, 0), n23 = n01;
@@ -114,8 +121,9 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
         comp(un, x) = __fmaf_rn(p, __fsub_rn(1.f, comp(un, x)), comp(un, x));
-        const bool gt = p > comp(mx, x);
-        comp(mx, x) = gt ? p : comp(mx, x);
+        comp(mx, x) = fmaxf(comp(mx, x), p);
+        const bool gt = p > __fmul_rn(comp(pc, x), kRouteTau1);
+        comp(pc, x) = gt ? p : comp(pc, x);
         comp(arg, x) = gt ? kk[u] : comp(arg, x);
       }
     }
@@ -230,6 +238,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
   float4 prod = make_float4(1.f, 1.f, 1.f, 1.f);
   float4 un = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 mx = make_float4(-1.f, -1.f, -1.f, -1.f);
+  float4 pc = mx;  // the routing champion's p (reading S7')
   int4 arg = make_int4(-1, -1, -1, -1);
   int4 zc = make_int4(0, 0, 0, 0);
   int4 n01 = make_int4(0, 0, 0, 0), n23 = n01;
@@ -259,8 +268,9 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
         comp(zc, x) += f == 0.f ? 1 : 0;
         comp(prod, x) = f == 0.f ? comp(prod, x) : __fmul_rn(comp(prod, x), f);
         comp(un, x) = __fmaf_rn(p, __fsub_rn(1.f, comp(un, x)), comp(un, x));
-        const bool gt = p > comp(mx, x);
-        comp(mx, x) = gt ? p : comp(mx, x);
+        comp(mx, x) = fmaxf(comp(mx, x), p);
+        const bool gt = p > __fmul_rn(comp(pc, x), kRouteTau1);
+        comp(pc, x) = gt ? p : comp(pc, x);
         comp(arg, x) = gt ? kk[u] : comp(arg, x);
       }
     }

@@ -248,6 +248,7 @@ struct smoothe_run {
   // graph
   cudaGraphExec_t graph_exec = nullptr;
   bool graph_failed = false;
+  int64_t graph_steps = 0;  // steps replayed from graph_exec
   bool poisoned = false;
   int steps_run = 0;
 };
@@ -558,10 +559,13 @@ void run_one_step(smoothe_run* r) {
       (void)cudaGetLastError();
       r->graph_exec = nullptr;
       r->graph_failed = true;  // fall back to direct launches (still all on the GPU)
+      std::fprintf(stderr, "[smoothe] warning: CUDA graph capture of the step failed; "
+                   "running direct launches (set SMOOTHE_GRAPH_DEBUG=1 for the reason)\n");
     }
   }
   if (use_graph && r->graph_exec) {
     SM_CUDA(cudaGraphLaunch(r->graph_exec, r->stream));
+    r->graph_steps++;
   } else {
     enqueue_step(r);
   }
@@ -931,6 +935,11 @@ smoothe_status smoothe_greedy(smoothe_egraph* g, const double* u, int32_t* choic
     } fr{o};
     SM_CUDA(cudaStreamCreateWithFlags(&fr.s, cudaStreamNonBlocking));
     std::vector<double> uh(u, u + hg.N);
+    // the worklist's fixpoint needs u >= 0: a negative cost on a cycle would
+    // lower a class's key on every pass (Bellman-Ford without termination)
+    for (int i = 0; i < hg.N; ++i)
+      SM_REQUIRE(std::isfinite(uh[i]) && uh[i] >= 0.0, SMOOTHE_E_INVALID_ARG,
+                 "greedy needs finite non-negative costs u");
     double* ud = upload(o, uh);
     double* cost = dalloc<double>(o, M);
     int32_t* ints = dalloc<int32_t>(o, (size_t)6 * M + 3 + grid);
@@ -1156,6 +1165,7 @@ smoothe_status smoothe_extract(smoothe_run* run, int32_t* choice, smoothe_summar
       out->steps_run = run->steps_run;
       out->K = run->K;
       out->last_loss = loss;
+      out->graph_mode = run->graph_failed ? -1 : (run->graph_steps > 0 ? 1 : 0);
       float ms = 0.f;
       const int bs = out->best_step;
       if (valid && bs >= 0 && (size_t)bs < run->ev_step.size() && bs < run->steps_run) {
@@ -1289,7 +1299,7 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     if (dump->route) {
       // Row t = sweep t + 1.  A class not recomputed in that sweep takes the
       // row of its version; version 0 (every p exactly 0, so every parent
-      // ties) is the lowest-id parent, the kernel's tie rule (S7), and -1 for
+      // ties) is the lowest-id parent, the kernel's tie rule (S7'), and -1 for
       // the root (q_root = 1 is not a decision, S3) and parentless classes.
       const HostGraph& hg = run->g->host;
       for (int t = 0; t < run->K; ++t)
@@ -1321,6 +1331,18 @@ smoothe_status smoothe_get_theta(smoothe_run* run, float* theta) {
     SM_REQUIRE(theta, SMOOTHE_E_INVALID_ARG, "NULL theta");
     copy_rows_d2h(theta, run->theta, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
     SM_CUDA(cudaStreamSynchronize(run->stream));
+  });
+}
+
+smoothe_status smoothe_get_state(smoothe_run* run, float* theta, float* m, float* v,
+                                 int32_t* steps_run) {
+  return guarded(run, [&] {
+    check_run(run);
+    if (theta) copy_rows_d2h(theta, run->theta, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
+    if (m) copy_rows_d2h(m, run->m, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
+    if (v) copy_rows_d2h(v, run->v, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+    if (steps_run) *steps_run = run->steps_run;
   });
 }
 

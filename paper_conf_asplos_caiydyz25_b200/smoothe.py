@@ -58,7 +58,7 @@ class _Summary(C.Structure):
     _fields_ = [("best_cost", C.c_double), ("best_seed", C.c_int64), ("best_step", C.c_int32),
                 ("valid", C.c_int32), ("steps_run", C.c_int32), ("K", C.c_int32),
                 ("time_to_best_s", C.c_double), ("step_time_s", C.c_double),
-                ("last_loss", C.c_double)]
+                ("last_loss", C.c_double), ("graph_mode", C.c_int32)]
 
 
 class _Dump(C.Structure):
@@ -98,6 +98,7 @@ _SIGS = {
     "smoothe_debug_step": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32,
                                      C.POINTER(_Dump)]),
     "smoothe_get_theta": (C.c_int, [C.c_void_p, C.c_void_p]),
+    "smoothe_get_state": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
     "smoothe_greedy": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
                                  C.POINTER(_Greedy)]),
     "smoothe_run_warm_start": (C.c_int, [C.c_void_p, C.c_void_p, C.c_float]),
@@ -309,6 +310,13 @@ class Run:
         out = np.zeros((self.egraph.N, self.B), np.float32)
         _check(lib().smoothe_get_theta(self._h, _p(out)))
         return out
+
+    def state(self):
+        """smoothe_get_state: (theta, m, v) [N][B] float32 and the steps run."""
+        th, m, v = (np.zeros((self.egraph.N, self.B), np.float32) for _ in range(3))
+        n = C.c_int32(0)
+        _check(lib().smoothe_get_state(self._h, _p(th), _p(m), _p(v), C.byref(n)))
+        return th, m, v, n.value
 
     def debug_step(self, theta=None, m=None, v=None, step_index=0, qstack=False, route=False):
         N, M, B = self.egraph.N, self.egraph.M, self.B

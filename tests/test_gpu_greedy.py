@@ -93,3 +93,17 @@ def test_planted_set_cover_beats_heuristic(sm, k):
     assert s["valid"] == 1 and s["best_cost"] == 2 * k
     run.close()
     g.close()
+
+
+def test_rejects_negative_or_nonfinite_costs(sm):
+    """A negative cost on a cycle would make the worklist relax forever: the
+    library refuses it up front (E_INVALID_ARG) and stays usable."""
+    eg = random_tiny(5100, "cyclic")
+    g = sm.load_egraph_from(eg)
+    for bad in (-1.0, float("nan"), float("inf")):
+        u = eg.u.copy()
+        u[1] = bad
+        with pytest.raises(Exception):
+            g.greedy(u)
+    g.greedy(eg.u)
+    g.close()
