@@ -291,6 +291,14 @@ class Run:
     def synchronize(self):
         _check(lib().smoothe_run_synchronize(self._h))
 
+    def summary(self):
+        """smoothe_extract without the extraction: the summary dict alone."""
+        s = _Summary()
+        st = lib().smoothe_extract(self._h, None, C.byref(s))
+        if st not in (OK, E_NO_VALID):
+            _check(st)
+        return {n: getattr(s, n) for n, _ in _Summary._fields_}
+
     def extract(self):
         """(choice [M] int32 with -1 for unselected classes, summary dict)."""
         choice = np.zeros(self.egraph.M, np.int32)

@@ -87,3 +87,34 @@ def test_global_best_gloo_world2():
     assert (c0, sd0, o0, ch0) == (11.0, 70, 1, [0, 6, 7])
     assert (c1, s1, o1, ch1) == (11.0, 4, 0, [0, 5, -1])
     assert (c2, o2, ch2) == (30.0, 1, [0, 1, 2])
+
+
+def _bench_dry(gpus):
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--dry-run-cpu",
+                          "--gpus", str(gpus), "--ttb-steps", "200", "--patience", "20"],
+                         capture_output=True, text=True, timeout=300, cwd=root)
+    assert out.returncode == 0, out.stderr[-2000:]
+    return json.loads([l for l in out.stdout.splitlines() if l.startswith("{")][-1])
+
+
+def test_bench_launcher_world2_global_patience():
+    """`bench.py --gpus 2` without torchrun re-executes itself with 2 ranks
+    (here on gloo, with bench's deterministic stand-in for the GPU run): the
+    line reports n_gpus = 2, every rank agrees on the best and its
+    extraction, and the ranks stop TOGETHER on the global patience (reading
+    S21): rank 0's own seeds stop improving at step 21 (it alone would stop at
+    step 48, as the 1-rank run does) but rank 1's keep improving until step
+    45, so both run 72 steps."""
+    one = _bench_dry(1)
+    assert one["n_gpus"] == 1 and one["steps_run"] == 48 and one["stopped_by"] == "patience"
+    two = _bench_dry(2)
+    assert two["n_gpus"] == 2 and len(two["all_ranks"]) == 2
+    keys = ("steps_run", "stopped_by", "best_cost", "best_step", "best_seed", "owner", "choice")
+    r0, r1 = two["all_ranks"]
+    assert all(r0[k] == r1[k] for k in keys)
+    assert (r0["best_seed"], r0["best_step"], r0["owner"], r0["steps_run"]) == (15, 45, 1, 72)
+    assert r0["choice"] == [15, 8]          # the owner's extraction, broadcast
