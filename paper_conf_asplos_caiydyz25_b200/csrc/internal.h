@@ -249,7 +249,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
-                          const int32_t* lastchg = nullptr);
+                          const int32_t* lastchg = nullptr, int32_t* cursor = nullptr);
 // sets the conditional handle to 1 iff some seed is not frozen (wm[s] == 0)
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h);

@@ -15,7 +15,12 @@
 //  * no division in the inner loops: the reverse sweep forms one reciprocal per
 //    e-node (an IEEE divide per edge or per node cost ~30% of the sweep);
 //  * deterministic: every output row has exactly one owner, no atomics.
+#include <cuda.h>
+
 #include <algorithm>
+#include <cstdlib>
+#include <mutex>
+#include <vector>
 
 #include "kcommon.cuh"
 
@@ -817,11 +822,335 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
                                 class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq);
 }
 
+// ---------------------------------------------------------------------------
+// The reverse sweep with its child rows staged by the tensor-memory
+// accelerator (128-seed slices, fixed K).  The per-lane
+// double buffer of the register kernel above (three gathered 512-byte rows
+// per child slot, 12 per batch of 4 slots) is what holds its occupancy to ~12
+// warps per SM at 124 registers.  Here each batch's rows come from three
+// TMA gather4 instructions (cp.async.bulk.tensor.2d ... tile::gather4: the 4
+// child rows of the batch for one array, 2 KB, into shared memory), issued by
+// one lane a batch ahead into a 2-stage ring per warp and completed on an
+// mbarrier: in-flight rows cost no registers, so 16 warps per SM each keep a
+// batch in flight.  Items are taken in order from a per-(sweep, seed slice)
+// cursor, so the warps in flight work on a compact window of classes whose
+// child rows share L2; the next item's first batch is requested while the
+// current item finishes.  The arithmetic, the e-node bookkeeping and the
+// epilogue are the register kernel's (same results bit for bit).
+// ---------------------------------------------------------------------------
+#ifndef SMOOTHE_RT_WARPS
+#define SMOOTHE_RT_WARPS 8   // warps per CTA
+#endif
+#ifndef SMOOTHE_RT_STAGES
+#define SMOOTHE_RT_STAGES 3  // ring stages per warp (batches in flight: stages - 1 ahead)
+#endif
+#ifndef SMOOTHE_RT_CTAS
+#define SMOOTHE_RT_CTAS 1    // CTAs per SM
+#endif
+constexpr int kRtWarps = SMOOTHE_RT_WARPS, kRtStages = SMOOTHE_RT_STAGES;
+constexpr int kRtRow = 512;                        // bytes of a 128-seed row
+constexpr int kRtStage = 3 * 4 * kRtRow;           // g, pi, am rows of a batch
+constexpr int kRtSmem = kRtWarps * (kRtStages * kRtStage + kRtStages * 8);
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAIT_%=;\n\t}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap* map, uint32_t bar, int x,
+                                            int4 rows) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(dst),
+      "l"(map), "r"(bar), "r"(x), "r"(rows.x), "r"(rows.y), "r"(rows.z), "r"(rows.w)
+      : "memory");
+}
+__device__ __forceinline__ int4 shfl4(int4 v, int src) {
+  return make_int4(__shfl_sync(0xffffffffu, v.x, src), __shfl_sync(0xffffffffu, v.y, src),
+                   __shfl_sync(0xffffffffu, v.z, src), __shfl_sync(0xffffffffu, v.w, src));
+}
+
+// One warp walks items it = w, w + T, w + 2T, ... (T warps in the slice's
+// grid).  Per item, lane l holds the child classes (pad_child) and e-node
+// (pad_batch_node) of the item's batch l (an item has at most 32 batches),
+// loaded with one coalesced request; the next item's header and index rows
+// are requested while the current item runs.  Batches flow through a ring of
+// kRtStages stages: batch n + kRtStages - 1 is requested before batch n is
+// consumed, across item boundaries.
+template <bool HI, bool HC>
+__global__ void __launch_bounds__(32 * kRtWarps, SMOOTHE_RT_CTAS) k_sweep_reverse_tma(
+    const __grid_constant__ CUtensorMap tm_g, const __grid_constant__ CUtensorMap tm_pi,
+    const __grid_constant__ CUtensorMap tm_am, int n_items, int Bp, int root,
+    const int4* __restrict__ items, const int32_t* __restrict__ class_item_ptr,
+    const int32_t* __restrict__ pad_child, const int32_t* __restrict__ pad_batch_node, float wI,
+    float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
+    const float* __restrict__ gq, float* __restrict__ gcp, float* __restrict__ gq_prev,
+    float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
+    const int32_t* __restrict__ wm, int32_t* __restrict__ cursor) {
+  constexpr int V = 4, S = kRtStages;
+  (void)cursor;
+  extern __shared__ __align__(128) unsigned char rt_smem[];
+  const int lane = threadIdx.x % 32, wi = threadIdx.x / 32;
+  unsigned char* ring = rt_smem + (size_t)wi * S * kRtStage;
+  const uint32_t bar0 = smem_addr(rt_smem + (size_t)kRtWarps * S * kRtStage + wi * 8 * S);
+  const int slice = blockIdx.y;
+  const int s0 = slice * 128 + lane * V, x0 = slice * 128;
+  const int T = gridDim.x * kRtWarps;
+  // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
+  Vec<V> keep, zero;
+  {
+    bool allw = true;
+#pragma unroll
+    for (int x = 0; x < V; ++x) {
+      const bool w = wm && __ldg(wm + s0 + x) != 0;
+      keep.v[x] = w ? 0.f : 1.f;
+      zero.v[x] = 0.f;
+      allw = allw && w;
+    }
+    if (__all_sync(0xffffffffu, allw)) return;
+  }
+  if (lane == 0) {
+#pragma unroll
+    for (int st = 0; st < S; ++st) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8 * st));
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  __syncwarp();
+  constexpr uint32_t kTx = (1 + (HI ? 1 : 0) + (HC ? 1 : 0)) * 4 * kRtRow;
+  uint32_t nb = 0, nc = 0;  // batches requested / consumed by this warp
+  // one lane requests a batch (child classes j4) into the next stage, whose
+  // previous batch every lane has consumed (__syncwarp; the generic-proxy
+  // reads ordered before the async-proxy writes by the proxy fence)
+  auto issue = [&](int4 j4) {
+    __syncwarp();
+    if (lane == 0) {
+      asm volatile("fence.proxy.async.shared::cta;");
+      const uint32_t st = nb % S, bar = bar0 + 8 * st;
+      const uint32_t dst = smem_addr(ring + (size_t)st * kRtStage);
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(kTx));
+      tma_gather4(dst, &tm_g, bar, x0, j4);
+      if (HI) tma_gather4(dst + 4 * kRtRow, &tm_pi, bar, x0, j4);
+      if (HC) tma_gather4(dst + 8 * kRtRow, &tm_am, bar, x0, j4);
+    }
+    ++nb;
+  };
+  auto active = [&](int4 c0, int4 c1) {  // the register kernel's exits
+    return !(c1.z > t - 1) && !((int64_t)t + c1.w <= K) && c0.y < c0.z;
+  };
+  // A queue of items whose batches are requested: the current item, and up
+  // to kRtStages - 1 batches of the following items.  Item state: header,
+  // the lane-distributed index rows, batches requested so far.
+  struct Item {
+    int it;
+    int4 c0, c1;
+    int4 jl;   // lane l: child classes of batch c0.y + l
+    int kl;    // lane l: e-node of batch c0.y + l
+    bool act;
+  };
+  auto load_item = [&](int it) {
+    Item m;
+    m.it = it;
+    m.c0 = make_int4(0, 0, 0, 0);
+    m.c1 = m.c0;
+    m.jl = m.c0;
+    m.kl = -1;
+    m.act = false;
+    if (it < n_items) {
+      m.c0 = items[2 * it];
+      m.c1 = items[2 * it + 1];
+      m.act = active(m.c0, m.c1);
+      if (m.act && m.c0.y + lane < m.c0.z) {
+        m.jl = ld4i(pad_child + 4 * (size_t)(m.c0.y + lane));
+        m.kl = pad_batch_node[m.c0.y + lane];
+      }
+    }
+    return m;
+  };
+  // request batches of the item queue [cur, nxt] up to S - 1 ahead of consumption
+  Item cur = load_item(blockIdx.x * kRtWarps + wi);
+  Item nxt = load_item(cur.it + T);
+  int cur_req = 0, nxt_req = 0;  // batches requested of cur / nxt
+  auto top_up = [&]() {
+    while ((int)(nb - nc) < S - 1) {
+      if (cur.act && cur_req < cur.c0.z - cur.c0.y) {
+        issue(shfl4(cur.jl, cur_req));
+        ++cur_req;
+      } else if (cur_req >= cur.c0.z - cur.c0.y || !cur.act) {
+        if (nxt.act && nxt_req < nxt.c0.z - nxt.c0.y) {
+          issue(shfl4(nxt.jl, nxt_req));
+          ++nxt_req;
+        } else {
+          break;
+        }
+      } else {
+        break;
+      }
+    }
+  };
+  while (cur.it < n_items) {
+    const int4 c0 = cur.c0, c1 = cur.c1;
+    const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
+    if (c1.z > t - 1) {  // q^{t-1}_{j'} = 0: nothing to add, g_q^{t-1}_{j'} never read
+    } else if ((int64_t)t + c1.w <= K) {  // reverse window (see k_sweep_reverse)
+      if ((int64_t)t + c1.w >= K - 1 && gq_prev && (info < 0 || cur.it == class_item_ptr[jp]))
+        stv<V>(gq_prev + (size_t)jp * Bp + s0, zero);
+    } else {
+      const bool piece = info >= 0 && (info & 1);
+      const Vec<V> qp = ldv<V>(q_prev + (size_t)jp * Bp + s0);
+      Vec<V> gqacc = zero, X = zero;
+      if (bb < be) {
+        top_up();
+        int k = c1.x;
+        if (l2_prefetch) {
+          const int nn = c1.y - k + 1;
+          const int lines = 2 * nn * V;
+          for (int l = lane; l < lines; l += 32) {
+            const int arr = l / (nn * V), r = l % (nn * V);
+            const float* base = arr ? gcp : cp;
+            const float* a = base + (size_t)(k + r / V) * Bp + x0 + (r % V) * 32;
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+          }
+        }
+        size_t ok = (size_t)k * Bp + s0;
+        Vec<V> cv = ldv_cs<V>(cp + ok), gc = piece ? zero : ldv_cs<V>(gcp + ok);
+        Vec<V> cvn = zero, gcn = zero;
+        Vec<V> rom, sI, cC;
+        auto node_consts = [&]() {
+#pragma unroll
+          for (int x = 0; x < V; ++x) {
+            const float om = __fsub_rn(1.f, __fmul_rn(cv.v[x], qp.v[x]));
+            const bool nz = om != 0.f;
+            float r;
+            asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
+            rom.v[x] = (HI && nz ? r : 1.f) * keep.v[x];
+            sI.v[x] = nz ? wI : -wI;
+            cC.v[x] = HI && nz ? wC * om : wC;
+          }
+        };
+        node_consts();
+        for (int b = bb; b < be; ++b) {
+          const int rb = b - bb;
+          const int knext = __shfl_sync(0xffffffffu, cur.kl, (rb + 1) & 31);
+          const int kn1 = rb + 1 < be - bb ? knext : -1;  // e-node of batch b+1 (-1: none)
+          if (kn1 >= 0 && kn1 != k) {
+            cvn = ldv_cs<V>(cp + (size_t)kn1 * Bp + s0);
+            if (!piece) gcn = ldv_cs<V>(gcp + (size_t)kn1 * Bp + s0);
+          }
+          const uint32_t st = nc % S;
+          mbar_wait(bar0 + 8 * st, (nc / S) & 1);
+          const unsigned char* stg = ring + (size_t)st * kRtStage;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const float4 g4 = reinterpret_cast<const float4*>(stg + u * kRtRow)[lane];
+            const float gA[4] = {g4.x, g4.y, g4.z, g4.w};
+            float PA[4] = {0.f, 0.f, 0.f, 0.f};
+            int aA[4] = {0, 0, 0, 0};
+            if (HI) {
+              const float4 p4 = reinterpret_cast<const float4*>(stg + (4 + u) * kRtRow)[lane];
+              PA[0] = p4.x; PA[1] = p4.y; PA[2] = p4.z; PA[3] = p4.w;
+            }
+            if (HC) {
+              const int4 a4 = reinterpret_cast<const int4*>(stg + (8 + u) * kRtRow)[lane];
+              aA[0] = a4.x; aA[1] = a4.y; aA[2] = a4.z; aA[3] = a4.w;
+            }
+#pragma unroll
+            for (int x = 0; x < V; ++x) {
+              if (HI) X.v[x] = fmaf(gA[x], fmaxf(sI.v[x] * PA[x], 0.f), X.v[x]);
+              if (HC && aA[x] == k) X.v[x] = fmaf(gA[x], cC.v[x], X.v[x]);
+            }
+          }
+          ++nc;
+          top_up();  // the stage just read is free: request the next batch
+          if (kn1 != k && !piece) {  // finalise e-node k
+#pragma unroll
+            for (int x = 0; x < V; ++x) {
+              const float gp = X.v[x] * rom.v[x];
+              gc.v[x] += gp * qp.v[x];
+              gqacc.v[x] += gp * cv.v[x];
+            }
+            stv_cs<V>(gcp + ok, gc);
+            if (kn1 >= 0) {
+              k = kn1;
+              ok = (size_t)k * Bp + s0;
+              cv = cvn;
+              gc = gcn;
+              node_consts();
+              X = zero;
+            }
+          }
+        }
+      }
+      Vec<V> pass = zero;
+      reverse_epilogue<V, HI, false>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X,
+                                     items, class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq);
+    }
+    // advance the queue: nxt becomes current (with the batches already requested)
+    cur = nxt;
+    cur_req = nxt_req;
+    nxt = load_item(cur.it + T);
+    nxt_req = 0;
+  }
+}
+
+// Tensor maps of the [M][Bp] rows the TMA reverse sweep gathers (box: one
+// 128-seed row), encoded on the host once per (pointer, shape) through the
+// driver entry point (the library links the static runtime only).
+static const CUtensorMap& row_map(const void* base, int M, int Bp, bool is_int) {
+  struct Key {
+    const void* p;
+    int M, Bp, i;
+    bool operator==(const Key& o) const { return p == o.p && M == o.M && Bp == o.Bp && i == o.i; }
+  };
+  static std::mutex mu;
+  static std::vector<std::pair<Key, CUtensorMap>> cache;
+  typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                               const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                               const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                               CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static EncodeFn encode = nullptr;
+  std::lock_guard<std::mutex> lk(mu);
+  const Key key{base, M, Bp, is_int ? 1 : 0};
+  for (auto& e : cache)
+    if (e.first == key) return e.second;
+  if (!encode) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    SM_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    SM_REQUIRE(fn && q == cudaDriverEntryPointSuccess, SMOOTHE_E_CUDA,
+               "cuTensorMapEncodeTiled unavailable");
+    encode = (EncodeFn)fn;
+  }
+  CUtensorMap m;
+  const cuuint64_t dims[2] = {(cuuint64_t)Bp, (cuuint64_t)M};
+  const cuuint64_t strides[1] = {(cuuint64_t)Bp * 4};
+  const cuuint32_t box[2] = {128, 1}, es[2] = {1, 1};
+  const CUresult r = encode(&m, is_int ? CU_TENSOR_MAP_DATA_TYPE_INT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                            2, const_cast<void*>(base), dims, strides, box, es,
+                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  SM_REQUIRE(r == CUDA_SUCCESS, SMOOTHE_E_CUDA, "cuTensorMapEncodeTiled failed");
+  if (cache.size() > 256) cache.erase(cache.begin());
+  cache.push_back({key, m});
+  return cache.back().second;
+}
+
+// Opt-in (SMOOTHE_REV_TMA=1): measured slower than the register kernel on C4
+// ("tried"); read at every host-side launch (A/B, tests).
+static bool reverse_tma_enabled() {
+  const char* e = std::getenv("SMOOTHE_REV_TMA");
+  return e && e[0] == '1';
+}
+
 void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t, int K,
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
-                          const int32_t* lastchg) {
+                          const int32_t* lastchg, int32_t* cursor) {
   float* out = write_gq_prev ? gq_prev : nullptr;
 #ifndef SMOOTHE_REV_VMAX
 #define SMOOTHE_REV_VMAX 4  // seeds per lane at Bp >= 128 (4: one warp per 128-seed slice)
@@ -831,6 +1160,22 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   // cp / g_cp rows are L2-prefetched per item only when they cannot stay
   // L2-resident (measured: +7% on C4 at 512 MB, -9% on C3 at 13 MB)
   const bool l2_prefetch = (double)sh.N * sh.Bp * sizeof(float) > 64e6;
+  if (V == 4 && !lastchg && cursor && reverse_tma_enabled()) {
+    const bool HI = a.wI != 0.f, HC = a.wC != 0.f;
+    const CUtensorMap& mg = row_map(gq, sh.M, sh.Bp, false);
+    const CUtensorMap& mp = row_map(HI ? (const void*)pi : (const void*)gq, sh.M, sh.Bp, false);
+    const CUtensorMap& ma = row_map(HC ? (const void*)am : (const void*)gq, sh.M, sh.Bp, true);
+    int dev = 0;
+    SM_CUDA(cudaGetDevice(&dev));
+    const dim3 grid(SMOOTHE_RT_CTAS * num_sms(dev), sh.Bp / 128);
+#define SM_RT(HI_, HC_)                                                                           do {                                                                                              static bool attr = false;                                                                       if (!attr) {                                                                                      SM_CUDA(cudaFuncSetAttribute(k_sweep_reverse_tma<HI_, HC_>,                                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kRtSmem));            attr = true;                                                                                  }                                                                                               k_sweep_reverse_tma<HI_, HC_><<<grid, 32 * kRtWarps, kRtSmem, s>>>(                                 mg, mp, ma, n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item),                       g.rev_class_item_ptr, g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, gcp,           out, rev_part, rev_cnt, l2_prefetch, t, K, wm, cursor);                                   } while (0)
+    if (HI && HC) SM_RT(true, true);
+    else if (HI) SM_RT(true, false);
+    else SM_RT(false, true);
+#undef SM_RT
+    SM_LAUNCH_CHECK();
+    return;
+  }
   const dim3 grid((n + kRevBlock / 32 - 1) / (kRevBlock / 32), sh.Bp / (32 * V));
 #define SM_REV3(VV, HI, HC, CV)                                                                \
   k_sweep_reverse<VV, HI, HC, CV><<<grid, kRevBlock, 0, s>>>(                                  \

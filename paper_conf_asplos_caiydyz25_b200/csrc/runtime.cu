@@ -219,6 +219,7 @@ struct smoothe_run {
   double* red_scratch = nullptr;  // 128 x Bp, reductions
   float* rev_part = nullptr;       // reverse sweep partial rows [rev_num_slots][Bp]
   int32_t* rev_cnt = nullptr;      // [M][seed slices] items finished (self-resetting)
+  int32_t* rev_cursor = nullptr;   // [K+2][Bp/128] item cursors of the TMA reverse sweeps (zeroed per step)
   // cost model
   float* u_f = nullptr;
   double* u_d = nullptr;
@@ -405,6 +406,7 @@ void enqueue_step(smoothe_run* r) {
 
   pm.mark(SMOOTHE_PHASE_FORWARD);
   launch_sweep_reset(s, sh, r->sw);
+  SM_CUDA(cudaMemsetAsync(r->rev_cursor, 0, sizeof(int32_t) * (r->K + 2) * std::max(1, sh.Bp / 128), s));
   // (when profiling, events bracket each sweep kernel: bench.py's roofline)
   auto kmark = [&](int which, int at) {
     if (!r->profiling) return;
@@ -488,7 +490,8 @@ void enqueue_step(smoothe_run* r) {
       launch_sweep_reverse(ss, sh, g, r->agg, t, sw.converge ? -1 : K, cur_q, sw.cur_pi,
                            sw.cur_am, sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
                            r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt,
-                           sw.converge && !sw.wmode ? sw.lastchg : nullptr);
+                           sw.converge && !sw.wmode ? sw.lastchg : nullptr,
+                           r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128));
     };
     if (r->in_capture && sw.wmode && t < K && g.num_rev_items >= 100000) {
       // in the captured step the plain sweep is a conditional node, skipped
@@ -511,7 +514,8 @@ void enqueue_step(smoothe_run* r) {
   }
   if (sw.wmode)  // the frozen sweeps' g_cp: one pass over the K-state with g = S
     launch_sweep_reverse(s, sh, g, r->agg, K, K, sw.kq, sw.kpi, sw.kam, nullptr, r->cp, sw.S,
-                         r->gcp, nullptr, false, r->rev_part, r->rev_cnt);
+                         r->gcp, nullptr, false, r->rev_part, r->rev_cnt, nullptr,
+                         r->rev_cursor + (size_t)(K + 1) * std::max(1, sh.Bp / 128));
 
   pm.mark(SMOOTHE_PHASE_UPDATE);
   launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
@@ -671,6 +675,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   if (r->overlap) r->red_scratch_d = dalloc<double>(o, (size_t)128 * sh.Bp);
   r->rev_part = dalloc<float>(o, (size_t)std::max(1, r->g->dev.rev_num_slots) * sh.Bp);
   r->rev_cnt = dalloc<int32_t>(o, (size_t)sh.M * std::max(1, sh.Bp / 32));  // per (class, warp seed slice)
+  r->rev_cursor = dalloc<int32_t>(o, (size_t)(r->K + 2) * std::max(1, sh.Bp / 128));
   r->dbg_p = nullptr;
 
   // cost model

@@ -637,3 +637,29 @@ def test_patience_stops_early(sm):
     run.steps(1000)
     _, s = run.extract()
     assert s["steps_run"] < 1000
+
+
+@pytest.mark.parametrize("name,B,G,agg,steps", [("C2", 128, 8, "hybrid", 6), ("C2", 256, 8, "independent", 4),
+                                                ("C3", 128, 8, "correlated", 3), ("C4", 128, 16, "hybrid", 3)])
+def test_reverse_tma_bit_identical(sm, monkeypatch, name, B, G, agg, steps):
+    """The TMA-staged reverse sweep (opt-in SMOOTHE_REV_TMA=1: gather4 into a
+    shared-memory ring, 128-seed slices) against the register kernel: the
+    same arithmetic in the same order, so theta after several steps, the
+    best extraction and a debug step's gradient are bit for bit equal."""
+    eg = make_config(name)
+    outs = []
+    for env in ("1", "0"):
+        monkeypatch.setenv("SMOOTHE_REV_TMA", env)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=17, assumption=agg))
+        run.steps(steps)
+        th = run.theta()
+        d = run.debug_step(th)
+        outs.append((run.theta(), run.extract(), d["grad_cp"]))
+        run.close()
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][2], outs[1][2])
+    assert np.array_equal(outs[0][1][0], outs[1][1][0])
+    assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
