@@ -258,6 +258,19 @@ SMOOTHE_API smoothe_status smoothe_run_warm_start(smoothe_run *run, const int32_
 /* theta [N][B] of the run as it stands (host copy). */
 SMOOTHE_API smoothe_status smoothe_get_theta(smoothe_run *run, float *theta);
 
+/* Per-step record of the run (PAPER.md:459-461 compare the
+ * relaxed loss with the sampled solutions along the optimisation): out[n][4]
+ * host, caller-owned, for steps 0 .. n-1 (n = min(steps run, 4096, max_steps)):
+ *   [0] min over the run's seeds of the relaxed cost f(p_b) at that step,
+ *   [1] its mean over the seeds,
+ *   [2] min over the seeds of the sampled (decoded) cost f_b(s) of that step
+ *       (+inf if no sample was valid),
+ *   [3] number of valid samples.
+ * Relaxed values are the step's loss terms (before the update); sampled ones
+ * decode the same theta (reading S17). */
+SMOOTHE_API smoothe_status smoothe_run_get_trace(smoothe_run *run, double *out, int32_t max_steps,
+                                                 int32_t *n_out);
+
 /* The optimiser state as it stands, host copies [N][B] (any pointer may be
  * NULL), and the number of steps run: a debug step from this state with
  * step_index = *steps_run continues the run exactly (tests: parity after

@@ -276,7 +276,8 @@ void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_sc
                           double beta1, double beta2, const int32_t* unused);
 void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, int Bp, float value);
 void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const double* f,
-                 const double* fextra, const double* h, double* ftot, double* loss);
+                 const double* fextra, const double* h, double* ftot, double* loss,
+                 const double* scal, double* trace, int trace_cap);
 // reached sets and validity masks (kernels_decode.cu); valid_out[W]
 void launch_decode(cudaStream_t s, const Shape& sh, const HostGraph& hg, const DevGraph& g,
                    const uint32_t* sel, const int32_t* choice, uint32_t* reach, uint32_t* settle,
@@ -299,7 +300,8 @@ int decode_cost_rows(const Shape& sh);
 void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
                         const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,
                         const int32_t* step_counter, double* best, int32_t* best_flag,
-                        double* valid_cost_out, uint8_t* valid_out);
+                        double* valid_cost_out, uint8_t* valid_out, double* trace = nullptr,
+                        int trace_cap = 0);
 void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice,
                           const uint32_t* reach, const double* best, const int32_t* best_flag,
                           int64_t seed_begin, int32_t* best_choice);

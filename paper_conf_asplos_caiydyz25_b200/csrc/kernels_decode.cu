@@ -313,21 +313,26 @@ __global__ void __launch_bounds__(256) k_best_update(
     int B, int W, int root, const uint32_t* __restrict__ settle, const double* __restrict__ dcost,
     const double* __restrict__ dextra, int64_t seed_begin, int32_t* __restrict__ counter,
     double* __restrict__ best, int32_t* __restrict__ flag, double* __restrict__ cost_out,
-    uint8_t* __restrict__ valid_out) {
+    uint8_t* __restrict__ valid_out, double* __restrict__ trace, int trace_cap) {
   __shared__ double sc[256];
   __shared__ int sb[256];
+  __shared__ int nvalid;
+  if (threadIdx.x == 0) nvalid = 0;
+  __syncthreads();
   double bc = INFINITY;
-  int bb = 0x7fffffff;
+  int bb = 0x7fffffff, nv = 0;
   for (int b = threadIdx.x; b < B; b += blockDim.x) {
     const bool ok = (settle[(size_t)root * W + (b >> 5)] >> (b & 31)) & 1u;
     const double c = ok ? dcost[b] + (dextra ? dextra[b] : 0.0) : INFINITY;
     if (cost_out) cost_out[b] = c;
     if (valid_out) valid_out[b] = ok ? 1 : 0;
+    nv += ok ? 1 : 0;
     if (c < bc) {
       bc = c;
       bb = b;
     }
   }
+  if (trace) atomicAdd(&nvalid, nv);
   sc[threadIdx.x] = bc;
   sb[threadIdx.x] = bb;
   __syncthreads();
@@ -344,6 +349,10 @@ __global__ void __launch_bounds__(256) k_best_update(
   }
   if (threadIdx.x == 0) {
     const int step = *counter;
+    if (trace && step < trace_cap) {  // the sampled side of the step's record (k_loss)
+      trace[4 * (size_t)step + 2] = sc[0];
+      trace[4 * (size_t)step + 3] = (double)nvalid;
+    }
     if (sc[0] < best[0]) {
       best[0] = sc[0];
       best[1] = (double)step;
@@ -361,10 +370,10 @@ __global__ void __launch_bounds__(256) k_best_update(
 void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
                         const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,
                         const int32_t* step_counter, double* best, int32_t* best_flag,
-                        double* valid_cost_out, uint8_t* valid_out) {
+                        double* valid_cost_out, uint8_t* valid_out, double* trace, int trace_cap) {
   k_best_update<<<1, 256, 0, s>>>(sh.B, sh.W, sh.root, settle, dcost_lin, dcost_extra, seed_begin,
                                   const_cast<int32_t*>(step_counter), best, best_flag,
-                                  valid_cost_out, valid_out);
+                                  valid_cost_out, valid_out, trace, trace_cap);
   SM_LAUNCH_CHECK();
 }
 

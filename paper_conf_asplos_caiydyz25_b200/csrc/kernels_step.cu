@@ -324,24 +324,36 @@ void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, in
 }
 
 // ftot[b] = f[b] + fextra[b];  L = sum_b ftot[b] + lambda * sum_g G h_g  (Eq. 10a; S12)
+// L = sum_b f_b + lambda sum_g G h_g (reading S12); with a trace, row
+// `step` (scal[2]) gets the relaxed side of the per-step record: min_b f(p_b)
+// and mean_b f(p_b) (the decode writes the sampled side, k_best_update).
 __global__ void k_loss(int B, int G, int ngroups, double lambda, const double* __restrict__ f,
                        const double* __restrict__ fextra, const double* __restrict__ h,
-                       double* __restrict__ ftot, double* __restrict__ loss) {
+                       double* __restrict__ ftot, double* __restrict__ loss,
+                       const double* __restrict__ scal, double* __restrict__ trace, int trace_cap) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
-  double L = 0.0;
+  double L = 0.0, mn = INFINITY;
   for (int b = 0; b < B; ++b) {
     const double v = f[b] + (fextra ? fextra[b] : 0.0);
     ftot[b] = v;
     L += v;
+    mn = fmin(mn, v);
   }
+  const double fsum = L;
   if (h)
     for (int g = 0; g < ngroups; ++g) L += lambda * G * h[g];
   *loss = L;
+  const int step = (int)scal[2];
+  if (trace && step < trace_cap) {
+    trace[4 * (size_t)step + 0] = mn;
+    trace[4 * (size_t)step + 1] = fsum / B;
+  }
 }
 
 void launch_loss(cudaStream_t s, int B, int G, int ngroups, double lambda, const double* f,
-                 const double* fextra, const double* h, double* ftot, double* loss) {
-  k_loss<<<1, 32, 0, s>>>(B, G, ngroups, lambda, f, fextra, h, ftot, loss);
+                 const double* fextra, const double* h, double* ftot, double* loss,
+                 const double* scal, double* trace, int trace_cap) {
+  k_loss<<<1, 32, 0, s>>>(B, G, ngroups, lambda, f, fextra, h, ftot, loss, scal, trace, trace_cap);
   SM_LAUNCH_CHECK();
 }
 
@@ -515,6 +527,7 @@ __global__ void k_step_prologue(const int32_t* __restrict__ counter, double* __r
   const double t = (double)(*counter + 1);
   scal[0] = 1.0 / (1.0 - pow(beta1, t));
   scal[1] = 1.0 / (1.0 - pow(beta2, t));
+  scal[2] = (double)*counter;  // this step's index (k_loss's trace row)
 }
 
 void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_scalars,

@@ -450,17 +450,34 @@ void launch_stack_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, f
   SM_LAUNCH_CHECK();
 }
 
-void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
-  const size_t MB = (size_t)sh.M * sh.Bp;
-  for (int b = 0; b < 2; ++b) {
-    SM_CUDA(cudaMemsetAsync(st.dirty[b], 0xff, sizeof(int32_t) * sh.M, s));
-    SM_CUDA(cudaMemsetAsync(st.chg[b], 0xff, sizeof(int32_t) * sh.M, s));
-    SM_CUDA(cudaMemsetAsync(st.qbuf[b], 0, sizeof(float) * MB, s));
+// Per-step reset of the forward's state in one kernel (instead of eight
+// memsets and a fill): stamps (dirty / chg, one allocation of 4 M) = -1,
+// lastver = 0, list_n = 0, both q ping-pong rows = e_root (qbuf[1] follows
+// qbuf[0] in one allocation).
+__global__ void k_sweep_reset(int M, int Bp, int root, int nlist, int32_t* __restrict__ stamps,
+                              int32_t* __restrict__ lastver, int32_t* __restrict__ list_n,
+                              float* __restrict__ qbuf) {
+  const int64_t MB = (int64_t)M * Bp, n0 = 4 * (int64_t)M, n1 = n0 + M, n2 = n1 + nlist,
+                n3 = n2 + 2 * MB;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n3;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    if (e < n0) stamps[e] = -1;
+    else if (e < n1) lastver[e - n0] = 0;
+    else if (e < n2) list_n[e - n1] = 0;
+    else {
+      const int64_t q = e - n2;
+      qbuf[q] = (q % MB) / Bp == root ? 1.f : 0.f;
+    }
   }
-  SM_CUDA(cudaMemsetAsync(st.lastver, 0, sizeof(int32_t) * sh.M, s));
-  SM_CUDA(cudaMemsetAsync(st.list_n, 0, sizeof(int32_t) * (st.K + 2), s));
-  // qbuf[1] = qbuf[0] + M Bp (one allocation)
-  launch_fill_rows(s, st.qbuf[0] + (size_t)sh.root * sh.Bp, (int64_t)MB, 2, sh.Bp, 1.0f);
+}
+
+void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
+  // stamps: dirty[0], dirty[1], chg[0], chg[1] are consecutive (alloc_state)
+  int dev = 0;
+  SM_CUDA(cudaGetDevice(&dev));
+  k_sweep_reset<<<4 * num_sms(dev), 256, 0, s>>>(sh.M, sh.Bp, sh.root, st.K + 2, st.dirty[0],
+                                                 st.lastver, st.list_n, st.qbuf[0]);
+  SM_LAUNCH_CHECK();
 }
 
 

@@ -31,6 +31,9 @@ namespace smoothe {
 static thread_local std::string g_last_error;
 void set_error(const std::string& msg) { g_last_error = msg; }
 
+// steps recorded by the per-step trace (relaxed vs sampled cost, E11)
+constexpr int kTraceCap = 4096;
+
 int64_t& launch_counter() {
   static int64_t counter = 0;
   return counter;
@@ -216,6 +219,7 @@ struct smoothe_run {
   double* best = nullptr;
   int32_t *best_flag = nullptr, *best_choice = nullptr, *counter = nullptr;
   double* scal = nullptr;
+  double* trace = nullptr;  // [kTraceCap][4] per-step record (smoothe_run_get_trace)
   double* red_scratch = nullptr;  // 128 x Bp, reductions
   float* rev_part = nullptr;       // reverse sweep partial rows [rev_num_slots][Bp]
   int32_t* rev_cnt = nullptr;      // [M][seed slices] items finished (self-resetting)
@@ -371,7 +375,7 @@ void enqueue_decode(smoothe_run* r, cudaStream_t ds, PhaseMarks* pm) {
   if (pm) pm->mark(SMOOTHE_PHASE_BEST);
   launch_best_update(ds, sh, r->settle, r->dcost, dextra, r->opt.seed_begin, r->counter, r->best,
                      r->best_flag, r->debug ? r->dbg_dcost : nullptr,
-                     r->debug ? r->dbg_valid : nullptr);
+                     r->debug ? r->dbg_valid : nullptr, r->trace, kTraceCap);
   launch_best_snapshot(ds, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
                        r->best_choice);
 }
@@ -451,7 +455,7 @@ void enqueue_step(smoothe_run* r) {
   }
   launch_loss(s, sh.B, r->G, r->ngroups, r->opt.lambda, r->f,
               r->cost_kind == SMOOTHE_COST_MLP ? r->fextra : nullptr, hg.num_scc > 0 ? r->h : nullptr,
-              r->ftot, r->loss);
+              r->ftot, r->loss, r->scal, r->trace, kTraceCap);
 
   pm.mark(SMOOTHE_PHASE_REVERSE);
   SweepState& sw = r->sw;
@@ -609,7 +613,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     w.list = dalloc<int2>(o, slots * sh.M);
     w.list_n = dalloc<int32_t>(o, slots + 1);
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < 2; ++b) {  // consecutive: k_sweep_reset fills all four at once
       w.dirty[b] = stamps + (size_t)b * sh.M;
       w.chg[b] = stamps + (size_t)(2 + b) * sh.M;
     }
@@ -670,7 +674,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->best_flag = dalloc<int32_t>(o, 1);
   r->best_choice = dalloc<int32_t>(o, sh.M);
   r->counter = dalloc<int32_t>(o, 1);
-  r->scal = dalloc<double>(o, 2);
+  r->scal = dalloc<double>(o, 3);
+  r->trace = dalloc<double>(o, 4 * (size_t)kTraceCap);
   r->red_scratch = dalloc<double>(o, (size_t)128 * sh.Bp);
   if (r->overlap) r->red_scratch_d = dalloc<double>(o, (size_t)128 * sh.Bp);
   r->rev_part = dalloc<float>(o, (size_t)std::max(1, r->g->dev.rev_num_slots) * sh.Bp);
@@ -748,6 +753,7 @@ void init_state(smoothe_run* r) {
   SM_CUDA(cudaMemsetAsync(r->fextra, 0, sizeof(double) * sh.Bp, s));
   SM_CUDA(cudaMemsetAsync(r->counter, 0, sizeof(int32_t), s));
   SM_CUDA(cudaMemsetAsync(r->rev_cnt, 0, sizeof(int32_t) * sh.M * std::max(1, sh.Bp / 32), s));
+  SM_CUDA(cudaMemsetAsync(r->trace, 0xff, sizeof(double) * 4 * kTraceCap, s));  // NaN: not run
   const double init_best[4] = {INFINITY, -1.0, -1.0, 0.0};
   SM_CUDA(cudaMemcpyAsync(r->best, init_best, sizeof(init_best), cudaMemcpyHostToDevice, s));
   SM_CUDA(cudaMemsetAsync(r->best_choice, 0xff, sizeof(int32_t) * sh.M, s));
@@ -1336,6 +1342,18 @@ smoothe_status smoothe_get_theta(smoothe_run* run, float* theta) {
     SM_REQUIRE(theta, SMOOTHE_E_INVALID_ARG, "NULL theta");
     copy_rows_d2h(theta, run->theta, run->sh.N, run->sh.B, run->sh.Bp, run->stream);
     SM_CUDA(cudaStreamSynchronize(run->stream));
+  });
+}
+
+smoothe_status smoothe_run_get_trace(smoothe_run* run, double* out, int32_t max_steps,
+                                     int32_t* n_out) {
+  return guarded(run, [&] {
+    check_run(run);
+    SM_REQUIRE(out && n_out && max_steps >= 0, SMOOTHE_E_INVALID_ARG, "bad trace arguments");
+    SM_CUDA(cudaStreamSynchronize(run->stream));
+    const int n = std::min({run->steps_run, kTraceCap, (int)max_steps});
+    if (n > 0) SM_CUDA(cudaMemcpy(out, run->trace, sizeof(double) * 4 * n, cudaMemcpyDeviceToHost));
+    *n_out = n;
   });
 }
 

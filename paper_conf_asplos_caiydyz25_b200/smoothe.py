@@ -99,6 +99,7 @@ _SIGS = {
                                      C.POINTER(_Dump)]),
     "smoothe_get_theta": (C.c_int, [C.c_void_p, C.c_void_p]),
     "smoothe_get_state": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
+    "smoothe_run_get_trace": (C.c_int, [C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p]),
     "smoothe_greedy": (C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
                                  C.POINTER(_Greedy)]),
     "smoothe_run_warm_start": (C.c_int, [C.c_void_p, C.c_void_p, C.c_float]),
@@ -318,6 +319,16 @@ class Run:
         out = np.zeros((self.egraph.N, self.B), np.float32)
         _check(lib().smoothe_get_theta(self._h, _p(out)))
         return out
+
+    def trace(self, max_steps: int = 4096):
+        """smoothe_run_get_trace: per-step relaxed vs sampled cost, dict of
+        arrays (relaxed_min, relaxed_mean, sampled_min, valid)."""
+        out = np.zeros((max_steps, 4), np.float64)
+        n = C.c_int32(0)
+        _check(lib().smoothe_run_get_trace(self._h, _p(out), int(max_steps), C.byref(n)))
+        t = out[: n.value]
+        return {"relaxed_min": t[:, 0], "relaxed_mean": t[:, 1], "sampled_min": t[:, 2],
+                "valid": t[:, 3].astype(np.int64)}
 
     def state(self):
         """smoothe_get_state: (theta, m, v) [N][B] float32 and the steps run."""

@@ -107,3 +107,33 @@ def test_rejects_negative_or_nonfinite_costs(sm):
             g.greedy(u)
     g.greedy(eg.u)
     g.close()
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_maxsat_reaches_brute_force_optimum(sm, seed):
+    """MaxSAT -> e-graph (gen/adversarial.py, Table 4):
+    the best sampled extraction is a truth assignment whose cost is minus its
+    satisfied weight, and on these 14-variable random 3-SAT instances it is
+    the maximum-weight assignment found by enumerating all 2^14 of them."""
+    import itertools
+    from gen.adversarial import random_maxsat
+    eg = random_maxsat(14, 60, 3, seed)
+    n, cls, ws = eg.meta["vars"], eg.meta["clause_list"], eg.meta["weights"]
+    lits = np.zeros((len(cls), n), np.int8)
+    for c, cl in enumerate(cls):
+        for l in cl:
+            lits[c, abs(l) - 1] = 1 if l > 0 else -1
+    bits = np.array(list(itertools.product([0, 1], repeat=n)), np.int8)  # [2^n][n]
+    sat = ((lits[None] == 1) & (bits[:, None] == 1)) | ((lits[None] == -1) & (bits[:, None] == 0))
+    best_sat = float((sat.any(axis=2) * np.asarray(ws)[None]).sum(axis=1).max())
+    g = sm.load_egraph_from(eg)
+    run = sm.optimize(g, sm.CostModel.from_input(eg), 64, 200,
+                      sm.Options(penalty_group=8, rng_key=7, lam=1.0))
+    choice, s = run.extract()
+    assert s["valid"] == 1
+    assign = [choice[1 + i] == int(eg.class_ptr[1 + i]) for i in range(n)]  # first e-node = true
+    satisfied = sum(w for cl, w in zip(cls, ws) if any(assign[abs(l) - 1] == (l > 0) for l in cl))
+    assert s["best_cost"] == -satisfied
+    assert -s["best_cost"] == best_sat
+    run.close()
+    g.close()

@@ -663,3 +663,30 @@ def test_reverse_tma_bit_identical(sm, monkeypatch, name, B, G, agg, steps):
     assert np.array_equal(outs[0][2], outs[1][2])
     assert np.array_equal(outs[0][1][0], outs[1][1][0])
     assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
+
+
+def test_step_trace_relaxed_vs_sampled(sm):
+    """The per-step record (smoothe_run_get_trace, E11 / PAPER.md:459-461):
+    row k holds min / mean over seeds of the relaxed f(p_b) and the min of the
+    sampled f_b(s) of step k; checked against a debug step taken as step k
+    (its own f and decoded costs), and the run's best is the minimum of the
+    sampled column at the recorded step."""
+    eg = make_config("C2")
+    g = sm.load_egraph_from(eg)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), 64, sm.Options(penalty_group=8, rng_key=23))
+    run.steps(9)
+    th, m, v, n = run.state()
+    d = run.debug_step(th, m, v, step_index=n)   # step 9
+    tr = run.trace()
+    assert len(tr["relaxed_min"]) == 10
+    assert tr["relaxed_min"][9] == d["f"].min()
+    assert tr["relaxed_mean"][9] == pytest.approx(d["f"].mean(), rel=1e-12)
+    ok = d["valid"] == 1
+    assert tr["valid"][9] == ok.sum()
+    assert tr["sampled_min"][9] == d["disc_cost"][ok].min()
+    _, s = run.extract()
+    smin = tr["sampled_min"]
+    assert s["best_cost"] == smin.min() and s["best_step"] == int(np.argmin(smin))
+    assert np.all(tr["relaxed_min"] <= tr["relaxed_mean"])
+    run.close()
+    g.close()
