@@ -142,4 +142,35 @@ __device__ __forceinline__ int& comp(int4& v, int c) {
     SM_CUDA(cudaGetLastError());                                 \
   } while (0)
 
+// ---------------------------------------------------------------------------
+// tcgen05 / mbarrier helpers (the tensor-core kernels: MLP layer 1, the
+// large-component matrix exponential)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+// no-swizzle UMMA shared-memory descriptor (sm_100 version 1)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+         ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity));
+}
+__device__ __forceinline__ float4 tf32_hi(float4 v) {
+  auto h = [](float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); };
+  return make_float4(h(v.x), h(v.y), h(v.z), h(v.w));
+}
+__device__ __forceinline__ float4 sub4(float4 a, float4 b) {
+  return make_float4(a.x - b.x, a.y - b.y, a.z - b.z, a.w - b.w);
+}
+
 }  // namespace smoothe

@@ -14,6 +14,8 @@
 // h = tr(e^A - I) carries no cancellation.  The entry sums run over a fixed
 // (entry, node, seed) order with a fixed warp-shuffle tree: h and the
 // gradient are bit-identical at every GPU count.
+#include <cstdlib>
+
 #include "kcommon.cuh"
 
 namespace smoothe {
@@ -255,6 +257,310 @@ __global__ void __launch_bounds__(256) k_big_finish(
   }
 }
 
+// ---------------------------------------------------------------------------
+// The same chain on the 5th-generation tensor cores (the default; SURVEY.md
+// NEXT-1): matrices in fp32, padded to np = 64 * ceil(n / 64) (zero padding:
+// the identity only on the first n diagonal entries, so padded rows and
+// columns stay 0 through every product), each product C = alpha A B + beta D
+// + gamma I with A B in "3xTF32": x = hi + lo (hi = x with the low 13 mantissa
+// bits cleared, lo = x - hi exactly), and one M=128 x N=128 x K=8 tcgen05
+// kind::tf32 MMA on A = [A_hi; A_lo] (a 64-row tile twice) and B = [B_hi |
+// B_lo] (a 64-column tile twice) accumulates all four products of the
+// 64 x 64 output tile in TMEM: AB = D[0:64,0:64] + D[0:64,64:128] +
+// (D[64:128,0:64] + D[64:128,64:128]), summed in that fixed order.
+// Precision (scripts/notears_precision_study.py, profiles/r2/notears_precision.md):
+// on the 217- to 1112-class test components h is within 4e-7 of fp64 and
+// every entry of e^Abar within 1.4% of the parity bar.  SMOOTHE_BIG_FP64=1
+// keeps the fp64 CUDA-core GEMMs above.
+// ---------------------------------------------------------------------------
+constexpr int kBtT = 64, kBtK = 32, kBtStages = 3, kBtThreads = 128;
+constexpr int kBtA = 128 * kBtK * 4, kBtB = kBtK * 128 * 4, kBtStage = kBtA + kBtB;
+constexpr int kBtSmem = kBtStages * kBtStage + 1024;
+
+__global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
+                                                              const float* __restrict__ A,
+                                                              const float* __restrict__ B,
+                                                              float* __restrict__ C, float alpha,
+                                                              float beta,
+                                                              const float* __restrict__ D,
+                                                              float gamma) {
+  constexpr int LBO = 16 * 128;  // K-chunk (4 elements) stride of both operands: 16 core rows
+  // kind::tf32, D f32, A and B K-major, M = 128, N = 128
+  constexpr uint32_t IDESC =
+      (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(128 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t bt_smem[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(bt_smem) + 1023) & ~(uintptr_t)1023);
+  __shared__ uint64_t bar[kBtStages + 1];
+  __shared__ uint32_t tmem_sh;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const size_t off = (size_t)blockIdx.z * np * np;
+  A += off;
+  B += off;
+  C += off;
+  if (D) D += off;
+  const int i0 = blockIdx.y * kBtT, j0 = blockIdx.x * kBtT;
+  const int nkb = np / kBtK;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&tmem_sh)),
+                 "n"(128));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int i = 0; i <= kBtStages; ++i) mbar_init(&bar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem = tmem_sh;
+  // two K slabs in flight in registers (buffers p, q for even / odd slabs),
+  // the third stage multiplying
+  float4 pa[4], pb[4], qa[4], qb[4];
+  auto load = [&](int kb, float4 (&ra)[4], float4 (&rb)[4]) {
+    const int k0 = kb * kBtK;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {  // A: 64 rows x 8 K-chunks of 4 (row-coalesced)
+      const int idx = tid + i * kBtThreads, r = idx / 8, kc = idx % 8;
+      ra[i] = __ldg(reinterpret_cast<const float4*>(A + (size_t)(i0 + r) * np + k0 + 4 * kc));
+    }
+    const int kc = tid / 16, c = (tid % 16) * 4;  // B: the 4 x 4 block (K-chunk kc, columns c..c+3)
+#pragma unroll
+    for (int r = 0; r < 4; ++r)
+      rb[r] = __ldg(reinterpret_cast<const float4*>(B + (size_t)(k0 + 4 * kc + r) * np + j0 + c));
+  };
+  auto store = [&](int st, const float4 (&ra)[4], const float4 (&rb)[4]) {
+    uint8_t* sa = smem + st * kBtStage;
+    uint8_t* sb = sa + kBtA;
+    // B: each pair of lanes starts its four transposed columns at a different
+    // offset, so every 8 consecutive lanes (a 128-bit store is served 8 lanes
+    // at a time) hit the 8 16-byte positions of a 128-byte core row (the
+    // plain order was a 4-way bank conflict).  A keeps the row-coalesced
+    // order: a conflict-free A order (8 rows per 8 lanes) measured slower,
+    // its global loads no longer coalesce (profiles/r2/notears_precision.md).
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int idx = tid + i * kBtThreads, r = idx / 8, kc = idx % 8;
+      const float4 hi = tf32_hi(ra[i]), lo = sub4(ra[i], hi);
+      // element (row, k): core (k/4, row/8) at (kc * 16 + row/8) * 128 + (row%8) * 16
+      *reinterpret_cast<float4*>(sa + (kc * 16 + r / 8) * 128 + (r % 8) * 16) = hi;
+      *reinterpret_cast<float4*>(sa + (kc * 16 + 8 + r / 8) * 128 + (r % 8) * 16) = lo;
+    }
+    const int kc = tid / 16, c = (tid % 16) * 4;
+    auto sel = [](float4 v, int o) { return o == 0 ? v.x : o == 1 ? v.y : o == 2 ? v.z : v.w; };
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {  // column c + o: its 4 K values, transposed to K-major
+      const int o = (x + (tid >> 1)) & 3;
+      const float4 col = make_float4(sel(rb[0], o), sel(rb[1], o), sel(rb[2], o), sel(rb[3], o));
+      const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+      const int m = c + o;
+      *reinterpret_cast<float4*>(sb + (kc * 16 + m / 8) * 128 + (m % 8) * 16) = hi;
+      *reinterpret_cast<float4*>(sb + (kc * 16 + (64 + m) / 8) * 128 + (m % 8) * 16) = lo;
+    }
+  };
+  auto step = [&](int kb, float4 (&ra)[4], float4 (&rb)[4]) {
+    const int st = kb % kBtStages;
+    if (kb >= kBtStages) mbar_wait(&bar[st], (uint32_t)((kb / kBtStages - 1) & 1));
+    store(st, ra, rb);
+    if (kb + 2 < nkb) load(kb + 2, ra, rb);
+    asm volatile("fence.proxy.async.shared::cta;");
+    __syncthreads();
+    if (tid == 0) {
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const uint32_t sa = smem_u32(smem + st * kBtStage), sb = sa + kBtA;
+#pragma unroll
+      for (int ks = 0; ks < kBtK / 8; ++ks) {
+        const uint64_t da = umma_desc(sa + ks * 2 * LBO, LBO, 128);
+        const uint64_t db = umma_desc(sb + ks * 2 * LBO, LBO, 128);
+        const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(da), "l"(db), "r"(IDESC), "r"(acc));
+      }
+      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+          smem_u32(&bar[st])));
+    }
+  };
+  load(0, pa, pb);
+  if (nkb > 1) load(1, qa, qb);
+  for (int kb = 0; kb < nkb; kb += 2) {  // np / 32 is even (np is a multiple of 64)
+    step(kb, pa, pb);
+    step(kb + 1, qa, qb);
+  }
+  if (tid == 0)
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+        smem_u32(&bar[kBtStages])));
+  mbar_wait(&bar[kBtStages], 0);
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  // warp w holds D rows 32w..32w+31: warps 2, 3 (the A_lo rows) hand their
+  // (lo*hi + lo*lo) to warps 0, 1 through shared memory (the stages are idle)
+  float* xch = reinterpret_cast<float*>(smem);  // [64][64 + 1]
+  auto ld16 = [&](uint32_t col, float* out) {
+    uint32_t v[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+          "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+          "=r"(v[14]), "=r"(v[15])
+        : "r"(tmem + ((uint32_t)(warp * 32) << 16) + col));
+    asm volatile("tcgen05.wait::ld.sync.aligned;");
+#pragma unroll
+    for (int x = 0; x < 16; ++x) out[x] = __uint_as_float(v[x]);
+  };
+  const int row = (warp & 1) * 32 + lane;  // output row within the tile
+  if (warp >= 2) {
+    for (int c = 0; c < 64; c += 16) {
+      float a[16], b[16];
+      ld16(c, a);
+      ld16(64 + c, b);
+#pragma unroll
+      for (int x = 0; x < 16; ++x) xch[row * 65 + c + x] = a[x] + b[x];
+    }
+  }
+  __syncthreads();
+  if (warp < 2) {
+    const int i = i0 + row;
+    for (int c = 0; c < 64; c += 16) {
+      float a[16], b[16];
+      ld16(c, a);
+      ld16(64 + c, b);
+#pragma unroll
+      for (int x = 0; x < 16; ++x) {
+        const int j = j0 + c + x;
+        const size_t o = (size_t)i * np + j;
+        float v = alpha * ((a[x] + b[x]) + xch[row * 65 + c + x]);
+        if (D) v += beta * D[o];
+        if (i == j && i < n) v += gamma;
+        C[o] = v;
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(128));
+}
+
+__global__ void __launch_bounds__(256) k_big_abar_f(
+    int Bp, int G, int g0, int np, float scale, int e0, int e1, const int32_t* __restrict__ ent_i,
+    const int32_t* __restrict__ ent_j, const int32_t* __restrict__ ent_node_ptr,
+    const int32_t* __restrict__ ent_node, const float* __restrict__ cp, float* __restrict__ X) {
+  const int lane = threadIdx.x & 31;
+  const int e = e0 + blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (e >= e1) return;
+  const int b0 = (g0 + blockIdx.y) * G;
+  double acc = 0.0;
+  for (int a = ent_node_ptr[e]; a < ent_node_ptr[e + 1]; ++a) {
+    const float* row = cp + (size_t)ent_node[a] * Bp + b0;
+    for (int b = lane; b < G; b += 32) acc += (double)row[b];
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+  if (lane == 0)
+    X[(size_t)blockIdx.y * np * np + (size_t)ent_i[e] * np + ent_j[e]] = (float)(acc / G * scale);
+}
+
+// T = I_n + c X over the batch (identity on the first n diagonal entries)
+__global__ void k_big_ipx_f(int n, int np, size_t total, float c, const float* __restrict__ X,
+                            float* __restrict__ T) {
+  const size_t nn = (size_t)np * np;
+  for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < total;
+       idx += (size_t)gridDim.x * blockDim.x) {
+    const size_t r = idx % nn, i = r / np;
+    T[idx] = c * X[idx] + (i == r % np && (int)i < n ? 1.f : 0.f);
+  }
+}
+
+__global__ void __launch_bounds__(256) k_big_finish_f(
+    int n, int np, int scc, int ngroups, int g0, double lambda, const float* __restrict__ Y,
+    int l0, int l1, const int32_t* __restrict__ slot_iloc, const int32_t* __restrict__ slot_jptr,
+    const int32_t* __restrict__ slot_jloc, double* __restrict__ h_part, float* __restrict__ pen) {
+  __shared__ double red[256];
+  const int grp = g0 + blockIdx.y;
+  Y += (size_t)blockIdx.y * np * np;
+  if (blockIdx.x == 0) {
+    double tr = 0.0;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) tr += (double)Y[(size_t)i * np + i];
+    red[threadIdx.x] = tr;
+    __syncthreads();
+    for (int o = blockDim.x / 2; o > 0; o >>= 1) {
+      if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) h_part[(size_t)scc * ngroups + grp] = red[0];
+  }
+  for (int l = l0 + blockIdx.x * blockDim.x + threadIdx.x; l < l1; l += gridDim.x * blockDim.x) {
+    const int il = slot_iloc[l];
+    double acc = 0.0;
+    for (int q = slot_jptr[l]; q < slot_jptr[l + 1]; ++q) {
+      const int jl = slot_jloc[q];
+      acc += (double)Y[(size_t)jl * np + il] + (jl == il ? 1.0 : 0.0);
+    }
+    pen[(size_t)l * ngroups + grp] = (float)(lambda * acc);
+  }
+}
+
+static bool big_fp64() {
+  const char* e = std::getenv("SMOOTHE_BIG_FP64");
+  return e && e[0] == '1';
+}
+
+static void launch_notears_big_tc(cudaStream_t s, const Shape& sh, const HostGraph& hg,
+                                  const DevGraph& g, int32_t G, double lambda, const float* cp,
+                                  double* h_part, float* pen, double* scratch_d, int gpb) {
+  const int ngroups = sh.B / G;
+  static bool attr = false;
+  if (!attr) {
+    SM_CUDA(cudaFuncSetAttribute(k_big_gemm_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, kBtSmem));
+    attr = true;
+  }
+  float* scratch = reinterpret_cast<float*>(scratch_d);
+  for (size_t t = 0; t < hg.big_scc.size(); ++t) {
+    const int scc = hg.big_scc[t], sq = hg.big_scc_sq[t];
+    const int n = hg.scc_class_ptr[scc + 1] - hg.scc_class_ptr[scc];
+    const int np = (n + kBtT - 1) / kBtT * kBtT;
+    const size_t nn = (size_t)np * np;
+    const int e0 = hg.ent_ptr[scc], e1 = hg.ent_ptr[scc + 1];
+    const int l0 = hg.slot_ptr[scc], l1 = hg.slot_ptr[scc + 1];
+    for (int g0 = 0; g0 < ngroups; g0 += gpb) {
+      const int gc = std::min(gpb, ngroups - g0);
+      float* X = scratch;
+      float* T = X + nn * gc;
+      float* U = T + nn * gc;
+      const dim3 gz(np / kBtT, np / kBtT, gc);
+      SM_CUDA(cudaMemsetAsync(X, 0, sizeof(float) * nn * gc, s));
+      if (e1 > e0) {
+        k_big_abar_f<<<dim3((e1 - e0 + 7) / 8, gc), 256, 0, s>>>(
+            sh.Bp, G, g0, np, (float)ldexp(1.0, -sq), e0, e1, g.ent_i, g.ent_j, g.ent_node_ptr,
+            g.ent_node, cp, X);
+        SM_LAUNCH_CHECK();
+      }
+      const int eg = (int)std::min<size_t>((nn * gc + 255) / 256, 148 * 8);
+      k_big_ipx_f<<<eg, 256, 0, s>>>(n, np, nn * gc, 1.f / kTaylorDeg, X, T);
+      SM_LAUNCH_CHECK();
+      for (int mdeg = kTaylorDeg - 1; mdeg >= 2; --mdeg) {  // T_m = I + X T_{m+1} / m
+        k_big_gemm_tc<<<gz, kBtThreads, kBtSmem, s>>>(n, np, X, T, U, 1.f / mdeg, 0.f, nullptr, 1.f);
+        SM_LAUNCH_CHECK();
+        std::swap(T, U);
+      }
+      k_big_gemm_tc<<<gz, kBtThreads, kBtSmem, s>>>(n, np, X, T, U, 1.f, 0.f, nullptr, 0.f);
+      SM_LAUNCH_CHECK();
+      float* Y = U;
+      float* Z = T;
+      for (int r = 0; r < sq; ++r) {  // e^{2A} - I = Y^2 + 2Y
+        k_big_gemm_tc<<<gz, kBtThreads, kBtSmem, s>>>(n, np, Y, Y, Z, 1.f, 2.f, Y, 0.f);
+        SM_LAUNCH_CHECK();
+        std::swap(Y, Z);
+      }
+      const int fb = std::max(1, std::min(148, (l1 - l0 + 255) / 256));
+      k_big_finish_f<<<dim3(fb, gc), 256, 0, s>>>(n, np, scc, ngroups, g0, lambda, Y, l0, l1,
+                                                  g.slot_iloc, g.slot_jptr, g.slot_jloc, h_part,
+                                                  pen);
+      SM_LAUNCH_CHECK();
+    }
+  }
+}
+
 size_t notears_big_scratch(const HostGraph& hg, int ngroups, int* groups_per_batch) {
   int nmax = 0;
   for (int s : hg.big_scc)
@@ -263,7 +569,9 @@ size_t notears_big_scratch(const HostGraph& hg, int ngroups, int* groups_per_bat
     *groups_per_batch = 0;
     return 0;
   }
-  const size_t per = 3 * sizeof(double) * (size_t)nmax * nmax;  // X, T, U per group
+  // X, T, U per group: fp64 n x n (SMOOTHE_BIG_FP64) or fp32 padded to np
+  const size_t np = (size_t)(nmax + kBtT - 1) / kBtT * kBtT;
+  const size_t per = big_fp64() ? 3 * sizeof(double) * (size_t)nmax * nmax : 3 * sizeof(float) * np * np;
   const size_t budget = (size_t)4 << 30;
   *groups_per_batch = (int)std::max<size_t>(1, std::min<size_t>(ngroups, budget / per));
   return per * *groups_per_batch;
@@ -339,9 +647,14 @@ void launch_notears(cudaStream_t s, const Shape& sh, const HostGraph& hg, const 
         g.ent_node, g.slot_ptr, g.slot_iloc, g.slot_jptr, g.slot_jloc, cp, h_part, pen);
     SM_LAUNCH_CHECK();
   }
-  if (!hg.big_scc.empty())
-    launch_notears_big(s, sh, hg, g, G, lambda, cp, h_part, pen, big_scratch,
-                       big_groups_per_batch);
+  if (!hg.big_scc.empty()) {
+    if (big_fp64())
+      launch_notears_big(s, sh, hg, g, G, lambda, cp, h_part, pen, big_scratch,
+                         big_groups_per_batch);
+    else
+      launch_notears_big_tc(s, sh, hg, g, G, lambda, cp, h_part, pen, big_scratch,
+                            big_groups_per_batch);
+  }
 }
 
 }  // namespace smoothe

@@ -340,13 +340,16 @@ def test_c2_aggregators(sm, orc, agg):
     compare_step(sm, orc, make_config("C2"), 64, 8, agg, seed=5)
 
 
-@pytest.mark.parametrize("p_back,G", [(0.06, 8), (0.1, 8), (0.15, 16), (0.06, 1)])
-def test_large_scc(sm, orc, p_back, G):
+@pytest.mark.parametrize("p_back,G,fp64", [(0.06, 8, "0"), (0.1, 8, "0"), (0.15, 16, "0"),
+                                           (0.06, 1, "0"), (0.1, 8, "1")])
+def test_large_scc(sm, orc, monkeypatch, p_back, G, fp64):
     """Components larger than 64 classes (217 / 702 / 1112 classes): the
-    global-memory penalty path (batched fp64 GEMMs) and the block-wide decode
+    global-memory penalty path (tcgen05 3xTF32 GEMMs by default, the fp64
+    CUDA-core GEMMs with SMOOTHE_BIG_FP64=1) and the block-wide decode
     closures.  The first half of the seeds favour the anchor e-nodes (children
     strictly deeper: a valid extraction), so both verdicts occur.  G = 1 is the
     exact per-seed penalty (no Eq. 11 averaging)."""
+    monkeypatch.setenv("SMOOTHE_BIG_FP64", fp64)
     eg = make_config("C2", scc_max=10**9, p_back=p_back)
     assert eg.meta["scc_max"] > 64
     B = 64
