@@ -389,7 +389,12 @@ def run_ours(args):
     torch.cuda.synchronize()
     ck = clocks.stop()
     ms = max_over_ranks(e0.elapsed_time(e1))
-    graph_mode = run.summary()["graph_mode"]
+    summ = run.summary()
+    graph_mode = summ["graph_mode"]
+    pools = {"rows_per_chunk": summ["pool_rows"], "peak_rows": summ["pool_peak_rows"],
+             "grows": summ["pool_grows"], "full_rows": (K + 1) * M,
+             "note": "version pools (DESIGN.md 6): rows per 128-seed chunk; the full stacks "
+                     "would hold (K+1) M"}
     if graph_mode != 1:
         log(f"[bench] WARNING: timed steps did not replay the CUDA graph (graph_mode {graph_mode})")
     units_rank = Bl * N * args.steps
@@ -515,6 +520,7 @@ def run_ours(args):
             "fwd_bwd_units_per_s": fwd_bwd_value,
             "fwd_bwd_ms_per_step": fwdbwd_ms_step,
             "graph_mode": graph_mode,
+            "version_pools": pools,
             "phases_ms_per_step": {k: v / max(1, prof["steps"]) for k, v in ph.items()},
             "profiled_ms_per_step": prof_ms / args.steps,
             "sweep_kernel_ms_per_step": {k: v / max(1, prof["steps"])

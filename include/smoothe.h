@@ -176,6 +176,9 @@ typedef struct {
   double time_to_best_s;   /* run creation -> end of best_step, CUDA events                */
   double step_time_s;      /* mean device time per step                                    */
   double last_loss;        /* L of the last step = sum_b f_b + lambda * sum_g G h_g (S12) */
+  int64_t pool_rows;       /* version-pool rows per seed chunk: capacity     */
+  int64_t pool_peak_rows;  /* most rows a chunk's forward took in one step so far          */
+  int32_t pool_grows;      /* times the pools grew (the overflowing steps were repeated)    */
   int32_t graph_mode;      /* how the steps ran: 1 = replayed from the captured CUDA graph, */
                            /* 0 = direct launches (use_graphs = 0, profiling or debug),     */
                            /* -1 = capture failed, fell back to direct launches (warned on  */

@@ -183,20 +183,27 @@ void launch_theta_init(cudaStream_t s, const Shape& sh, uint64_t key, int64_t se
                        float* theta, float* m, float* v);
 void launch_softmax_argmax(cudaStream_t s, const Shape& sh, const DevGraph& g, const float* theta,
                            float* cp, int32_t* choice, uint32_t* sel);
-// Per-run sweep state (kernels_sweep.cu, "change propagation").  Stacks are
-// indexed by version: slot t holds the rows of the classes recomputed in
-// forward sweep t, listed in list[t] with their previous version (slot 0:
-// q^0 = e_root, pi = 1, am = first parent).
+// Per-run sweep state (kernels_sweep.cu, "change propagation").  Versions
+// live in pools: per seed chunk c (wc = min(Bp, 128) seeds,
+// nchunk = Bp / wc) a pool of cap rows [cap][wc] for each of q, pi, am, rows
+// [0, M) holding version 0 (q^0 = e_root, pi = 1, am = first parent); a class
+// recomputed in forward sweep t takes the next row and is listed in
+// list[c][t] with its previous row.  A step whose chunk needs more than cap
+// rows is aborted and repeated after the host grows the pools.
 struct SweepState {
-  float* qstack = nullptr;    // [K+1][M][Bp]
-  float* pistack = nullptr;   // [K+1][M][Bp] (NULL for the correlated aggregator)
-  int32_t* astack = nullptr;  // [K+1][M][Bp]
+  float* qpool = nullptr;     // [nchunk][cap][wc]
+  float* pipool = nullptr;    // [nchunk][cap][wc] (NULL for the correlated aggregator)
+  int32_t* apool = nullptr;   // [nchunk][cap][wc]
+  int64_t cap = 0;            // rows per chunk pool
+  int nchunk = 1, wc = 0;
+  int32_t* pool_n = nullptr;  // [nchunk] rows taken this step (beyond cap: overflow)
+  int32_t* lastrow = nullptr; // [nchunk][M] current row of each class (during the forward)
+  int4* list = nullptr;       // [nchunk][K+1][M] (class, previous row, new row, -) of sweep t
+  int32_t* list_n = nullptr;  // [nchunk][K+2] list lengths
+  int32_t* abort_flag = nullptr;  // [0] this step overflowed a pool, [1] steps aborted, [2] max rows taken
   float* qbuf[2] = {nullptr, nullptr};  // complete q^t rows, buffer t & 1
   float* cur_pi = nullptr;    // [M][Bp] pi^t of every class during reverse sweep t
   int32_t* cur_am = nullptr;  // [M][Bp]
-  int32_t* lastver = nullptr; // [M] last version of each class (during the forward)
-  int2* list = nullptr;       // [K+1][M] (class, previous version) recomputed in sweep t
-  int32_t* list_n = nullptr;  // [K+2] list lengths
   int K = 0, num_sms = 148;
   int32_t* dirty[2] = {nullptr, nullptr};  // [M] stamp t: recompute in sweep t
   int32_t* chg[2] = {nullptr, nullptr};    // [M] stamp t: q row changed in sweep t
@@ -216,8 +223,8 @@ struct SweepState {
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).
 void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
-void launch_stack_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, float* pi0,
-                           int32_t* am0);
+// version 0 of every class in rows [0, M) of each chunk's pool (run creation, pool growth)
+void launch_pool_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, const SweepState& st);
 // Forward sweep t: q^t (qbuf[t & 1]) from q^{t-1} and versions t of the stacks.
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const SweepState& st, const float* cp);
@@ -271,7 +278,8 @@ size_t notears_big_scratch(const HostGraph& hg, int ngroups, int* groups_per_bat
 void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,
                    const float* gcp, const float* pen, float* theta, float* m, float* v,
                    const double* step_scalars, int32_t optimizer, float lr, float beta1,
-                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out);
+                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out,
+                   const int32_t* abort_flag);
 void launch_step_prologue(cudaStream_t s, int32_t* step_counter, double* step_scalars,
                           double beta1, double beta2, const int32_t* unused);
 void launch_fill_rows(cudaStream_t s, float* base, int64_t stride, int count, int Bp, float value);
@@ -297,6 +305,9 @@ void launch_greedy(cudaStream_t s, const HostGraph& hg, const DevGraph& g, int g
 void launch_warm_start(cudaStream_t s, int M, int Bp, const int32_t* choice, float bias,
                        float* theta);
 int decode_cost_rows(const Shape& sh);
+// after the step (main stream): keep-best commit of the step's candidate (best[4..5])
+void launch_best_commit(cudaStream_t s, int32_t* counter, double* best, int32_t* flag,
+                        int32_t* abort_flag, const int32_t* pool_n, int nchunk);
 void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,
                         const double* dcost_lin, const double* dcost_extra, int64_t seed_begin,
                         const int32_t* step_counter, double* best, int32_t* best_flag,

@@ -353,18 +353,46 @@ __global__ void __launch_bounds__(256) k_best_update(
       trace[4 * (size_t)step + 2] = sc[0];
       trace[4 * (size_t)step + 3] = (double)nvalid;
     }
-    if (sc[0] < best[0]) {
-      best[0] = sc[0];
-      best[1] = (double)step;
-      best[2] = (double)(seed_begin + sb[0]);
-      best[3] = 0.0;
-      *flag = 1;
-    } else {
-      best[3] += 1.0;
-      *flag = 0;
-    }
-    *counter = step + 1;
+    best[4] = sc[0];  // the step's candidate; k_best_commit decides once the step is complete
+    best[5] = (double)(seed_begin + sb[0]);
   }
+}
+
+// Commit the step's candidate (cost, step, global seed) after the whole step
+// ran (main stream): lexicographic keep-best (reading S20), patience counter
+// best[3], step counter.  A step aborted by a full version pool (its update
+// was skipped, it will be repeated) commits nothing and is counted in
+// abort_flag[1]; abort_flag[2] tracks the most pool rows any chunk took.
+__global__ void k_best_commit(int32_t* __restrict__ counter, double* __restrict__ best,
+                              int32_t* __restrict__ flag, int32_t* __restrict__ abort_flag,
+                              const int32_t* __restrict__ pool_n, int nchunk) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (abort_flag) {
+    for (int c = 0; c < nchunk; ++c) abort_flag[2] = max(abort_flag[2], pool_n[c]);
+    if (abort_flag[0]) {
+      *flag = 0;
+      abort_flag[1] += 1;
+      return;
+    }
+  }
+  const int step = *counter;
+  if (best[4] < best[0]) {
+    best[0] = best[4];
+    best[1] = (double)step;
+    best[2] = best[5];
+    best[3] = 0.0;
+    *flag = 1;
+  } else {
+    best[3] += 1.0;
+    *flag = 0;
+  }
+  *counter = step + 1;
+}
+
+void launch_best_commit(cudaStream_t s, int32_t* counter, double* best, int32_t* flag,
+                        int32_t* abort_flag, const int32_t* pool_n, int nchunk) {
+  k_best_commit<<<1, 32, 0, s>>>(counter, best, flag, abort_flag, pool_n, nchunk);
+  SM_LAUNCH_CHECK();
 }
 
 void launch_best_update(cudaStream_t s, const Shape& sh, const uint32_t* settle,

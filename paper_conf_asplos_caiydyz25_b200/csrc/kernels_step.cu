@@ -550,7 +550,9 @@ __global__ void __launch_bounds__(kBlock) k_update(
     const float* __restrict__ cp, const float* __restrict__ gcp, const float* __restrict__ pen,
     float* __restrict__ theta, float* __restrict__ m, float* __restrict__ v,
     const double* __restrict__ scal, int optimizer, float lr, float beta1, float beta2, float eps,
-    float* __restrict__ gth_out, float* __restrict__ gcp_out) {
+    float* __restrict__ gth_out, float* __restrict__ gcp_out, const int32_t* __restrict__ abort_flag) {
+  // a step aborted by a full version pool is repeated: leave theta, m, v as they are
+  if (abort_flag && *abort_flag) return;
   constexpr int R = kBlock / LPR;
   const int lane = threadIdx.x % LPR, sub = threadIdx.x / LPR;
   const int s0 = blockIdx.y * (4 * LPR) + lane * 4;
@@ -625,13 +627,14 @@ __global__ void __launch_bounds__(kBlock) k_update(
 void launch_update(cudaStream_t s, const Shape& sh, const DevGraph& g, int32_t G, const float* cp,
                    const float* gcp, const float* pen, float* theta, float* m, float* v,
                    const double* step_scalars, int32_t optimizer, float lr, float beta1,
-                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out) {
+                   float beta2, float eps, float* grad_theta_out, float* grad_cp_out,
+                   const int32_t* abort_flag) {
   const int ngroups = (sh.B + G - 1) / G;
   SM_DISPATCH_LPR(sh.Bp, {
     k_update<LPR><<<class_grid(sh.M, sh.Bp, LPR, g.num_big), kBlock, 0, s>>>(
         sh.M, sh.Bp, G, ngroups, g.class_ptr, g.big_class, g.num_big, pen ? g.node_slot : nullptr,
         cp, gcp, pen, theta, m,
-        v, step_scalars, optimizer, lr, beta1, beta2, eps, grad_theta_out, grad_cp_out);
+        v, step_scalars, optimizer, lr, beta1, beta2, eps, grad_theta_out, grad_cp_out, abort_flag);
   });
   SM_LAUNCH_CHECK();
 }

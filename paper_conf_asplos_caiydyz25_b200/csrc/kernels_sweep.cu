@@ -60,11 +60,52 @@ constexpr float kRouteTau1 = 1.0f + 1.0f / 1024.0f;
 //
 //   q_prev / q_cur   complete rows q^{t-1} / q^t (ping-pong; a class that
 //                    changed in t-1 but is not recomputed copies its row)
-//   q_slot, pi_slot, am_slot   version t of the stacks, written only by the
-//                    classes recomputed in this sweep; they are appended to
-//                    the list of sweep t with their previous version
-//                    (lastver; 0: the all-zero input, slot 0)
+//   P                the version pools (pooled version stacks):
+//                    a recomputed class takes the next row of its seed
+//                    chunk's pool for its q / pi / am rows and is listed for
+//                    sweep t with its previous row (publish_version)
 // ---------------------------------------------------------------------------
+// Pooled versions: per seed chunk c (wc seeds) a pool of cap rows; rows
+// [0, M) hold version 0 of every class (q^0 = e_root, pi = 1, am = the first
+// parent).  The row group's leader takes the next row of its chunk's pool,
+// every lane writes its seeds of the q / pi / am rows, and the leader lists
+// (class, previous row, new row) for sweep t.  A full pool gives no row: the
+// step is marked aborted (its update is skipped; the host grows the pool and
+// repeats the step, smoothe_run_steps).
+struct PoolArgs {
+  float* q;
+  float* pi;  // NULL for the correlated aggregator
+  int32_t* am;
+  int64_t cap;
+  int wc, M, K;
+  int32_t* pool_n;      // [nchunk] rows taken this step (may exceed cap: overflow)
+  int32_t* lastrow;     // [nchunk][M]
+  int4* list;           // [nchunk][K+1][M]
+  int32_t* list_n;      // [nchunk][K+2]
+  int32_t* abort_flag;  // [0]: this step overflowed
+};
+template <int LPR>
+__device__ __forceinline__ void publish_version(const PoolArgs& P, int t, int j, int gl,
+                                                unsigned gm, float4 qo, float4 po, int4 arg) {
+  const int c = blockIdx.y;
+  int r = 0;
+  if (gl == 0) r = atomicAdd(P.pool_n + c, 1);
+  r = __shfl_sync(gm, r, (int)(threadIdx.x % 32) / LPR * LPR);  // from the group's leader
+  if (r >= P.cap) {
+    if (gl == 0) P.abort_flag[0] = 1;
+    return;
+  }
+  const size_t o = ((size_t)c * P.cap + r) * P.wc + gl * 4;
+  stcs4(P.q + o, qo);
+  if (P.pi) stcs4(P.pi + o, po);
+  stcs4i(P.am + o, arg);
+  if (gl == 0) {
+    int32_t* lr = P.lastrow + (size_t)c * P.M + j;
+    const int n = atomicAdd(P.list_n + (size_t)c * (P.K + 2) + t, 1);
+    P.list[((size_t)c * (P.K + 1) + t) * P.M + n] = make_int4(j, *lr, r, 0);
+    *lr = r;
+  }
+}
 // read-only path for the gathers (as the former kernel-parameter version got)
 __device__ __forceinline__ float4 ldg4(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
 __device__ __forceinline__ int4 ldg4i(const int32_t* p) { return __ldg(reinterpret_cast<const int4*>(p)); }
@@ -72,22 +113,18 @@ __device__ __forceinline__ int4 ldg4i(const int32_t* p) { return __ldg(reinterpr
 #define SM_FWD_PARAMS                                                                        \
   int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,                   \
       const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,                 \
-      const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,                     \
-      int32_t* __restrict__ lastver, int32_t* __restrict__ list_n, int2* __restrict__ list,    \
+      const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur, PoolArgs P,          \
       const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,        \
       const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,  \
       float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,                \
-      float* __restrict__ q_cur, float* __restrict__ q_slot, float* __restrict__ pi_slot,      \
-      int32_t* __restrict__ am_slot
+      float* __restrict__ q_cur
 #define SM_FWD_ARGS                                                                            \
-  M, Bp, root, t, all, dmin, dirty_cur, dirty_next, chg_prev, chg_cur, lastver, list_n, list,  \
-      cls_child_ptr, cls_child, pad_par_ptr, pad_par, wI, wC, cp, q_prev, q_cur, q_slot,       \
-      pi_slot, am_slot
+  M, Bp, root, t, all, dmin, dirty_cur, dirty_next, chg_prev, chg_cur, P, cls_child_ptr,       \
+      cls_child, pad_par_ptr, pad_par, wI, wC, cp, q_prev, q_cur
 
 // Recompute class j (its row group: LPR lanes, this lane's 4 seeds from s0).
 template <int LPR>
-__device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int s0, bool leader,
-                                              unsigned gm) {
+__device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int s0, unsigned gm) {
   const size_t o = (size_t)j * Bp + s0;
   const float4 qold = ldg4(q_prev + o);
   // (node, class) pairs in batches of 4; padding pairs (N, root) read the zero
@@ -142,13 +179,7 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
     comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
   st4(q_cur + o, qo);
-  stcs4(q_slot + o, qo);
-  if (pi_slot) stcs4(pi_slot + o, po);
-  if (leader) {
-    list[atomicAdd(list_n + t, 1)] = make_int2(j, lastver[j]);
-    lastver[j] = t;
-  }
-  stcs4i(am_slot + o, arg);
+  publish_version<LPR>(P, t, j, gl, gm, qo, po, arg);
   // bitwise change of the row (any seed of this chunk); chunks of a class write
   // the same stamps, so concurrent stores are benign
   const bool ne = __float_as_uint(qo.x) != __float_as_uint(qold.x) ||
@@ -176,7 +207,6 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(SM_FWD_PARAMS) {
   const int sh = (int)(threadIdx.x % 32) / LPR * LPR;
   const unsigned gm = LPR == 32 ? 0xffffffffu : ((1u << LPR) - 1u) << sh;
   const int s0 = blockIdx.y * (4 * LPR) + gl * 4;
-  const bool lead = gl == 0 && blockIdx.y == 0;
   // the warp iterates together (row groups of LPR < 32 lanes share it): loop
   // bounds from the warp's first row group, and the union of the groups' work
   // bits, so the row groups of a warp run their classes side by side
@@ -200,7 +230,7 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(SM_FWD_PARAMS) {
       if (!((wb >> i) & 1u)) continue;
       const int j = (int)((r0 + i) * G + g);
       if ((db >> i) & 1u) {
-        forward_class<LPR>(SM_FWD_ARGS, j, gl, s0, lead, gm);
+        forward_class<LPR>(SM_FWD_ARGS, j, gl, s0, gm);
       } else {  // q^t_j = q^{t-1}_j, which q_cur (written two sweeps ago) lacks
         const size_t o = (size_t)j * Bp + s0;
         st4(q_cur + o, ld4(q_prev + o));
@@ -218,17 +248,14 @@ template <int LPR>
 __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
     int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,
-    const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur,
-    int32_t* __restrict__ lastver, int32_t* __restrict__ list_n, int2* __restrict__ list,
+    const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur, PoolArgs P,
     const int32_t* __restrict__ cls_child_ptr, const int32_t* __restrict__ cls_child,
     const int32_t* __restrict__ pad_par_ptr, const int32_t* __restrict__ pad_par, float wI,
     float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
-    float* __restrict__ q_cur, float* __restrict__ q_slot, float* __restrict__ pi_slot,
-    int32_t* __restrict__ am_slot) {
+    float* __restrict__ q_cur) {
   const int j = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
   if (j >= M) return;
   const int gl = threadIdx.x % LPR;
-  const bool leader = gl == 0 && blockIdx.y == 0;
   const int s0 = blockIdx.y * (4 * LPR) + gl * 4;
   const size_t o = (size_t)j * Bp + s0;
   const bool dirty = j != root && (all || (t == 1 ? __ldg(dmin + j) == 1 : dirty_cur[j] == t));
@@ -289,20 +316,14 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
     comp(po, x) = z == 0 ? comp(prod, x) : (z == 1 ? -comp(prod, x) : 0.f);
   }
   st4(q_cur + o, qo);
-  stcs4(q_slot + o, qo);
-  if (pi_slot) stcs4(pi_slot + o, po);
-  if (leader) {
-    list[atomicAdd(list_n + t, 1)] = make_int2(j, lastver[j]);
-    lastver[j] = t;
-  }
-  stcs4i(am_slot + o, arg);
+  const unsigned gm = LPR == 32 ? 0xffffffffu : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
+  publish_version<LPR>(P, t, j, gl, gm, qo, po, arg);
   // bitwise change of the row (any seed of this chunk); chunks of a class write
   // the same stamps, so concurrent stores are benign
   const bool ne = __float_as_uint(qo.x) != __float_as_uint(qold.x) ||
                   __float_as_uint(qo.y) != __float_as_uint(qold.y) ||
                   __float_as_uint(qo.z) != __float_as_uint(qold.z) ||
                   __float_as_uint(qo.w) != __float_as_uint(qold.w);
-  const unsigned gm = LPR == 32 ? 0xffffffffu : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
   if (__ballot_sync(gm, ne) == 0u) return;
   if (gl == 0) chg_cur[j] = t;
   for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
@@ -323,11 +344,28 @@ static int forward_grid(int device) {
   return b;
 }
 
+static PoolArgs pool_args(const Shape& sh, const SweepState& st) {
+  PoolArgs P;
+  P.q = st.qpool;
+  P.pi = st.pipool;
+  P.am = st.apool;
+  P.cap = st.cap;
+  P.wc = st.wc;
+  P.M = sh.M;
+  P.K = st.K;
+  P.pool_n = st.pool_n;
+  P.lastrow = st.lastrow;
+  P.list = st.list;
+  P.list_n = st.list_n;
+  P.abort_flag = st.abort_flag;
+  return P;
+}
+
 void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a, int t,
                           const SweepState& st, const float* cp) {
-  const size_t MB = (size_t)sh.M * sh.Bp;
   int dev = 0;
   SM_CUDA(cudaGetDevice(&dev));
+  const PoolArgs P = pool_args(sh, st);
   SM_DISPATCH_LPR(sh.Bp, {
     const int rows_per_block = kSweepBlock / LPR;
     const int need = (sh.M + rows_per_block - 1) / rows_per_block;
@@ -336,17 +374,13 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
     if (need <= cap)
       k_sweep_forward_direct<LPR><<<grid, kSweepBlock, 0, s>>>(
           sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
-          st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n, st.list + (size_t)t * sh.M,
-          g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp,
-          t == 1 ? st.qstack : st.qbuf[(t - 1) & 1], st.qbuf[t & 1], st.qstack + (size_t)t * MB,
-          st.pistack ? st.pistack + (size_t)t * MB : nullptr, st.astack + (size_t)t * MB);
+          st.chg[(t - 1) & 1], st.chg[t & 1], P, g.cls_child_ptr, g.cls_child, g.pad_par_ptr,
+          g.pad_par, a.wI, a.wC, cp, st.qbuf[(t - 1) & 1], st.qbuf[t & 1]);
     else
       k_sweep_forward<LPR><<<grid, kSweepBlock, 0, s>>>(
           sh.M, sh.Bp, sh.root, t, st.all ? 1 : 0, g.dmin, st.dirty[t & 1], st.dirty[(t + 1) & 1],
-          st.chg[(t - 1) & 1], st.chg[t & 1], st.lastver, st.list_n, st.list + (size_t)t * sh.M,
-          g.cls_child_ptr, g.cls_child, g.pad_par_ptr, g.pad_par, a.wI, a.wC, cp,
-          t == 1 ? st.qstack : st.qbuf[(t - 1) & 1], st.qbuf[t & 1], st.qstack + (size_t)t * MB,
-          st.pistack ? st.pistack + (size_t)t * MB : nullptr, st.astack + (size_t)t * MB);
+          st.chg[(t - 1) & 1], st.chg[t & 1], P, g.cls_child_ptr, g.cls_child, g.pad_par_ptr,
+          g.pad_par, a.wI, a.wC, cp, st.qbuf[(t - 1) & 1], st.qbuf[t & 1]);
   });
   SM_LAUNCH_CHECK();
 }
@@ -354,43 +388,49 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // Before reverse sweep t: the reverse reads q^{t-1} (its own class) and
 // pi^t / am^t (child classes) from complete rows cur_q / cur_pi / cur_am.
 // Going from sweep t+1 to t, only the classes recomputed in forward sweep t+1
-// (pi, am) or t (q) change version: copy their previous version's rows (the
-// forward's lists, so the work is proportional to the recomputed classes).
-// t == K fills cur_pi / cur_am from every class's last version (cur_q is the
-// forward's complete q^{K-1} buffer).
+// (pi, am) or t (q) change version: copy their previous version's pool rows
+// (the forward's lists, so the work is proportional to the recomputed
+// classes).  t == K fills cur_pi / cur_am from every class's last row (cur_q
+// is the forward's complete q^{K-1} buffer).  Grid y = seed chunk = pool.
 template <int LPR>
-__global__ void __launch_bounds__(kBlock) k_rev_restore_all(
-    int M, int Bp, const int32_t* __restrict__ lastver, const float* __restrict__ pistack,
-    const int32_t* __restrict__ astack, float* __restrict__ cur_pi, int32_t* __restrict__ cur_am) {
+__global__ void __launch_bounds__(kBlock) k_rev_restore_all(int M, int Bp, PoolArgs P,
+                                                           float* __restrict__ cur_pi,
+                                                           int32_t* __restrict__ cur_am) {
   const RowGroup<LPR> rg;
   const int j = rg.row;
   if (j >= M) return;
-  const size_t MB = (size_t)M * Bp, o = (size_t)j * Bp + rg.s0;
-  const size_t v = (size_t)lastver[j];
-  if (cur_pi) st4(cur_pi + o, ld4(pistack + v * MB + o));
-  st4i(cur_am + o, ld4i(astack + v * MB + o));
+  const int c = blockIdx.y;
+  const size_t o = (size_t)j * Bp + rg.s0;
+  const size_t src = ((size_t)c * P.cap + P.lastrow[(size_t)c * M + j]) * P.wc + (rg.s0 - c * P.wc);
+  if (cur_pi) st4(cur_pi + o, ld4(P.pi + src));
+  st4i(cur_am + o, ld4i(P.am + src));
 }
 
 template <int LPR>
-__global__ void __launch_bounds__(kBlock) k_rev_transition(
-    int M, int Bp, const int32_t* __restrict__ n_pa, const int2* __restrict__ l_pa,
-    const int32_t* __restrict__ n_q, const int2* __restrict__ l_q, const float* __restrict__ qstack,
-    const float* __restrict__ pistack, const int32_t* __restrict__ astack, float* __restrict__ cur_q,
-    float* __restrict__ cur_pi, int32_t* __restrict__ cur_am, int32_t* __restrict__ wm) {
+__global__ void __launch_bounds__(kBlock) k_rev_transition(int M, int Bp, int t, PoolArgs P,
+                                                          float* __restrict__ cur_q,
+                                                          float* __restrict__ cur_pi,
+                                                          int32_t* __restrict__ cur_am,
+                                                          int32_t* __restrict__ wm) {
   const int groups = gridDim.x * (kBlock / LPR);
-  const int n1 = *n_pa, n = n1 + *n_q;
-  const size_t MB = (size_t)M * Bp;
-  const int s0 = blockIdx.y * (4 * LPR) + (threadIdx.x % LPR) * 4;
+  const int c = blockIdx.y;
+  const int32_t* ln = P.list_n + (size_t)c * (P.K + 2);
+  const int4* l_pa = P.list + ((size_t)c * (P.K + 1) + t + 1) * M;  // recomputed in sweep t+1
+  const int4* l_q = P.list + ((size_t)c * (P.K + 1) + t) * M;       // recomputed in sweep t
+  const int n1 = ln[t + 1], n = n1 + ln[t];
+  const int gl = threadIdx.x % LPR;
+  const int s0 = c * (4 * LPR) + gl * 4;
+  const size_t pbase = (size_t)c * P.cap;
   for (int i = blockIdx.x * (kBlock / LPR) + (int)threadIdx.x / LPR; i < n; i += groups) {
     if (i < n1) {
-      const int2 e = l_pa[i];
-      const size_t o = (size_t)e.x * Bp + s0, src = (size_t)e.y * MB + o;
-      if (cur_pi) st4(cur_pi + o, ld4(pistack + src));
-      st4i(cur_am + o, ld4i(astack + src));
+      const int4 e = l_pa[i];
+      const size_t o = (size_t)e.x * Bp + s0, src = (pbase + e.y) * P.wc + gl * 4;
+      if (cur_pi) st4(cur_pi + o, ld4(P.pi + src));
+      st4i(cur_am + o, ld4i(P.am + src));
     } else {
-      const int2 e = l_q[i - n1];
+      const int4 e = l_q[i - n1];
       const size_t o = (size_t)e.x * Bp + s0;
-      const float4 prev = ld4(qstack + (size_t)e.y * MB + o);
+      const float4 prev = ld4(P.q + (pbase + e.y) * P.wc + gl * 4);
       if (wm) {  // a seed whose q row changed in forward sweep t leaves the K-state
         const float4 now = ld4(cur_q + o);
 #pragma unroll
@@ -407,66 +447,76 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(
 void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
                            const SweepState& st) {
   (void)g;
+  const PoolArgs P = pool_args(sh, st);
   SM_DISPATCH_LPR(sh.Bp, {
     if (t == K) {
-      k_rev_restore_all<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-          sh.M, sh.Bp, st.lastver, st.pistack, st.astack, st.cur_pi, st.cur_am);
+      k_rev_restore_all<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, P,
+                                                                            st.cur_pi, st.cur_am);
     } else {
       const dim3 grid(2 * st.num_sms, num_chunks(sh.Bp));
-      k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(
-          sh.M, sh.Bp, st.list_n + t + 1, st.list + (size_t)(t + 1) * sh.M, st.list_n + t,
-          st.list + (size_t)t * sh.M, st.qstack, st.pistack, st.astack, st.qbuf[(K - 1) & 1],
-          st.cur_pi, st.cur_am, st.wmode ? st.wm : nullptr);
+      k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, t, P, st.qbuf[(K - 1) & 1],
+                                                    st.cur_pi, st.cur_am,
+                                                    st.wmode ? st.wm : nullptr);
     }
   });
   SM_LAUNCH_CHECK();
 }
 
-// Version 0 of the stacks (a class never recomputed: every parent's q is 0):
-// pi = +1 (every factor 1 - 0 is non-zero), am = the first (lowest-id) parent,
-// the forward kernel's tie rule; -1 for the root and parentless classes.
+// Version 0 of every class in rows [0, M) of each chunk's pool (a class never
+// recomputed: every parent's q is 0): q = e_root, pi = +1 (every factor 1 - 0
+// is non-zero), am = the first (lowest-id) parent, the forward kernel's tie
+// rule; -1 for the root and parentless classes.
 template <int LPR>
-__global__ void __launch_bounds__(kBlock) k_stack_version0(int M, int Bp, int root,
-                                                           const int32_t* __restrict__ pad_par_ptr,
-                                                           const int32_t* __restrict__ pad_par,
-                                                           float* __restrict__ pi0,
-                                                           int32_t* __restrict__ am0) {
+__global__ void __launch_bounds__(kBlock) k_pool_version0(int M, int root,
+                                                          const int32_t* __restrict__ pad_par_ptr,
+                                                          const int32_t* __restrict__ pad_par,
+                                                          PoolArgs P) {
   const RowGroup<LPR> rg;
   const int j = rg.row;
   if (j >= M) return;
-  const size_t o = (size_t)j * Bp + rg.s0;
+  const int c = blockIdx.y;
+  const size_t o = ((size_t)c * P.cap + j) * P.wc + (rg.s0 - c * P.wc);
   const int e0 = pad_par_ptr[j];
   const int a = j != root && e0 < pad_par_ptr[j + 1] ? pad_par[2 * (size_t)e0] : -1;
-  if (pi0) st4(pi0 + o, make_float4(1.f, 1.f, 1.f, 1.f));
-  st4i(am0 + o, make_int4(a, a, a, a));
+  const float q0 = j == root ? 1.f : 0.f;
+  st4(P.q + o, make_float4(q0, q0, q0, q0));
+  if (P.pi) st4(P.pi + o, make_float4(1.f, 1.f, 1.f, 1.f));
+  st4i(P.am + o, make_int4(a, a, a, a));
 }
 
-void launch_stack_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, float* pi0,
-                           int32_t* am0) {
+void launch_pool_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, const SweepState& st) {
+  const PoolArgs P = pool_args(sh, st);
   SM_DISPATCH_LPR(sh.Bp, {
-    k_stack_version0<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(
-        sh.M, sh.Bp, sh.root, g.pad_par_ptr, g.pad_par, pi0, am0);
+    k_pool_version0<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.root, g.pad_par_ptr,
+                                                                       g.pad_par, P);
   });
   SM_LAUNCH_CHECK();
 }
 
-// Per-step reset of the forward's state in one kernel (instead of eight
-// memsets and a fill): stamps (dirty / chg, one allocation of 4 M) = -1,
-// lastver = 0, list_n = 0, both q ping-pong rows = e_root (qbuf[1] follows
-// qbuf[0] in one allocation).
-__global__ void k_sweep_reset(int M, int Bp, int root, int nlist, int32_t* __restrict__ stamps,
-                              int32_t* __restrict__ lastver, int32_t* __restrict__ list_n,
-                              float* __restrict__ qbuf) {
-  const int64_t MB = (int64_t)M * Bp, n0 = 4 * (int64_t)M, n1 = n0 + M, n2 = n1 + nlist,
-                n3 = n2 + 2 * MB;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n3;
-       e += (int64_t)gridDim.x * blockDim.x) {
+// Per-step reset of the forward's state in one kernel (instead of a dozen
+// memsets and a fill): stamps (dirty / chg, one allocation of 4 M) = -1, both
+// q ping-pong rows = e_root (qbuf[1] follows qbuf[0] in one allocation), and
+// per seed chunk: the pool's rows taken = M (version 0), every class's row =
+// its version 0, list lengths 0; the step's abort flag 0.
+__global__ void k_sweep_reset(int M, int Bp, int root, int nchunk, int K,
+                              int32_t* __restrict__ stamps, float* __restrict__ qbuf,
+                              int32_t* __restrict__ pool_n, int32_t* __restrict__ lastrow,
+                              int32_t* __restrict__ list_n, int32_t* __restrict__ abort_flag) {
+  const int64_t MB = (int64_t)M * Bp, n0 = 4 * (int64_t)M, n1 = n0 + 2 * MB,
+                n2 = n1 + (int64_t)nchunk * M, n3 = n2 + (int64_t)nchunk * (K + 2);
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e0 == 0) abort_flag[0] = 0;
+  if (e0 < nchunk) pool_n[e0] = M;
+  for (int64_t e = e0; e < n3; e += stride) {
     if (e < n0) stamps[e] = -1;
-    else if (e < n1) lastver[e - n0] = 0;
-    else if (e < n2) list_n[e - n1] = 0;
-    else {
-      const int64_t q = e - n2;
+    else if (e < n1) {
+      const int64_t q = e - n0;
       qbuf[q] = (q % MB) / Bp == root ? 1.f : 0.f;
+    } else if (e < n2) {
+      lastrow[e - n1] = (int32_t)((e - n1) % M);
+    } else {
+      list_n[e - n2] = 0;
     }
   }
 }
@@ -475,8 +525,9 @@ void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
   // stamps: dirty[0], dirty[1], chg[0], chg[1] are consecutive (alloc_state)
   int dev = 0;
   SM_CUDA(cudaGetDevice(&dev));
-  k_sweep_reset<<<4 * num_sms(dev), 256, 0, s>>>(sh.M, sh.Bp, sh.root, st.K + 2, st.dirty[0],
-                                                 st.lastver, st.list_n, st.qbuf[0]);
+  k_sweep_reset<<<4 * num_sms(dev), 256, 0, s>>>(sh.M, sh.Bp, sh.root, st.nchunk, st.K,
+                                                 st.dirty[0], st.qbuf[0], st.pool_n, st.lastrow,
+                                                 st.list_n, st.abort_flag);
   SM_LAUNCH_CHECK();
 }
 
@@ -1315,7 +1366,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
     const int32_t* __restrict__ lastchg) {
   const RowGroup<LPR, kWBlock> rg;
-  if (frozen_count && blockIdx.x == 0 && threadIdx.x == 0) {  // profiling: a working launch?
+  if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {  // profiling: a working launch?
     bool any = false;
     for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
     if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
@@ -1496,42 +1547,38 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
 
 // Converge mode: lastchg[s] = max over sweeps t and classes j recomputed in t of
 // t if version t of q_j differs from its previous version in seed s.  Grid
-// (x: entries, y: sweep t - 1, z: seed chunk); per-block flags, one atomicMax
-// per seed and block.
+// (x: entries, y: sweep t - 1, z: seed chunk = pool); per-block flags, one
+// atomicMax per seed and block.
 template <int LPR>
-__global__ void __launch_bounds__(kBlock) k_last_change(int M, int Bp,
-                                                       const int32_t* __restrict__ list_n,
-                                                       const int2* __restrict__ list,
-                                                       const float* __restrict__ qstack,
+__global__ void __launch_bounds__(kBlock) k_last_change(int M, PoolArgs P,
                                                        int32_t* __restrict__ lastchg) {
   __shared__ int flag[4 * LPR];
-  const int t = blockIdx.y + 1;
+  const int t = blockIdx.y + 1, c = blockIdx.z;
   const int gl = threadIdx.x % LPR, sub = threadIdx.x / LPR;
-  const int s0 = blockIdx.z * (4 * LPR) + gl * 4;
   if (threadIdx.x < 4 * LPR) flag[threadIdx.x] = 0;
   __syncthreads();
-  const int n = list_n[t];
-  const size_t MB = (size_t)M * Bp;
-  const int2* lt = list + (size_t)t * M;
+  const int n = P.list_n[(size_t)c * (P.K + 2) + t];
+  const int4* lt = P.list + ((size_t)c * (P.K + 1) + t) * M;
+  const size_t pbase = (size_t)c * P.cap;
   for (int e = blockIdx.x * (kBlock / LPR) + sub; e < n; e += gridDim.x * (kBlock / LPR)) {
-    const int2 en = lt[e];
-    const size_t o = (size_t)en.x * Bp + s0;
-    const float4 a = ld4(qstack + (size_t)t * MB + o), b = ld4(qstack + (size_t)en.y * MB + o);
+    const int4 en = lt[e];
+    const float4 a = ld4(P.q + (pbase + en.z) * P.wc + gl * 4),
+                 b = ld4(P.q + (pbase + en.y) * P.wc + gl * 4);
 #pragma unroll
     for (int x = 0; x < 4; ++x)
       if (__float_as_uint(comp(a, x)) != __float_as_uint(comp(b, x))) flag[gl * 4 + x] = 1;
   }
   __syncthreads();
   if (threadIdx.x < 4 * LPR && flag[threadIdx.x])
-    atomicMax(lastchg + blockIdx.z * (4 * LPR) + threadIdx.x, t);
+    atomicMax(lastchg + c * (4 * LPR) + threadIdx.x, t);
 }
 
 void launch_last_change(cudaStream_t s, const Shape& sh, const SweepState& st) {
   SM_CUDA(cudaMemsetAsync(st.lastchg, 0, sizeof(int32_t) * sh.Bp, s));
+  const PoolArgs P = pool_args(sh, st);
   SM_DISPATCH_LPR(sh.Bp, {
     const dim3 grid(64, st.K, num_chunks(sh.Bp));
-    k_last_change<LPR><<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, st.list_n, st.list, st.qstack,
-                                                st.lastchg);
+    k_last_change<LPR><<<grid, kBlock, 0, s>>>(sh.M, P, st.lastchg);
   });
   SM_LAUNCH_CHECK();
 }

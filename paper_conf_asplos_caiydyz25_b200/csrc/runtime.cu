@@ -166,6 +166,16 @@ static T* upload(RunMem& m, const std::vector<T>& v, int64_t* bytes = nullptr) {
 }
 
 // a freed run's blocks replace the device's cache
+void runmem_free(RunMem& m, void* p) {  // one block, back to the driver
+  for (size_t i = 0; i < m.p.size(); ++i)
+    if (m.p[i] == p) {
+      cudaFree(p);
+      m.p.erase(m.p.begin() + i);
+      m.n.erase(m.n.begin() + i);
+      return;
+    }
+}
+
 void runmem_recycle(RunMem& m) {
   cache_release(m.device);
   DevCache& c = dev_cache();
@@ -254,6 +264,8 @@ struct smoothe_run {
   cudaGraphExec_t graph_exec = nullptr;
   bool graph_failed = false;
   int64_t graph_steps = 0;  // steps replayed from graph_exec
+  int64_t pool_high = 0;    // most version-pool rows a chunk took in a step (checked steps)
+  int32_t pool_grows = 0;   // times the pools grew
   bool poisoned = false;
   int steps_run = 0;
 };
@@ -376,8 +388,6 @@ void enqueue_decode(smoothe_run* r, cudaStream_t ds, PhaseMarks* pm) {
   launch_best_update(ds, sh, r->settle, r->dcost, dextra, r->opt.seed_begin, r->counter, r->best,
                      r->best_flag, r->debug ? r->dbg_dcost : nullptr,
                      r->debug ? r->dbg_valid : nullptr, r->trace, kTraceCap);
-  launch_best_snapshot(ds, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
-                       r->best_choice);
 }
 
 void enqueue_step(smoothe_run* r) {
@@ -525,7 +535,7 @@ void enqueue_step(smoothe_run* r) {
   launch_update(s, sh, g, r->G, r->cp, r->gcp, hg.num_scc > 0 ? r->pen : nullptr, r->theta, r->m,
                 r->v, r->scal, r->opt.optimizer, (float)r->opt.lr, (float)r->opt.beta1,
                 (float)r->opt.beta2, (float)r->opt.eps, r->debug ? r->dbg_gth : nullptr,
-                r->debug ? r->dbg_gcp : nullptr);
+                r->debug ? r->dbg_gcp : nullptr, r->sw.abort_flag);
 
   if (!overlap_now) {
     pm.mark(SMOOTHE_PHASE_DECODE);
@@ -533,6 +543,11 @@ void enqueue_step(smoothe_run* r) {
   } else {
     SM_CUDA(cudaStreamWaitEvent(s, r->ev_join, 0));
   }
+  // keep-best of the complete step (an aborted step commits nothing)
+  launch_best_commit(s, r->counter, r->best, r->best_flag, r->sw.abort_flag, r->sw.pool_n,
+                     r->sw.nchunk);
+  launch_best_snapshot(s, sh, r->choice, r->reach, r->best, r->best_flag, r->opt.seed_begin,
+                       r->best_choice);
   pm.finish();
   if (r->profiling) {
     r->prof_launch_total += launch_counter() - l0;
@@ -583,6 +598,60 @@ void run_one_step(smoothe_run* r) {
   r->steps_run++;
 }
 
+// Version pools.  All (K + 1) M rows per chunk -- the stacks of
+// a full recompute -- when that is small; else a fraction of it
+// (SMOOTHE_POOL_FRAC, default 0.25 of the K sweeps, measured: the forward
+// recomputes ~5-40% of the classes per sweep on C4 / C5, more late in a run)
+// that smoothe_run_steps grows when a step overflows.
+int64_t initial_pool_rows(const smoothe_run* r) {
+  const Shape& sh = r->sh;
+  const int64_t full = ((int64_t)r->K + 1) * sh.M;
+  const double bytes = (double)full * sh.Bp * 4.0 * (r->agg.wI != 0.f ? 3 : 2);
+  const char* e = std::getenv("SMOOTHE_POOL_FRAC");
+  if (!e && bytes <= 4e9) return full;
+  const double frac = e ? std::atof(e) : 0.25;
+  return std::min<int64_t>(full, sh.M + (int64_t)std::ceil(frac * r->K * sh.M));
+}
+
+void alloc_pools(smoothe_run* r, int64_t cap) {
+  SweepState& w = r->sw;
+  for (void* p : {(void*)w.qpool, (void*)w.pipool, (void*)w.apool})
+    if (p) runmem_free(r->owned, p);
+  w.qpool = w.pipool = nullptr;
+  w.apool = nullptr;
+  w.cap = cap;
+  const size_t n = (size_t)w.nchunk * cap * w.wc;
+  w.qpool = dalloc<float>(r->owned, n);
+  if (r->agg.wI != 0.f) w.pipool = dalloc<float>(r->owned, n);
+  w.apool = dalloc<int32_t>(r->owned, n);
+}
+
+// After steps were enqueued: if any step overflowed a version pool (it was
+// aborted: no update, no keep-best), grow the pools to 1.25x the most rows a
+// chunk asked for (at least 1.5x), re-initialise version 0, drop the captured
+// graph (its pointers changed) and return the number of aborted steps, which
+// the caller repeats.  Synchronises the run's stream.
+int pool_check_grow(smoothe_run* r) {
+  SweepState& w = r->sw;
+  int32_t f[4];
+  SM_CUDA(cudaMemcpyAsync(f, w.abort_flag, sizeof(f), cudaMemcpyDeviceToHost, r->stream));
+  SM_CUDA(cudaStreamSynchronize(r->stream));
+  r->pool_high = std::max<int64_t>(r->pool_high, f[2]);
+  if (f[1] == 0) return 0;
+  const int64_t full = ((int64_t)r->K + 1) * r->sh.M;
+  const int64_t want = std::max<int64_t>((int64_t)(1.25 * f[2]) + 1, (int64_t)(1.5 * w.cap));
+  if (w.cap >= full) throw Failure{SMOOTHE_E_STATE, "version pool overflow at full capacity"};
+  alloc_pools(r, std::min(full, want));
+  launch_pool_version0(r->stream, r->sh, r->g->dev, w);
+  SM_CUDA(cudaMemsetAsync(w.abort_flag, 0, sizeof(int32_t) * 2, r->stream));
+  if (r->graph_exec) {
+    SM_CUDA(cudaGraphExecDestroy(r->graph_exec));
+    r->graph_exec = nullptr;
+  }
+  r->pool_grows++;
+  return f[1];
+}
+
 void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   const Shape& sh = r->sh;
   const HostGraph& hg = r->g->host;
@@ -598,20 +667,20 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     const char* env = std::getenv("SMOOTHE_SWEEP_ALL");
     w.all = env && env[0] == '1';
     const size_t slots = (size_t)r->K + 1;
-    w.qstack = dalloc<float>(o, slots * MB);
-    if (r->agg.wI != 0.f) {
-      w.pistack = dalloc<float>(o, slots * MB);
-      w.cur_pi = dalloc<float>(o, MB);
-    }
-    w.astack = dalloc<int32_t>(o, slots * MB);
+    if (r->agg.wI != 0.f) w.cur_pi = dalloc<float>(o, MB);
     w.cur_am = dalloc<int32_t>(o, MB);
     w.qbuf[0] = dalloc<float>(o, 2 * MB);
     w.qbuf[1] = w.qbuf[0] + MB;
     w.K = r->K;
     w.num_sms = num_sms(r->device);
-    w.lastver = dalloc<int32_t>(o, sh.M);
-    w.list = dalloc<int2>(o, slots * sh.M);
-    w.list_n = dalloc<int32_t>(o, slots + 1);
+    w.wc = std::min(sh.Bp, 128);
+    w.nchunk = sh.Bp / w.wc;
+    w.lastrow = dalloc<int32_t>(o, (size_t)w.nchunk * sh.M);
+    w.list = dalloc<int4>(o, (size_t)w.nchunk * slots * sh.M);
+    w.list_n = dalloc<int32_t>(o, (size_t)w.nchunk * (slots + 1));
+    w.pool_n = dalloc<int32_t>(o, w.nchunk);
+    w.abort_flag = dalloc<int32_t>(o, 4);
+    alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
     for (int b = 0; b < 2; ++b) {  // consecutive: k_sweep_reset fills all four at once
       w.dirty[b] = stamps + (size_t)b * sh.M;
@@ -629,7 +698,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.W = dalloc<float>(o, (size_t)r->g->dev.num_cedge * sh.Bp);
       w.S = dalloc<float>(o, MB);
       w.kq = dalloc<float>(o, MB);
-      if (w.pistack) w.kpi = dalloc<float>(o, MB);
+      if (r->agg.wI != 0.f) w.kpi = dalloc<float>(o, MB);
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
       w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
@@ -670,7 +739,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   r->dcost_part = dalloc<double>(o, (size_t)r->dcost_rows * sh.Bp);
   r->dcost = dalloc<double>(o, sh.Bp);
   r->dextra = dalloc<double>(o, sh.Bp);
-  r->best = dalloc<double>(o, 4);
+  r->best = dalloc<double>(o, 6);  // (cost, step, seed, steps since), the step's candidate (cost, seed)
   r->best_flag = dalloc<int32_t>(o, 1);
   r->best_choice = dalloc<int32_t>(o, sh.M);
   r->counter = dalloc<int32_t>(o, 1);
@@ -740,13 +809,12 @@ void init_state(smoothe_run* r) {
   const size_t MB = (size_t)sh.M * sh.Bp;
   launch_theta_init(s, sh, r->opt.rng_key, r->opt.seed_begin, r->theta, r->m, r->v);
   SM_CUDA(cudaMemsetAsync(r->cp + (size_t)sh.N * sh.Bp, 0, sizeof(float) * sh.Bp, s));
-  // version 0 of the stacks (never overwritten: sweeps write slots 1..K):
+  // version 0 in the pools (never overwritten: sweeps take rows from M on):
   // q^0 = e_root; pi = 1; am = the first parent, -1 for the root, whose rows
   // therefore match no e-node, so padding slots (which point at the root) take
   // no correlated term
-  SM_CUDA(cudaMemsetAsync(r->sw.qstack, 0, sizeof(float) * MB, s));
-  launch_fill_rows(s, r->sw.qstack + (size_t)sh.root * sh.Bp, (int64_t)MB, 1, sh.Bp, 1.0f);
-  launch_stack_version0(s, sh, r->g->dev, r->sw.pistack, r->sw.astack);
+  launch_pool_version0(s, sh, r->g->dev, r->sw);
+  SM_CUDA(cudaMemsetAsync(r->sw.abort_flag, 0, sizeof(int32_t) * 4, s));
   SM_CUDA(cudaMemsetAsync(r->gq[0], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->gq[1], 0, sizeof(float) * MB, s));
   SM_CUDA(cudaMemsetAsync(r->pen, 0, sizeof(float), s));
@@ -754,7 +822,7 @@ void init_state(smoothe_run* r) {
   SM_CUDA(cudaMemsetAsync(r->counter, 0, sizeof(int32_t), s));
   SM_CUDA(cudaMemsetAsync(r->rev_cnt, 0, sizeof(int32_t) * sh.M * std::max(1, sh.Bp / 32), s));
   SM_CUDA(cudaMemsetAsync(r->trace, 0xff, sizeof(double) * 4 * kTraceCap, s));  // NaN: not run
-  const double init_best[4] = {INFINITY, -1.0, -1.0, 0.0};
+  const double init_best[6] = {INFINITY, -1.0, -1.0, 0.0, INFINITY, -1.0};
   SM_CUDA(cudaMemcpyAsync(r->best, init_best, sizeof(init_best), cudaMemcpyHostToDevice, s));
   SM_CUDA(cudaMemsetAsync(r->best_choice, 0xff, sizeof(int32_t) * sh.M, s));
   SM_CUDA(cudaStreamSynchronize(s));
@@ -1122,16 +1190,26 @@ smoothe_status smoothe_run_steps(smoothe_run* run, int32_t steps) {
       SM_CUDA(cudaStreamWaitEvent(run->stream, join, 0));
     }
     const bool checks = run->opt.patience > 0 || run->opt.time_limit_s > 0;
-    for (int32_t i = 0; i < steps; ++i) {
-      run_one_step(run);
-      if (checks && ((i + 1) % 8 == 0 || i + 1 == steps)) {
-        double best[4];
-        SM_CUDA(cudaMemcpyAsync(best, run->best, sizeof(best), cudaMemcpyDeviceToHost, run->stream));
-        SM_CUDA(cudaStreamSynchronize(run->stream));
-        if (run->opt.patience > 0 && best[3] >= run->opt.patience) break;
-        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - run->t_create).count();
-        if (run->opt.time_limit_s > 0 && el >= run->opt.time_limit_s) break;
+    const bool growable = run->sw.cap < ((int64_t)run->K + 1) * run->sh.M;
+    int32_t left = steps;
+    while (left > 0) {
+      int32_t done = 0;
+      bool stop = false;
+      for (; done < left && !stop; ++done) {
+        run_one_step(run);
+        if (checks && ((done + 1) % 8 == 0 || done + 1 == left)) {
+          double best[4];
+          SM_CUDA(cudaMemcpyAsync(best, run->best, sizeof(best), cudaMemcpyDeviceToHost, run->stream));
+          SM_CUDA(cudaStreamSynchronize(run->stream));
+          if (run->opt.patience > 0 && best[3] >= run->opt.patience) stop = true;
+          const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - run->t_create).count();
+          if (run->opt.time_limit_s > 0 && el >= run->opt.time_limit_s) stop = true;
+        }
       }
+      // steps aborted by a full version pool are repeated on grown pools
+      const int aborted = growable ? pool_check_grow(run) : 0;
+      run->steps_run -= aborted;
+      left = stop ? 0 : aborted;
     }
     if (user) {
       SM_CUDA(cudaEventRecord(join, run->stream));
@@ -1177,6 +1255,11 @@ smoothe_status smoothe_extract(smoothe_run* run, int32_t* choice, smoothe_summar
       out->K = run->K;
       out->last_loss = loss;
       out->graph_mode = run->graph_failed ? -1 : (run->graph_steps > 0 ? 1 : 0);
+      int32_t f[4];
+      SM_CUDA(cudaMemcpy(f, run->sw.abort_flag, sizeof(f), cudaMemcpyDeviceToHost));
+      out->pool_rows = run->sw.cap;
+      out->pool_peak_rows = std::max<int64_t>(run->pool_high, f[2]);
+      out->pool_grows = run->pool_grows;
       float ms = 0.f;
       const int bs = out->best_step;
       if (valid && bs >= 0 && (size_t)bs < run->ev_step.size() && bs < run->steps_run) {
@@ -1225,7 +1308,10 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     run->debug = true;
     try {
       // the step overwrites theta; keep the input's cp etc. from the step itself
+      // (a step aborted by a full version pool left theta, m, v and the step
+      // counter as they were: grow the pools and take it again)
       enqueue_step(run);
+      while (pool_check_grow(run) > 0) enqueue_step(run);
     } catch (...) {
       run->debug = false;
       for (void* p : scratch) cudaFree(p);
@@ -1242,26 +1328,47 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
     copy_rows_d2h(dump->theta_out, run->theta, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->m_out, run->m, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->v_out, run->v, sh.N, sh.B, sh.Bp, s);
-    // version stacks: slot t holds the classes recomputed in sweep t; the rest
-    // of row t is filled from ver on the host below
-    // ver[t][j]: the version holding class j's rows at sweep t, rebuilt from
-    // the forward's lists of recomputed classes
-    std::vector<int32_t> ver;
+    // q stack / routes from the version pools: per seed chunk, the row of
+    // class j at sweep t is its last version listed up to sweep t (rows
+    // [0, M): version 0), rebuilt from the forward's lists on the host
     if (dump->qstack || dump->route) {
-      std::vector<int32_t> ln(run->K + 2);
-      std::vector<int2> lst((size_t)(run->K + 1) * sh.M);
-      SM_CUDA(cudaMemcpyAsync(ln.data(), run->sw.list_n, sizeof(int32_t) * ln.size(), cudaMemcpyDeviceToHost, s));
-      SM_CUDA(cudaMemcpyAsync(lst.data(), run->sw.list, sizeof(int2) * lst.size(), cudaMemcpyDeviceToHost, s));
-      SM_CUDA(cudaStreamSynchronize(s));
-      ver.assign((size_t)(run->K + 1) * sh.M, 0);
-      for (int t = 1; t <= run->K; ++t) {
-        std::copy(ver.begin() + (size_t)(t - 1) * sh.M, ver.begin() + (size_t)t * sh.M,
-                  ver.begin() + (size_t)t * sh.M);
-        for (int i = 0; i < ln[t]; ++i) ver[(size_t)t * sh.M + lst[(size_t)t * sh.M + i].x] = t;
+      const SweepState& w = run->sw;
+      const int K = run->K;
+      std::vector<int32_t> ln((size_t)w.nchunk * (K + 2));
+      std::vector<int4> lst((size_t)w.nchunk * (K + 1) * sh.M);
+      std::vector<float> qp(dump->qstack ? (size_t)w.cap * w.wc : 0);
+      std::vector<int32_t> ap(dump->route ? (size_t)w.cap * w.wc : 0);
+      SM_CUDA(cudaMemcpyAsync(ln.data(), w.list_n, sizeof(int32_t) * ln.size(), cudaMemcpyDeviceToHost, s));
+      SM_CUDA(cudaMemcpyAsync(lst.data(), w.list, sizeof(int4) * lst.size(), cudaMemcpyDeviceToHost, s));
+      std::vector<int32_t> row(sh.M);
+      for (int c = 0; c < w.nchunk; ++c) {
+        if (dump->qstack)
+          SM_CUDA(cudaMemcpyAsync(qp.data(), w.qpool + (size_t)c * w.cap * w.wc,
+                                  sizeof(float) * qp.size(), cudaMemcpyDeviceToHost, s));
+        if (dump->route)
+          SM_CUDA(cudaMemcpyAsync(ap.data(), w.apool + (size_t)c * w.cap * w.wc,
+                                  sizeof(int32_t) * ap.size(), cudaMemcpyDeviceToHost, s));
+        SM_CUDA(cudaStreamSynchronize(s));
+        const int b0 = c * w.wc, b1 = std::min(sh.B, b0 + w.wc);
+        for (int j = 0; j < sh.M; ++j) row[j] = j;
+        for (int t = 0; t <= K; ++t) {
+          if (t > 0)
+            for (int i = 0; i < ln[(size_t)c * (K + 2) + t]; ++i) {
+              const int4 e = lst[((size_t)c * (K + 1) + t) * sh.M + i];
+              row[e.x] = e.z;
+            }
+          for (int j = 0; j < sh.M; ++j) {
+            const size_t src = (size_t)row[j] * w.wc;
+            if (dump->qstack)
+              for (int b = b0; b < b1; ++b)
+                dump->qstack[((size_t)t * sh.M + j) * sh.B + b] = qp[src + (b - b0)];
+            if (dump->route && t > 0)  // route row t - 1 = sweep t
+              for (int b = b0; b < b1; ++b)
+                dump->route[((size_t)(t - 1) * sh.M + j) * sh.B + b] = ap[src + (b - b0)];
+          }
+        }
       }
     }
-    if (dump->qstack)
-      copy_rows_d2h(dump->qstack, run->sw.qstack, (run->K + 1) * sh.M, sh.B, sh.Bp, s);
     if (dump->f) SM_CUDA(cudaMemcpyAsync(dump->f, run->ftot, sizeof(double) * sh.B, cudaMemcpyDeviceToHost, s));
     if (dump->h) {
       if (run->g->host.num_scc > 0)
@@ -1285,10 +1392,6 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       }
       for (int b = 0; b < sh.B; ++b) dump->sweeps[b] = std::min(run->K, lc[b] + 1);
     }
-    if (dump->route && run->K > 0)  // rows of sweep t + 1 = slot t + 1
-      SM_CUDA(cudaMemcpy2DAsync(dump->route, sizeof(int32_t) * sh.B, run->sw.astack + MB,
-                                sizeof(int32_t) * sh.Bp, sizeof(int32_t) * sh.B,
-                                (size_t)run->K * sh.M, cudaMemcpyDeviceToHost, s));
     std::vector<uint32_t> rbits;
     if (dump->reached) {
       rbits.resize((size_t)sh.M * sh.W);
@@ -1299,33 +1402,6 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       for (int j = 0; j < sh.M; ++j)
         for (int b = 0; b < sh.B; ++b)
           dump->reached[(size_t)j * sh.B + b] = (rbits[(size_t)j * sh.W + (b >> 5)] >> (b & 31)) & 1u;
-    if (dump->qstack)  // row t of a class not recomputed in sweep t = its version's row
-      for (int t = 1; t <= run->K; ++t)
-        for (int j = 0; j < sh.M; ++j) {
-          const int v = ver[(size_t)t * sh.M + j];
-          if (v != t)
-            std::memcpy(dump->qstack + ((size_t)t * sh.M + j) * sh.B,
-                        dump->qstack + ((size_t)v * sh.M + j) * sh.B, sizeof(float) * sh.B);
-        }
-    if (dump->route) {
-      // Row t = sweep t + 1.  A class not recomputed in that sweep takes the
-      // row of its version; version 0 (every p exactly 0, so every parent
-      // ties) is the lowest-id parent, the kernel's tie rule (S7'), and -1 for
-      // the root (q_root = 1 is not a decision, S3) and parentless classes.
-      const HostGraph& hg = run->g->host;
-      for (int t = 0; t < run->K; ++t)
-        for (int j = 0; j < sh.M; ++j) {
-          const int v = ver[(size_t)(t + 1) * sh.M + j];
-          if (v == t + 1) continue;
-          int32_t* row = dump->route + ((size_t)t * sh.M + j) * sh.B;
-          if (v > 0) {
-            std::memcpy(row, dump->route + ((size_t)(v - 1) * sh.M + j) * sh.B, sizeof(int32_t) * sh.B);
-          } else {
-            const int32_t a = j != sh.root && hg.par_ptr[j + 1] > hg.par_ptr[j] ? hg.par_node[hg.par_ptr[j]] : -1;
-            for (int b = 0; b < sh.B; ++b) row[b] = a;
-          }
-        }
-    }
     if ((size_t)run->steps_run < run->ev_step.size())
       SM_CUDA(cudaEventRecord(run->ev_step[run->steps_run], s));
     for (void* p : scratch) SM_CUDA(cudaFree(p));

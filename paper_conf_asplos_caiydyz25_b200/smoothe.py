@@ -58,7 +58,8 @@ class _Summary(C.Structure):
     _fields_ = [("best_cost", C.c_double), ("best_seed", C.c_int64), ("best_step", C.c_int32),
                 ("valid", C.c_int32), ("steps_run", C.c_int32), ("K", C.c_int32),
                 ("time_to_best_s", C.c_double), ("step_time_s", C.c_double),
-                ("last_loss", C.c_double), ("graph_mode", C.c_int32)]
+                ("last_loss", C.c_double), ("pool_rows", C.c_int64), ("pool_peak_rows", C.c_int64),
+                ("pool_grows", C.c_int32), ("graph_mode", C.c_int32)]
 
 
 class _Dump(C.Structure):

@@ -693,3 +693,37 @@ def test_step_trace_relaxed_vs_sampled(sm):
     assert np.all(tr["relaxed_min"] <= tr["relaxed_mean"])
     run.close()
     g.close()
+
+
+@pytest.mark.parametrize("name,B,G,steps", [("C2", 64, 8, 6), ("C3", 128, 8, 3), ("C5", 64, 8, 3)])
+def test_version_pool_growth_bit_identical(sm, monkeypatch, name, B, G, steps):
+    """Pooled version stacks: a run whose pools start far too
+    small (SMOOTHE_POOL_FRAC=0.01) aborts the overflowing steps (no update, no
+    keep-best), grows the pools and repeats them; theta, the best extraction
+    and a debug step's q stack and routes (rebuilt from the pools) are bit
+    for bit those of a run with pools for every sweep (SMOOTHE_POOL_FRAC=1)."""
+    eg = make_config(name)
+    outs = []
+    for frac in ("0.01", "1"):
+        monkeypatch.setenv("SMOOTHE_POOL_FRAC", frac)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=31))
+        run.steps(steps)
+        th, m, v, n = run.state()
+        assert n == steps
+        small = eg.num_nodes < 10000
+        d = run.debug_step(th, m, v, step_index=n, qstack=small, route=small)
+        ch, s = run.extract()
+        outs.append((th, ch, s, d))
+        run.close()
+        g.close()
+    (t0, c0, s0, d0), (t1, c1, s1, d1) = outs
+    assert s0["pool_grows"] > 0 and s1["pool_grows"] == 0
+    assert s0["pool_rows"] < s1["pool_rows"] or s1["pool_rows"] == s0["pool_rows"]
+    assert np.array_equal(t0, t1) and np.array_equal(c0, c1)
+    for k in ("best_cost", "best_step", "best_seed", "steps_run"):
+        assert s0[k] == s1[k], k
+    for k in ("qstack", "route", "grad_cp", "theta_out", "qK"):
+        if k in d0:
+            assert np.array_equal(d0[k], d1[k]), k
