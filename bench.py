@@ -448,6 +448,27 @@ def run_ours(args):
                              "valid": gr["valid"], "linear_cost_only": eg.mlp is not None
                              or eg.quad is not None}
 
+    # the config's whole seed batch on this one GPU (P = 1; C4:
+    # 1024 seeds), graph-timed like the headline: the per-GPU slice above is
+    # the 8-GPU configuration's
+    p1 = None
+    if world == 1 and not args.no_p1_leg and spec["seeds"] > Bl:
+        prun = sm.run_create(g, cost, spec["seeds"], options(converge=args.converge))
+        prun.steps(3)
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        prun.steps(3)
+        q1.record(stream)
+        torch.cuda.synchronize()
+        pms = q0.elapsed_time(q1) / 3
+        ps = prun.summary()
+        p1 = {"seeds": spec["seeds"], "steps": 3, "warmup": 3, "ms_per_step": pms,
+              "value": spec["seeds"] * N / (pms * 1e-3), "unit": UNIT,
+              "version_pool_rows_per_chunk": ps["pool_rows"], "pool_grows": ps["pool_grows"]}
+        prun.close()
+        sm.release_cached_memory(local)
+
     # the same workload in convergence mode (reading S1b, an option, not the
     # headline: the north star fixes the number of iterations)
     conv = None
@@ -528,6 +549,7 @@ def run_ours(args):
             "gpu_launches": prof["launches"],
             "time_to_best": ttb,
             "converge_mode": conv,
+            "single_gpu_full_batch": p1,
             "roofline": roof, "e2e": e2e, "cpu_baseline": cb, "clocks": ck,
         }
         print(json.dumps(line), flush=True)
@@ -617,6 +639,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--converge", action="store_true",
                     help="reading S1b: each seed's sweeps stop at convergence (not the default K)")
+    ap.add_argument("--no-p1-leg", action="store_true",
+                    help="skip the config's whole seed batch on one GPU")
     ap.add_argument("--no-converge-leg", action="store_true",
                     help="skip the extra convergence-mode measurement")
     ap.add_argument("--ttb-steps", type=int, default=1000,

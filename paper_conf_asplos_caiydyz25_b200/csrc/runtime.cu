@@ -600,8 +600,8 @@ void run_one_step(smoothe_run* r) {
 
 // Version pools.  All (K + 1) M rows per chunk -- the stacks of
 // a full recompute -- when that is small; else a fraction of it
-// (SMOOTHE_POOL_FRAC, default 0.25 of the K sweeps, measured: the forward
-// recomputes ~5-40% of the classes per sweep on C4 / C5, more late in a run)
+// (SMOOTHE_POOL_FRAC, default 0.15 of the K sweeps; measured on C4: a step
+// recomputes 7% of (K+1) M class rows early in a run, more later)
 // that smoothe_run_steps grows when a step overflows.
 int64_t initial_pool_rows(const smoothe_run* r) {
   const Shape& sh = r->sh;
@@ -609,7 +609,7 @@ int64_t initial_pool_rows(const smoothe_run* r) {
   const double bytes = (double)full * sh.Bp * 4.0 * (r->agg.wI != 0.f ? 3 : 2);
   const char* e = std::getenv("SMOOTHE_POOL_FRAC");
   if (!e && bytes <= 4e9) return full;
-  const double frac = e ? std::atof(e) : 0.25;
+  const double frac = e ? std::atof(e) : 0.15;
   return std::min<int64_t>(full, sh.M + (int64_t)std::ceil(frac * r->K * sh.M));
 }
 
