@@ -94,6 +94,8 @@ def main():
         lines.append(f"| {k} | {n} | {t * 1e3:.2f} | {100 * t / tot:.1f}% | {1e6 * t / n:.1f} |")
     traffic_path = os.path.join(ROOT, "profiles", "traffic.json")
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+    l2_path = os.path.join(ROOT, "profiles", "l2.json")
+    l2 = json.load(open(l2_path)) if os.path.exists(l2_path) else {}
     for rp in reps:
         for d in capture(rp):
             lines += ["", f"## `ncu --set full` capture: {d['kernel']} ({os.path.basename(rp)})", "",
@@ -107,10 +109,14 @@ def main():
                         else "forward" if "forward" in d["kernel"] else d["kernel"])
                 traffic.setdefault(cfg, {})[kind] = b
                 lines.append(f"| traffic (read + write) per launch | {b / 1e9:.3f} GB |")
+            if "L2 hit rate %" in d:  # bench.py reports it for L2-resident configs
+                l2.setdefault(cfg, {})[d["kernel"]] = float(d["L2 hit rate %"][0].replace(",", ""))
     with open(os.path.join(ROOT, "profiles", f"{tag}_{cfg}.md"), "w") as fh:
         fh.write("\n".join(lines) + "\n")
     with open(traffic_path, "w") as fh:
         json.dump(traffic, fh, indent=1)
+    with open(l2_path, "w") as fh:
+        json.dump(l2, fh, indent=1)
     print("\n".join(lines))
 
 
