@@ -332,12 +332,6 @@ __global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
   auto store = [&](int st, const float4 (&ra)[4], const float4 (&rb)[4]) {
     uint8_t* sa = smem + st * kBtStage;
     uint8_t* sb = sa + kBtA;
-    // B: each pair of lanes starts its four transposed columns at a different
-    // offset, so every 8 consecutive lanes (a 128-bit store is served 8 lanes
-    // at a time) hit the 8 16-byte positions of a 128-byte core row (the
-    // plain order was a 4-way bank conflict).  A keeps the row-coalesced
-    // order: a conflict-free A order (8 rows per 8 lanes) measured slower,
-    // its global loads no longer coalesce (profiles/r2/notears_precision.md).
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       const int idx = tid + i * kBtThreads, r = idx / 8, kc = idx % 8;
@@ -346,14 +340,14 @@ __global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
       *reinterpret_cast<float4*>(sa + (kc * 16 + r / 8) * 128 + (r % 8) * 16) = hi;
       *reinterpret_cast<float4*>(sa + (kc * 16 + 8 + r / 8) * 128 + (r % 8) * 16) = lo;
     }
+    // (bank-conflict-free store orders for A and B measured slower: they cost
+    // the loads' coalescing or extra selects, and shared stores are not the limit)
     const int kc = tid / 16, c = (tid % 16) * 4;
-    auto sel = [](float4 v, int o) { return o == 0 ? v.x : o == 1 ? v.y : o == 2 ? v.z : v.w; };
 #pragma unroll
-    for (int x = 0; x < 4; ++x) {  // column c + o: its 4 K values, transposed to K-major
-      const int o = (x + (tid >> 1)) & 3;
-      const float4 col = make_float4(sel(rb[0], o), sel(rb[1], o), sel(rb[2], o), sel(rb[3], o));
+    for (int x = 0; x < 4; ++x) {  // column c + x: its 4 K values, transposed to K-major
+      const float4 col = make_float4(comp(rb[0], x), comp(rb[1], x), comp(rb[2], x), comp(rb[3], x));
       const float4 hi = tf32_hi(col), lo = sub4(col, hi);
-      const int m = c + o;
+      const int m = c + x;
       *reinterpret_cast<float4*>(sb + (kc * 16 + m / 8) * 128 + (m % 8) * 16) = hi;
       *reinterpret_cast<float4*>(sb + (kc * 16 + (64 + m) / 8) * 128 + (m % 8) * 16) = lo;
     }
