@@ -1,6 +1,7 @@
 // Internal declarations of libsmoothe (not part of the ABI).
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -321,6 +322,7 @@ void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice
 // z1_part: [nsplit][128][Bp] split-K partials of the tensor-core layer 1
 // (nsplit = mlp_nsplit(device) CTAs per seed chunk); z1: [H1][Bp]
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
+                    const float* W1t,
                     const float* b1, const float* W2, const float* b2, const float* W3,
                     const float* b3, const float* p, float* z1_part, float* z1, double* f_mlp,
                     float* gz1, int32_t nsplit);
@@ -330,5 +332,10 @@ void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1
 
 int num_sms(int device);
 int64_t& launch_counter();
+
+// 2-D tensor map (tma.cu): dims {inner, outer} elements of fp32 / int32,
+// rows row_bytes apart, box {box_inner, box_outer}; cached
+const CUtensorMap& tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
+                                 uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
 
 }  // namespace smoothe

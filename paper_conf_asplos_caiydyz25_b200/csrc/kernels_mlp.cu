@@ -5,6 +5,8 @@
 // (2*H1*N*B flop) and g_p[k][b] += sum_h W1[h][k] gz1[h][b] (same); both run
 // on the tensor cores.  Split-K partial sums are reduced in a fixed order, so
 // results are deterministic.
+#include <cstdlib>
+
 #include "kcommon.cuh"
 
 namespace smoothe {
@@ -222,6 +224,223 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
 }
 
+// ---------------------------------------------------------------------------
+// Layer 1 with TMA-fed, warp-specialised stages (the default; SMOOTHE_MLP_TMA=0
+// keeps the register-staged kernel above).  Raw fp32 tiles come in by TMA --
+// W1^T [32 e-nodes x 64 hidden] (the run keeps W1 transposed, zero-padded to
+// 64 hidden units, so a tile is 8 KB of contiguous memory; W1's own rows
+// gave 64 pieces of 128 bytes, measured no faster than the register kernel)
+// and p [32 e-nodes x Bc seeds], e-nodes past N zero-filled by the TMA --
+// into a ring of kRawStages; four
+// converter warps split each raw tile into hi / lo and lay it out in the
+// canonical no-swizzle K-major UMMA layouts of a ring of kMmaStages; one
+// thread issues the MMAs (as in k_mlp_l1_tc: A = [W1_hi; W1_lo], B = [p_hi |
+// p_lo], all four products in one M=128 x N=2Bc x K=8 MMA), tcgen05.commit
+// releases each stage; the converter warps read the accumulator back (warp w
+// owns TMEM lanes 32 (w % 4)..).  Output: z1_part as k_mlp_l1_tc.
+//   warp 0: TMA producer, warp 1: MMA issuer, warps 2..5: converters + epilogue
+// ---------------------------------------------------------------------------
+constexpr int kTmKB = 32;  // e-nodes per stage
+
+template <int BC>
+__host__ __device__ constexpr int tm_raw_stages() { return BC >= 128 ? 4 : BC >= 64 ? 6 : 8; }
+template <int BC>
+__host__ __device__ constexpr int tm_mma_stages() { return BC >= 128 ? 2 : BC >= 64 ? 3 : 4; }
+template <int BC>
+__host__ __device__ constexpr int tm_smem() {
+  return tm_raw_stages<BC>() * (64 * kTmKB * 4 + kTmKB * BC * 4) +
+         tm_mma_stages<BC>() * (128 * kTmKB * 4 + kTmKB * 2 * BC * 4) + 1024;
+}
+
+template <int BC>
+__global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ CUtensorMap tm_w,
+                                                      const __grid_constant__ CUtensorMap tm_p,
+                                                      int N, int Bp, int nsplit,
+                                                      float* __restrict__ z1_part) {
+  constexpr int NM = 2 * BC;
+  constexpr int RS = tm_raw_stages<BC>(), MS = tm_mma_stages<BC>();
+  constexpr int RAW_A = 64 * kTmKB * 4, RAW_B = kTmKB * BC * 4, RAW = RAW_A + RAW_B;
+  constexpr int A_BYTES = 128 * kTmKB * 4, B_BYTES = kTmKB * NM * 4, MMA = A_BYTES + B_BYTES;
+  constexpr int A_LBO = 16 * 128, B_LBO = (NM / 8) * 128;
+  constexpr uint32_t TMEM_COLS = NM <= 32 ? 32 : NM <= 64 ? 64 : NM <= 128 ? 128 : 256;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
+                             ((uint32_t)(128 >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t tm_smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(tm_smem_raw) + 1023) & ~(uintptr_t)1023);
+  uint8_t* raw = smem;                 // RS x RAW
+  uint8_t* mma = smem + RS * RAW;      // MS x MMA (1 KB aligned: RAW is a multiple of 1 KB)
+  __shared__ uint64_t raw_full[RS], raw_empty[RS], mma_full[MS], mma_empty[MS], acc_full;
+  __shared__ uint32_t tmem_sh;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int seed0 = blockIdx.y * BC;
+  const int64_t per = (((int64_t)N + nsplit - 1) / nsplit + kTmKB - 1) / kTmKB * kTmKB;
+  const int64_t kb64 = (int64_t)blockIdx.x * per;
+  const int k_begin = (int)(kb64 < N ? kb64 : N);
+  const int k_end = (int)(k_begin + per < N ? k_begin + per : N);
+  const int nkb = (k_end - k_begin + kTmKB - 1) / kTmKB;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&tmem_sh)),
+                 "n"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int i = 0; i < RS; ++i) {
+      mbar_init(&raw_full[i], 1);
+      mbar_init(&raw_empty[i], 4);  // one arrival per converter warp
+    }
+    for (int i = 0; i < MS; ++i) {
+      mbar_init(&mma_full[i], 4);
+      mbar_init(&mma_empty[i], 1);  // tcgen05.commit
+    }
+    mbar_init(&acc_full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem = tmem_sh;
+
+  if (warp == 0) {  // TMA producer
+    if (lane == 0)
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int st = kb % RS;
+        if (kb >= RS) mbar_wait(&raw_empty[st], (uint32_t)((kb / RS - 1) & 1));
+        const uint32_t dst = smem_u32(raw + st * RAW), bar = smem_u32(&raw_full[st]);
+        const int k0 = k_begin + kb * kTmKB;
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(RAW));
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+            " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+            "l"(&tm_w), "r"(0), "r"(k0), "r"(bar)
+            : "memory");
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+            " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst + RAW_A),
+            "l"(&tm_p), "r"(seed0), "r"(k0), "r"(bar)
+            : "memory");
+      }
+  } else if (warp == 1) {  // MMA issuer
+    if (lane == 0) {
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int st = kb % MS;
+        mbar_wait(&mma_full[st], (uint32_t)((kb / MS) & 1));
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        const uint32_t sa = smem_u32(mma + st * MMA), sb = sa + A_BYTES;
+#pragma unroll
+        for (int ks = 0; ks < kTmKB / 8; ++ks) {
+          const uint64_t da = umma_desc(sa + ks * 2 * A_LBO, A_LBO, 128);
+          const uint64_t db = umma_desc(sb + ks * 2 * B_LBO, B_LBO, 128);
+          const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
+          asm volatile(
+              "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+              "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+              "l"(da), "l"(db), "r"(IDESC), "r"(acc));
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+            smem_u32(&mma_empty[st])));
+      }
+      if (nkb > 0)
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+            smem_u32(&acc_full)));
+      else
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_full)));
+    }
+  } else {  // converters (128 threads), then the epilogue
+    const int ct = tid - 64;
+    for (int kb = 0; kb < nkb; ++kb) {
+      const int rs = kb % RS, ms = kb % MS;
+      mbar_wait(&raw_full[rs], (uint32_t)((kb / RS) & 1));
+      if (kb >= MS) mbar_wait(&mma_empty[ms], (uint32_t)((kb / MS - 1) & 1));
+      const uint8_t* ra = raw + rs * RAW;
+      const uint8_t* rb = ra + RAW_A;
+      uint8_t* sa = mma + ms * MMA;
+      uint8_t* sb = sa + A_BYTES;
+      // A: raw (k, h) at (k * 64 + h) * 4; one 4 x 4 block (K chunk kc,
+      // hidden units hc..hc+3) per thread, transposed to K-major
+      {
+        const int kc = ct / 16, hc = (ct % 16) * 4;
+        float4 r4[4];
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+          r4[r] = *reinterpret_cast<const float4*>(ra + ((4 * kc + r) * 64 + hc) * 4);
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+          // (rotating each lane pair's column order removes the 4-way bank
+          // conflicts of these stores but measured 65 -> 97 us: the shared
+          // stores are conflicted yet cheaper than the selects)
+          const float4 col = make_float4(comp(r4[0], x), comp(r4[1], x), comp(r4[2], x), comp(r4[3], x));
+          const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+          const int h = hc + x;
+          *reinterpret_cast<float4*>(sa + (kc * 16 + h / 8) * 128 + (h % 8) * 16) = hi;
+          *reinterpret_cast<float4*>(sa + (kc * 16 + 8 + h / 8) * 128 + (h % 8) * 16) = lo;
+        }
+      }
+      // B: raw (k, s) at (k * BC + s) * 4; 4 x 4 blocks transposed to K-major
+      constexpr int BBLK = (kTmKB / 4) * (BC / 4);
+      for (int blk = ct; blk < BBLK; blk += 128) {
+        const int kc = blk / (BC / 4), n = (blk % (BC / 4)) * 4;
+        float4 r4[4];
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+          r4[r] = *reinterpret_cast<const float4*>(rb + ((4 * kc + r) * BC + n) * 4);
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+          const float4 col = make_float4(comp(r4[0], x), comp(r4[1], x), comp(r4[2], x), comp(r4[3], x));
+          const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+          const int m = n + x;
+          *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + m / 8) * 128 + (m % 8) * 16) = hi;
+          *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + (BC + m) / 8) * 128 + (m % 8) * 16) = lo;
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;");
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&raw_empty[rs])));
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&mma_full[ms])));
+      }
+    }
+    mbar_wait(&acc_full, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    const int q = warp % 4;  // TMEM lanes 32q .. 32q + 31 = D rows
+    const int row = q * 32 + lane;
+    float* out = z1_part + ((size_t)blockIdx.x * 128 + row) * Bp + seed0;
+    if (nkb == 0) {
+#pragma unroll
+      for (int c = 0; c < BC; c += 4) *reinterpret_cast<float4*>(out + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+#pragma unroll
+    for (int c = 0; c < BC && nkb > 0; c += 16) {
+      uint32_t v[16], w[16];
+      const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + c;
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+            "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+            "=r"(v[14]), "=r"(v[15])
+          : "r"(ta));
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]),
+            "=r"(w[7]), "=r"(w[8]), "=r"(w[9]), "=r"(w[10]), "=r"(w[11]), "=r"(w[12]), "=r"(w[13]),
+            "=r"(w[14]), "=r"(w[15])
+          : "r"(ta + BC));
+      asm volatile("tcgen05.wait::ld.sync.aligned;");
+#pragma unroll
+      for (int x = 0; x < 16; x += 4)
+        *reinterpret_cast<float4*>(out + c + x) =
+            make_float4(__uint_as_float(v[x]) + __uint_as_float(w[x]),
+                        __uint_as_float(v[x + 1]) + __uint_as_float(w[x + 1]),
+                        __uint_as_float(v[x + 2]) + __uint_as_float(w[x + 2]),
+                        __uint_as_float(v[x + 3]) + __uint_as_float(w[x + 3]));
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+}
+
 // z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h
 __global__ void k_mlp_reduce(int Bp, int H1, int nsplit, const float* __restrict__ b1,
                              const float* __restrict__ z1_part, float* __restrict__ z1) {
@@ -412,11 +631,34 @@ __global__ void __launch_bounds__(kTcThreads) k_mlp_l1_back_tc(int N, int Bp, in
 int mlp_nsplit(int device) { return num_sms(device); }
 
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
+                    const float* W1t,
                     const float* b1, const float* W2, const float* b2, const float* W3,
                     const float* b3, const float* p, float* z1_part, float* z1, double* f_mlp,
                     float* gz1, int32_t nsplit) {
   const int Bc = sh.Bp < 128 ? sh.Bp : 128;
   const dim3 grid(nsplit, sh.Bp / Bc);
+  const char* tenv = std::getenv("SMOOTHE_MLP_TMA");
+  const bool tma = !(tenv && tenv[0] == '0') && W1t;
+  if (tma) {
+    const CUtensorMap& tw = tensor_map_2d(W1t, false, 64, (uint64_t)sh.N, 64 * 4, 64, kTmKB);
+    const CUtensorMap& tp = tensor_map_2d(p, false, (uint64_t)sh.Bp, (uint64_t)sh.N,
+                                          (uint64_t)sh.Bp * 4, (uint32_t)Bc, kTmKB);
+#define SM_L1T(BCV)                                                                             \
+  do {                                                                                          \
+    static bool attr = false;                                                                   \
+    if (!attr) {                                                                                \
+      SM_CUDA(cudaFuncSetAttribute(k_mlp_l1_tma<BCV>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                   tm_smem<BCV>()));                                            \
+      attr = true;                                                                              \
+    }                                                                                           \
+    k_mlp_l1_tma<BCV><<<grid, 192, tm_smem<BCV>(), s>>>(tw, tp, sh.N, sh.Bp, nsplit, z1_part);  \
+  } while (0)
+    if (Bc == 128) SM_L1T(128);
+    else if (Bc == 64) SM_L1T(64);
+    else SM_L1T(32);
+#undef SM_L1T
+    SM_LAUNCH_CHECK();
+  } else {
 #define SM_L1(BCV)                                                                              \
   do {                                                                                          \
     constexpr int smem = tc_stages<BCV>() * (128 * kTcKB * 4 + kTcKB * 2 * BCV * 4) + 1024;     \
@@ -433,6 +675,7 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
   else SM_L1(32);
 #undef SM_L1
   SM_LAUNCH_CHECK();
+  }
   k_mlp_reduce<<<(H1 * sh.Bp + 255) / 256, 256, 0, s>>>(sh.Bp, H1, nsplit, b1, z1_part, z1);
   SM_LAUNCH_CHECK();
   k_mlp_head<<<(sh.Bp + 127) / 128, 128, 0, s>>>(sh.Bp, H1, H2, z1, W2, b2, W3, b3, f_mlp, gz1);

@@ -1165,46 +1165,10 @@ __global__ void __launch_bounds__(32 * kRtWarps, SMOOTHE_RT_CTAS) k_sweep_revers
   }
 }
 
-// Tensor maps of the [M][Bp] rows the TMA reverse sweep gathers (box: one
-// 128-seed row), encoded on the host once per (pointer, shape) through the
-// driver entry point (the library links the static runtime only).
+// Tensor map of the [M][Bp] rows the TMA reverse sweep gathers (box: one
+// 128-seed row)
 static const CUtensorMap& row_map(const void* base, int M, int Bp, bool is_int) {
-  struct Key {
-    const void* p;
-    int M, Bp, i;
-    bool operator==(const Key& o) const { return p == o.p && M == o.M && Bp == o.Bp && i == o.i; }
-  };
-  static std::mutex mu;
-  static std::vector<std::pair<Key, CUtensorMap>> cache;
-  typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
-                               const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
-                               const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
-                               CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-  static EncodeFn encode = nullptr;
-  std::lock_guard<std::mutex> lk(mu);
-  const Key key{base, M, Bp, is_int ? 1 : 0};
-  for (auto& e : cache)
-    if (e.first == key) return e.second;
-  if (!encode) {
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    SM_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
-    SM_REQUIRE(fn && q == cudaDriverEntryPointSuccess, SMOOTHE_E_CUDA,
-               "cuTensorMapEncodeTiled unavailable");
-    encode = (EncodeFn)fn;
-  }
-  CUtensorMap m;
-  const cuuint64_t dims[2] = {(cuuint64_t)Bp, (cuuint64_t)M};
-  const cuuint64_t strides[1] = {(cuuint64_t)Bp * 4};
-  const cuuint32_t box[2] = {128, 1}, es[2] = {1, 1};
-  const CUresult r = encode(&m, is_int ? CU_TENSOR_MAP_DATA_TYPE_INT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
-                            2, const_cast<void*>(base), dims, strides, box, es,
-                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  SM_REQUIRE(r == CUDA_SUCCESS, SMOOTHE_E_CUDA, "cuTensorMapEncodeTiled failed");
-  if (cache.size() > 256) cache.erase(cache.begin());
-  cache.push_back({key, m});
-  return cache.back().second;
+  return tensor_map_2d(base, is_int, (uint64_t)Bp, (uint64_t)M, (uint64_t)Bp * 4, 128, 1);
 }
 
 // Opt-in (SMOOTHE_REV_TMA=1): measured slower than the register kernel on C4

@@ -239,6 +239,7 @@ struct smoothe_run {
   double* u_d = nullptr;
   int32_t *q_ptr = nullptr, *q_nbr = nullptr;
   float* q_w = nullptr;
+  float* W1t = nullptr;  // W1^T [N][64]
   float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr, *W3 = nullptr, *b3 = nullptr;
   float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *z1 = nullptr,
         *gz1 = nullptr;
@@ -380,7 +381,7 @@ void enqueue_decode(smoothe_run* r, cudaStream_t ds, PhaseMarks* pm) {
     dextra = r->dextra;
   } else if (r->cost_kind == SMOOTHE_COST_MLP) {
     launch_decode_s(ds, sh, g, r->sel, r->reach, r->sbin);
-    launch_mlp_fwd(ds, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
+    launch_mlp_fwd(ds, sh, r->H1, r->H2, r->W1, r->W1t, r->b1, r->W2, r->b2, r->W3, r->b3, r->sbin,
                    z1p, z1, r->dextra, nullptr, r->nsplit);
     dextra = r->dextra;
   }
@@ -449,7 +450,7 @@ void enqueue_step(smoothe_run* r) {
   } else {
     launch_materialize_p_f(s, sh, g, r->u_f, r->cp, qK, r->p, r->f_part);
     launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0, r->red_scratch);
-    launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
+    launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->W1t, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
                    r->z1_part, r->z1, r->fextra, r->gz1, r->nsplit);
     launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
     launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
@@ -787,6 +788,12 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   if (r->cost_kind == SMOOTHE_COST_MLP) {
     const int H1 = r->H1, H2 = r->H2;
     r->W1 = upload(o, std::vector<float>(cost->W1, cost->W1 + (size_t)H1 * sh.N));
+    {  // W1^T [N][64] (zero-padded hidden units): the TMA layer-1 kernel's K-contiguous tiles
+      std::vector<float> t((size_t)sh.N * 64, 0.f);
+      for (int h = 0; h < H1; ++h)
+        for (int k = 0; k < sh.N; ++k) t[(size_t)k * 64 + h] = cost->W1[(size_t)h * sh.N + k];
+      r->W1t = upload(o, t);
+    }
     r->b1 = upload(o, std::vector<float>(cost->b1, cost->b1 + H1));
     r->W2 = upload(o, std::vector<float>(cost->W2, cost->W2 + (size_t)H2 * H1));
     r->b2 = upload(o, std::vector<float>(cost->b2, cost->b2 + H2));
