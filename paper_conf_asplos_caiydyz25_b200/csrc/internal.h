@@ -335,7 +335,7 @@ int64_t& launch_counter();
 
 // 2-D tensor map (tma.cu): dims {inner, outer} elements of fp32 / int32,
 // rows row_bytes apart, box {box_inner, box_outer}; cached
-const CUtensorMap& tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
-                                 uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
+CUtensorMap tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
+                          uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
 
 }  // namespace smoothe

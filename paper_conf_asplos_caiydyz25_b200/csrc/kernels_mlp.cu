@@ -185,6 +185,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
       asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&bar[kTcStages])));
   }
   mbar_wait(&bar[kTcStages], 0);
+  __syncwarp();  // lanes leave the wait loop separately: converge before .sync.aligned tcgen05 ops
   asm volatile("tcgen05.fence::after_thread_sync;");
   // warp w reads TMEM lanes 32w..32w+31 = D rows; thread = one row
   const int row = warp * 32 + lane;
@@ -220,8 +221,10 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0)
+  if (warp == 0) {
+    __syncwarp();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -401,6 +404,7 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
       }
     }
     mbar_wait(&acc_full, 0);
+    __syncwarp();  // lanes leave the wait loop separately: converge before .sync.aligned tcgen05 ops
     asm volatile("tcgen05.fence::after_thread_sync;");
     const int q = warp % 4;  // TMEM lanes 32q .. 32q + 31 = D rows
     const int row = q * 32 + lane;
@@ -437,8 +441,10 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0)
+  if (warp == 0) {
+    __syncwarp();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+  }
 }
 
 // z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h
@@ -591,6 +597,7 @@ __global__ void __launch_bounds__(kTcThreads) k_mlp_l1_back_tc(int N, int Bp, in
         smem_u32(&bar)));
   }
   mbar_wait(&bar, 0);
+  __syncwarp();  // lanes leave the wait loop separately: converge before .sync.aligned tcgen05 ops
   asm volatile("tcgen05.fence::after_thread_sync;");
   const int m = warp * 32 + lane, k = k0 + m;
   const float uk = k < N ? __ldg(u + k) : 0.f;
@@ -624,8 +631,10 @@ __global__ void __launch_bounds__(kTcThreads) k_mlp_l1_back_tc(int N, int Bp, in
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0)
+  if (warp == 0) {
+    __syncwarp();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+  }
 }
 
 int mlp_nsplit(int device) { return num_sms(device); }
@@ -640,8 +649,8 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
   const char* tenv = std::getenv("SMOOTHE_MLP_TMA");
   const bool tma = !(tenv && tenv[0] == '0') && W1t;
   if (tma) {
-    const CUtensorMap& tw = tensor_map_2d(W1t, false, 64, (uint64_t)sh.N, 64 * 4, 64, kTmKB);
-    const CUtensorMap& tp = tensor_map_2d(p, false, (uint64_t)sh.Bp, (uint64_t)sh.N,
+    const CUtensorMap tw = tensor_map_2d(W1t, false, 64, (uint64_t)sh.N, 64 * 4, 64, kTmKB);
+    const CUtensorMap tp = tensor_map_2d(p, false, (uint64_t)sh.Bp, (uint64_t)sh.N,
                                           (uint64_t)sh.Bp * 4, (uint32_t)Bc, kTmKB);
 #define SM_L1T(BCV)                                                                             \
   do {                                                                                          \

@@ -386,6 +386,7 @@ __global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
         smem_u32(&bar[kBtStages])));
   mbar_wait(&bar[kBtStages], 0);
+  __syncwarp();  // lanes leave the wait loop separately: converge before .sync.aligned tcgen05 ops
   asm volatile("tcgen05.fence::after_thread_sync;");
   // warp w holds D rows 32w..32w+31: warps 2, 3 (the A_lo rows) hand their
   // (lo*hi + lo*lo) to warps 0, 1 through shared memory (the stages are idle)
@@ -432,7 +433,10 @@ __global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(128));
+  if (warp == 0) {
+    __syncwarp();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(128));
+  }
 }
 
 __global__ void __launch_bounds__(256) k_big_abar_f(

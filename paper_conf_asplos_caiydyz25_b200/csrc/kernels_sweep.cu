@@ -1167,7 +1167,7 @@ __global__ void __launch_bounds__(32 * kRtWarps, SMOOTHE_RT_CTAS) k_sweep_revers
 
 // Tensor map of the [M][Bp] rows the TMA reverse sweep gathers (box: one
 // 128-seed row)
-static const CUtensorMap& row_map(const void* base, int M, int Bp, bool is_int) {
+static CUtensorMap row_map(const void* base, int M, int Bp, bool is_int) {
   return tensor_map_2d(base, is_int, (uint64_t)Bp, (uint64_t)M, (uint64_t)Bp * 4, 128, 1);
 }
 
@@ -1194,9 +1194,9 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   const bool l2_prefetch = (double)sh.N * sh.Bp * sizeof(float) > 64e6;
   if (V == 4 && !lastchg && cursor && reverse_tma_enabled()) {
     const bool HI = a.wI != 0.f, HC = a.wC != 0.f;
-    const CUtensorMap& mg = row_map(gq, sh.M, sh.Bp, false);
-    const CUtensorMap& mp = row_map(HI ? (const void*)pi : (const void*)gq, sh.M, sh.Bp, false);
-    const CUtensorMap& ma = row_map(HC ? (const void*)am : (const void*)gq, sh.M, sh.Bp, true);
+    const CUtensorMap mg = row_map(gq, sh.M, sh.Bp, false);
+    const CUtensorMap mp = row_map(HI ? (const void*)pi : (const void*)gq, sh.M, sh.Bp, false);
+    const CUtensorMap ma = row_map(HC ? (const void*)am : (const void*)gq, sh.M, sh.Bp, true);
     int dev = 0;
     SM_CUDA(cudaGetDevice(&dev));
     const dim3 grid(SMOOTHE_RT_CTAS * num_sms(dev), sh.Bp / 128);

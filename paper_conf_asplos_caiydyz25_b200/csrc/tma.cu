@@ -11,8 +11,11 @@
 
 namespace smoothe {
 
-const CUtensorMap& tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
-                                 uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer) {
+// Returned by value: the cache is a growing vector, so a reference into it
+// would dangle as soon as a later call adds an entry (a second map encoded
+// for the same launch corrupted the first one's copy: illegal instruction).
+CUtensorMap tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
+                          uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer) {
   struct Entry {
     const void* p;
     bool i;
