@@ -434,6 +434,38 @@ void enqueue_step(smoothe_run* r) {
     launch_sweep_forward(s, sh, g, r->agg, t, r->sw, r->cp);
     kmark(0, 1);
   }
+  if (r->profiling && std::getenv("SMOOTHE_FREEZE_STATS")) {
+    // diagnostic (stderr): per class the last forward sweep that recomputed
+    // it, and F_i = the first reverse sweep (going down) at which class i's
+    // reverse item no longer sees final rows: max(last(i) + 1, max_j last(j))
+    std::vector<int32_t> ln(K + 2);
+    std::vector<int4> lst((size_t)(K + 1) * sh.M);
+    SM_CUDA(cudaMemcpyAsync(ln.data(), r->sw.list_n, sizeof(int32_t) * ln.size(), cudaMemcpyDeviceToHost, s));
+    SM_CUDA(cudaMemcpyAsync(lst.data(), r->sw.list, sizeof(int4) * lst.size(), cudaMemcpyDeviceToHost, s));
+    SM_CUDA(cudaStreamSynchronize(s));
+    std::vector<int32_t> last(sh.M, 0);
+    for (int t = 1; t <= K; ++t)
+      for (int i = 0; i < ln[t]; ++i) last[lst[(size_t)t * sh.M + i].x] = t;
+    std::vector<int64_t> hist(K + 2, 0), lasth(K + 2, 0);
+    int64_t items_plain = 0;
+    for (int j = 0; j < sh.M; ++j) {
+      int F = last[j] + 1;
+      for (int c = hg.cls_child_ptr[j]; c < hg.cls_child_ptr[j + 1]; ++c)
+        F = std::max(F, last[hg.cls_child[c]]);
+      F = std::min(F, K + 1);
+      hist[F]++;
+      lasth[last[j]]++;
+      items_plain += F - 1;  // reverse sweeps t < F_i
+    }
+    int64_t seedf = 0;
+    for (int t = 0; t <= K; ++t) if (ln[t] > 0) seedf = t;
+    std::fprintf(stderr, "[freeze] K=%d last recompute sweep (any class) %lld; mean F %.2f; "
+                 "plain (class,sweep) pairs %.3f of K*M\n", K, (long long)seedf,
+                 (double)items_plain / sh.M + 1.0, (double)items_plain / ((double)K * sh.M));
+    std::fprintf(stderr, "[freeze] F histogram (F: classes):");
+    for (int t = 0; t <= K + 1; ++t) if (hist[t]) std::fprintf(stderr, " %d:%lld", t, (long long)hist[t]);
+    std::fprintf(stderr, "\n");
+  }
 
   pm.mark(SMOOTHE_PHASE_COST);
   const float* qK = r->sw.qbuf[K & 1];

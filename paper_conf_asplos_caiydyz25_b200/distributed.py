@@ -44,7 +44,7 @@ def global_best(run, dist=None, device=None):
     best_step, best_seed, time_to_best_s, owner and choice (numpy int32 [M])."""
     choice, s = run.extract()
     cost = s["best_cost"] if s["valid"] else math.inf
-    if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
+    if dist is None or not dist.is_initialized():
         return {"best_cost": cost, "best_step": s["best_step"], "best_seed": s["best_seed"],
                 "time_to_best_s": s["time_to_best_s"], "owner": 0, "choice": choice}
     import torch
@@ -74,7 +74,7 @@ def _gather_best(run, dist, device, extra=0.0):
     s = run.summary()
     cost = s["best_cost"] if s["valid"] else math.inf
     rec = (cost, float(s["best_step"]), float(s["best_seed"]), float(extra))
-    if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
+    if dist is None or not dist.is_initialized():
         return [rec + (0.0,)]
     import torch
     mine = torch.tensor(rec + (float(dist.get_rank()),), dtype=torch.float64, device=device)
