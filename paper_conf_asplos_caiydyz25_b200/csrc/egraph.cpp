@@ -10,6 +10,9 @@
 #include <algorithm>
 #include <cstring>
 
+#include <exception>
+#include <thread>
+
 #include "internal.h"
 
 namespace {
@@ -230,6 +233,14 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   g.cls_child_ptr = sptr;
   g.cls_child = sadj;
   lt("scc");
+  // The analysis below runs in two threads: (A) hmax, components, penalty
+  // slots, K_auto and the decode levels; (B, this thread) padded layouts,
+  // class edges, dmin and the padded parent lists.  They write disjoint
+  // fields of g and only read the CSR / CSC arrays built above; the reverse
+  // items need both (hmax, dmin) and run after the join.
+  std::exception_ptr thread_error;
+  std::thread thread_a([&]() {
+    try {
   // hmax_j: the longest walk from class j in the class graph, i.e. the
   // largest L with g_q^{K-L}_j possibly non-zero in the reverse sweeps
   // (INT32_MAX when j can reach a cycle).  Kahn's algorithm on out-degrees:
@@ -302,7 +313,6 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
       g.scc_class[fill[s]++] = j;
     }
   }
-  lt("hmax+scc lists");
   // Abar entries and penalty slots per component
   g.ent_ptr.assign(1, 0);
   g.ent_node_ptr.assign(1, 0);
@@ -354,7 +364,6 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   }
   g.K_auto = k_auto(g, sptr, sadj, comp);
 
-  lt("abar slots+k_auto");
   // decode schedule: condensation levels reachable from the root (Kahn order)
   {
     std::vector<int32_t> cptr, cadj;
@@ -410,7 +419,17 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     }
   }
 
-  lt("decode levels");
+    } catch (...) {
+      thread_error = std::current_exception();
+    }
+  });
+  struct Joiner {
+    std::thread& t;
+    ~Joiner() {
+      if (t.joinable()) t.join();
+    }
+  } joiner{thread_a};
+
   // padded sweep layouts (multiples of 4 entries per list)
   g.pad_child_ptr.assign(N + 1, 0);
   for (int32_t i = 0; i < N; ++i) {
@@ -506,6 +525,22 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
   });
 
   lt("dmin");
+  // pad parents (thread B) before the join
+  g.pad_par_ptr.assign(M + 1, 0);
+  for (int32_t j = 0; j < M; ++j) {
+    const int32_t n = g.par_ptr[j + 1] - g.par_ptr[j];
+    g.pad_par_ptr[j + 1] = g.pad_par_ptr[j] + ((n + 3) & ~3);
+  }
+  g.pad_par.resize(2 * (size_t)g.pad_par_ptr[M]);
+  for (int32_t j = 0; j < M; ++j)
+    for (int32_t s = g.pad_par_ptr[j], e = g.par_ptr[j]; s < g.pad_par_ptr[j + 1]; ++s, ++e) {
+      const bool real = e < g.par_ptr[j + 1];
+      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
+      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
+    }
+  thread_a.join();
+  if (thread_error) std::rethrow_exception(thread_error);
+  lt("join (components, levels)");
   // reverse-sweep work items: runs of <= kRevChunk batches of one class, cut at
   // e-node boundaries; an e-node with more batches is cut into pieces of its own
   {
@@ -556,20 +591,7 @@ void build_host_graph(int32_t M, int32_t N, const int32_t* class_ptr, const int6
     }
     g.rev_class_item_ptr[j + 1] = g.rev_class_item_ptr[j] + n;
   }
-
-  g.pad_par_ptr.assign(M + 1, 0);
-  for (int32_t j = 0; j < M; ++j) {
-    const int32_t n = g.par_ptr[j + 1] - g.par_ptr[j];
-    g.pad_par_ptr[j + 1] = g.pad_par_ptr[j] + ((n + 3) & ~3);
-  }
-  g.pad_par.resize(2 * (size_t)g.pad_par_ptr[M]);
-  for (int32_t j = 0; j < M; ++j)
-    for (int32_t s = g.pad_par_ptr[j], e = g.par_ptr[j]; s < g.pad_par_ptr[j + 1]; ++s, ++e) {
-      const bool real = e < g.par_ptr[j + 1];
-      g.pad_par[2 * (size_t)s] = real ? g.par_node[e] : N;
-      g.pad_par[2 * (size_t)s + 1] = real ? g.par_class[e] : root;
-    }
-  lt("rev items+pad parents");
+  lt("rev items");
 }
 
 }  // namespace smoothe

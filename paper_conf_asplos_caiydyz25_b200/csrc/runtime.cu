@@ -916,11 +916,13 @@ smoothe_status smoothe_load_egraph(int32_t num_classes, int32_t num_nodes, const
       SM_CUDA(cudaGetDeviceCount(&ndev));
       SM_REQUIRE(device_ordinal < ndev, SMOOTHE_E_INVALID_ARG, "device ordinal out of range");
       SM_CUDA(cudaSetDevice(device_ordinal));
-      cudaDeviceProp prop;
-      SM_CUDA(cudaGetDeviceProperties(&prop, device_ordinal));
-      SM_REQUIRE(prop.major == 10, SMOOTHE_E_CUDA,
-                 "libsmoothe is built for sm_100a; device has sm_" + std::to_string(prop.major) +
-                     std::to_string(prop.minor));
+      // (two attribute queries: cudaGetDeviceProperties took ~150 ms of the load)
+      int major = 0, minor = 0;
+      SM_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device_ordinal));
+      SM_CUDA(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device_ordinal));
+      SM_REQUIRE(major == 10, SMOOTHE_E_CUDA,
+                 "libsmoothe is built for sm_100a; device has sm_" + std::to_string(major) +
+                     std::to_string(minor));
       lap("device query");
       const HostGraph& h = g->host;
       DevGraph& d = g->dev;
