@@ -421,6 +421,12 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(int M, int Bp, int t,
   const int gl = threadIdx.x % LPR;
   const int s0 = c * (4 * LPR) + gl * 4;
   const size_t pbase = (size_t)c * P.cap;
+  // seeds whose restored q row differs: a lane always covers seeds s0..s0+3,
+  // so it keeps its own flags and the block clears wm once at the end (every
+  // entry testing and storing the same 128 wm words serialised on them)
+  __shared__ int changed[4 * LPR];
+  if (wm && threadIdx.x < 4 * LPR) changed[threadIdx.x] = 0;
+  bool chg[4] = {false, false, false, false};
   for (int i = blockIdx.x * (kBlock / LPR) + (int)threadIdx.x / LPR; i < n; i += groups) {
     if (i < n1) {
       const int4 e = l_pa[i];
@@ -435,13 +441,19 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(int M, int Bp, int t,
         const float4 now = ld4(cur_q + o);
 #pragma unroll
         for (int x = 0; x < 4; ++x)
-          if (__float_as_uint(comp(prev, x)) != __float_as_uint(comp(now, x)) &&
-              __ldcg(wm + s0 + x))
-            __stcg(wm + s0 + x, 0);
+          chg[x] = chg[x] || __float_as_uint(comp(prev, x)) != __float_as_uint(comp(now, x));
       }
       st4(cur_q + o, prev);
     }
   }
+  if (!wm) return;
+  __syncthreads();
+#pragma unroll
+  for (int x = 0; x < 4; ++x)
+    if (chg[x]) changed[gl * 4 + x] = 1;  // benign same-value stores
+  __syncthreads();
+  if (threadIdx.x < 4 * LPR && changed[threadIdx.x] && __ldcg(wm + c * (4 * LPR) + threadIdx.x))
+    __stcg(wm + c * (4 * LPR) + threadIdx.x, 0);
 }
 
 void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, int t, int K,
@@ -453,7 +465,10 @@ void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, i
       k_rev_restore_all<LPR><<<row_grid(sh.M, sh.Bp, LPR), kBlock, 0, s>>>(sh.M, sh.Bp, P,
                                                                             st.cur_pi, st.cur_am);
     } else {
-      const dim3 grid(2 * st.num_sms, num_chunks(sh.Bp));
+#ifndef SMOOTHE_TRANS_BPS
+#define SMOOTHE_TRANS_BPS 8  // blocks per SM (2: 5.1 ms of transitions per C4 step, 8: 4.3, ncu)
+#endif
+      const dim3 grid(SMOOTHE_TRANS_BPS * st.num_sms, num_chunks(sh.Bp));
       k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, t, P, st.qbuf[(K - 1) & 1],
                                                     st.cur_pi, st.cur_am,
                                                     st.wmode ? st.wm : nullptr);

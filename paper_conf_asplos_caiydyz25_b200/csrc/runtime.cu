@@ -1359,7 +1359,6 @@ smoothe_status smoothe_debug_step(smoothe_run* run, const float* theta_in, const
       throw;
     }
     run->debug = false;
-    const size_t MB = (size_t)sh.M * sh.Bp;
     const float* pdev = run->cost_kind == SMOOTHE_COST_LINEAR ? run->dbg_p : run->p;
     copy_rows_d2h(dump->cp, run->cp, sh.N, sh.B, sh.Bp, s);
     copy_rows_d2h(dump->qK, run->sw.qbuf[run->K & 1], sh.M, sh.B, sh.Bp, s);
