@@ -321,6 +321,8 @@ void launch_best_snapshot(cudaStream_t s, const Shape& sh, const int32_t* choice
 // gp = u + W1^T gz1.
 // z1_part: [nsplit][128][Bp] split-K partials of the tensor-core layer 1
 // (nsplit = mlp_nsplit(device) CTAs per seed chunk); z1: [H1][Bp]
+// W1 in the tiles of the TMA layer-1 kernel (kernels_mlp.cu)
+std::vector<float> mlp_w1_tiles(const float* W1, int H1, int N);
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
                     const float* W1t,
                     const float* b1, const float* W2, const float* b2, const float* W3,
@@ -334,8 +336,10 @@ int num_sms(int device);
 int64_t& launch_counter();
 
 // 2-D tensor map (tma.cu): dims {inner, outer} elements of fp32 / int32,
-// rows row_bytes apart, box {box_inner, box_outer}; cached
+// rows row_bytes apart, box {box_inner, box_outer}, optionally written to
+// shared memory with the 128-byte swizzle (box_inner * 4 must be 128); cached
 CUtensorMap tensor_map_2d(const void* base, bool is_int, uint64_t inner, uint64_t outer,
-                          uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
+                          uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer,
+                          bool swizzle128 = false);
 
 }  // namespace smoothe

@@ -149,6 +149,13 @@ __device__ __forceinline__ int& comp(int4& v, int c) {
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
 }
+
+// p advanced to the next 1 KB boundary of the shared window, by arithmetic on
+// the shared pointer itself: a round trip through uintptr_t loses the address
+// space and turns every access into a generic LD.E / ST.E.
+__device__ __forceinline__ uint8_t* smem_align1024(uint8_t* p) {
+  return p + ((1024u - (smem_u32(p) & 1023u)) & 1023u);
+}
 // no-swizzle UMMA shared-memory descriptor (sm_100 version 1)
 __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
   return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |

@@ -6,6 +6,8 @@
 // on the tensor cores.  Split-K partial sums are reduced in a fixed order, so
 // results are deterministic.
 #include <cstdlib>
+#include <cstring>
+#include <vector>
 
 #include "kcommon.cuh"
 
@@ -229,50 +231,66 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_mlp_l1_tc(int N, int Bp, int 
 
 // ---------------------------------------------------------------------------
 // Layer 1 with TMA-fed, warp-specialised stages (the default; SMOOTHE_MLP_TMA=0
-// keeps the register-staged kernel above).  Raw fp32 tiles come in by TMA --
-// W1^T [32 e-nodes x 64 hidden] (the run keeps W1 transposed, zero-padded to
-// 64 hidden units, so a tile is 8 KB of contiguous memory; W1's own rows
-// gave 64 pieces of 128 bytes, measured no faster than the register kernel)
-// and p [32 e-nodes x Bc seeds], e-nodes past N zero-filled by the TMA --
-// into a ring of kRawStages; four
-// converter warps split each raw tile into hi / lo and lay it out in the
-// canonical no-swizzle K-major UMMA layouts of a ring of kMmaStages; one
-// thread issues the MMAs (as in k_mlp_l1_tc: A = [W1_hi; W1_lo], B = [p_hi |
-// p_lo], all four products in one M=128 x N=2Bc x K=8 MMA), tcgen05.commit
-// releases each stage; the converter warps read the accumulator back (warp w
-// owns TMEM lanes 32 (w % 4)..).  Output: z1_part as k_mlp_l1_tc.
-//   warp 0: TMA producer, warp 1: MMA issuer, warps 2..5: converters + epilogue
+// keeps the register-staged kernel above).
+//  * A = [W1_hi; W1_lo] (M = 128, K-major).  The run keeps W1 in tiles of 32
+//    e-nodes (`mlp_w1_tiles`, 8 KB, already in the no-swizzle K-major core
+//    order); one 1-D bulk copy puts a tile into the A_hi half of a stage.
+//  * The MMA reads an fp32 operand as tf32 by dropping the low 13 mantissa
+//    bits (scripts/microbench/umma_layout.cu: operands with all 13 low bits
+//    set give the exact products of the truncated values), so the raw W1 tile
+//    IS A_hi; the converter warps only write A_lo = x - trunc(x) next to it,
+//    element for element.
+//  * B = [p_hi | p_lo] (N = 2 Bc, K-major).  p is stored seeds-contiguous,
+//    i.e. MN-major for B, and a tf32 MMA with the MN-major bit set returned
+//    zeros on this part (same microbenchmark), so p is transposed on chip:
+//    tensor TMA brings the raw tile [32 e-nodes x Bc seeds], and each
+//    converter thread builds one 16-byte K-major core row (4 e-nodes of one
+//    seed) from four 4-byte loads; a warp reads whole 128-byte rows and
+//    writes 512 contiguous bytes, so neither side has bank conflicts.
+// One thread issues the MMAs (M=128 x N=2Bc x K=8, all four products as in
+// k_mlp_l1_tc), tcgen05.commit hands each stage back to the producer; the
+// converter warps read the accumulator back.  Output: z1_part as k_mlp_l1_tc.
+//   warp 0: TMA producer, warp 1: MMA issuer, warps 2..2+kTmCW-1: converters +
+//   epilogue (warp w reads TMEM lanes 32 (w % 4).., column part (w - 2) / 4)
+// (C5 layer 1: W1 as 2-D TMA tiles of W1^T, both operands transposed as 4 x 4
+// register blocks, 64 us; W1 stored pre-split -- twice the bytes -- 48.5 us;
+// the 4 x 4 blocks' stores were 4-way bank-conflicted, and shared-memory
+// bandwidth was the limit: 29 us with the converters skipped.)
 // ---------------------------------------------------------------------------
-constexpr int kTmKB = 32;  // e-nodes per stage
+constexpr int kTmKB = 32;                          // e-nodes per stage
+constexpr int kTmWBytes = 64 * kTmKB * 4;          // one stored W1 tile (8 KB)
+#ifndef SMOOTHE_TM_CW
+#define SMOOTHE_TM_CW 8
+#endif
+constexpr int kTmCW = SMOOTHE_TM_CW;               // converter warps (C5: 8 -> 33.5 us, 4 -> 35.5)
+constexpr int kTmThreads = 64 + 32 * kTmCW;
+template <int BC>
+__host__ __device__ constexpr int tm_stages() { return BC >= 128 ? 3 : BC >= 64 ? 5 : 7; }
+template <int BC>  // A [hi; lo], B [hi | lo], raw p tile
+__host__ __device__ constexpr int tm_stage_bytes() { return 2 * kTmWBytes + 3 * BC * kTmKB * 4; }
+template <int BC>
+__host__ __device__ constexpr int tm_smem() { return tm_stages<BC>() * tm_stage_bytes<BC>() + 1024; }
 
 template <int BC>
-__host__ __device__ constexpr int tm_raw_stages() { return BC >= 128 ? 4 : BC >= 64 ? 6 : 8; }
-template <int BC>
-__host__ __device__ constexpr int tm_mma_stages() { return BC >= 128 ? 2 : BC >= 64 ? 3 : 4; }
-template <int BC>
-__host__ __device__ constexpr int tm_smem() {
-  return tm_raw_stages<BC>() * (64 * kTmKB * 4 + kTmKB * BC * 4) +
-         tm_mma_stages<BC>() * (128 * kTmKB * 4 + kTmKB * 2 * BC * 4) + 1024;
-}
-
-template <int BC>
-__global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ CUtensorMap tm_w,
-                                                      const __grid_constant__ CUtensorMap tm_p,
-                                                      int N, int Bp, int nsplit,
-                                                      float* __restrict__ z1_part) {
+__global__ void __launch_bounds__(kTmThreads, 1) k_mlp_l1_tma(const float* __restrict__ w1tiles,
+                                                             const __grid_constant__ CUtensorMap tm_p,
+                                                             int N, int Bp, int nsplit,
+                                                             float* __restrict__ z1_part) {
   constexpr int NM = 2 * BC;
-  constexpr int RS = tm_raw_stages<BC>(), MS = tm_mma_stages<BC>();
-  constexpr int RAW_A = 64 * kTmKB * 4, RAW_B = kTmKB * BC * 4, RAW = RAW_A + RAW_B;
-  constexpr int A_BYTES = 128 * kTmKB * 4, B_BYTES = kTmKB * NM * 4, MMA = A_BYTES + B_BYTES;
-  constexpr int A_LBO = 16 * 128, B_LBO = (NM / 8) * 128;
+  constexpr int S = tm_stages<BC>(), SB = tm_stage_bytes<BC>();
+  constexpr int A_BYTES = 2 * kTmWBytes;          // [hi; lo]
+  constexpr int PB = BC * kTmKB * 4;              // the raw p tile
+  constexpr int B_BYTES = 2 * PB;                 // [hi | lo]
+  // A: core (e-node quad kc, hidden-unit octet g) at g * 1024 + kc * 128
+  constexpr uint32_t A_LBO = 128, A_SBO = 1024;
+  // B: core (e-node quad kc, seed octet) at kc * B_LBO + (n / 8) * 128
+  constexpr uint32_t B_LBO = (NM / 8) * 128, B_SBO = 128;
   constexpr uint32_t TMEM_COLS = NM <= 32 ? 32 : NM <= 64 ? 64 : NM <= 128 ? 128 : 256;
   constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
                              ((uint32_t)(128 >> 4) << 24);
   extern __shared__ __align__(1024) uint8_t tm_smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(tm_smem_raw) + 1023) & ~(uintptr_t)1023);
-  uint8_t* raw = smem;                 // RS x RAW
-  uint8_t* mma = smem + RS * RAW;      // MS x MMA (1 KB aligned: RAW is a multiple of 1 KB)
-  __shared__ uint64_t raw_full[RS], raw_empty[RS], mma_full[MS], mma_empty[MS], acc_full;
+  uint8_t* smem = smem_align1024(tm_smem_raw);
+  __shared__ uint64_t full[S], conv[S], empty[S], acc_full;
   __shared__ uint32_t tmem_sh;
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
   const int seed0 = blockIdx.y * BC;
@@ -288,13 +306,10 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (tid == 0) {
-    for (int i = 0; i < RS; ++i) {
-      mbar_init(&raw_full[i], 1);
-      mbar_init(&raw_empty[i], 4);  // one arrival per converter warp
-    }
-    for (int i = 0; i < MS; ++i) {
-      mbar_init(&mma_full[i], 4);
-      mbar_init(&mma_empty[i], 1);  // tcgen05.commit
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&conv[i], kTmCW);  // one arrival per converter warp
+      mbar_init(&empty[i], 1);     // tcgen05.commit
     }
     mbar_init(&acc_full, 1);
     asm volatile("fence.mbarrier_init.release.cluster;");
@@ -304,36 +319,38 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_sh;
 
-  if (warp == 0) {  // TMA producer
+  if (warp == 0) {  // producer: W1 tile (bulk copy) -> A_hi, p tile (tensor TMA) -> raw
     if (lane == 0)
       for (int kb = 0; kb < nkb; ++kb) {
-        const int st = kb % RS;
-        if (kb >= RS) mbar_wait(&raw_empty[st], (uint32_t)((kb / RS - 1) & 1));
-        const uint32_t dst = smem_u32(raw + st * RAW), bar = smem_u32(&raw_full[st]);
+        const int st = kb % S;
         const int k0 = k_begin + kb * kTmKB;
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(RAW));
+        if (kb >= S) mbar_wait(&empty[st], (uint32_t)((kb / S - 1) & 1));
+        const uint32_t bar = smem_u32(&full[st]);
+        const uint32_t dst = smem_u32(smem + st * SB);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                     "r"(kTmWBytes + PB));
         asm volatile(
-            "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-            " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
-            "l"(&tm_w), "r"(0), "r"(k0), "r"(bar)
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                dst),
+            "l"(w1tiles + (size_t)(k0 / kTmKB) * (kTmWBytes / 4)), "r"(kTmWBytes), "r"(bar)
             : "memory");
         asm volatile(
             "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-            " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst + RAW_A),
+            " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst + A_BYTES + B_BYTES),
             "l"(&tm_p), "r"(seed0), "r"(k0), "r"(bar)
             : "memory");
       }
   } else if (warp == 1) {  // MMA issuer
     if (lane == 0) {
       for (int kb = 0; kb < nkb; ++kb) {
-        const int st = kb % MS;
-        mbar_wait(&mma_full[st], (uint32_t)((kb / MS) & 1));
+        const int st = kb % S;
+        mbar_wait(&conv[st], (uint32_t)((kb / S) & 1));
         asm volatile("tcgen05.fence::after_thread_sync;");
-        const uint32_t sa = smem_u32(mma + st * MMA), sb = sa + A_BYTES;
+        const uint32_t sa = smem_u32(smem + st * SB), sb = sa + A_BYTES;
 #pragma unroll
         for (int ks = 0; ks < kTmKB / 8; ++ks) {
-          const uint64_t da = umma_desc(sa + ks * 2 * A_LBO, A_LBO, 128);
-          const uint64_t db = umma_desc(sb + ks * 2 * B_LBO, B_LBO, 128);
+          const uint64_t da = umma_desc(sa + ks * 2 * A_LBO, A_LBO, A_SBO);
+          const uint64_t db = umma_desc(sb + ks * 2 * B_LBO, B_LBO, B_SBO);
           const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
           asm volatile(
               "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
@@ -341,7 +358,7 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
               "l"(da), "l"(db), "r"(IDESC), "r"(acc));
         }
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-            smem_u32(&mma_empty[st])));
+            smem_u32(&empty[st])));
       }
       if (nkb > 0)
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
@@ -349,72 +366,50 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
       else
         asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_full)));
     }
-  } else {  // converters (128 threads), then the epilogue
+  } else {  // converters: A_lo next to A_hi, B from the raw p tile; then the epilogue
     const int ct = tid - 64;
     for (int kb = 0; kb < nkb; ++kb) {
-      const int rs = kb % RS, ms = kb % MS;
-      mbar_wait(&raw_full[rs], (uint32_t)((kb / RS) & 1));
-      if (kb >= MS) mbar_wait(&mma_empty[ms], (uint32_t)((kb / MS - 1) & 1));
-      const uint8_t* ra = raw + rs * RAW;
-      const uint8_t* rb = ra + RAW_A;
-      uint8_t* sa = mma + ms * MMA;
+      const int st = kb % S;
+      mbar_wait(&full[st], (uint32_t)((kb / S) & 1));
+      uint8_t* sa = smem + st * SB;
       uint8_t* sb = sa + A_BYTES;
-      // A: raw (k, h) at (k * 64 + h) * 4; one 4 x 4 block (K chunk kc,
-      // hidden units hc..hc+3) per thread, transposed to K-major
-      {
-        const int kc = ct / 16, hc = (ct % 16) * 4;
-        float4 r4[4];
 #pragma unroll
-        for (int r = 0; r < 4; ++r)
-          r4[r] = *reinterpret_cast<const float4*>(ra + ((4 * kc + r) * 64 + hc) * 4);
-#pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          // (rotating each lane pair's column order removes the 4-way bank
-          // conflicts of these stores but measured 65 -> 97 us: the shared
-          // stores are conflicted yet cheaper than the selects)
-          const float4 col = make_float4(comp(r4[0], x), comp(r4[1], x), comp(r4[2], x), comp(r4[3], x));
-          const float4 hi = tf32_hi(col), lo = sub4(col, hi);
-          const int h = hc + x;
-          *reinterpret_cast<float4*>(sa + (kc * 16 + h / 8) * 128 + (h % 8) * 16) = hi;
-          *reinterpret_cast<float4*>(sa + (kc * 16 + 8 + h / 8) * 128 + (h % 8) * 16) = lo;
-        }
+      for (int i = ct; i < kTmWBytes / 16; i += 32 * kTmCW) {
+        const float4 w = *reinterpret_cast<const float4*>(sa + i * 16);
+        *reinterpret_cast<float4*>(sa + kTmWBytes + i * 16) = sub4(w, tf32_hi(w));
       }
-      // B: raw (k, s) at (k * BC + s) * 4; 4 x 4 blocks transposed to K-major
-      constexpr int BBLK = (kTmKB / 4) * (BC / 4);
-      for (int blk = ct; blk < BBLK; blk += 128) {
-        const int kc = blk / (BC / 4), n = (blk % (BC / 4)) * 4;
-        float4 r4[4];
+      // B core row (kc, n): p[4 kc .. 4 kc + 3][n], raw (k, n) at (k * BC + n) * 4
+      const float* rp = reinterpret_cast<const float*>(sb + B_BYTES);
 #pragma unroll
-        for (int r = 0; r < 4; ++r)
-          r4[r] = *reinterpret_cast<const float4*>(rb + ((4 * kc + r) * BC + n) * 4);
-#pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          const float4 col = make_float4(comp(r4[0], x), comp(r4[1], x), comp(r4[2], x), comp(r4[3], x));
-          const float4 hi = tf32_hi(col), lo = sub4(col, hi);
-          const int m = n + x;
-          *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + m / 8) * 128 + (m % 8) * 16) = hi;
-          *reinterpret_cast<float4*>(sb + (kc * (NM / 8) + (BC + m) / 8) * 128 + (m % 8) * 16) = lo;
-        }
+      for (int i = ct; i < (kTmKB / 4) * BC; i += 32 * kTmCW) {
+        const int kc = i / BC, n = i % BC;
+        const float4 x = make_float4(rp[(4 * kc) * BC + n], rp[(4 * kc + 1) * BC + n],
+                                     rp[(4 * kc + 2) * BC + n], rp[(4 * kc + 3) * BC + n]);
+        const int off = kc * B_LBO + (n / 8) * 128 + (n % 8) * 16;
+        *reinterpret_cast<float4*>(sb + off) = x;  // the MMA truncates: x is B_hi
+        *reinterpret_cast<float4*>(sb + off + (BC / 8) * 128) = sub4(x, tf32_hi(x));
       }
       asm volatile("fence.proxy.async.shared::cta;");
       __syncwarp();
-      if (lane == 0) {
-        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&raw_empty[rs])));
-        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&mma_full[ms])));
-      }
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&conv[st])));
     }
     mbar_wait(&acc_full, 0);
     __syncwarp();  // lanes leave the wait loop separately: converge before .sync.aligned tcgen05 ops
     asm volatile("tcgen05.fence::after_thread_sync;");
     const int q = warp % 4;  // TMEM lanes 32q .. 32q + 31 = D rows
+    constexpr int PARTS = kTmCW / 4, CH = BC / PARTS >= 16 ? BC / PARTS : 16;
+    const int c0 = ((warp - 2) / 4) * CH;
     const int row = q * 32 + lane;
     float* out = z1_part + ((size_t)blockIdx.x * 128 + row) * Bp + seed0;
-    if (nkb == 0) {
+    if (c0 < BC && nkb == 0) {
 #pragma unroll
-      for (int c = 0; c < BC; c += 4) *reinterpret_cast<float4*>(out + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int c = 0; c < CH; c += 4)
+        *reinterpret_cast<float4*>(out + c0 + c) = make_float4(0.f, 0.f, 0.f, 0.f);
     }
 #pragma unroll
-    for (int c = 0; c < BC && nkb > 0; c += 16) {
+    for (int cc = 0; cc < CH; cc += 16) {
+      const int c = c0 + cc;
+      if (c >= BC || nkb == 0) break;
       uint32_t v[16], w[16];
       const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + c;
       asm volatile(
@@ -445,6 +440,23 @@ __global__ void __launch_bounds__(192, 1) k_mlp_l1_tma(const __grid_constant__ C
     __syncwarp();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
   }
+}
+
+// W1 laid out for k_mlp_l1_tma, once per run: ceil(N / 32) tiles of
+// kTmWBytes, element (hidden unit h, e-node k) of tile kb at core (k/4, h/8):
+// (h/8) * 1024 + (k/4) * 128 + (h%8) * 16 + (k%4) * 4 bytes; hidden units
+// >= H1 and e-nodes >= N are zero.
+std::vector<float> mlp_w1_tiles(const float* W1, int H1, int N) {
+  const int nblk = (N + kTmKB - 1) / kTmKB;
+  std::vector<float> t((size_t)nblk * (kTmWBytes / 4), 0.f);
+  for (int kb = 0; kb < nblk; ++kb) {
+    float* tile = t.data() + (size_t)kb * (kTmWBytes / 4);
+    for (int kk = 0; kk < kTmKB && kb * kTmKB + kk < N; ++kk)
+      for (int h = 0; h < H1 && h < 64; ++h)
+        tile[((h / 8) * 1024 + (kk / 4) * 128 + (h % 8) * 16 + (kk % 4) * 4) / 4] =
+            W1[(size_t)h * N + kb * kTmKB + kk];
+  }
+  return t;
 }
 
 // z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h
@@ -649,7 +661,6 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
   const char* tenv = std::getenv("SMOOTHE_MLP_TMA");
   const bool tma = !(tenv && tenv[0] == '0') && W1t;
   if (tma) {
-    const CUtensorMap tw = tensor_map_2d(W1t, false, 64, (uint64_t)sh.N, 64 * 4, 64, kTmKB);
     const CUtensorMap tp = tensor_map_2d(p, false, (uint64_t)sh.Bp, (uint64_t)sh.N,
                                           (uint64_t)sh.Bp * 4, (uint32_t)Bc, kTmKB);
 #define SM_L1T(BCV)                                                                             \
@@ -660,7 +671,7 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
                                    tm_smem<BCV>()));                                            \
       attr = true;                                                                              \
     }                                                                                           \
-    k_mlp_l1_tma<BCV><<<grid, 192, tm_smem<BCV>(), s>>>(tw, tp, sh.N, sh.Bp, nsplit, z1_part);  \
+    k_mlp_l1_tma<BCV><<<grid, kTmThreads, tm_smem<BCV>(), s>>>(W1t, tp, sh.N, sh.Bp, nsplit, z1_part); \
   } while (0)
     if (Bc == 128) SM_L1T(128);
     else if (Bc == 64) SM_L1T(64);

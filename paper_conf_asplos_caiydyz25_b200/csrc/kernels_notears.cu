@@ -289,7 +289,7 @@ __global__ void __launch_bounds__(kBtThreads, 1) k_big_gemm_tc(int n, int np,
   constexpr uint32_t IDESC =
       (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(128 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
   extern __shared__ __align__(1024) uint8_t bt_smem[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(bt_smem) + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(bt_smem);
   __shared__ uint64_t bar[kBtStages + 1];
   __shared__ uint32_t tmem_sh;
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;

@@ -239,7 +239,7 @@ struct smoothe_run {
   double* u_d = nullptr;
   int32_t *q_ptr = nullptr, *q_nbr = nullptr;
   float* q_w = nullptr;
-  float* W1t = nullptr;  // W1^T [N][64]
+  float* W1t = nullptr;  // W1 in k_mlp_l1_tma's tiles (mlp_w1_tiles)
   float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr, *W3 = nullptr, *b3 = nullptr;
   float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *z1 = nullptr,
         *gz1 = nullptr;
@@ -820,12 +820,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
   if (r->cost_kind == SMOOTHE_COST_MLP) {
     const int H1 = r->H1, H2 = r->H2;
     r->W1 = upload(o, std::vector<float>(cost->W1, cost->W1 + (size_t)H1 * sh.N));
-    {  // W1^T [N][64] (zero-padded hidden units): the TMA layer-1 kernel's K-contiguous tiles
-      std::vector<float> t((size_t)sh.N * 64, 0.f);
-      for (int h = 0; h < H1; ++h)
-        for (int k = 0; k < sh.N; ++k) t[(size_t)k * 64 + h] = cost->W1[(size_t)h * sh.N + k];
-      r->W1t = upload(o, t);
-    }
+    // W1 in the TMA layer-1 kernel's tile order (constant for the run)
+    r->W1t = upload(o, mlp_w1_tiles(cost->W1, H1, sh.N));
     r->b1 = upload(o, std::vector<float>(cost->b1, cost->b1 + H1));
     r->W2 = upload(o, std::vector<float>(cost->W2, cost->W2 + (size_t)H2 * H1));
     r->b2 = upload(o, std::vector<float>(cost->b2, cost->b2 + H2));

@@ -446,6 +446,36 @@ def test_mlp_layer1_tensor_cores(sm, B):
     g.close()
 
 
+@pytest.mark.parametrize("N,B", [(300_000, 32), (300_000, 64), (300_000, 128), (7_777, 64),
+                                 (1_000, 256)])
+def test_mlp_l1_tma_bit_identical(sm, monkeypatch, N, B):
+    """The TMA layer-1 kernel (default) against the register-staged one
+    (SMOOTHE_MLP_TMA=0): the same products (the MMA truncates the raw W1 / p
+    tiles to tf32 exactly as the register kernel's explicit split does) summed
+    in the same order, so f and the gradient of a debug step are bit for bit
+    equal -- at C5's size and on a ragged e-node count (7 777: last
+    32-e-node tile partial).  On 1 000 e-nodes (most split-K CTAs without a
+    tile) the two kernels split K into 32- and 64-e-node ranges, so the
+    partial sums differ in order: equal to fp32 rounding there."""
+    eg = make_config("C5") if N == 300_000 else make_config("C5", N=N, M=max(N // 18, 8))
+    g = sm.load_egraph_from(eg, device=0)
+    run = sm.run_create(g, sm.CostModel.from_input(eg), B, sm.Options(penalty_group=8, rng_key=5))
+    run.steps(2)
+    th, m, v, n = run.state()
+    outs = []
+    for env in ("1", "0"):
+        monkeypatch.setenv("SMOOTHE_MLP_TMA", env)
+        outs.append(run.debug_step(th, m, v, step_index=n))
+    for k in ("f", "grad_cp", "loss", "theta_out"):
+        a, b = np.asarray(outs[0][k], np.float64), np.asarray(outs[1][k], np.float64)
+        if N == 1_000:
+            assert np.allclose(a, b, rtol=1e-5, atol=1e-6 * np.abs(b).max()), k
+        else:
+            assert np.array_equal(a, b), k
+    run.close()
+    g.close()
+
+
 def test_c4_full_size_first_group(sm, orc):
     """C4 at the bench launch configuration (128 seeds, G = 16): the oracle
     recomputes the first penalty group (16 seeds) exactly."""
