@@ -329,8 +329,10 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
                     const float* b3, const float* p, float* z1_part, float* z1, double* f_mlp,
                     float* gz1, int32_t nsplit);
 int mlp_nsplit(int device);
-void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* u,
-                    const float* gz1, float* gp);
+// W1^T in the tiles of the TMA layer-1 backward kernel (kernels_mlp.cu)
+std::vector<float> mlp_w1_back_tiles(const float* W1, int H1, int N);
+void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* W1b,
+                    const float* u, const float* gz1, float* gp, int32_t nsms);
 
 int num_sms(int device);
 int64_t& launch_counter();

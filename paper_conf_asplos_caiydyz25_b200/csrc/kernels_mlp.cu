@@ -649,6 +649,233 @@ __global__ void __launch_bounds__(kTcThreads) k_mlp_l1_back_tc(int N, int Bp, in
   }
 }
 
+// ---------------------------------------------------------------------------
+// Backward of layer 1, persistent and TMA-fed (the default; SMOOTHE_MLP_TMA=0
+// keeps k_mlp_l1_back_tc): the same products in the same order as
+// k_mlp_l1_back_tc, so g_p is bit for bit the same.  Per CTA: one seed chunk
+// and every gridDim.x-th tile of 128 e-nodes.
+//  * B = [gz1_hi | gz1_lo] (K = 64 hidden units) is built once per CTA and
+//    stays in shared memory.
+//  * A_hi = the W1^T tile, kept by the run in the K-major core order
+//    (`mlp_w1_back_tiles`, 32 KB per tile): one bulk copy, used raw (the MMA
+//    truncates to tf32); converter warps write A_lo = x - trunc(x) next to it.
+//  * The accumulator is double-buffered in TMEM, so the epilogue of tile i
+//    overlaps the MMAs of tile i + 1; the epilogue adds u, writes the tile
+//    into a 128-byte-swizzled staging buffer (conflict-free) and one thread
+//    stores it with tensor TMA (rows past N clipped).
+//   warp 0: producer, warp 1: MMA issuer, warps 2-5: converters, warps 6-9: epilogue
+// ---------------------------------------------------------------------------
+constexpr int kBkABytes = 128 * kMlpMaxH1 * 4;  // one W1^T tile (32 KB)
+constexpr int kBkThreads = 64 + 8 * 32;
+template <int BC>
+__host__ __device__ constexpr int bk_stages() { return BC >= 128 ? 1 : 2; }
+template <int BC>
+__host__ __device__ constexpr int bk_smem() {
+  return bk_stages<BC>() * 2 * kBkABytes + kMlpMaxH1 * 2 * BC * 4 + 128 * BC * 4 + 1024;
+}
+
+template <int BC>
+__global__ void __launch_bounds__(kBkThreads, 1) k_mlp_l1_back_tma(const float* __restrict__ w1b,
+                                                                  const __grid_constant__ CUtensorMap tm_gp,
+                                                                  int N, int Bp, int H1,
+                                                                  const float* __restrict__ u,
+                                                                  const float* __restrict__ gz1) {
+  constexpr int NM = 2 * BC, KH = kMlpMaxH1, S = bk_stages<BC>();
+  constexpr uint32_t A_LBO = 16 * 128, B_LBO = (NM / 8) * 128;
+  constexpr uint32_t TMEM_COLS = 2 * NM <= 32 ? 32 : 2 * NM <= 64 ? 64 : 2 * NM <= 128 ? 128 : 2 * NM <= 256 ? 256 : 512;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NM >> 3) << 17) |
+                             ((uint32_t)(128 >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t bk_smem_raw[];
+  uint8_t* smem = smem_align1024(bk_smem_raw);
+  uint8_t* sA = smem;                                // S x [hi 32 KB | lo 32 KB]
+  uint8_t* sB = smem + S * 2 * kBkABytes;            // KH x 2BC, K-major
+  uint8_t* stg = sB + KH * NM * 4;                   // BC/32 blocks of [128 rows][128 B], swizzled
+  __shared__ uint64_t a_full[S], a_conv[S], a_empty[S], acc_full[2], acc_empty[2];
+  __shared__ uint32_t tmem_sh;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int seed0 = blockIdx.y * BC;
+  const int ntiles = (N + 127) / 128;
+  const int nt = blockIdx.x < ntiles ? (ntiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&tmem_sh)),
+                 "n"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&a_full[i], 1);
+      mbar_init(&a_conv[i], 4);
+      mbar_init(&a_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_empty[i], 4);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  // B: hidden h (K), column c (N) -> core (h/4, c/8) at ((h/4) * NM/8 + c/8) * 128 + (c%8) * 16 + (h%4) * 4
+  for (int blk = tid; blk < (KH / 4) * (BC / 4); blk += kBkThreads) {
+    const int hc = blk / (BC / 4), n0 = (blk % (BC / 4)) * 4;
+    float4 r[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int h = hc * 4 + i;
+      r[i] = h < H1 ? *reinterpret_cast<const float4*>(gz1 + (size_t)h * Bp + seed0 + n0)
+                    : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const int c = n0 + x;
+      const float4 col = make_float4(comp(r[0], x), comp(r[1], x), comp(r[2], x), comp(r[3], x));
+      const float4 hi = tf32_hi(col), lo = sub4(col, hi);
+      *reinterpret_cast<float4*>(sB + (hc * (NM / 8) + c / 8) * 128 + (c % 8) * 16) = hi;
+      *reinterpret_cast<float4*>(sB + (hc * (NM / 8) + (BC + c) / 8) * 128 + (c % 8) * 16) = lo;
+    }
+  }
+  asm volatile("fence.proxy.async.shared::cta;");
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem = tmem_sh;
+
+  if (warp == 0) {  // producer
+    if (lane == 0)
+      for (int i = 0; i < nt; ++i) {
+        const int st = i % S, tile = blockIdx.x + i * gridDim.x;
+        if (i >= S) mbar_wait(&a_empty[st], (uint32_t)((i / S - 1) & 1));
+        const uint32_t bar = smem_u32(&a_full[st]);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(kBkABytes));
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_u32(sA + st * 2 * kBkABytes)),
+            "l"(w1b + (size_t)tile * (kBkABytes / 4)), "r"(kBkABytes), "r"(bar)
+            : "memory");
+      }
+  } else if (warp == 1) {  // MMA issuer
+    if (lane == 0)
+      for (int i = 0; i < nt; ++i) {
+        const int st = i % S, d = i & 1;
+        mbar_wait(&a_conv[st], (uint32_t)((i / S) & 1));
+        if (i >= 2) mbar_wait(&acc_empty[d], (uint32_t)((i / 2 - 1) & 1));
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        const uint32_t ah = smem_u32(sA + st * 2 * kBkABytes), al = ah + kBkABytes, bb = smem_u32(sB);
+#pragma unroll
+        for (int ks = 0; ks < KH / 8; ++ks) {
+          const uint64_t db = umma_desc(bb + ks * 2 * B_LBO, B_LBO, 128);
+#pragma unroll
+          for (int part = 0; part < 2; ++part) {
+            const uint64_t da = umma_desc((part ? al : ah) + ks * 2 * A_LBO, A_LBO, 128);
+            const uint32_t acc = (ks > 0 || part > 0) ? 1u : 0u;
+            asm volatile(
+                "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem + d * NM),
+                "l"(da), "l"(db), "r"(IDESC), "r"(acc));
+          }
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+            smem_u32(&a_empty[st])));
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+            smem_u32(&acc_full[d])));
+      }
+  } else if (warp < 6) {  // converters: A_lo next to A_hi
+    const int ct = tid - 64;
+    for (int i = 0; i < nt; ++i) {
+      const int st = i % S;
+      mbar_wait(&a_full[st], (uint32_t)((i / S) & 1));
+      uint8_t* ah = sA + st * 2 * kBkABytes;
+#pragma unroll 4
+      for (int j = ct; j < kBkABytes / 16; j += 128) {
+        const float4 x = *reinterpret_cast<const float4*>(ah + j * 16);
+        *reinterpret_cast<float4*>(ah + kBkABytes + j * 16) = sub4(x, tf32_hi(x));
+      }
+      asm volatile("fence.proxy.async.shared::cta;");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&a_conv[st])));
+    }
+  } else {  // epilogue: g_p = u + D_hi + D_lo -> swizzled staging -> tensor TMA store
+    const int et = tid - 192, q = warp % 4, m = q * 32 + lane;
+    for (int i = 0; i < nt; ++i) {
+      const int d = i & 1, tile = blockIdx.x + i * gridDim.x;
+      if (i > 0) {  // the previous tile's store has read the staging buffer
+        if (et == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+      }
+      mbar_wait(&acc_full[d], (uint32_t)((i / 2) & 1));
+      __syncwarp();
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const int k = tile * 128 + m;
+      const float uk = k < N ? __ldg(u + k) : 0.f;
+#pragma unroll
+      for (int c = 0; c < BC; c += 16) {
+        uint32_t v[16], w[16];
+        const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + d * NM + c;
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+              "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+              "=r"(v[14]), "=r"(v[15])
+            : "r"(ta));
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]),
+              "=r"(w[7]), "=r"(w[8]), "=r"(w[9]), "=r"(w[10]), "=r"(w[11]), "=r"(w[12]), "=r"(w[13]),
+              "=r"(w[14]), "=r"(w[15])
+            : "r"(ta + BC));
+        asm volatile("tcgen05.wait::ld.sync.aligned;");
+        uint8_t* rowp = stg + (c / 32) * (128 * 128) + m * 128;
+#pragma unroll
+        for (int x = 0; x < 16; x += 4) {
+          const int j = ((c % 32) + x) / 4;  // 16-byte chunk within the 128-byte row
+          *reinterpret_cast<float4*>(rowp + ((j ^ (m % 8)) * 16)) =
+              make_float4(uk + (__uint_as_float(v[x]) + __uint_as_float(w[x])),
+                          uk + (__uint_as_float(v[x + 1]) + __uint_as_float(w[x + 1])),
+                          uk + (__uint_as_float(v[x + 2]) + __uint_as_float(w[x + 2])),
+                          uk + (__uint_as_float(v[x + 3]) + __uint_as_float(w[x + 3])));
+        }
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_empty[d])));
+      asm volatile("fence.proxy.async.shared::cta;");
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (et == 0) {
+#pragma unroll
+        for (int jb = 0; jb < BC / 32; ++jb)
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
+                           &tm_gp),
+                       "r"(seed0 + 32 * jb), "r"(tile * 128), "r"(smem_u32(stg + jb * 128 * 128))
+                       : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+    }
+    if (et == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 0) {
+    __syncwarp();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TMEM_COLS));
+  }
+}
+
+// W1^T laid out for k_mlp_l1_back_tma, once per run: ceil(N / 128) tiles of
+// kBkABytes, element (e-node m of the tile, hidden unit h) at core (h/4, m/8):
+// ((h/4) * 16 + m/8) * 128 + (m%8) * 16 + (h%4) * 4 bytes (k_mlp_l1_back_tc's
+// A layout); hidden units >= H1 and e-nodes >= N are zero.
+std::vector<float> mlp_w1_back_tiles(const float* W1, int H1, int N) {
+  const int ntiles = (N + 127) / 128;
+  std::vector<float> t((size_t)ntiles * (kBkABytes / 4), 0.f);
+  for (int tl = 0; tl < ntiles; ++tl) {
+    float* tile = t.data() + (size_t)tl * (kBkABytes / 4);
+    for (int h = 0; h < H1 && h < kMlpMaxH1; ++h)
+      for (int m = 0; m < 128 && tl * 128 + m < N; ++m)
+        tile[(((h / 4) * 16 + m / 8) * 128 + (m % 8) * 16 + (h % 4) * 4) / 4] =
+            W1[(size_t)h * N + tl * 128 + m];
+  }
+  return t;
+}
+
 int mlp_nsplit(int device) { return num_sms(device); }
 
 void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, const float* W1,
@@ -702,9 +929,34 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
   SM_LAUNCH_CHECK();
 }
 
-void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* u,
-                    const float* gz1, float* gp) {
+void launch_mlp_bwd(cudaStream_t s, const Shape& sh, int32_t H1, const float* W1, const float* W1b,
+                    const float* u, const float* gz1, float* gp, int32_t nsms) {
   const int Bc = sh.Bp < 128 ? sh.Bp : 128;
+  const char* tenv = std::getenv("SMOOTHE_MLP_TMA");
+  if (!(tenv && tenv[0] == '0') && W1b) {
+    const int nchunks = sh.Bp / Bc, ntiles = (sh.N + 127) / 128;
+    int gx = nsms / nchunks;
+    gx = gx < 1 ? 1 : gx > ntiles ? ntiles : gx;
+    const dim3 grid(gx, nchunks);
+    const CUtensorMap tg = tensor_map_2d(gp, false, (uint64_t)sh.Bp, (uint64_t)sh.N,
+                                          (uint64_t)sh.Bp * 4, 32, 128, true);
+#define SM_L1BT(BCV)                                                                             \
+  do {                                                                                           \
+    static bool attr = false;                                                                    \
+    if (!attr) {                                                                                 \
+      SM_CUDA(cudaFuncSetAttribute(k_mlp_l1_back_tma<BCV>,                                       \
+                                   cudaFuncAttributeMaxDynamicSharedMemorySize, bk_smem<BCV>()));\
+      attr = true;                                                                               \
+    }                                                                                            \
+    k_mlp_l1_back_tma<BCV><<<grid, kBkThreads, bk_smem<BCV>(), s>>>(W1b, tg, sh.N, sh.Bp, H1, u, gz1); \
+  } while (0)
+    if (Bc == 128) SM_L1BT(128);
+    else if (Bc == 64) SM_L1BT(64);
+    else SM_L1BT(32);
+#undef SM_L1BT
+    SM_LAUNCH_CHECK();
+    return;
+  }
   const dim3 grid((sh.N + 127) / 128, sh.Bp / Bc);
 #define SM_L1B(BCV)                                                                              \
   do {                                                                                           \

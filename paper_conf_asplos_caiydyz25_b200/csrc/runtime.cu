@@ -240,6 +240,7 @@ struct smoothe_run {
   int32_t *q_ptr = nullptr, *q_nbr = nullptr;
   float* q_w = nullptr;
   float* W1t = nullptr;  // W1 in k_mlp_l1_tma's tiles (mlp_w1_tiles)
+  float* W1b = nullptr;  // W1^T in k_mlp_l1_back_tma's tiles (mlp_w1_back_tiles)
   float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr, *W3 = nullptr, *b3 = nullptr;
   float *p = nullptr, *gp = nullptr, *sbin = nullptr, *z1_part = nullptr, *z1 = nullptr,
         *gz1 = nullptr;
@@ -484,7 +485,7 @@ void enqueue_step(smoothe_run* r) {
     launch_reduce_rows_f64(s, r->f_part, r->rows_M, sh.Bp, r->f, 1.0, r->red_scratch);
     launch_mlp_fwd(s, sh, r->H1, r->H2, r->W1, r->W1t, r->b1, r->W2, r->b2, r->W3, r->b3, r->p,
                    r->z1_part, r->z1, r->fextra, r->gz1, r->nsplit);
-    launch_mlp_bwd(s, sh, r->H1, r->W1, r->u_f, r->gz1, r->gp);
+    launch_mlp_bwd(s, sh, r->H1, r->W1, r->W1b, r->u_f, r->gz1, r->gp, r->nsplit);
     launch_cost_gp(s, sh, g, r->gp, r->cp, qK, r->gcp, gqK);
   }
 
@@ -822,6 +823,7 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     r->W1 = upload(o, std::vector<float>(cost->W1, cost->W1 + (size_t)H1 * sh.N));
     // W1 in the TMA layer-1 kernel's tile order (constant for the run)
     r->W1t = upload(o, mlp_w1_tiles(cost->W1, H1, sh.N));
+    r->W1b = upload(o, mlp_w1_back_tiles(cost->W1, H1, sh.N));
     r->b1 = upload(o, std::vector<float>(cost->b1, cost->b1 + H1));
     r->W2 = upload(o, std::vector<float>(cost->W2, cost->W2 + (size_t)H2 * H1));
     r->b2 = upload(o, std::vector<float>(cost->b2, cost->b2 + H2));
