@@ -459,43 +459,65 @@ std::vector<float> mlp_w1_tiles(const float* W1, int H1, int N) {
   return t;
 }
 
-// z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h
-__global__ void k_mlp_reduce(int Bp, int H1, int nsplit, const float* __restrict__ b1,
-                             const float* __restrict__ z1_part, float* __restrict__ z1) {
-  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= H1 * Bp) return;
-  const int h = idx / Bp, b = idx % Bp;
+// z1[h][b] = b1[h] + sum over CTAs (in order) of rows h and 64 + h.  One
+// block per hidden unit and 32 seeds: 8 warps stage the per-CTA terms
+// (coalesced, all loads in flight) in shared memory, then warp 0 adds them in
+// CTA order (the in-order sum over 148 CTAs was latency-bound: 34 us on C5).
+constexpr int kRedMaxSplit = 256;
+__global__ void __launch_bounds__(256) k_mlp_reduce(int Bp, int H1, int nsplit, const float* __restrict__ b1,
+                                                    const float* __restrict__ z1_part, float* __restrict__ z1) {
+  __shared__ float xs[kRedMaxSplit][33];
+  const int h = blockIdx.x, b = blockIdx.y * 32 + threadIdx.x % 32, w = threadIdx.x / 32;
+  const size_t cs = (size_t)128 * Bp, lo = (size_t)64 * Bp;
+  const float* q = z1_part + (size_t)h * Bp + b;
+  for (int c = w; c < nsplit; c += 8) xs[c][threadIdx.x % 32] = q[c * cs] + q[c * cs + lo];
+  __syncthreads();
+  if (w != 0) return;
   float acc = 0.f;
-  for (int c = 0; c < nsplit; ++c) {
-    const float* q = z1_part + (size_t)c * 128 * Bp;
-    acc += q[(size_t)h * Bp + b] + q[(size_t)(64 + h) * Bp + b];
-  }
-  z1[idx] = b1[h] + acc;
+  for (int c = 0; c < nsplit; ++c) acc += xs[c][threadIdx.x];
+  z1[(size_t)h * Bp + b] = b1[h] + acc;
 }
 
-// Per seed: layers 2-3, f_mlp, and gz1 = d f_mlp / d z1.
-__global__ void k_mlp_head(int Bp, int H1, int H2, const float* __restrict__ z1g,
-                           const float* __restrict__ W2, const float* __restrict__ b2,
-                           const float* __restrict__ W3, const float* __restrict__ b3,
-                           double* __restrict__ f_mlp, float* __restrict__ gz1) {
-  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+// Per seed (one warp, lanes over hidden units): layers 2-3, f_mlp, and
+// gz1 = d f_mlp / d z1.  Layer-2 sums are warp trees in a fixed order.
+__global__ void __launch_bounds__(128) k_mlp_head(int Bp, int H1, int H2, const float* __restrict__ z1g,
+                                                  const float* __restrict__ W2, const float* __restrict__ b2,
+                                                  const float* __restrict__ W3, const float* __restrict__ b3,
+                                                  double* __restrict__ f_mlp, float* __restrict__ gz1) {
+  const int b = blockIdx.x * 4 + threadIdx.x / 32, lane = threadIdx.x % 32;
   if (b >= Bp) return;
-  float z1[kMlpMaxH1], z2[kMlpMaxH2];
-  for (int h = 0; h < H1; ++h) z1[h] = z1g[(size_t)h * Bp + b];
-  float y = b3[0];
-  for (int h2 = 0; h2 < H2; ++h2) {
-    float acc = b2[h2];
-    for (int h = 0; h < H1; ++h) acc += W2[h2 * H1 + h] * fmaxf(z1[h], 0.f);
-    z2[h2] = acc;
-    y += W3[h2] * fmaxf(acc, 0.f);
+  constexpr int HL = kMlpMaxH1 / 32;  // hidden units per lane: lane, lane + 32
+  float z1[HL];
+#pragma unroll
+  for (int r = 0; r < HL; ++r) {
+    const int h = lane + 32 * r;
+    z1[r] = h < H1 ? z1g[(size_t)h * Bp + b] : 0.f;
   }
-  f_mlp[b] = (double)y;
+  float y = b3[0];
+  uint32_t pos = 0;  // bit h2: z2[h2] > 0
+  for (int h2 = 0; h2 < H2; ++h2) {
+    float part = 0.f;
+#pragma unroll
+    for (int r = 0; r < HL; ++r) {
+      const int h = lane + 32 * r;
+      if (h < H1) part = fmaf(W2[h2 * H1 + h], fmaxf(z1[r], 0.f), part);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+    const float z2 = b2[h2] + part;
+    y += W3[h2] * fmaxf(z2, 0.f);
+    if (z2 > 0.f) pos |= 1u << h2;
+  }
+  if (lane == 0) f_mlp[b] = (double)y;
   if (gz1) {
-    for (int h = 0; h < H1; ++h) {
+#pragma unroll
+    for (int r = 0; r < HL; ++r) {
+      const int h = lane + 32 * r;
+      if (h >= H1) continue;
       float acc = 0.f;
       for (int h2 = 0; h2 < H2; ++h2)
-        if (z2[h2] > 0.f) acc += W2[h2 * H1 + h] * W3[h2];
-      gz1[(size_t)h * Bp + b] = z1[h] > 0.f ? acc : 0.f;  // ReLU'(0) = 0 (S25)
+        if (pos >> h2 & 1u) acc += W2[h2 * H1 + h] * W3[h2];
+      gz1[(size_t)h * Bp + b] = z1[r] > 0.f ? acc : 0.f;  // ReLU'(0) = 0 (S25)
     }
   }
 }
@@ -923,9 +945,10 @@ void launch_mlp_fwd(cudaStream_t s, const Shape& sh, int32_t H1, int32_t H2, con
 #undef SM_L1
   SM_LAUNCH_CHECK();
   }
-  k_mlp_reduce<<<(H1 * sh.Bp + 255) / 256, 256, 0, s>>>(sh.Bp, H1, nsplit, b1, z1_part, z1);
+  SM_REQUIRE(nsplit <= kRedMaxSplit, SMOOTHE_E_CUDA, "k_mlp_reduce: more split-K partials than SMs expected");
+  k_mlp_reduce<<<dim3(H1, sh.Bp / 32), 256, 0, s>>>(sh.Bp, H1, nsplit, b1, z1_part, z1);
   SM_LAUNCH_CHECK();
-  k_mlp_head<<<(sh.Bp + 127) / 128, 128, 0, s>>>(sh.Bp, H1, H2, z1, W2, b2, W3, b3, f_mlp, gz1);
+  k_mlp_head<<<(sh.Bp + 3) / 4, 128, 0, s>>>(sh.Bp, H1, H2, z1, W2, b2, W3, b3, f_mlp, gz1);
   SM_LAUNCH_CHECK();
 }
 
