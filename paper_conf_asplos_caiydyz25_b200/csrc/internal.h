@@ -221,6 +221,14 @@ struct SweepState {
   int32_t* lastchg = nullptr;
   float *W = nullptr, *S = nullptr, *kq = nullptr, *kpi = nullptr, *wpart = nullptr;
   int32_t *kam = nullptr, *wm = nullptr;
+  // live[t] [K + 2], zeroed per step: some g_q^t value is non-zero (set by the
+  // reverse-phase writers; sweeps whose input is all zero are skipped).
+  // NULL with SMOOTHE_GLIVE=0.
+  int32_t* glive = nullptr;
+  // gstamp[t & 1][row][chunk] = t: sweep t + 1 wrote a non-zero g_q^t row
+  // (by parity: sweep t reads t & 1 and writes (t - 1) & 1; never reset, a
+  // stale match only costs a read).  NULL with SMOOTHE_GLIVE=0.
+  int32_t* gstamp = nullptr;
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).
 void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
@@ -257,7 +265,9 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
-                          const int32_t* lastchg = nullptr, int32_t* cursor = nullptr);
+                          const int32_t* lastchg = nullptr, int32_t* cursor = nullptr,
+                          const int32_t* live_in = nullptr, int32_t* live_out = nullptr,
+                          int32_t* gstamp = nullptr);
 // sets the conditional handle to 1 iff some seed is not frozen (wm[s] == 0)
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h);

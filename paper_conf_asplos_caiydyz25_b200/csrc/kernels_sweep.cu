@@ -392,6 +392,25 @@ void launch_sweep_forward(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // (the forward's lists, so the work is proportional to the recomputed
 // classes).  t == K fills cur_pi / cur_am from every class's last row (cur_q
 // is the forward's complete q^{K-1} buffer).  Grid y = seed chunk = pool.
+// Dead gradients: the reverse sweeps are linear in g_q
+// with no source term after the loss, so once every g_q^t row is zero, sweep t
+// and all later ones add nothing.  live[t] (zeroed per step) is set by any
+// writer that stores a non-zero g_q^t value; the kernels of reverse sweep t
+// (transition, plain, frozen, combine) return at once when live_in = &live[t]
+// is still 0.  (On C4 the gradient underflows to zero from sweep ~60 down.)
+__device__ __forceinline__ bool g_dead(const int32_t* live_in) {
+  return live_in && __ldcg(live_in) == 0;
+}
+// lane `leader` of the (sub)warp `mask` marks live_out when any lane's row is
+// non-zero, and stamps the row (stamp = t - 1 for a g_q^{t-1} row, NULL: none)
+// so that k_wspmv can skip the W rows of children whose g_q^t is all zero
+__device__ __forceinline__ void g_mark(int32_t* live_out, unsigned mask, bool nz, bool leader,
+                                       int32_t* stamp = nullptr, int tval = 0) {
+  if (__any_sync(mask, nz) && leader) {
+    if (live_out && __ldcg(live_out) == 0) __stcg(live_out, 1);
+    if (stamp) __stcg(stamp, tval);
+  }
+}
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_rev_restore_all(int M, int Bp, PoolArgs P,
                                                            float* __restrict__ cur_pi,
@@ -411,7 +430,9 @@ __global__ void __launch_bounds__(kBlock) k_rev_transition(int M, int Bp, int t,
                                                           float* __restrict__ cur_q,
                                                           float* __restrict__ cur_pi,
                                                           int32_t* __restrict__ cur_am,
-                                                          int32_t* __restrict__ wm) {
+                                                          int32_t* __restrict__ wm,
+                                                          const int32_t* __restrict__ live_in) {
+  if (g_dead(live_in)) return;  // reverse sweep t and all later ones add nothing
   const int groups = gridDim.x * (kBlock / LPR);
   const int c = blockIdx.y;
   const int32_t* ln = P.list_n + (size_t)c * (P.K + 2);
@@ -471,7 +492,8 @@ void launch_rev_transition(cudaStream_t s, const Shape& sh, const DevGraph& g, i
       const dim3 grid(SMOOTHE_TRANS_BPS * st.num_sms, num_chunks(sh.Bp));
       k_rev_transition<LPR><<<grid, kBlock, 0, s>>>(sh.M, sh.Bp, t, P, st.qbuf[(K - 1) & 1],
                                                     st.cur_pi, st.cur_am,
-                                                    st.wmode ? st.wm : nullptr);
+                                                    st.wmode ? st.wm : nullptr,
+                                                    st.glive ? st.glive + t : nullptr);
     }
   });
   SM_LAUNCH_CHECK();
@@ -516,12 +538,14 @@ void launch_pool_version0(cudaStream_t s, const Shape& sh, const DevGraph& g, co
 __global__ void k_sweep_reset(int M, int Bp, int root, int nchunk, int K,
                               int32_t* __restrict__ stamps, float* __restrict__ qbuf,
                               int32_t* __restrict__ pool_n, int32_t* __restrict__ lastrow,
-                              int32_t* __restrict__ list_n, int32_t* __restrict__ abort_flag) {
+                              int32_t* __restrict__ list_n, int32_t* __restrict__ abort_flag,
+                              int32_t* __restrict__ glive) {
   const int64_t MB = (int64_t)M * Bp, n0 = 4 * (int64_t)M, n1 = n0 + 2 * MB,
                 n2 = n1 + (int64_t)nchunk * M, n3 = n2 + (int64_t)nchunk * (K + 2);
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (e0 == 0) abort_flag[0] = 0;
+  if (glive && e0 < K + 2) glive[e0] = 0;
   if (e0 < nchunk) pool_n[e0] = M;
   for (int64_t e = e0; e < n3; e += stride) {
     if (e < n0) stamps[e] = -1;
@@ -542,7 +566,7 @@ void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
   SM_CUDA(cudaGetDevice(&dev));
   k_sweep_reset<<<4 * num_sms(dev), 256, 0, s>>>(sh.M, sh.Bp, sh.root, st.nchunk, st.K,
                                                  st.dirty[0], st.qbuf[0], st.pool_n, st.lastrow,
-                                                 st.list_n, st.abort_flag);
+                                                 st.list_n, st.abort_flag, st.glive);
   SM_LAUNCH_CHECK();
 }
 
@@ -623,6 +647,14 @@ __device__ __forceinline__ Vec<V> ldv_cg(const float* p) {  // L2 only: rows oth
   return r;
 }
 
+template <int V>
+__device__ __forceinline__ bool any_nz(const Vec<V>& v) {
+  bool nz = false;
+#pragma unroll
+  for (int x = 0; x < V; ++x) nz = nz || v.v[x] != 0.f;
+  return nz;
+}
+
 // Outputs of one reverse-sweep item: g_q^{t-1}_{j'} directly (the class's only
 // item), else its partial row, and the class's last item to finish combines.
 // CONV (convergence mode without the frozen-sweep path): seeds with pass = 1
@@ -651,14 +683,18 @@ __device__ __forceinline__ void reverse_epilogue(
     const Vec<V>& gqacc, const Vec<V>& X, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const float* __restrict__ cp,
     float* __restrict__ gcp, float* __restrict__ gq_prev, float* __restrict__ part,
-    int32_t* __restrict__ cnt, const Vec<V>& pass, const float* __restrict__ gq) {
+    int32_t* __restrict__ cnt, const Vec<V>& pass, const float* __restrict__ gq,
+    int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp, int t) {
   Vec<V> zero;
+  int32_t* st = gstamp ? gstamp + (size_t)jp * gridDim.y + blockIdx.y : nullptr;  // [row][chunk]
 #pragma unroll
   for (int x = 0; x < V; ++x) zero.v[x] = 0.f;
   if (info < 0) {  // the class's only item
-    if (gq_prev)
-      stv<V>(gq_prev + (size_t)jp * Bp + s0,
-             jp == root ? zero : pass_through<V, CONV>(gqacc, pass, gq, jp, Bp, s0));
+    if (gq_prev) {
+      const Vec<V> o = jp == root ? zero : pass_through<V, CONV>(gqacc, pass, gq, jp, Bp, s0);
+      stv<V>(gq_prev + (size_t)jp * Bp + s0, o);
+      g_mark(live_out, 0xffffffffu, any_nz<V>(o), lane == 0, st, t - 1);
+    }
     return;
   }
   stv<V>(part + (size_t)(info >> 1) * Bp + s0, piece ? X : gqacc);
@@ -701,9 +737,11 @@ __device__ __forceinline__ void reverse_epilogue(
     }
     stv<V>(gcp + ok, gc);
   }
-  if (gq_prev)
-    stv<V>(gq_prev + (size_t)jp * Bp + s0,
-           jp == root ? zero : pass_through<V, CONV>(acc, pass, gq, jp, Bp, s0));
+  if (gq_prev) {
+    const Vec<V> o = jp == root ? zero : pass_through<V, CONV>(acc, pass, gq, jp, Bp, s0);
+    stv<V>(gq_prev + (size_t)jp * Bp + s0, o);
+    g_mark(live_out, 0xffffffffu, any_nz<V>(o), lane == 0, st, t - 1);
+  }
 }
 
 // One warp per work item (HostGraph::rev_item): a run of batches of class j'.
@@ -731,9 +769,11 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
     const float* __restrict__ q_prev, const float* __restrict__ gq, const float* __restrict__ pi,
     const int32_t* __restrict__ am, float* __restrict__ gcp, float* __restrict__ gq_prev,
     float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
-    const int32_t* __restrict__ wm, const int32_t* __restrict__ lastchg) {
+    const int32_t* __restrict__ wm, const int32_t* __restrict__ lastchg,
+    const int32_t* __restrict__ live_in, int32_t* __restrict__ live_out,
+    int32_t* __restrict__ gstamp) {
   const int it = blockIdx.x * (kRevBlock / 32) + (int)threadIdx.x / 32;
-  if (it >= n_items) return;
+  if (it >= n_items || g_dead(live_in)) return;
   const int lane = threadIdx.x % 32;
   // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
   Vec<V> keep, pass;
@@ -775,6 +815,8 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
 #pragma unroll
         for (int x = 0; x < V; ++x) g.v[x] = 0.f;
       stv<V>(gq_prev + (size_t)jp * Bp + s0, g);
+      g_mark(live_out, 0xffffffffu, any_nz<V>(g), lane == 0,
+             gstamp ? gstamp + (size_t)jp * gridDim.y + blockIdx.y : nullptr, t - 1);
     }
     return;
   }
@@ -902,7 +944,8 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
     }
   }
   reverse_epilogue<V, HI, CONV>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X, items,
-                                class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq);
+                                class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq, live_out,
+                                gstamp, t);
 }
 
 // ---------------------------------------------------------------------------
@@ -975,9 +1018,12 @@ __global__ void __launch_bounds__(32 * kRtWarps, SMOOTHE_RT_CTAS) k_sweep_revers
     float wC, const float* __restrict__ cp, const float* __restrict__ q_prev,
     const float* __restrict__ gq, float* __restrict__ gcp, float* __restrict__ gq_prev,
     float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
-    const int32_t* __restrict__ wm, int32_t* __restrict__ cursor) {
+    const int32_t* __restrict__ wm, int32_t* __restrict__ cursor,
+    const int32_t* __restrict__ live_in, int32_t* __restrict__ live_out,
+    int32_t* __restrict__ gstamp) {
   constexpr int V = 4, S = kRtStages;
   (void)cursor;
+  if (g_dead(live_in)) return;
   extern __shared__ __align__(128) unsigned char rt_smem[];
   const int lane = threadIdx.x % 32, wi = threadIdx.x / 32;
   unsigned char* ring = rt_smem + (size_t)wi * S * kRtStage;
@@ -1170,7 +1216,8 @@ __global__ void __launch_bounds__(32 * kRtWarps, SMOOTHE_RT_CTAS) k_sweep_revers
       }
       Vec<V> pass = zero;
       reverse_epilogue<V, HI, false>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X,
-                                     items, class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq);
+                                     items, class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq,
+                                     live_out, gstamp, t);
     }
     // advance the queue: nxt becomes current (with the batches already requested)
     cur = nxt;
@@ -1197,8 +1244,10 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const float* q_prev, const float* pi, const int32_t* am,
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
-                          const int32_t* lastchg, int32_t* cursor) {
+                          const int32_t* lastchg, int32_t* cursor, const int32_t* live_in,
+                          int32_t* live_out, int32_t* gstamp) {
   float* out = write_gq_prev ? gq_prev : nullptr;
+  if (!out) live_out = gstamp = nullptr;
 #ifndef SMOOTHE_REV_VMAX
 #define SMOOTHE_REV_VMAX 4  // seeds per lane at Bp >= 128 (4: one warp per 128-seed slice)
 #endif
@@ -1215,7 +1264,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
     int dev = 0;
     SM_CUDA(cudaGetDevice(&dev));
     const dim3 grid(SMOOTHE_RT_CTAS * num_sms(dev), sh.Bp / 128);
-#define SM_RT(HI_, HC_)                                                                           do {                                                                                              static bool attr = false;                                                                       if (!attr) {                                                                                      SM_CUDA(cudaFuncSetAttribute(k_sweep_reverse_tma<HI_, HC_>,                                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kRtSmem));            attr = true;                                                                                  }                                                                                               k_sweep_reverse_tma<HI_, HC_><<<grid, 32 * kRtWarps, kRtSmem, s>>>(                                 mg, mp, ma, n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item),                       g.rev_class_item_ptr, g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, gcp,           out, rev_part, rev_cnt, l2_prefetch, t, K, wm, cursor);                                   } while (0)
+#define SM_RT(HI_, HC_)                                                                           do {                                                                                              static bool attr = false;                                                                       if (!attr) {                                                                                      SM_CUDA(cudaFuncSetAttribute(k_sweep_reverse_tma<HI_, HC_>,                                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kRtSmem));            attr = true;                                                                                  }                                                                                               k_sweep_reverse_tma<HI_, HC_><<<grid, 32 * kRtWarps, kRtSmem, s>>>(                                 mg, mp, ma, n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item),                       g.rev_class_item_ptr, g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, gcp,           out, rev_part, rev_cnt, l2_prefetch, t, K, wm, cursor, live_in, live_out, gstamp);                                   } while (0)
     if (HI && HC) SM_RT(true, true);
     else if (HI) SM_RT(true, false);
     else SM_RT(false, true);
@@ -1228,7 +1277,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
   k_sweep_reverse<VV, HI, HC, CV><<<grid, kRevBlock, 0, s>>>(                                  \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,             \
-      rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg)
+      rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg, live_in, live_out, gstamp)
 #define SM_REV2(VV, HI, HC)                                                                    \
   do {                                                                                         \
     if (lastchg) SM_REV3(VV, HI, HC, true);                                                    \
@@ -1343,17 +1392,23 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     const int32_t* __restrict__ cls_child, const float* __restrict__ W,
     const int32_t* __restrict__ wm, const float* __restrict__ gq, float* __restrict__ S,
     float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
-    const int32_t* __restrict__ lastchg) {
+    const int32_t* __restrict__ lastchg, const int32_t* __restrict__ live_in,
+    int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
+    const int32_t* __restrict__ gstamp_in) {
   const RowGroup<LPR, kWBlock> rg;
   if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {  // profiling: a working launch?
     bool any = false;
     for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
     if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
   }
-  if (rg.row >= n_items) return;
+  if (rg.row >= n_items || g_dead(live_in)) return;
   const int4 w4 = ld4i(wm + rg.s0);
   const unsigned gm = LPR == 32 ? 0xffffffffu
                                 : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
+  const bool lead = threadIdx.x % LPR == 0;
+  // g_q^t_j may be non-zero only if sweep t + 1 stamped row j with t (every
+  // writer of a non-zero row does); sweep K reads the cost's g_q^K rows
+  const bool check = gstamp_in && live_in;
   if (!__any_sync(gm, (w4.x | w4.y | w4.z | w4.w) != 0)) return;  // row-group uniform
   const int4 itm = items[rg.row];
   const int i = itm.x, e0 = itm.y, e1 = itm.z, slot = itm.w;
@@ -1389,6 +1444,8 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
         if (!comp(w4, x)) comp(o, x) = comp(cur, x);
     }
     st4(gq_prev + oi, o);
+    g_mark(live_out, gm, o.x != 0.f || o.y != 0.f || o.z != 0.f || o.w != 0.f, lead,
+           gstamp ? gstamp + (size_t)i * gridDim.y + blockIdx.y : nullptr, t - 1);
     return;
   }
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -1399,6 +1456,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   for (int c0 = e0; c0 < e1; c0 += LPR) {
     const int n = min(LPR, e1 - c0);
     const int myj = gl < n ? __ldg(cls_child + c0 + gl) : 0;
+    const int myl = !check || (gl < n && __ldcg(gstamp_in + (size_t)myj * gridDim.y + blockIdx.y) == t);
     const float* wrow = W + (size_t)c0 * Bp + rg.s0;
     constexpr int DP = LPR == 32 ? SMOOTHE_WSPMV_DEPTH32 : SMOOTHE_WSPMV_DEPTH;
     for (int u = 0; u < n; u += DP) {  // DP edges in flight; the last batch predicated
@@ -1406,7 +1464,8 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
 #pragma unroll
       for (int v = 0; v < DP; ++v) {
         const int j = __shfl_sync(gm, myj, (u + v) & (LPR - 1), LPR);
-        if (u + v < n) {
+        const int lv = __shfl_sync(gm, myl, (u + v) & (LPR - 1), LPR);
+        if (u + v < n && lv) {  // a child whose g_q^t is all zero adds nothing: no W load
           wv[v] = STREAM ? ldcs4(wrow + (size_t)(u + v) * Bp) : ld4(wrow + (size_t)(u + v) * Bp);
           gv[v] = ld4(gq + (size_t)j * Bp + rg.s0);
         } else {
@@ -1442,6 +1501,8 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
       if (!comp(w4, x)) comp(o, x) = comp(cur, x);
   }
   st4(gq_prev + oi, o);
+  g_mark(live_out, gm, o.x != 0.f || o.y != 0.f || o.z != 0.f || o.w != 0.f, lead,
+         gstamp ? gstamp + (size_t)i * gridDim.y + blockIdx.y : nullptr, t - 1);
 }
 
 // g_q^{t-1}_i of the classes split into several chunks: their partial rows in
@@ -1451,9 +1512,13 @@ __global__ void __launch_bounds__(kBlock) k_wcombine(
     int n_multi, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ wmulti, const int32_t* __restrict__ wmulti_ptr,
     const int32_t* __restrict__ wm, const float* __restrict__ part, float* __restrict__ gq_prev,
-    const int32_t* __restrict__ lastchg, const float* __restrict__ gq) {
+    const int32_t* __restrict__ lastchg, const float* __restrict__ gq,
+    const int32_t* __restrict__ live_in, int32_t* __restrict__ live_out,
+    int32_t* __restrict__ gstamp) {
   const RowGroup<LPR> rg;
-  if (rg.row >= n_multi) return;
+  if (rg.row >= n_multi || g_dead(live_in)) return;
+  const unsigned gm = LPR == 32 ? 0xffffffffu
+                                : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
   const int4 w4 = ld4i(wm + rg.s0);
   if (!(w4.x | w4.y | w4.z | w4.w)) return;
   const int i = wmulti[rg.row];
@@ -1490,6 +1555,9 @@ __global__ void __launch_bounds__(kBlock) k_wcombine(
       if (!comp(w4, x)) comp(o, x) = comp(cur, x);
   }
   st4(gq_prev + oi, o);
+  g_mark(live_out, gm, o.x != 0.f || o.y != 0.f || o.z != 0.f || o.w != 0.f,
+         threadIdx.x % LPR == 0, gstamp ? gstamp + (size_t)i * gridDim.y + blockIdx.y : nullptr,
+         t - 1);
 }
 
 void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
@@ -1498,10 +1566,16 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
   // room to spare, where it stays resident across the frozen sweeps (C5: 69 MB)
   const bool stream = (double)g.num_cedge * sh.Bp * sizeof(float) > 96e6;
   const int4* items = reinterpret_cast<const int4*>(g.witem);
+  const int32_t* live_in = st.glive && t < st.K ? st.glive + t : nullptr;
+  int32_t* live_out = st.glive && gq_prev ? st.glive + (t - 1) : nullptr;
+  // stamps by sweep parity: sweep t reads buffer t & 1 while writing (t - 1) & 1
+  const size_t sm_n = (size_t)st.nchunk * sh.M;
+  int32_t* gstamp = gq_prev && st.gstamp ? st.gstamp + ((t - 1) & 1) * sm_n : nullptr;
+  const int32_t* gstamp_in = st.gstamp ? st.gstamp + (t & 1) * sm_n : nullptr;
 #define SM_WSPMV(ST, CV)                                                                       \
   k_wspmv<LPR, ST, CV><<<grid, kWBlock, 0, s>>>(                                               \
       g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W, st.wm, \
-      gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg)
+      gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out, gstamp, gstamp_in)
   SM_DISPATCH_LPR(sh.Bp, {
     const dim3 grid = row_grid(g.num_witems, sh.Bp, LPR, kWBlock);
     if (st.converge) {
@@ -1516,7 +1590,7 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
       SM_LAUNCH_CHECK();
       k_wcombine<LPR><<<row_grid(g.num_wmulti, sh.Bp, LPR), kBlock, 0, s>>>(
           g.num_wmulti, sh.Bp, sh.root, t, g.dmin, g.wmulti, g.wmulti_ptr, st.wm, st.wpart,
-          gq_prev, st.converge ? st.lastchg : nullptr, gq);
+          gq_prev, st.converge ? st.lastchg : nullptr, gq, live_in, live_out, gstamp);
     }
   });
 #undef SM_WSPMV

@@ -539,7 +539,10 @@ void enqueue_step(smoothe_run* r) {
                            sw.cur_am, sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
                            r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt,
                            sw.converge && !sw.wmode ? sw.lastchg : nullptr,
-                           r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128));
+                           r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128),
+                           sw.glive && t < K ? sw.glive + t : nullptr,
+                           sw.glive && t > 1 ? sw.glive + (t - 1) : nullptr,
+                           sw.gstamp ? sw.gstamp + ((t - 1) & 1) * (size_t)sw.nchunk * sh.M : nullptr);
     };
     if (r->in_capture && sw.wmode && t < K && g.num_rev_items >= 100000) {
       // in the captured step the plain sweep is a conditional node, skipped
@@ -714,6 +717,14 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     w.list_n = dalloc<int32_t>(o, (size_t)w.nchunk * (slots + 1));
     w.pool_n = dalloc<int32_t>(o, w.nchunk);
     w.abort_flag = dalloc<int32_t>(o, 4);
+    {
+      const char* genv = std::getenv("SMOOTHE_GLIVE");
+      if (!(genv && genv[0] == '0')) {
+        w.glive = dalloc<int32_t>(o, slots + 1);
+        w.gstamp = dalloc<int32_t>(o, 2 * (size_t)w.nchunk * sh.M);
+        SM_CUDA(cudaMemset(w.gstamp, 0xFF, sizeof(int32_t) * 2 * w.nchunk * sh.M));
+      }
+    }
     alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
     for (int b = 0; b < 2; ++b) {  // consecutive: k_sweep_reset fills all four at once

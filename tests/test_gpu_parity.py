@@ -698,6 +698,36 @@ def test_reverse_tma_bit_identical(sm, monkeypatch, name, B, G, agg, steps):
     assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
 
 
+@pytest.mark.parametrize("name,B,G,agg,steps,conv", [
+    ("C2", 64, 8, "hybrid", 6, 0), ("C3", 32, 8, "correlated", 4, 0), ("C5", 64, 8, "hybrid", 4, 0),
+    ("C4", 32, 16, "hybrid", 3, 0), ("C4", 128, 16, "independent", 2, 0), ("C5", 64, 8, "hybrid", 3, 1)])
+def test_dead_gradient_skip_identical(sm, monkeypatch, name, B, G, agg, steps, conv):
+    """Reverse sweeps whose input g_q^t is all zero (live flag unset) are
+    skipped (default) against running every sweep (SMOOTHE_GLIVE=0): the
+    sweeps are linear in g_q with no source term, so theta after several
+    steps, a debug step's gradient and the best extraction are equal
+    (skipping can only leave a -0 where +0 would be added: compared as
+    values, so -0 == +0)."""
+    eg = make_config(name)
+    outs = []
+    for env in ("1", "0"):
+        monkeypatch.setenv("SMOOTHE_GLIVE", env)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=19, assumption=agg, converge=bool(conv)))
+        run.steps(steps)
+        th, m, v, n = run.state()
+        d = run.debug_step(th, m, v, step_index=n)
+        outs.append((run.theta(), run.extract(), d["grad_cp"], d["grad_theta"]))
+        run.close()
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][2], outs[1][2])
+    assert np.array_equal(outs[0][3], outs[1][3])
+    assert np.array_equal(outs[0][1][0], outs[1][1][0])
+    assert outs[0][1][1]["best_cost"] == outs[1][1][1]["best_cost"]
+
+
 def test_step_trace_relaxed_vs_sampled(sm):
     """The per-step record (smoothe_run_get_trace, E11 / PAPER.md:459-461):
     row k holds min / mean over seeds of the relaxed f(p_b) and the min of the
