@@ -281,17 +281,34 @@ def roofline(args, eg, prof, Bl, K, steps_ms):
     units_launch = Bl * N
     peak, peak_src = measured_peaks()
     extra = {}
+    alg_override = None
     if dom == "frozen":
         nwork = max(1, prof.get("frozen_sweeps", 0))
         per_launch_ms = kms[dom] / nwork
         unit_8d = bm["reverse_sweep"]
         C_edges = len(class_graph(eg)[0])
         w_bytes = Bl * (4.0 * C_edges + 16.0 * M)
-        extra["frac_kernel_model"] = w_bytes / (per_launch_ms * 1e-3) / 1e9 / peak
-        extra["kernel_model"] = ("one W row per class edge + g_q^t, S read/write, g_q^{t-1}: "
-                                 "B_l (4 C + 16 M) bytes per launch, C = %d class edges" % C_edges)
+        extra["frac_full_stream_model"] = w_bytes / (per_launch_ms * 1e-3) / 1e9 / peak
+        extra["full_stream_model"] = ("one W row per class edge + g_q^t, S read/write, g_q^{t-1}: "
+                                      "B_l (4 C + 16 M) bytes per launch, C = %d class edges" % C_edges)
         extra["working_launches_per_step"] = nwork / max(1, prof["steps"])
         kname = "k_wspmv"
+        # dead-gradient skipping: a launch moves only the W rows
+        # of children whose g_q^t is live, the g_q^t / S rows of live rows and
+        # the g_q^{t-1} rows it writes -- counted on the device per launch
+        le, lr, rw = (prof.get(k, 0) for k in ("frozen_live_edges", "frozen_live_rows",
+                                                 "frozen_rows_written"))
+        if le + lr + rw > 0:
+            wc = min(128, Bl)
+            live_bytes = 4.0 * wc * (le + 3.0 * lr + rw) / nwork
+            extra["live_model"] = ("4 x seeds-per-chunk x (live class edges + 3 live rows + rows "
+                                   "written) per launch, counted per launch on the device")
+            extra["live_units_per_launch"] = {"class_edges": le / nwork, "rows_read": lr / nwork,
+                                              "rows_written": rw / nwork}
+            extra["live_bytes_per_launch"] = live_bytes
+            extra["frac_8d_full_model"] = (bm["reverse_sweep"] * Bl * N / (per_launch_ms * 1e-3)
+                                           / 1e9 / peak)
+            alg_override = live_bytes
     else:
         per_launch_ms = kms[dom] / max(1, kn[dom])
         unit_8d = bm["forward_sweep" if dom == "forward" else "reverse_sweep"]
@@ -302,6 +319,8 @@ def roofline(args, eg, prof, Bl, K, steps_ms):
         extra["active_node_frac"], extra["active_class_frac"] = fn, fc
         kname = f"k_sweep_{dom}"
     alg = unit_8d * units_launch
+    if alg_override is not None:  # bytes the launch must move (see above)
+        alg = alg_override
     achieved = alg / (per_launch_ms * 1e-3) / 1e9
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": ncu_traffic(args.config, dom), "kernel": kname,
@@ -309,7 +328,9 @@ def roofline(args, eg, prof, Bl, K, steps_ms):
             "alg_bytes_per_launch": alg, "avg_launch_ms": per_launch_ms,
             "kernel_share_of_profiled_step": kms[dom] / max(1e-9, sum(ph.values())),
             "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json), copy bandwidth",
-            "bytes_model": "SURVEY.md 8(d) streaming model per sweep", **extra}
+            "bytes_model": ("live bytes of the frozen sweep (dead-gradient skipping): live_model"
+                            if alg_override is not None else
+                            "SURVEY.md 8(d) streaming model per sweep"), **extra}
     cp_mb = N * Bl * 4 / 1e6
     if cp_mb < 64:   # 8(d): L2-resident configs report the L2 hit rate, not a DRAM fraction
         roof["l2_resident"] = True

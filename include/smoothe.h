@@ -310,7 +310,15 @@ typedef struct {
      reverse sweeps)                                    */
   double sweep_kernel_ms[3];
   int64_t sweep_kernel_launches[3];
-  int64_t frozen_sweeps;     /* k_wspmv launches with at least one frozen seed */
+  int64_t frozen_sweeps;     /* k_wspmv launches with at least one frozen seed
+                                and a live input (g_q^t not all zero)           */
+  /* units (row or class edge x seed chunk of min(Bp, 128) seeds) those
+     launches move, summed over them (dead-gradient skipping):
+     class edges whose W row is loaded (child's g_q^t live), rows whose
+     g_q^t / S are read and S written, rows whose g_q^{t-1} is written      */
+  int64_t frozen_live_edges;
+  int64_t frozen_live_rows;
+  int64_t frozen_rows_written;
 } smoothe_profile;
 
 SMOOTHE_API smoothe_status smoothe_run_profile(smoothe_run *run, int32_t enable);

@@ -271,12 +271,17 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // sets the conditional handle to 1 iff some seed is not frozen (wm[s] == 0)
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h);
+// sets the conditional handle to 1 iff *flag != 0
+void launch_flag_if(cudaStream_t s, const int32_t* flag, cudaGraphConditionalHandle h);
 // W from the K-state rows (before reverse sweep K)
 void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                    const SweepState& st, const float* cp);
 // frozen reverse sweep t for the seeds with wm set: g_q^{t-1} = W g_q^t, S += g_q^t
 void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
                   const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count);
+// profiling: live units of frozen sweep t into out[0..2] (kernels_sweep.cu)
+void launch_count_live(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
+                       const SweepState& st, int64_t* out);
 // converge mode: lastchg[s] from the forward's version lists (per seed, the
 // last sweep whose recomputed q rows differ from their previous versions)
 void launch_last_change(cudaStream_t s, const Shape& sh, const SweepState& st);

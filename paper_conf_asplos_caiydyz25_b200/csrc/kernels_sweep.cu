@@ -1396,7 +1396,8 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
     const int32_t* __restrict__ gstamp_in) {
   const RowGroup<LPR, kWBlock> rg;
-  if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {  // profiling: a working launch?
+  if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 &&
+      !g_dead(live_in)) {  // profiling: a working launch?
     bool any = false;
     for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
     if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
@@ -1422,7 +1423,9 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     cp4 = make_int4(w4.x && t > lc.x + 1, w4.y && t > lc.y + 1, w4.z && t > lc.z + 1,
                     w4.w && t > lc.w + 1);
   }
-  if (d <= t && e0 == cls_child_ptr[i]) {  // first item: S_i += g_q^t_i (a valid row)
+  if (d <= t && e0 == cls_child_ptr[i] &&
+      (!check || __ldcg(gstamp_in + (size_t)i * gridDim.y + blockIdx.y) == t)) {
+    // first item: S_i += g_q^t_i (a valid, non-zero row)
     const float4 gi = ld4(gq + oi);
     float4 si = ld4(S + oi);
 #pragma unroll
@@ -1456,17 +1459,23 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   for (int c0 = e0; c0 < e1; c0 += LPR) {
     const int n = min(LPR, e1 - c0);
     const int myj = gl < n ? __ldg(cls_child + c0 + gl) : 0;
-    const int myl = !check || (gl < n && __ldcg(gstamp_in + (size_t)myj * gridDim.y + blockIdx.y) == t);
+    const bool myl = gl < n && (!check || __ldcg(gstamp_in + (size_t)myj * gridDim.y + blockIdx.y) == t);
+    // the row group's live children (a child whose g_q^t is all zero adds
+    // nothing: no W or g_q load), visited in ascending order, DP in flight
+    unsigned lm = __ballot_sync(gm, myl);
+    if (LPR < 32) lm = (lm >> ((threadIdx.x % 32) / LPR * LPR)) & (LPR == 32 ? 0xffffffffu : (1u << LPR) - 1u);
     const float* wrow = W + (size_t)c0 * Bp + rg.s0;
     constexpr int DP = LPR == 32 ? SMOOTHE_WSPMV_DEPTH32 : SMOOTHE_WSPMV_DEPTH;
-    for (int u = 0; u < n; u += DP) {  // DP edges in flight; the last batch predicated
+    while (lm) {
       float4 wv[DP], gv[DP];
 #pragma unroll
       for (int v = 0; v < DP; ++v) {
-        const int j = __shfl_sync(gm, myj, (u + v) & (LPR - 1), LPR);
-        const int lv = __shfl_sync(gm, myl, (u + v) & (LPR - 1), LPR);
-        if (u + v < n && lv) {  // a child whose g_q^t is all zero adds nothing: no W load
-          wv[v] = STREAM ? ldcs4(wrow + (size_t)(u + v) * Bp) : ld4(wrow + (size_t)(u + v) * Bp);
+        const int e = lm ? __ffs(lm) - 1 : 0;
+        const bool has = lm != 0;
+        lm &= lm - 1;
+        const int j = __shfl_sync(gm, myj, e, LPR);
+        if (has) {
+          wv[v] = STREAM ? ldcs4(wrow + (size_t)e * Bp) : ld4(wrow + (size_t)e * Bp);
           gv[v] = ld4(gq + (size_t)j * Bp + rg.s0);
         } else {
           wv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -1560,6 +1569,50 @@ __global__ void __launch_bounds__(kBlock) k_wcombine(
          t - 1);
 }
 
+// Profiling only (bench.py's roofline of k_wspmv): the (row, seed chunk)
+// units frozen sweep t actually moves: out[0] += class edges (i, j) with i
+// inside the window (dmin_i <= t - 1) and g_q^t_j live (W row loaded),
+// out[1] += rows with a live g_q^t_i inside the window (g_q^t and S read, S
+// written), out[2] += rows written (dmin_i <= t - 1).  stamp_in NULL: all live.
+__global__ void k_count_live(int64_t n_cedge, int M, int nchunk, int t,
+                             const int32_t* __restrict__ cedge_class,
+                             const int32_t* __restrict__ cls_child,
+                             const int32_t* __restrict__ dmin, const int32_t* __restrict__ stamp_in,
+                             const int32_t* __restrict__ live_in, int64_t* __restrict__ out) {
+  if (g_dead(live_in)) return;  // the sweep is skipped
+  const int64_t ne = n_cedge * nchunk, nr = (int64_t)M * nchunk;
+  unsigned long long c[3] = {0, 0, 0};
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < ne + nr;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    if (e < ne) {
+      const int64_t ce = e / nchunk;
+      const int ch = (int)(e % nchunk), i = cedge_class[ce], j = cls_child[ce];
+      c[0] += dmin[i] <= t - 1 && (!stamp_in || stamp_in[(size_t)j * nchunk + ch] == t);
+    } else {
+      const int64_t r = e - ne;
+      const int i = (int)(r / nchunk), ch = (int)(r % nchunk);
+      c[1] += dmin[i] <= t && (!stamp_in || stamp_in[(size_t)i * nchunk + ch] == t);
+      c[2] += dmin[i] <= t - 1;
+    }
+  }
+#pragma unroll
+  for (int x = 0; x < 3; ++x) {
+    for (int o = 16; o > 0; o >>= 1) c[x] += __shfl_xor_sync(0xffffffffu, c[x], o);
+    if (threadIdx.x % 32 == 0 && c[x])
+      atomicAdd(reinterpret_cast<unsigned long long*>(out + x), c[x]);
+  }
+}
+
+void launch_count_live(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
+                       const SweepState& st, int64_t* out) {
+  const size_t sm_n = (size_t)st.nchunk * sh.M;
+  const int32_t* stamp_in = st.gstamp && t < st.K ? st.gstamp + (t & 1) * sm_n : nullptr;
+  k_count_live<<<4 * st.num_sms, 256, 0, s>>>(g.num_cedge, sh.M, st.nchunk, t, g.cedge_class,
+                                              g.cls_child, g.dmin, stamp_in,
+                                              st.glive && t < st.K ? st.glive + t : nullptr, out);
+  SM_LAUNCH_CHECK();
+}
+
 void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
                   const SweepState& st, const float* gq, float* gq_prev, int64_t* frozen_count) {
   // W streams from HBM once per sweep (evict-first) unless it fits in L2 with
@@ -1650,6 +1703,15 @@ __global__ void k_any_unfrozen(cudaGraphConditionalHandle h, const int32_t* __re
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h) {
   k_any_unfrozen<<<1, 256, 0, s>>>(h, wm, sh.B);
+  SM_LAUNCH_CHECK();
+}
+
+__global__ void k_flag_if(cudaGraphConditionalHandle h, const int32_t* __restrict__ flag) {
+  cudaGraphSetConditional(h, __ldcg(flag) != 0 ? 1u : 0u);
+}
+
+void launch_flag_if(cudaStream_t s, const int32_t* flag, cudaGraphConditionalHandle h) {
+  k_flag_if<<<1, 1, 0, s>>>(h, flag);
   SM_LAUNCH_CHECK();
 }
 

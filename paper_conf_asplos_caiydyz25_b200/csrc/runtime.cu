@@ -206,6 +206,7 @@ struct smoothe_run {
   cudaStream_t stream2 = nullptr;
   // graph capture: conditional bodies are captured on their own stream
   cudaStream_t stream_body = nullptr;
+  cudaStream_t stream_body2 = nullptr;  // nested conditional bodies
   bool in_capture = false;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_pen = nullptr;
   bool overlap = false;
@@ -504,64 +505,80 @@ void enqueue_step(smoothe_run* r) {
   pm.mark(SMOOTHE_PHASE_REVERSE);
   SweepState& sw = r->sw;
   const float* cur_q = sw.qbuf[(K - 1) & 1];
+  // In the captured step of a large graph (C4), each sweep t < K is a
+  // conditional node on live[t] (the sweep's input g_q^t not all zero), so
+  // the sweeps after the gradient has died launch nothing; the plain kernel
+  // inside is itself conditional on some seed being unfrozen.  (Direct
+  // launches: every kernel of a dead sweep returns at once.)
+  const bool big = r->in_capture && g.num_rev_items >= 100000;
   for (int t = K; t >= 1; --t) {
-    launch_rev_transition(s, sh, g, t, K, sw);
-    if (sw.wmode && t == K) {  // K-state rows, W, every seed frozen at t = K
-      SM_CUDA(cudaMemcpyAsync(sw.kq, cur_q, sizeof(float) * MB, cudaMemcpyDeviceToDevice, s));
-      if (sw.kpi)
-        SM_CUDA(cudaMemcpyAsync(sw.kpi, sw.cur_pi, sizeof(float) * MB, cudaMemcpyDeviceToDevice, s));
-      SM_CUDA(cudaMemcpyAsync(sw.kam, sw.cur_am, sizeof(int32_t) * MB, cudaMemcpyDeviceToDevice, s));
-      SM_CUDA(cudaMemsetAsync(sw.wm, 1, sizeof(int32_t) * sh.Bp, s));
-      SM_CUDA(cudaMemsetAsync(sw.S, 0, sizeof(float) * MB, s));
-      launch_wbuild(s, sh, g, r->agg, sw, r->cp);
-    }
-    if (sw.converge && t == K) launch_last_change(s, sh, sw);
-    if (sw.wmode && r->profiling && std::getenv("SMOOTHE_REV_W_STATS")) {
-      // diagnostic: seeds still frozen before reverse sweep t (stderr, one line per sweep)
-      std::vector<int32_t> h(sh.Bp);
-      SM_CUDA(cudaMemcpyAsync(h.data(), sw.wm, sizeof(int32_t) * sh.Bp, cudaMemcpyDeviceToHost, s));
-      SM_CUDA(cudaStreamSynchronize(s));
-      int n = 0, slices = 0;
-      for (int b = 0; b < sh.B; ++b) n += h[b] != 0;
-      for (int c = 0; c * 128 < sh.Bp; ++c) {
-        bool all = true;
-        for (int b = c * 128; b < std::min(sh.Bp, (c + 1) * 128); ++b) all = all && h[b] != 0;
-        slices += all;
+    auto sweep = [&](cudaStream_t ss, cudaStream_t sbody) {
+      launch_rev_transition(ss, sh, g, t, K, sw);
+      if (sw.wmode && t == K) {  // K-state rows, W, every seed frozen at t = K
+        SM_CUDA(cudaMemcpyAsync(sw.kq, cur_q, sizeof(float) * MB, cudaMemcpyDeviceToDevice, ss));
+        if (sw.kpi)
+          SM_CUDA(cudaMemcpyAsync(sw.kpi, sw.cur_pi, sizeof(float) * MB, cudaMemcpyDeviceToDevice, ss));
+        SM_CUDA(cudaMemcpyAsync(sw.kam, sw.cur_am, sizeof(int32_t) * MB, cudaMemcpyDeviceToDevice, ss));
+        SM_CUDA(cudaMemsetAsync(sw.wm, 1, sizeof(int32_t) * sh.Bp, ss));
+        SM_CUDA(cudaMemsetAsync(sw.S, 0, sizeof(float) * MB, ss));
+        launch_wbuild(ss, sh, g, r->agg, sw, r->cp);
       }
-      fprintf(stderr, "[wstats] t=%d frozen_seeds=%d full_slices=%d\n", t, n, slices);
-    }
-    kmark(1, 0);
-    // converge mode: a seed's loss reads q^{t*} (t* = its convergence sweep),
-    // so the reverse window (g_q^t_j = 0 while t + hmax_j <= K) does not hold
-    // for K; no window then (the window argument with t* would be per seed)
-    auto plain = [&](cudaStream_t ss) {
-      launch_sweep_reverse(ss, sh, g, r->agg, t, sw.converge ? -1 : K, cur_q, sw.cur_pi,
-                           sw.cur_am, sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
-                           r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt,
-                           sw.converge && !sw.wmode ? sw.lastchg : nullptr,
-                           r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128),
-                           sw.glive && t < K ? sw.glive + t : nullptr,
-                           sw.glive && t > 1 ? sw.glive + (t - 1) : nullptr,
-                           sw.gstamp ? sw.gstamp + ((t - 1) & 1) * (size_t)sw.nchunk * sh.M : nullptr);
+      if (sw.converge && t == K) launch_last_change(ss, sh, sw);
+      if (sw.wmode && r->profiling && std::getenv("SMOOTHE_REV_W_STATS")) {
+        // diagnostic: seeds still frozen before reverse sweep t (stderr, one line per sweep)
+        std::vector<int32_t> h(sh.Bp);
+        SM_CUDA(cudaMemcpyAsync(h.data(), sw.wm, sizeof(int32_t) * sh.Bp, cudaMemcpyDeviceToHost, ss));
+        SM_CUDA(cudaStreamSynchronize(ss));
+        int n = 0, slices = 0;
+        for (int b = 0; b < sh.B; ++b) n += h[b] != 0;
+        for (int c = 0; c * 128 < sh.Bp; ++c) {
+          bool all = true;
+          for (int b = c * 128; b < std::min(sh.Bp, (c + 1) * 128); ++b) all = all && h[b] != 0;
+          slices += all;
+        }
+        fprintf(stderr, "[wstats] t=%d frozen_seeds=%d full_slices=%d\n", t, n, slices);
+      }
+      kmark(1, 0);
+      // converge mode: a seed's loss reads q^{t*} (t* = its convergence sweep),
+      // so the reverse window (g_q^t_j = 0 while t + hmax_j <= K) does not hold
+      // for K; no window then (the window argument with t* would be per seed)
+      auto plain = [&](cudaStream_t ps) {
+        launch_sweep_reverse(ps, sh, g, r->agg, t, sw.converge ? -1 : K, cur_q, sw.cur_pi,
+                             sw.cur_am, sw.wmode ? sw.wm : nullptr, r->cp, r->gq[t & 1], r->gcp,
+                             r->gq[(t - 1) & 1], t > 1, r->rev_part, r->rev_cnt,
+                             sw.converge && !sw.wmode ? sw.lastchg : nullptr,
+                             r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128),
+                             sw.glive && t < K ? sw.glive + t : nullptr,
+                             sw.glive && t > 1 ? sw.glive + (t - 1) : nullptr,
+                             sw.gstamp ? sw.gstamp + ((t - 1) & 1) * (size_t)sw.nchunk * sh.M : nullptr);
+      };
+      if (big && sw.wmode && t < K) {
+        // the plain sweep is a conditional node, skipped (no launch of its
+        // blocks) once every seed is frozen; only for large grids (C4: 171k
+        // items, 114.0 -> 108.3 ms per step), where an empty launch costs
+        // more than the conditional (C5: 6.58 -> 7.10 ms)
+        enqueue_if(
+            ss, sbody,
+            [&](cudaGraphConditionalHandle h) { launch_any_unfrozen(ss, sh, sw.wm, h); }, plain);
+      } else {
+        plain(ss);
+      }
+      kmark(1, 1);
+      if (sw.wmode) {
+        if (r->profiling) launch_count_live(ss, sh, g, t, sw, r->frozen_count + 1);
+        kmark(2, 0);
+        launch_wspmv(ss, sh, g, t, sw, r->gq[t & 1], t > 1 ? r->gq[(t - 1) & 1] : nullptr,
+                     r->profiling ? r->frozen_count : nullptr);
+        kmark(2, 1);
+      }
     };
-    if (r->in_capture && sw.wmode && t < K && g.num_rev_items >= 100000) {
-      // in the captured step the plain sweep is a conditional node, skipped
-      // (no launch of its blocks) once every seed is frozen; only for large
-      // grids (C4: 171k items, 114.0 -> 108.3 ms per step), where an empty
-      // launch costs more than the conditional (C5: 6.58 -> 7.10 ms)
+    if (big && sw.glive && t < K)
       enqueue_if(
           s, r->stream_body,
-          [&](cudaGraphConditionalHandle h) { launch_any_unfrozen(s, sh, sw.wm, h); }, plain);
-    } else {
-      plain(s);
-    }
-    kmark(1, 1);
-    if (sw.wmode) {
-      kmark(2, 0);
-      launch_wspmv(s, sh, g, t, sw, r->gq[t & 1], t > 1 ? r->gq[(t - 1) & 1] : nullptr,
-                   r->profiling ? r->frozen_count : nullptr);
-      kmark(2, 1);
-    }
+          [&](cudaGraphConditionalHandle h) { launch_flag_if(s, sw.glive + t, h); },
+          [&](cudaStream_t bs) { sweep(bs, r->stream_body2); });
+    else
+      sweep(s, r->stream_body);
   }
   if (sw.wmode)  // the frozen sweeps' g_cp: one pass over the K-state with g = S
     launch_sweep_reverse(s, sh, g, r->agg, K, K, sw.kq, sw.kpi, sw.kam, nullptr, r->cp, sw.S,
@@ -747,8 +764,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
       w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
-      r->frozen_count = dalloc<int64_t>(o, 1);
-      SM_CUDA(cudaMemset(r->frozen_count, 0, sizeof(int64_t)));
+      r->frozen_count = dalloc<int64_t>(o, 4);  // launches, live edges / rows, rows written
+      SM_CUDA(cudaMemset(r->frozen_count, 0, 4 * sizeof(int64_t)));
     }
   }
   r->gq[0] = dalloc<float>(o, MB);
@@ -1202,6 +1219,7 @@ smoothe_status smoothe_run_create(smoothe_egraph* g, const smoothe_cost_model* c
       r->overlap = !(ov && ov[0] == '0');
     }
     SM_CUDA(cudaStreamCreateWithFlags(&r->stream_body, cudaStreamNonBlocking));
+    SM_CUDA(cudaStreamCreateWithFlags(&r->stream_body2, cudaStreamNonBlocking));
     if (r->overlap) {
       SM_CUDA(cudaStreamCreateWithFlags(&r->stream2, cudaStreamNonBlocking));
       SM_CUDA(cudaEventCreateWithFlags(&r->ev_fork, cudaEventDisableTiming));
@@ -1501,7 +1519,8 @@ smoothe_status smoothe_run_profile(smoothe_run* run, int32_t enable) {
     run->profiling = enable != 0;
     run->prof_ev.clear();
     for (auto& v : run->prof_kev) v.clear();
-    if (run->frozen_count) SM_CUDA(cudaMemsetAsync(run->frozen_count, 0, sizeof(int64_t), run->stream));
+    if (run->frozen_count)
+      SM_CUDA(cudaMemsetAsync(run->frozen_count, 0, 4 * sizeof(int64_t), run->stream));
     run->prof_pool_used = 0;
     std::memset(run->prof_launch, 0, sizeof(run->prof_launch));
     run->prof_launch_total = 0;
@@ -1524,7 +1543,7 @@ smoothe_status smoothe_run_get_profile(smoothe_run* run, smoothe_profile* out) {
     }
     for (int ph = 0; ph < SMOOTHE_NUM_PHASES; ++ph) out->phase_launches[ph] = run->prof_launch[ph];
     if (run->frozen_count)
-      SM_CUDA(cudaMemcpy(&out->frozen_sweeps, run->frozen_count, sizeof(int64_t),
+      SM_CUDA(cudaMemcpy(&out->frozen_sweeps, run->frozen_count, 4 * sizeof(int64_t),
                          cudaMemcpyDeviceToHost));
     for (int w = 0; w < 3; ++w) {
       for (const auto& ev : run->prof_kev[w]) {
@@ -1554,6 +1573,7 @@ void smoothe_free_run(smoothe_run* run) {
   if (run->stream) cudaStreamDestroy(run->stream);
   if (run->stream2) cudaStreamDestroy(run->stream2);
   if (run->stream_body) cudaStreamDestroy(run->stream_body);
+  if (run->stream_body2) cudaStreamDestroy(run->stream_body2);
   if (run->ev_fork) cudaEventDestroy(run->ev_fork);
   if (run->ev_join) cudaEventDestroy(run->ev_join);
   if (run->ev_pen) cudaEventDestroy(run->ev_pen);

@@ -77,7 +77,8 @@ class _Profile(C.Structure):
     _fields_ = [("phase_ms", C.c_double * 8), ("phase_launches", C.c_int64 * 8),
                 ("steps", C.c_int64), ("launches", C.c_int64), ("num_seeds_padded", C.c_int32),
                 ("sweep_kernel_ms", C.c_double * 3), ("sweep_kernel_launches", C.c_int64 * 3),
-                ("frozen_sweeps", C.c_int64)]
+                ("frozen_sweeps", C.c_int64), ("frozen_live_edges", C.c_int64),
+                ("frozen_live_rows", C.c_int64), ("frozen_rows_written", C.c_int64)]
 
 
 _lib = None
@@ -371,7 +372,9 @@ class Run:
                 "sweep_kernel_launches": {"forward": p.sweep_kernel_launches[0],
                                           "reverse": p.sweep_kernel_launches[1],
                                           "frozen": p.sweep_kernel_launches[2]},
-                "frozen_sweeps": p.frozen_sweeps}
+                "frozen_sweeps": p.frozen_sweeps, "frozen_live_edges": p.frozen_live_edges,
+                "frozen_live_rows": p.frozen_live_rows,
+                "frozen_rows_written": p.frozen_rows_written}
 
     def close(self):
         if self._h:
