@@ -229,6 +229,24 @@ struct SweepState {
   // (by parity: sweep t reads t & 1 and writes (t - 1) & 1; never reset, a
   // stale match only costs a read).  NULL with SMOOTHE_GLIVE=0.
   int32_t* gstamp = nullptr;
+  // fchg[t] [K + 2], zeroed per step: some q row changed (bitwise) in forward
+  // sweep t.  Once a sweep changes nothing, every later sweep is the identity
+  // (no class is dirty, no row to copy forward): in the captured step of a
+  // large graph, forward sweep t is a conditional node on fchg[t - 1].  NULL
+  // with SMOOTHE_FSKIP=0.
+  int32_t* fchg = nullptr;
+  // k_wspmv as one wave of persistent row groups striding over the work items
+  // (default for >= 100k items; SMOOTHE_WSPMV_PERSIST=0 / 1 forces)
+  bool wpersist = false;
+  // captured step of a large graph (>= 100k reverse items): conditional nodes
+  // cost ~15 us each, so sweeps are gated in blocks: forward sweeps
+  // [t, t + fblock) by one IF on fchg[t - 1] (0: no gating), reverse sweeps
+  // (t - rblock, t] by one IF on live[t]; the plain reverse kernel runs as one
+  // wave of persistent warps (an all-frozen sweep then costs a few us) unless
+  // plain_if, which puts it under an IF on "some seed unfrozen"
+  // (SMOOTHE_FBLOCK, SMOOTHE_RBLOCK, SMOOTHE_PLAIN_IF)
+  int fblock = 0, rblock = 8;
+  bool plain_if = false;
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).
 void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
@@ -267,7 +285,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
                           const int32_t* lastchg = nullptr, int32_t* cursor = nullptr,
                           const int32_t* live_in = nullptr, int32_t* live_out = nullptr,
-                          int32_t* gstamp = nullptr);
+                          int32_t* gstamp = nullptr, bool persist = false);
 // sets the conditional handle to 1 iff some seed is not frozen (wm[s] == 0)
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h);

@@ -83,6 +83,7 @@ struct PoolArgs {
   int4* list;           // [nchunk][K+1][M]
   int32_t* list_n;      // [nchunk][K+2]
   int32_t* abort_flag;  // [0]: this step overflowed
+  int32_t* fchg;        // [K+2] or NULL: fchg[t] = 1 once some q row changed in sweep t
 };
 template <int LPR>
 __device__ __forceinline__ void publish_version(const PoolArgs& P, int t, int j, int gl,
@@ -187,7 +188,10 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
                   __float_as_uint(qo.z) != __float_as_uint(qold.z) ||
                   __float_as_uint(qo.w) != __float_as_uint(qold.w);
   if (__ballot_sync(gm, ne) == 0u) return;
-  if (gl == 0) chg_cur[j] = t;
+  if (gl == 0) {
+    chg_cur[j] = t;
+    if (P.fchg && __ldcg(P.fchg + t) == 0) __stcg(P.fchg + t, 1);
+  }
   for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
     dirty_next[cls_child[c]] = t + 1;
 }
@@ -325,7 +329,10 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
                   __float_as_uint(qo.z) != __float_as_uint(qold.z) ||
                   __float_as_uint(qo.w) != __float_as_uint(qold.w);
   if (__ballot_sync(gm, ne) == 0u) return;
-  if (gl == 0) chg_cur[j] = t;
+  if (gl == 0) {
+    chg_cur[j] = t;
+    if (P.fchg && __ldcg(P.fchg + t) == 0) __stcg(P.fchg + t, 1);
+  }
   for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
     dirty_next[cls_child[c]] = t + 1;
 }
@@ -358,6 +365,7 @@ static PoolArgs pool_args(const Shape& sh, const SweepState& st) {
   P.list = st.list;
   P.list_n = st.list_n;
   P.abort_flag = st.abort_flag;
+  P.fchg = st.fchg;
   return P;
 }
 
@@ -539,13 +547,14 @@ __global__ void k_sweep_reset(int M, int Bp, int root, int nchunk, int K,
                               int32_t* __restrict__ stamps, float* __restrict__ qbuf,
                               int32_t* __restrict__ pool_n, int32_t* __restrict__ lastrow,
                               int32_t* __restrict__ list_n, int32_t* __restrict__ abort_flag,
-                              int32_t* __restrict__ glive) {
+                              int32_t* __restrict__ glive, int32_t* __restrict__ fchg) {
   const int64_t MB = (int64_t)M * Bp, n0 = 4 * (int64_t)M, n1 = n0 + 2 * MB,
                 n2 = n1 + (int64_t)nchunk * M, n3 = n2 + (int64_t)nchunk * (K + 2);
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (e0 == 0) abort_flag[0] = 0;
   if (glive && e0 < K + 2) glive[e0] = 0;
+  if (fchg && e0 < K + 2) fchg[e0] = 0;
   if (e0 < nchunk) pool_n[e0] = M;
   for (int64_t e = e0; e < n3; e += stride) {
     if (e < n0) stamps[e] = -1;
@@ -566,7 +575,7 @@ void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st) {
   SM_CUDA(cudaGetDevice(&dev));
   k_sweep_reset<<<4 * num_sms(dev), 256, 0, s>>>(sh.M, sh.Bp, sh.root, st.nchunk, st.K,
                                                  st.dirty[0], st.qbuf[0], st.pool_n, st.lastrow,
-                                                 st.list_n, st.abort_flag, st.glive);
+                                                 st.list_n, st.abort_flag, st.glive, st.fchg);
   SM_LAUNCH_CHECK();
 }
 
@@ -761,7 +770,7 @@ constexpr int kRevBlock = SMOOTHE_REV_BLOCK;
 #ifndef SMOOTHE_REV_MINB4
 #define SMOOTHE_REV_MINB4 (6 * 64 / SMOOTHE_REV_BLOCK)  // min resident blocks per SM at V = 4
 #endif
-template <int V, bool HI, bool HC, bool CONV>
+template <int V, bool HI, bool HC, bool CONV, bool PERSIST = false>
 __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64 / kRevBlock) k_sweep_reverse(
     int n_items, int Bp, int root, const int4* __restrict__ items,
     const int32_t* __restrict__ class_item_ptr, const int32_t* __restrict__ pad_child,
@@ -771,9 +780,9 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
     float* __restrict__ part, int32_t* __restrict__ cnt, bool l2_prefetch, int t, int K,
     const int32_t* __restrict__ wm, const int32_t* __restrict__ lastchg,
     const int32_t* __restrict__ live_in, int32_t* __restrict__ live_out,
-    int32_t* __restrict__ gstamp) {
-  const int it = blockIdx.x * (kRevBlock / 32) + (int)threadIdx.x / 32;
-  if (it >= n_items || g_dead(live_in)) return;
+    int32_t* __restrict__ gstamp, int stride) {
+  const int it0 = blockIdx.x * (kRevBlock / 32) + (int)threadIdx.x / 32;
+  if (it0 >= n_items || g_dead(live_in)) return;
   const int lane = threadIdx.x % 32;
   // seeds in a frozen sweep (wm set) are the W kernel's: no contribution here
   Vec<V> keep, pass;
@@ -803,6 +812,10 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
     }
     if (__all_sync(0xffffffffu, allw)) return;
   }
+  // stride = n_items: one item per warp; else persistent warps (one wave of
+  // blocks) take items it0, it0 + stride, ... (an all-frozen sweep then costs
+  // one wave of blocks that exit at once instead of a block per two items)
+  auto item = [&](const int it) {
   const int4 c0 = items[2 * it], c1 = items[2 * it + 1];
   if (c1.z > t - 1) return;  // q^{t-1}_{j'} = 0: nothing to add, g_q^{t-1}_{j'} never read
   const int jp = c0.x, bb = c0.y, be = c0.z, info = c0.w;
@@ -946,6 +959,12 @@ __global__ void __launch_bounds__(kRevBlock, V == 4 ? SMOOTHE_REV_MINB4 : 8 * 64
   reverse_epilogue<V, HI, CONV>(lane, jp, info, piece, Bp, root, s0, keep, qp, gqacc, X, items,
                                 class_item_ptr, cp, gcp, gq_prev, part, cnt, pass, gq, live_out,
                                 gstamp, t);
+  };
+  if (PERSIST) {
+    for (int it = it0; it < n_items; it += stride) item(it);
+  } else {
+    item(it0);
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -1245,7 +1264,7 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
                           const int32_t* wm, const float* cp, const float* gq, float* gcp,
                           float* gq_prev, bool write_gq_prev, float* rev_part, int32_t* rev_cnt,
                           const int32_t* lastchg, int32_t* cursor, const int32_t* live_in,
-                          int32_t* live_out, int32_t* gstamp) {
+                          int32_t* live_out, int32_t* gstamp, bool persist) {
   float* out = write_gq_prev ? gq_prev : nullptr;
   if (!out) live_out = gstamp = nullptr;
 #ifndef SMOOTHE_REV_VMAX
@@ -1272,12 +1291,33 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
     SM_LAUNCH_CHECK();
     return;
   }
-  const dim3 grid((n + kRevBlock / 32 - 1) / (kRevBlock / 32), sh.Bp / (32 * V));
+  dim3 grid((n + kRevBlock / 32 - 1) / (kRevBlock / 32), sh.Bp / (32 * V));
+  int stride = n;
+  persist = persist && V == 4 && !lastchg;
+  if (persist) {  // one wave of resident blocks
+    int dev = 0;
+    SM_CUDA(cudaGetDevice(&dev));
+    static int wave[64] = {0};
+    int& nb = wave[dev & 63];
+    if (!nb) {
+      SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+          &nb, k_sweep_reverse<4, true, true, false, true>, kRevBlock, 0));
+      nb = std::max(1, nb) * num_sms(dev);
+    }
+    grid.x = std::min<unsigned>(grid.x, (unsigned)nb);
+    stride = (int)grid.x * (kRevBlock / 32);
+  }
 #define SM_REV3(VV, HI, HC, CV)                                                                \
+  if (VV == 4 && !CV && persist)                                                               \
+    k_sweep_reverse<VV, HI, HC, CV, VV == 4 && !CV><<<grid, kRevBlock, 0, s>>>(                \
+        n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,    \
+        g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,           \
+        rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg, live_in, live_out, gstamp, stride); \
+  else                                                                                         \
   k_sweep_reverse<VV, HI, HC, CV><<<grid, kRevBlock, 0, s>>>(                                  \
       n, sh.Bp, sh.root, reinterpret_cast<const int4*>(g.rev_item), g.rev_class_item_ptr,      \
       g.pad_child, g.pad_batch_node, a.wI, a.wC, cp, q_prev, gq, pi, am, gcp, out,             \
-      rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg, live_in, live_out, gstamp)
+      rev_part, rev_cnt, l2_prefetch, t, K, wm, lastchg, live_in, live_out, gstamp, stride)
 #define SM_REV2(VV, HI, HC)                                                                    \
   do {                                                                                         \
     if (lastchg) SM_REV3(VV, HI, HC, true);                                                    \
@@ -1385,41 +1425,25 @@ constexpr int kWBlock = SMOOTHE_WSPMV_BLOCK;
 #ifndef SMOOTHE_WSPMV_DEPTH32
 #define SMOOTHE_WSPMV_DEPTH32 4
 #endif
+// One W work item (row group of LPR lanes; rows [s0, s0 + 4) of its seeds).
 template <int LPR, bool STREAM, bool CONV>
-__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : SMOOTHE_WSPMV_MINB16) k_wspmv(
-    int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+__device__ __forceinline__ void wspmv_item(
+    int row, int s0, int Bp, int root, int t, const int32_t* __restrict__ dmin,
     const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
-    const int32_t* __restrict__ cls_child, const float* __restrict__ W,
-    const int32_t* __restrict__ wm, const float* __restrict__ gq, float* __restrict__ S,
-    float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
-    const int32_t* __restrict__ lastchg, const int32_t* __restrict__ live_in,
+    const int32_t* __restrict__ cls_child, const float* __restrict__ W, int4 w4, unsigned gm,
+    bool lead, bool check, const float* __restrict__ gq, float* __restrict__ S,
+    float* __restrict__ gq_prev, float* __restrict__ part, const int32_t* __restrict__ lastchg,
     int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
     const int32_t* __restrict__ gstamp_in) {
-  const RowGroup<LPR, kWBlock> rg;
-  if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 &&
-      !g_dead(live_in)) {  // profiling: a working launch?
-    bool any = false;
-    for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
-    if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
-  }
-  if (rg.row >= n_items || g_dead(live_in)) return;
-  const int4 w4 = ld4i(wm + rg.s0);
-  const unsigned gm = LPR == 32 ? 0xffffffffu
-                                : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
-  const bool lead = threadIdx.x % LPR == 0;
-  // g_q^t_j may be non-zero only if sweep t + 1 stamped row j with t (every
-  // writer of a non-zero row does); sweep K reads the cost's g_q^K rows
-  const bool check = gstamp_in && live_in;
-  if (!__any_sync(gm, (w4.x | w4.y | w4.z | w4.w) != 0)) return;  // row-group uniform
-  const int4 itm = items[rg.row];
+  const int4 itm = items[row];
   const int i = itm.x, e0 = itm.y, e1 = itm.z, slot = itm.w;
   const int d = __ldg(dmin + i);
-  const size_t oi = (size_t)i * Bp + rg.s0;
+  const size_t oi = (size_t)i * Bp + s0;
   // converge mode: a frozen seed's sweeps after its convergence sweep
   // lastchg + 1 were never performed: its g_q passes through unchanged
   int4 cp4 = make_int4(0, 0, 0, 0);  // copy mode per seed
   if (CONV) {
-    const int4 lc = ld4i(lastchg + rg.s0);
+    const int4 lc = ld4i(lastchg + s0);
     cp4 = make_int4(w4.x && t > lc.x + 1, w4.y && t > lc.y + 1, w4.z && t > lc.z + 1,
                     w4.w && t > lc.w + 1);
   }
@@ -1464,7 +1488,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     // nothing: no W or g_q load), visited in ascending order, DP in flight
     unsigned lm = __ballot_sync(gm, myl);
     if (LPR < 32) lm = (lm >> ((threadIdx.x % 32) / LPR * LPR)) & (LPR == 32 ? 0xffffffffu : (1u << LPR) - 1u);
-    const float* wrow = W + (size_t)c0 * Bp + rg.s0;
+    const float* wrow = W + (size_t)c0 * Bp + s0;
     constexpr int DP = LPR == 32 ? SMOOTHE_WSPMV_DEPTH32 : SMOOTHE_WSPMV_DEPTH;
     while (lm) {
       float4 wv[DP], gv[DP];
@@ -1476,7 +1500,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
         const int j = __shfl_sync(gm, myj, e, LPR);
         if (has) {
           wv[v] = STREAM ? ldcs4(wrow + (size_t)e * Bp) : ld4(wrow + (size_t)e * Bp);
-          gv[v] = ld4(gq + (size_t)j * Bp + rg.s0);
+          gv[v] = ld4(gq + (size_t)j * Bp + s0);
         } else {
           wv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
           gv[v] = wv[v];
@@ -1492,7 +1516,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     }
   }
   if (slot >= 0) {  // one chunk of a long class: k_wcombine adds the chunks
-    st4(part + (size_t)slot * Bp + rg.s0, acc);
+    st4(part + (size_t)slot * Bp + s0, acc);
     return;
   }
   if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -1512,6 +1536,43 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   st4(gq_prev + oi, o);
   g_mark(live_out, gm, o.x != 0.f || o.y != 0.f || o.z != 0.f || o.w != 0.f, lead,
          gstamp ? gstamp + (size_t)i * gridDim.y + blockIdx.y : nullptr, t - 1);
+}
+
+
+template <int LPR, bool STREAM, bool CONV, bool PERSIST>
+__global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 / kWBlock : SMOOTHE_WSPMV_MINB16) k_wspmv(
+    int n_items, int Bp, int root, int t, const int32_t* __restrict__ dmin,
+    const int4* __restrict__ items, const int32_t* __restrict__ cls_child_ptr,
+    const int32_t* __restrict__ cls_child, const float* __restrict__ W,
+    const int32_t* __restrict__ wm, const float* __restrict__ gq, float* __restrict__ S,
+    float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
+    const int32_t* __restrict__ lastchg, const int32_t* __restrict__ live_in,
+    int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
+    const int32_t* __restrict__ gstamp_in) {
+  const RowGroup<LPR, kWBlock> rg;
+  if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 &&
+      !g_dead(live_in)) {  // profiling: a working launch?
+    bool any = false;
+    for (int b = 0; b < Bp && !any; ++b) any = wm[b] != 0;
+    if (any) atomicAdd(reinterpret_cast<unsigned long long*>(frozen_count), 1ull);
+  }
+  if (rg.row >= n_items || g_dead(live_in)) return;
+  const int4 w4 = ld4i(wm + rg.s0);
+  const unsigned gm = LPR == 32 ? 0xffffffffu
+                                : ((1u << LPR) - 1u) << ((threadIdx.x % 32) / LPR * LPR);
+  const bool lead = threadIdx.x % LPR == 0;
+  // g_q^t_j may be non-zero only if sweep t + 1 stamped row j with t (every
+  // writer of a non-zero row does); sweep K reads the cost's g_q^K rows
+  const bool check = gstamp_in && live_in;
+  if (!__any_sync(gm, (w4.x | w4.y | w4.z | w4.w) != 0)) return;  // row-group uniform
+  // persistent launches (one wave of resident blocks): row group g takes
+  // items g, g + G, ... (round robin keeps the items in flight a compact
+  // window); otherwise one item per row group
+  const int G = PERSIST ? gridDim.x * (kWBlock / LPR) : n_items;
+  for (int row = rg.row; row < n_items; row += G)
+    wspmv_item<LPR, STREAM, CONV>(row, rg.s0, Bp, root, t, dmin, items, cls_child_ptr, cls_child,
+                                  W, w4, gm, lead, check, gq, S, gq_prev, part, lastchg, live_out,
+                                  gstamp, gstamp_in);
 }
 
 // g_q^{t-1}_i of the classes split into several chunks: their partial rows in
@@ -1626,11 +1687,31 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
   int32_t* gstamp = gq_prev && st.gstamp ? st.gstamp + ((t - 1) & 1) * sm_n : nullptr;
   const int32_t* gstamp_in = st.gstamp ? st.gstamp + (t & 1) * sm_n : nullptr;
 #define SM_WSPMV(ST, CV)                                                                       \
-  k_wspmv<LPR, ST, CV><<<grid, kWBlock, 0, s>>>(                                               \
+  if (persist) {                                                                               \
+    static int wave[64] = {0};                                                                 \
+    int& nb = wave[dev & 63];                                                                  \
+    if (!nb) {                                                                                 \
+      SM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_wspmv<LPR, ST, CV, true>,   \
+                                                            kWBlock, 0));                      \
+      nb = std::max(1, nb) * num_sms(dev);                                                     \
+    }                                                                                          \
+    grid.x = std::min<unsigned>(grid.x, (unsigned)nb);                                         \
+    k_wspmv<LPR, ST, CV, true><<<grid, kWBlock, 0, s>>>(                                       \
+        g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,    \
+        st.wm, gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out,       \
+        gstamp, gstamp_in);                                                                    \
+  } else                                                                                       \
+  k_wspmv<LPR, ST, CV, false><<<grid, kWBlock, 0, s>>>(                                        \
       g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W, st.wm, \
       gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out, gstamp, gstamp_in)
+  // persistent row groups (one wave of resident blocks striding over the
+  // items) for large item counts: the launch of ~85k blocks costs ~45 us per
+  // sweep on C4 (SMOOTHE_WSPMV_PERSIST=0 / 1 forces)
+  const bool persist = st.wpersist;
+  int dev = 0;
+  SM_CUDA(cudaGetDevice(&dev));
   SM_DISPATCH_LPR(sh.Bp, {
-    const dim3 grid = row_grid(g.num_witems, sh.Bp, LPR, kWBlock);
+    dim3 grid = row_grid(g.num_witems, sh.Bp, LPR, kWBlock);
     if (st.converge) {
       if (stream) SM_WSPMV(true, true);
       else SM_WSPMV(false, true);

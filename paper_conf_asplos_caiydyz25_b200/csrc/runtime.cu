@@ -431,10 +431,30 @@ void enqueue_step(smoothe_run* r) {
     else r->prof_kev[which].back()[1] = pool_event(r);
     SM_CUDA(cudaEventRecord(r->prof_kev[which].back()[at], s));
   };
-  for (int t = 1; t <= K; ++t) {
+  // In the captured step of a large graph, forward sweeps [t, t + fblock)
+  // (t >= 2) are one conditional node on fchg[t - 1]: once a sweep changes no
+  // q row, it and every later sweep are the identity (C4: the rows freeze by
+  // sweep ~46 of 207), so the blocks after it launch nothing.  Gated in blocks
+  // because a conditional node costs more than an empty sweep (~10 us).
+  // (Direct launches: the kernels of such a sweep find no dirty class.)
+  const bool big = r->in_capture && g.num_rev_items >= 100000;
+  const int fb = big && r->sw.fchg ? r->sw.fblock : 0;
+  for (int t = 1; t <= K;) {
+    if (fb > 0 && t >= 2) {
+      const int t1 = std::min(K + 1, t + fb);
+      enqueue_if(
+          s, r->stream_body,
+          [&](cudaGraphConditionalHandle h) { launch_flag_if(s, r->sw.fchg + (t - 1), h); },
+          [&](cudaStream_t bs) {
+            for (int u = t; u < t1; ++u) launch_sweep_forward(bs, sh, g, r->agg, u, r->sw, r->cp);
+          });
+      t = t1;
+      continue;
+    }
     kmark(0, 0);
     launch_sweep_forward(s, sh, g, r->agg, t, r->sw, r->cp);
     kmark(0, 1);
+    ++t;
   }
   if (r->profiling && std::getenv("SMOOTHE_FREEZE_STATS")) {
     // diagnostic (stderr): per class the last forward sweep that recomputed
@@ -510,9 +530,7 @@ void enqueue_step(smoothe_run* r) {
   // the sweeps after the gradient has died launch nothing; the plain kernel
   // inside is itself conditional on some seed being unfrozen.  (Direct
   // launches: every kernel of a dead sweep returns at once.)
-  const bool big = r->in_capture && g.num_rev_items >= 100000;
-  for (int t = K; t >= 1; --t) {
-    auto sweep = [&](cudaStream_t ss, cudaStream_t sbody) {
+  auto sweep = [&](int t, cudaStream_t ss, cudaStream_t sbody) {
       launch_rev_transition(ss, sh, g, t, K, sw);
       if (sw.wmode && t == K) {  // K-state rows, W, every seed frozen at t = K
         SM_CUDA(cudaMemcpyAsync(sw.kq, cur_q, sizeof(float) * MB, cudaMemcpyDeviceToDevice, ss));
@@ -550,13 +568,13 @@ void enqueue_step(smoothe_run* r) {
                              r->rev_cursor + (size_t)t * std::max(1, sh.Bp / 128),
                              sw.glive && t < K ? sw.glive + t : nullptr,
                              sw.glive && t > 1 ? sw.glive + (t - 1) : nullptr,
-                             sw.gstamp ? sw.gstamp + ((t - 1) & 1) * (size_t)sw.nchunk * sh.M : nullptr);
+                             sw.gstamp ? sw.gstamp + ((t - 1) & 1) * (size_t)sw.nchunk * sh.M : nullptr,
+                             big && sw.wmode && t < K && !sw.plain_if);
       };
-      if (big && sw.wmode && t < K) {
-        // the plain sweep is a conditional node, skipped (no launch of its
-        // blocks) once every seed is frozen; only for large grids (C4: 171k
-        // items, 114.0 -> 108.3 ms per step), where an empty launch costs
-        // more than the conditional (C5: 6.58 -> 7.10 ms)
+      if (big && sw.wmode && t < K && sw.plain_if) {
+        // the plain sweep as a conditional node, skipped once every seed is
+        // frozen (the default instead launches it as one wave of persistent
+        // warps, which exit at once then: cheaper than the conditional)
         enqueue_if(
             ss, sbody,
             [&](cudaGraphConditionalHandle h) { launch_any_unfrozen(ss, sh, sw.wm, h); }, plain);
@@ -572,13 +590,24 @@ void enqueue_step(smoothe_run* r) {
         kmark(2, 1);
       }
     };
-    if (big && sw.glive && t < K)
+  // In the captured step of a large graph, reverse sweeps (t - rblock, t]
+  // (t < K) are one conditional node on live[t]: the sweeps after the
+  // gradient has died launch nothing (the kernels of a dead sweep inside a
+  // live block return at once)
+  for (int t = K; t >= 1;) {
+    if (big && sw.glive && t < K) {
+      const int t1 = std::max(0, t - sw.rblock);
       enqueue_if(
           s, r->stream_body,
           [&](cudaGraphConditionalHandle h) { launch_flag_if(s, sw.glive + t, h); },
-          [&](cudaStream_t bs) { sweep(bs, r->stream_body2); });
-    else
-      sweep(s, r->stream_body);
+          [&](cudaStream_t bs) {
+            for (int u = t; u > t1; --u) sweep(u, bs, r->stream_body2);
+          });
+      t = t1;
+    } else {
+      sweep(t, s, r->stream_body);
+      --t;
+    }
   }
   if (sw.wmode)  // the frozen sweeps' g_cp: one pass over the K-state with g = S
     launch_sweep_reverse(s, sh, g, r->agg, K, K, sw.kq, sw.kpi, sw.kam, nullptr, r->cp, sw.S,
@@ -742,6 +771,16 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
         SM_CUDA(cudaMemset(w.gstamp, 0xFF, sizeof(int32_t) * 2 * w.nchunk * sh.M));
       }
     }
+    {
+      auto envi = [](const char* k, int d) {
+        const char* e = std::getenv(k);
+        return e && e[0] ? std::atoi(e) : d;
+      };
+      w.fblock = w.all ? 0 : envi("SMOOTHE_FBLOCK", 16);
+      w.rblock = std::max(1, envi("SMOOTHE_RBLOCK", 8));
+      w.plain_if = envi("SMOOTHE_PLAIN_IF", 0) != 0;
+      if (w.fblock > 0) w.fchg = dalloc<int32_t>(o, slots + 1);
+    }
     alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
     for (int b = 0; b < 2; ++b) {  // consecutive: k_sweep_reset fills all four at once
@@ -757,6 +796,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
     // converged seed's g_q through, without it the reverse kernel does
     w.wmode = (wenv ? wenv[0] == '1' : r->K >= 48) && r->g->dev.num_cedge > 0;
     if (w.wmode) {
+      const char* penv = std::getenv("SMOOTHE_WSPMV_PERSIST");
+      w.wpersist = penv ? penv[0] == '1' : r->g->dev.num_witems >= 100000;
       w.W = dalloc<float>(o, (size_t)r->g->dev.num_cedge * sh.Bp);
       w.S = dalloc<float>(o, MB);
       w.kq = dalloc<float>(o, MB);
