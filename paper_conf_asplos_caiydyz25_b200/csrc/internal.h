@@ -238,6 +238,10 @@ struct SweepState {
   // k_wspmv as one wave of persistent row groups striding over the work items
   // (default for >= 100k items; SMOOTHE_WSPMV_PERSIST=0 / 1 forces)
   bool wpersist = false;
+  // [w_num_slots][nchunk] arrival counters of the long classes' chunks (the
+  // last chunk combines; zero between launches).  NULL: k_wcombine
+  // (SMOOTHE_WFUSE=0)
+  int32_t* wcnt = nullptr;
   // captured step of a large graph (>= 100k reverse items): conditional nodes
   // cost ~15 us each, so sweeps are gated in blocks: forward sweeps
   // [t, t + fblock) by one IF on fchg[t - 1] (0: no gating), reverse sweeps

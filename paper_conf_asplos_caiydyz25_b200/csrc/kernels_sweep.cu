@@ -1434,7 +1434,7 @@ __device__ __forceinline__ void wspmv_item(
     bool lead, bool check, const float* __restrict__ gq, float* __restrict__ S,
     float* __restrict__ gq_prev, float* __restrict__ part, const int32_t* __restrict__ lastchg,
     int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
-    const int32_t* __restrict__ gstamp_in) {
+    const int32_t* __restrict__ gstamp_in, int32_t* __restrict__ wcnt) {
   const int4 itm = items[row];
   const int i = itm.x, e0 = itm.y, e1 = itm.z, slot = itm.w;
   const int d = __ldg(dmin + i);
@@ -1515,9 +1515,32 @@ __device__ __forceinline__ void wspmv_item(
       }
     }
   }
-  if (slot >= 0) {  // one chunk of a long class: k_wcombine adds the chunks
+  if (slot >= 0) {  // one chunk of a long class
     st4(part + (size_t)slot * Bp + s0, acc);
-    return;
+    if (CONV || !wcnt) return;  // k_wcombine adds the chunks
+    // the class's last chunk to finish adds the partial rows in slot order
+    // (k_wcombine's order: bit-identical) and writes g_q^{t-1}_i.  Chunks sit
+    // at ptr + 64 k (slots first + k), so the first slot and the count follow
+    // from the class's child range; one counter per (class, seed chunk),
+    // reset by the last arriver.
+    const int ptr = cls_child_ptr[i], nsl = (cls_child_ptr[i + 1] - ptr + kWChunk - 1) / kWChunk;
+    const int first = slot - (e0 - ptr) / kWChunk;
+    __threadfence();
+    __syncwarp(gm);
+    int last = 0;
+    int32_t* c = wcnt + (size_t)first * gridDim.y + blockIdx.y;
+    if (lead) last = atomicAdd(c, 1) == nsl - 1;
+    if (!__shfl_sync(gm, last, (threadIdx.x % 32) / LPR * LPR)) return;
+    __threadfence();
+    if (lead) *c = 0;
+    acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int sl = first; sl < first + nsl; ++sl) {
+      const float4 p = __ldcg(reinterpret_cast<const float4*>(part + (size_t)sl * Bp + s0));
+      acc.x += p.x;
+      acc.y += p.y;
+      acc.z += p.z;
+      acc.w += p.w;
+    }
   }
   if (i == root) acc = make_float4(0.f, 0.f, 0.f, 0.f);
   float4 o = acc;
@@ -1548,7 +1571,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
     float* __restrict__ gq_prev, float* __restrict__ part, int64_t* __restrict__ frozen_count,
     const int32_t* __restrict__ lastchg, const int32_t* __restrict__ live_in,
     int32_t* __restrict__ live_out, int32_t* __restrict__ gstamp,
-    const int32_t* __restrict__ gstamp_in) {
+    const int32_t* __restrict__ gstamp_in, int32_t* __restrict__ wcnt) {
   const RowGroup<LPR, kWBlock> rg;
   if (frozen_count && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 &&
       !g_dead(live_in)) {  // profiling: a working launch?
@@ -1572,7 +1595,7 @@ __global__ void __launch_bounds__(kWBlock, LPR == 32 ? SMOOTHE_WSPMV_MINB * 64 /
   for (int row = rg.row; row < n_items; row += G)
     wspmv_item<LPR, STREAM, CONV>(row, rg.s0, Bp, root, t, dmin, items, cls_child_ptr, cls_child,
                                   W, w4, gm, lead, check, gq, S, gq_prev, part, lastchg, live_out,
-                                  gstamp, gstamp_in);
+                                  gstamp, gstamp_in, wcnt);
 }
 
 // g_q^{t-1}_i of the classes split into several chunks: their partial rows in
@@ -1699,15 +1722,19 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
     k_wspmv<LPR, ST, CV, true><<<grid, kWBlock, 0, s>>>(                                       \
         g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W,    \
         st.wm, gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out,       \
-        gstamp, gstamp_in);                                                                    \
+        gstamp, gstamp_in, wcnt);                                                              \
   } else                                                                                       \
   k_wspmv<LPR, ST, CV, false><<<grid, kWBlock, 0, s>>>(                                        \
       g.num_witems, sh.Bp, sh.root, t, g.dmin, items, g.cls_child_ptr, g.cls_child, st.W, st.wm, \
-      gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out, gstamp, gstamp_in)
+      gq, st.S, gq_prev, st.wpart, frozen_count, st.lastchg, live_in, live_out, gstamp, gstamp_in, \
+      wcnt)
   // persistent row groups (one wave of resident blocks striding over the
   // items) for large item counts: the launch of ~85k blocks costs ~45 us per
   // sweep on C4 (SMOOTHE_WSPMV_PERSIST=0 / 1 forces)
   const bool persist = st.wpersist;
+  // long classes: the last chunk combines inside k_wspmv (no k_wcombine
+  // launch per sweep) except in convergence mode
+  int32_t* wcnt = st.wcnt && !st.converge && gq_prev ? st.wcnt : nullptr;
   int dev = 0;
   SM_CUDA(cudaGetDevice(&dev));
   SM_DISPATCH_LPR(sh.Bp, {
@@ -1720,7 +1747,7 @@ void launch_wspmv(cudaStream_t s, const Shape& sh, const DevGraph& g, int t,
       else SM_WSPMV(false, false);
     }
 
-    if (g.num_wmulti > 0 && gq_prev) {
+    if (g.num_wmulti > 0 && gq_prev && !wcnt) {
       SM_LAUNCH_CHECK();
       k_wcombine<LPR><<<row_grid(g.num_wmulti, sh.Bp, LPR), kBlock, 0, s>>>(
           g.num_wmulti, sh.Bp, sh.root, t, g.dmin, g.wmulti, g.wmulti_ptr, st.wm, st.wpart,

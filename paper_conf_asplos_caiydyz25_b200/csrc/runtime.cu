@@ -805,6 +805,12 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.kam = dalloc<int32_t>(o, MB);
       w.wm = dalloc<int32_t>(o, sh.Bp);
       w.wpart = dalloc<float>(o, (size_t)std::max(1, r->g->dev.w_num_slots) * sh.Bp);
+      const char* fuse = std::getenv("SMOOTHE_WFUSE");
+      if (!(fuse && fuse[0] == '0') && r->g->dev.w_num_slots > 0) {
+        const size_t nc = (size_t)r->g->dev.w_num_slots * w.nchunk;
+        w.wcnt = dalloc<int32_t>(o, nc);
+        SM_CUDA(cudaMemset(w.wcnt, 0, sizeof(int32_t) * nc));
+      }
       r->frozen_count = dalloc<int64_t>(o, 4);  // launches, live edges / rows, rows written
       SM_CUDA(cudaMemset(r->frozen_count, 0, 4 * sizeof(int64_t)));
     }

@@ -536,6 +536,44 @@ def test_c4_graph_replay_and_direct_launches_identical(sm):
         assert outs[0][2][k] == outs[1][2][k], k
 
 
+@pytest.mark.parametrize("name,B,G,env", [
+    ("C4", 128, 16, {"SMOOTHE_WSPMV_PERSIST": "0"}),
+    ("C4", 128, 16, {"SMOOTHE_WFUSE": "0"}),
+    ("C4", 128, 16, {"SMOOTHE_RBLOCK": "1", "SMOOTHE_FBLOCK": "0", "SMOOTHE_PLAIN_IF": "1",
+                     "SMOOTHE_WSPMV_PERSIST": "0", "SMOOTHE_WFUSE": "0"}),
+    ("C5", 64, 8, {"SMOOTHE_WFUSE": "0"})])
+def test_schedule_variants_identical(sm, monkeypatch, name, B, G, env):
+    """The benchmarked C4 schedule at 128 seeds (graph replay; forward sweeps
+    gated in blocks of 16 and reverse sweeps in blocks of 8 by conditional
+    nodes; persistent k_wspmv whose last chunk of a long class combines the
+    partial rows; persistent plain reverse) against the plainer schedules it
+    replaced (per-item k_wspmv blocks, k_wcombine launches, one conditional
+    per reverse sweep, the plain sweep under its own conditional, ungated
+    forward), and C5's fused combine against k_wcombine: theta after 3 steps
+    and the best extraction bit for bit (the schedule never changes which sums
+    are formed or their order)."""
+    eg = make_config(name)
+    outs = []
+    for e in ({}, env):
+        for k in env:
+            monkeypatch.delenv(k, raising=False)
+        for k, v in e.items():
+            monkeypatch.setenv(k, v)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), B,
+                            sm.Options(penalty_group=G, rng_key=0x5EED0128))
+        run.steps(3)
+        ch, s = run.extract()
+        assert s["graph_mode"] == 1
+        outs.append((run.theta(), ch, s))
+        run.close()
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][1], outs[1][1])
+    for k in ("best_cost", "best_step", "best_seed", "last_loss"):
+        assert outs[0][2][k] == outs[1][2][k], k
+
+
 def test_graphs_and_direct_launches_identical(sm):
     eg = make_config("C2")
     outs = []
