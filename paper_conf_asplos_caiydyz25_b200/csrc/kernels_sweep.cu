@@ -203,8 +203,13 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
 // only those with work: recompute (dirty) or copy the q row (changed in the
 // previous sweep, not dirty now).  A frozen sweep is thus a few loads per row
 // group instead of one thread block per 2 classes.
+#ifndef SMOOTHE_FWD_MINB
+#define SMOOTHE_FWD_MINB 16  // min resident blocks per SM of the persistent forward (72 -> 64
+                            // registers, small spills: C4 44.6 -> 43.5 ms per step; 14 / 18 / 20:
+                            // 44.2 / 46.6 / 53.6)
+#endif
 template <int LPR>
-__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(SM_FWD_PARAMS) {
+__global__ void __launch_bounds__(kSweepBlock, SMOOTHE_FWD_MINB) k_sweep_forward(SM_FWD_PARAMS) {
   const int gl = threadIdx.x % LPR;
   const int G = gridDim.x * (kSweepBlock / LPR);
   const int g = blockIdx.x * (kSweepBlock / LPR) + (int)threadIdx.x / LPR;
@@ -248,8 +253,11 @@ __global__ void __launch_bounds__(kSweepBlock) k_sweep_forward(SM_FWD_PARAMS) {
 // same as forward_class; kept as a kernel of its own because the inlined
 // version schedules its loads worse (measured 15% slower on C5, same
 // instruction and sector counts, more long-scoreboard stalls).
+#ifndef SMOOTHE_FWDD_MINB
+#define SMOOTHE_FWDD_MINB 1
+#endif
 template <int LPR>
-__global__ void __launch_bounds__(kSweepBlock) k_sweep_forward_direct(
+__global__ void __launch_bounds__(kSweepBlock, SMOOTHE_FWDD_MINB) k_sweep_forward_direct(
     int M, int Bp, int root, int t, int all, const int32_t* __restrict__ dmin,
     const int32_t* __restrict__ dirty_cur, int32_t* __restrict__ dirty_next,
     const int32_t* __restrict__ chg_prev, int32_t* __restrict__ chg_cur, PoolArgs P,

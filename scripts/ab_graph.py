@@ -27,6 +27,7 @@ def main():
     eg = make_config(name)
     g = sm.load_egraph_from(eg, device=0)
     res = {v: [] for v in variants}
+    stream = torch.cuda.Stream()  # a real stream: handle 0 (legacy default) means none
     for rnd in range(3):
         for v in variants:
             saved = {}
@@ -34,15 +35,16 @@ def main():
                 k, val = kv.split("=")
                 saved[k] = os.environ.get(k)
                 os.environ[k] = val
-            opts = sm.Options(lam=float(np.mean(eg.u)), penalty_group=spec["group"], rng_key=rng_key(name))
+            opts = sm.Options(lam=float(np.mean(eg.u)), penalty_group=spec["group"], rng_key=rng_key(name),
+                              cuda_stream=stream.cuda_stream)
             run = sm.run_create(g, sm.CostModel.from_input(eg), spec["seeds_per_gpu"], opts)
             run.steps(3)
             run.synchronize()
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
+            e0.record(stream)
             run.steps(n)
-            e1.record()
+            e1.record(stream)
             run.synchronize()
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / n
