@@ -230,7 +230,7 @@ struct SweepState {
   // stale match only costs a read).  NULL with SMOOTHE_GLIVE=0.
   int32_t* gstamp = nullptr;
   // fchg[t] [K + 2], zeroed per step: some q row changed (bitwise) in forward
-  // sweep t.  Once a sweep changes nothing, every later sweep is the identity
+  // sweep t; fchg[0] = the last such sweep.  Once a sweep changes nothing, every later sweep is the identity
   // (no class is dirty, no row to copy forward): in the captured step of a
   // large graph, forward sweep t is a conditional node on fchg[t - 1].  NULL
   // with SMOOTHE_FSKIP=0.
@@ -251,6 +251,10 @@ struct SweepState {
   // (SMOOTHE_FBLOCK, SMOOTHE_RBLOCK, SMOOTHE_PLAIN_IF)
   int fblock = 0, rblock = 8;
   bool plain_if = false;
+  // reverse blocks as a switch node whose k_wspmv-only body skips the
+  // transitions and the plain kernel above the last changing forward sweep
+  // (SMOOTHE_RSWITCH=0: the plain IF)
+  bool rswitch = true;
 };
 // Reset the per-step sweep state (stamps, q buffers = q^0).
 void launch_sweep_reset(cudaStream_t s, const Shape& sh, const SweepState& st);
@@ -295,6 +299,8 @@ void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h);
 // sets the conditional handle to 1 iff *flag != 0
 void launch_flag_if(cudaStream_t s, const int32_t* flag, cudaGraphConditionalHandle h);
+void launch_rev_switch(cudaStream_t s, const int32_t* live, const int32_t* fchg, int t_low,
+                       cudaGraphConditionalHandle h);
 // W from the K-state rows (before reverse sweep K)
 void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                    const SweepState& st, const float* cp);

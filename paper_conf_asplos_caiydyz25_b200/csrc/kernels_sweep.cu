@@ -190,7 +190,10 @@ __device__ __forceinline__ void forward_class(SM_FWD_PARAMS, int j, int gl, int 
   if (__ballot_sync(gm, ne) == 0u) return;
   if (gl == 0) {
     chg_cur[j] = t;
-    if (P.fchg && __ldcg(P.fchg + t) == 0) __stcg(P.fchg + t, 1);
+    if (P.fchg && __ldcg(P.fchg + t) == 0) {  // fchg[0]: the last sweep with a change
+      __stcg(P.fchg + t, 1);
+      atomicMax(P.fchg, t);
+    }
   }
   for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
     dirty_next[cls_child[c]] = t + 1;
@@ -339,7 +342,10 @@ __global__ void __launch_bounds__(kSweepBlock, SMOOTHE_FWDD_MINB) k_sweep_forwar
   if (__ballot_sync(gm, ne) == 0u) return;
   if (gl == 0) {
     chg_cur[j] = t;
-    if (P.fchg && __ldcg(P.fchg + t) == 0) __stcg(P.fchg + t, 1);
+    if (P.fchg && __ldcg(P.fchg + t) == 0) {  // fchg[0]: the last sweep with a change
+      __stcg(P.fchg + t, 1);
+      atomicMax(P.fchg, t);
+    }
   }
   for (int c = cls_child_ptr[j] + gl, ce = cls_child_ptr[j + 1]; c < ce; c += LPR)
     dirty_next[cls_child[c]] = t + 1;
@@ -1819,6 +1825,23 @@ __global__ void k_any_unfrozen(cudaGraphConditionalHandle h, const int32_t* __re
 void launch_any_unfrozen(cudaStream_t s, const Shape& sh, const int32_t* wm,
                          cudaGraphConditionalHandle h) {
   k_any_unfrozen<<<1, 256, 0, s>>>(h, wm, sh.B);
+  SM_LAUNCH_CHECK();
+}
+
+// Reverse sweeps (t_low - 1, t] as a switch node: 2 (no body) when g_q^t is all
+// zero, 1 (the whole sweeps) when a sweep of the block lies within one of the
+// last forward sweep that changed a q row (fchg[0]) -- only there can a
+// transition restore a row or a seed be unfrozen --, else 0 (k_wspmv alone:
+// every seed frozen, no version to restore)
+__global__ void k_rev_switch(cudaGraphConditionalHandle h, const int32_t* __restrict__ live,
+                             const int32_t* __restrict__ fchg, int t_low) {
+  const unsigned v = __ldcg(live) == 0 ? 2u : (t_low <= __ldcg(fchg) + 1 ? 1u : 0u);
+  cudaGraphSetConditional(h, v);
+}
+
+void launch_rev_switch(cudaStream_t s, const int32_t* live, const int32_t* fchg, int t_low,
+                       cudaGraphConditionalHandle h) {
+  k_rev_switch<<<1, 1, 0, s>>>(h, live, fchg, t_low);
   SM_LAUNCH_CHECK();
 }
 

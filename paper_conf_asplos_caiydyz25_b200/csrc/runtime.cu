@@ -360,6 +360,36 @@ void enqueue_if(cudaStream_t s, cudaStream_t sb, SetF set, BodyF body) {
   SM_CUDA(cudaStreamUpdateCaptureDependencies(s, &node, 1, cudaStreamSetCaptureDependencies));
 }
 
+// A two-body switch node: `set` launches the kernel that sets the handle;
+// value 0 runs body0, 1 runs body1, anything else nothing.
+template <class SetF, class B0, class B1>
+void enqueue_switch2(cudaStream_t s, cudaStream_t sb, SetF set, B0 body0, B1 body1) {
+  cudaStreamCaptureStatus st;
+  cudaGraph_t graph = nullptr;
+  const cudaGraphNode_t* deps = nullptr;
+  size_t ndeps = 0;
+  SM_CUDA(cudaStreamGetCaptureInfo(s, &st, nullptr, &graph, &deps, &ndeps));
+  cudaGraphConditionalHandle h;
+  SM_CUDA(cudaGraphConditionalHandleCreate(&h, graph, 0, 0));
+  set(h);
+  SM_CUDA(cudaStreamGetCaptureInfo(s, &st, nullptr, &graph, &deps, &ndeps));
+  cudaGraphNodeParams p = {};
+  p.type = cudaGraphNodeTypeConditional;
+  p.conditional.handle = h;
+  p.conditional.type = cudaGraphCondTypeSwitch;
+  p.conditional.size = 2;
+  cudaGraphNode_t node;
+  SM_CUDA(cudaGraphAddNode(&node, graph, deps, ndeps, &p));
+  cudaGraph_t b0 = p.conditional.phGraph_out[0], b1 = p.conditional.phGraph_out[1];
+  SM_CUDA(cudaStreamBeginCaptureToGraph(sb, b0, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
+  body0(sb);
+  SM_CUDA(cudaStreamEndCapture(sb, &b0));
+  SM_CUDA(cudaStreamBeginCaptureToGraph(sb, b1, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
+  body1(sb);
+  SM_CUDA(cudaStreamEndCapture(sb, &b1));
+  SM_CUDA(cudaStreamUpdateCaptureDependencies(s, &node, 1, cudaStreamSetCaptureDependencies));
+}
+
 // Decode (P279, P103-111), its discrete cost and keep-best (P297) on stream ds.
 // With the decode stream (overlap), it uses its own scratch buffers.
 void enqueue_decode(smoothe_run* r, cudaStream_t ds, PhaseMarks* pm) {
@@ -595,7 +625,26 @@ void enqueue_step(smoothe_run* r) {
   // gradient has died launch nothing (the kernels of a dead sweep inside a
   // live block return at once)
   for (int t = K; t >= 1;) {
-    if (big && sw.glive && t < K) {
+    if (big && sw.glive && t < K && sw.wmode && sw.fchg && sw.rswitch) {
+      // a switch node: nothing (dead), k_wspmv alone (every seed frozen and
+      // no row to restore: the block lies above the last forward sweep with
+      // a change), or the whole sweeps
+      const int t1 = std::max(0, t - sw.rblock);
+      enqueue_switch2(
+          s, r->stream_body,
+          [&](cudaGraphConditionalHandle h) {
+            launch_rev_switch(s, sw.glive + t, sw.fchg, t1 + 1, h);
+          },
+          [&](cudaStream_t bs) {
+            for (int u = t; u > t1; --u)
+              launch_wspmv(bs, sh, g, u, sw, r->gq[u & 1], u > 1 ? r->gq[(u - 1) & 1] : nullptr,
+                           nullptr);
+          },
+          [&](cudaStream_t bs) {
+            for (int u = t; u > t1; --u) sweep(u, bs, r->stream_body2);
+          });
+      t = t1;
+    } else if (big && sw.glive && t < K) {
       const int t1 = std::max(0, t - sw.rblock);
       enqueue_if(
           s, r->stream_body,
@@ -779,7 +828,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.fblock = w.all ? 0 : envi("SMOOTHE_FBLOCK", 16);
       w.rblock = std::max(1, envi("SMOOTHE_RBLOCK", 8));
       w.plain_if = envi("SMOOTHE_PLAIN_IF", 0) != 0;
-      if (w.fblock > 0) w.fchg = dalloc<int32_t>(o, slots + 1);
+      w.rswitch = envi("SMOOTHE_RSWITCH", 1) != 0;
+      if (!w.all) w.fchg = dalloc<int32_t>(o, slots + 1);
     }
     alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);

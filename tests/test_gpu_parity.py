@@ -536,16 +536,19 @@ def test_c4_graph_replay_and_direct_launches_identical(sm):
         assert outs[0][2][k] == outs[1][2][k], k
 
 
-@pytest.mark.parametrize("name,B,G,env", [
-    ("C4", 128, 16, {"SMOOTHE_WSPMV_PERSIST": "0"}),
-    ("C4", 128, 16, {"SMOOTHE_WFUSE": "0"}),
-    ("C4", 128, 16, {"SMOOTHE_RBLOCK": "1", "SMOOTHE_FBLOCK": "0", "SMOOTHE_PLAIN_IF": "1",
-                     "SMOOTHE_WSPMV_PERSIST": "0", "SMOOTHE_WFUSE": "0"}),
-    ("C5", 64, 8, {"SMOOTHE_WFUSE": "0"})])
-def test_schedule_variants_identical(sm, monkeypatch, name, B, G, env):
+@pytest.mark.parametrize("name,B,G,conv,env", [
+    ("C4", 128, 16, False, {"SMOOTHE_WSPMV_PERSIST": "0"}),
+    ("C4", 128, 16, False, {"SMOOTHE_WFUSE": "0"}),
+    ("C4", 128, 16, False, {"SMOOTHE_RSWITCH": "0"}),
+    ("C4", 128, 16, True, {"SMOOTHE_RSWITCH": "0"}),
+    ("C4", 128, 16, False, {"SMOOTHE_RBLOCK": "1", "SMOOTHE_FBLOCK": "0", "SMOOTHE_PLAIN_IF": "1",
+                            "SMOOTHE_WSPMV_PERSIST": "0", "SMOOTHE_WFUSE": "0", "SMOOTHE_RSWITCH": "0"}),
+    ("C5", 64, 8, False, {"SMOOTHE_WFUSE": "0"})])
+def test_schedule_variants_identical(sm, monkeypatch, name, B, G, conv, env):
     """The benchmarked C4 schedule at 128 seeds (graph replay; forward sweeps
     gated in blocks of 16 and reverse sweeps in blocks of 8 by conditional
-    nodes; persistent k_wspmv whose last chunk of a long class combines the
+    nodes -- a reverse block above the last forward sweep that changed a row
+    runs k_wspmv alone --; persistent k_wspmv whose last chunk of a long class combines the
     partial rows; persistent plain reverse) against the plainer schedules it
     replaced (per-item k_wspmv blocks, k_wcombine launches, one conditional
     per reverse sweep, the plain sweep under its own conditional, ungated
@@ -561,7 +564,7 @@ def test_schedule_variants_identical(sm, monkeypatch, name, B, G, env):
             monkeypatch.setenv(k, v)
         g = sm.load_egraph_from(eg)
         run = sm.run_create(g, sm.CostModel.from_input(eg), B,
-                            sm.Options(penalty_group=G, rng_key=0x5EED0128))
+                            sm.Options(penalty_group=G, rng_key=0x5EED0128, converge=conv))
         run.steps(3)
         ch, s = run.extract()
         assert s["graph_mode"] == 1
