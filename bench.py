@@ -309,6 +309,13 @@ def roofline(args, eg, prof, Bl, K, steps_ms):
             extra["frac_8d_full_model"] = (bm["reverse_sweep"] * Bl * N / (per_launch_ms * 1e-3)
                                            / 1e9 / peak)
             alg_override = live_bytes
+            # the committed ncu capture (profiles/traffic.json) is of one fully
+            # live frozen sweep (launch 20 of a step: every class edge live);
+            # its own live bytes are the full stream, against which traffic
+            # shows re-reads
+            extra["traffic_launch"] = ("ncu --set full of one fully live frozen sweep (every class "
+                                       "edge live): compare with full_stream_model's bytes")
+            extra["full_stream_bytes"] = w_bytes
     else:
         per_launch_ms = kms[dom] / max(1, kn[dom])
         unit_8d = bm["forward_sweep" if dom == "forward" else "reverse_sweep"]
