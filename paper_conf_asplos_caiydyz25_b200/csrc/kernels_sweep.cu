@@ -1373,8 +1373,13 @@ void launch_sweep_reverse(cudaStream_t s, const Shape& sh, const DevGraph& g, Ag
 // rows forward sweep t recomputed) clears wm[s] when a restored row differs
 // in seed s.  Decisions are per seed, so results do not depend on the batch.
 // ---------------------------------------------------------------------------
-// One row group per class edge (i, j): W_ij = sum over its e-nodes k (ascending)
-// of cp_k c_kj, with pi_j / am_j / q_i loaded once.
+// One row group per EP class edges (i, j), interleaved so that their loads
+// are in flight together (the kernel is bound by its dependent gathers):
+// W_ij = sum over the edge's e-nodes k (ascending) of cp_k c_kj, with pi_j /
+// am_j / q_i loaded once per edge.
+#ifndef SMOOTHE_WBUILD_EP
+#define SMOOTHE_WBUILD_EP 2
+#endif
 template <int LPR>
 __global__ void __launch_bounds__(kBlock) k_wbuild(
     int64_t n_cedge, int Bp, float wI, float wC, const int32_t* __restrict__ cedge_class,
@@ -1382,38 +1387,68 @@ __global__ void __launch_bounds__(kBlock) k_wbuild(
     const int32_t* __restrict__ cls_child, const float* __restrict__ cp,
     const float* __restrict__ kq, const float* __restrict__ kpi, const int32_t* __restrict__ kam,
     float* __restrict__ W) {
+  constexpr int EP = SMOOTHE_WBUILD_EP;
   const RowGroup<LPR> rg;
-  const int64_t ce = (int64_t)blockIdx.x * (kBlock / LPR) + rg.sub;
-  if (ce >= n_cedge) return;
+  const int64_t ce0 = ((int64_t)blockIdx.x * (kBlock / LPR) + rg.sub) * EP;
+  if (ce0 >= n_cedge) return;
   const bool HI = wI != 0.f, HC = wC != 0.f;
-  const int i = cedge_class[ce], j = cls_child[ce];
-  const float4 qp = ld4(kq + (size_t)i * Bp + rg.s0);
-  const float4 P = HI ? ld4(kpi + (size_t)j * Bp + rg.s0) : make_float4(0.f, 0.f, 0.f, 0.f);
-  const int4 A = ld4i(kam + (size_t)j * Bp + rg.s0);
-  float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (int a = cedge_ptr[ce]; a < cedge_ptr[ce + 1]; ++a) {
-    const int k = cedge_node[a];
-    const float4 cv = ld4(cp + (size_t)k * Bp + rg.s0);
+  int64_t ce[EP];
+  int i[EP], j[EP], a0[EP], a1[EP];
 #pragma unroll
-    for (int x = 0; x < 4; ++x) {  // node_consts of k_sweep_reverse, then c_kj
-      const float om = __fsub_rn(1.f, __fmul_rn(comp(cv, x), comp(qp, x)));
-      const bool nz = om != 0.f;
-      float r;
-      asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
-      const float rom = HI && nz ? r : 1.f;
-      const float cC = HI && nz ? wC * om : wC;
-      float c = HI ? wI * fmaxf((nz ? 1.f : -1.f) * comp(P, x), 0.f) : 0.f;
-      if (HC && comp(A, x) == k) c += cC;
-      comp(w, x) = fmaf(comp(cv, x), c * rom, comp(w, x));
+  for (int e = 0; e < EP; ++e) {
+    ce[e] = ce0 + e < n_cedge ? ce0 + e : ce0;  // a tail pair repeats its first edge (same value)
+    i[e] = cedge_class[ce[e]];
+    j[e] = cls_child[ce[e]];
+    a0[e] = cedge_ptr[ce[e]];
+    a1[e] = cedge_ptr[ce[e] + 1];
+  }
+  float4 qp[EP], P[EP], w[EP];
+  int4 A[EP];
+#pragma unroll
+  for (int e = 0; e < EP; ++e) {
+    qp[e] = ld4(kq + (size_t)i[e] * Bp + rg.s0);
+    P[e] = HI ? ld4(kpi + (size_t)j[e] * Bp + rg.s0) : make_float4(0.f, 0.f, 0.f, 0.f);
+    A[e] = ld4i(kam + (size_t)j[e] * Bp + rg.s0);
+    w[e] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  int n = 0;
+#pragma unroll
+  for (int e = 0; e < EP; ++e) n = max(n, a1[e] - a0[e]);
+  for (int u = 0; u < n; ++u) {
+    int k[EP];
+    float4 cv[EP];
+#pragma unroll
+    for (int e = 0; e < EP; ++e) {
+      k[e] = a0[e] + u < a1[e] ? cedge_node[a0[e] + u] : -1;
+      if (k[e] >= 0) cv[e] = ld4(cp + (size_t)k[e] * Bp + rg.s0);
+    }
+#pragma unroll
+    for (int e = 0; e < EP; ++e) {
+      if (k[e] < 0) continue;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {  // node_consts of k_sweep_reverse, then c_kj
+        const float om = __fsub_rn(1.f, __fmul_rn(comp(cv[e], x), comp(qp[e], x)));
+        const bool nz = om != 0.f;
+        float r;
+        asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(om));
+        const float rom = HI && nz ? r : 1.f;
+        const float cC = HI && nz ? wC * om : wC;
+        float c = HI ? wI * fmaxf((nz ? 1.f : -1.f) * comp(P[e], x), 0.f) : 0.f;
+        if (HC && comp(A[e], x) == k[e]) c += cC;
+        comp(w[e], x) = fmaf(comp(cv[e], x), c * rom, comp(w[e], x));
+      }
     }
   }
-  st4(W + (size_t)ce * Bp + rg.s0, w);
+#pragma unroll
+  for (int e = 0; e < EP; ++e)
+    if (ce0 + e < n_cedge) st4(W + (size_t)ce[e] * Bp + rg.s0, w[e]);
 }
 
 void launch_wbuild(cudaStream_t s, const Shape& sh, const DevGraph& g, Agg a,
                    const SweepState& st, const float* cp) {
   SM_DISPATCH_LPR(sh.Bp, {
-    k_wbuild<LPR><<<row_grid((int)g.num_cedge, sh.Bp, LPR), kBlock, 0, s>>>(
+    k_wbuild<LPR><<<row_grid((int)((g.num_cedge + SMOOTHE_WBUILD_EP - 1) / SMOOTHE_WBUILD_EP),
+                             sh.Bp, LPR), kBlock, 0, s>>>(
         g.num_cedge, sh.Bp, a.wI, a.wC, g.cedge_class, g.cedge_ptr, g.cedge_node, g.cls_child,
         cp, st.kq, st.kpi, st.kam, st.W);
   });
