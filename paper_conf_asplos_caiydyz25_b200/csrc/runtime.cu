@@ -833,7 +833,8 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.rblock = std::max(1, envi("SMOOTHE_RBLOCK", 8));
       w.plain_if = envi("SMOOTHE_PLAIN_IF", 0) != 0;
       w.rswitch = envi("SMOOTHE_RSWITCH", 1) != 0;
-      if (!w.all) w.fchg = dalloc<int32_t>(o, slots + 1);
+      // (the change flags feed the conditional nodes of large graphs only)
+      if (!w.all && r->g->dev.num_rev_items >= 100000) w.fchg = dalloc<int32_t>(o, slots + 1);
     }
     alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);
