@@ -249,6 +249,7 @@ struct SweepState {
   // wave of persistent warps (an all-frozen sweep then costs a few us) unless
   // plain_if, which puts it under an IF on "some seed unfrozen"
   // (SMOOTHE_FBLOCK, SMOOTHE_RBLOCK, SMOOTHE_PLAIN_IF)
+  bool big_sched = false;  // the gated schedule below (>= 100k reverse items; SMOOTHE_BIG_SCHED)
   int fblock = 0, rblock = 8;
   bool plain_if = false;
   // reverse blocks as a switch node whose k_wspmv-only body skips the

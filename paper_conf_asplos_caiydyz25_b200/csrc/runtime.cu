@@ -467,7 +467,7 @@ void enqueue_step(smoothe_run* r) {
   // sweep ~46 of 207), so the blocks after it launch nothing.  Gated in blocks
   // because a conditional node costs more than an empty sweep (~10 us).
   // (Direct launches: the kernels of such a sweep find no dirty class.)
-  const bool big = r->in_capture && g.num_rev_items >= 100000;
+  const bool big = r->in_capture && r->sw.big_sched;
   const int fb = big && r->sw.fchg ? r->sw.fblock : 0;
   for (int t = 1; t <= K;) {
     if (fb > 0 && t >= 2) {
@@ -834,7 +834,12 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.plain_if = envi("SMOOTHE_PLAIN_IF", 0) != 0;
       w.rswitch = envi("SMOOTHE_RSWITCH", 1) != 0;
       // (the change flags feed the conditional nodes of large graphs only)
-      if (!w.all && r->g->dev.num_rev_items >= 100000) w.fchg = dalloc<int32_t>(o, slots + 1);
+      // large graphs (>= 100k reverse items) get the gated schedule of the
+      // captured step; SMOOTHE_BIG_SCHED=1 / 0 forces it on / off (tests and
+      // sanitizer runs of the gated schedule on small graphs)
+      const int bs = envi("SMOOTHE_BIG_SCHED", -1);
+      w.big_sched = bs >= 0 ? bs != 0 : r->g->dev.num_rev_items >= 100000;
+      if (!w.all && w.big_sched) w.fchg = dalloc<int32_t>(o, slots + 1);
     }
     alloc_pools(r, initial_pool_rows(r));
     int32_t* stamps = dalloc<int32_t>(o, 4 * (size_t)sh.M);

@@ -593,6 +593,43 @@ def test_schedule_variants_identical(sm, monkeypatch, name, B, G, conv, env):
         assert outs[0][2][k] == outs[1][2][k], k
 
 
+@pytest.mark.parametrize("agg,conv", [("hybrid", False), ("independent", False), ("correlated", False),
+                                      ("hybrid", True)])
+def test_gated_schedule_small_graph(sm, orc, monkeypatch, agg, conv):
+    """The large-graph schedule of the captured step (forward / reverse
+    sweeps gated in blocks by conditional and switch nodes, persistent
+    k_wspmv and plain reverse, dead-gradient skipping, frozen sweeps) forced
+    on C2 with K = 150 (SMOOTHE_BIG_SCHED=1): bit for bit the ungated graph
+    and direct launches after 5 steps, then a debug step from that state
+    against the oracle."""
+    eg = make_config("C2")
+    for k, v in (("SMOOTHE_GLIVE", "1"), ("SMOOTHE_REV_W", "1"), ("SMOOTHE_WSPMV_PERSIST", "1"),
+                 ("SMOOTHE_RBLOCK", "4"), ("SMOOTHE_FBLOCK", "4")):
+        monkeypatch.setenv(k, v)
+    outs = []
+    for big, graphs in (("1", True), ("0", True), ("1", False)):
+        monkeypatch.setenv("SMOOTHE_BIG_SCHED", big)
+        g = sm.load_egraph_from(eg)
+        run = sm.run_create(g, sm.CostModel.from_input(eg), 64,
+                            sm.Options(penalty_group=8, rng_key=0x5EED0150, prop_iters=150,
+                                       assumption=agg, converge=conv, use_graphs=graphs))
+        run.steps(5)
+        ch, s = run.extract()
+        assert s["graph_mode"] == (1 if graphs else 0)
+        outs.append((run.theta(), ch, s, run.state()))
+        run.close()
+        g.close()
+    for o in outs[1:]:
+        assert np.array_equal(outs[0][0], o[0])
+        assert np.array_equal(outs[0][1], o[1])
+        for k in ("best_cost", "best_step", "best_seed", "last_loss"):
+            assert outs[0][2][k] == o[2][k], k
+    if not conv:
+        th, m, v, n = outs[0][3]
+        compare_step(sm, orc, eg, 64, 8, agg=agg, theta=th, m=m, v=v, step_index=n, K=150,
+                     label=f"C2_gated_{agg}")
+
+
 def test_graphs_and_direct_launches_identical(sm):
     eg = make_config("C2")
     outs = []
