@@ -833,10 +833,10 @@ void alloc_state(smoothe_run* r, const smoothe_cost_model* cost) {
       w.rblock = std::max(1, envi("SMOOTHE_RBLOCK", 8));
       w.plain_if = envi("SMOOTHE_PLAIN_IF", 0) != 0;
       w.rswitch = envi("SMOOTHE_RSWITCH", 1) != 0;
-      // (the change flags feed the conditional nodes of large graphs only)
       // large graphs (>= 100k reverse items) get the gated schedule of the
-      // captured step; SMOOTHE_BIG_SCHED=1 / 0 forces it on / off (tests and
-      // sanitizer runs of the gated schedule on small graphs)
+      // captured step, whose conditional nodes read the forward change flags;
+      // SMOOTHE_BIG_SCHED=1 / 0 forces it on / off (tests of the gated
+      // schedule on small graphs)
       const int bs = envi("SMOOTHE_BIG_SCHED", -1);
       w.big_sched = bs >= 0 ? bs != 0 : r->g->dev.num_rev_items >= 100000;
       if (!w.all && w.big_sched) w.fchg = dalloc<int32_t>(o, slots + 1);
